@@ -1,0 +1,191 @@
+/*
+ * ascetic.h — C ABI of libascetic.so, the B200-native hot path of Ascetic
+ * (Tang et al., "Ascetic: Enhancing Cross-Iterations Data Efficiency in
+ * Out-of-Memory Graph Processing on GPUs", ICPP '21).
+ *
+ * Citations: "P:NNN" = line NNN of the paper text; "§8(x)" = SURVEY.md.
+ *
+ * What the library does, per iteration of a push-based vertex-centric BSP
+ * algorithm over a CSR graph whose edges exceed a capped device budget
+ * (§3.1):
+ *   1. GenDataMap: StaticMap = Active AND Static, On-demand Map = StaticMap XOR
+ *      Active (Fig. 4), compacted into a hit queue and the
+ *      on-demand request sized by degrees.
+ *   2. Static Computing on the resident Static Region (Fig. 4 (3))
+ *      overlapped with the On-demand transfer (Fig. 5).
+ *   3. On-demand Computing on chunks of the On-demand Region, fragmented when the
+ *      request exceeds the region (§3.3; Fig. 4 (5)).
+ *   4. Next active set "generated based on the connected edges".
+ * The device memory split follows Eq. 1/Eq. 2 (§3.3, K = 10 %,
+ * P:856-859) with the front prefix as initial static content (§5).
+ *
+ * Conventions for every call:
+ *   - returns ASCETIC_OK (0) or a negative ascetic_status; no C++ exception
+ *     crosses the ABI; ascetic_last_error() gives a thread-local message.
+ *   - one context per process (one GPU per process); calls are NOT thread-safe.
+ *   - host pointers are plain host memory; the library never frees caller memory.
+ *   - state machine: UNLOADED --load_csr--> LOADED --set_budget--> READY
+ *     --run--> READY (run and set_budget may repeat); out-of-order => ESTATE.
+ */
+#ifndef ASCETIC_H
+#define ASCETIC_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    ASCETIC_OK = 0,
+    ASCETIC_EINVAL = -1,       /* bad argument (message says which) */
+    ASCETIC_ESTATE = -2,       /* call out of order */
+    ASCETIC_ENOMEM = -3,       /* device allocation failed, or budget too small for a chunk */
+    ASCETIC_EHOSTMEM = -4,     /* host pin / allocation failed */
+    ASCETIC_ECUDA = -5,        /* CUDA runtime error (message has cudaGetErrorString) */
+    ASCETIC_ENCCL = -6,        /* collective error (multi-GPU) */
+    ASCETIC_EUNSUPPORTED = -7  /* feature not built */
+} ascetic_status;
+
+typedef enum { ASCETIC_BFS = 0, ASCETIC_SSSP = 1, ASCETIC_CC = 2, ASCETIC_PR = 3 } ascetic_algo;
+
+/* load_csr flags */
+enum {
+    ASCETIC_SYMMETRIC = 1u,   /* caller asserts both directions are stored; required for CC and PR */
+    ASCETIC_COPY = 2u,        /* copy into library-owned pinned memory instead of pinning in place */
+    ASCETIC_VALIDATE = 4u,    /* O(m) check that every neighbour id < n */
+    ASCETIC_PAIRS = 8u        /* nbr holds 2m uint32: interleaved (id, weight) per arc */
+};
+
+/* Tuning knobs (ascetic_set_option). None changes what is computed or the
+ * per-iteration payload bytes; they change chunking and the transfer mechanism. */
+typedef enum {
+    ASCETIC_OPT_CHUNK_CAP = 1,     /* bytes; 0 = from the placer (C/2). Clamped to the placer's cap, multiple of 16 */
+    ASCETIC_OPT_XFER_MODE = 2,     /* 0 = auto, 1 = zero-copy SM gather only, 2 = copy-engine DMA of runs only */
+    ASCETIC_OPT_DMA_MIN_RUN = 3,   /* bytes: auto mode uses DMA when every run piece averages >= this */
+    ASCETIC_OPT_OVERLAP = 4,       /* 1 (default) = static compute overlaps the transfer; 0 = serialize (ablation, Fig. 8) */
+    ASCETIC_OPT_KEEP_STATIC = 5,   /* 1 = keep the Static Region filled across runs (fill counted once) ; default 0 */
+    ASCETIC_OPT_HUB_DEGREE = 6,    /* hit-queue degree at/above which a list is split across CTAs (default 2048) */
+    ASCETIC_OPT_TIMING = 7         /* 1 (default) = per-iteration phase timing with CUDA events */
+} ascetic_option;
+
+typedef struct {
+    int32_t algo;
+    uint32_t iterations;          /* executed expansions with non-empty A_t (PR: max_iters) */
+    uint64_t n, m;                /* vertices, stored arcs */
+    uint32_t b_e;                 /* payload bytes per arc: 4, or 8 with ASCETIC_PAIRS */
+    uint32_t rank, world;
+    uint64_t s;                   /* static vertices are [0, s) (front prefix) */
+    uint64_t budget_bytes;        /* B: Static + On-demand edge regions */
+    uint64_t static_reserved;     /* Ms = R*B floored to 16 KiB */
+    uint64_t static_bytes;        /* b_e * off[s] actually resident */
+    uint64_t ondemand_bytes;      /* C = B - Ms */
+    uint64_t chunk_cap;           /* bytes per on-demand chunk buffer (2 buffers) */
+    double static_fraction_used;  /* R */
+    uint64_t h2d_payload_bytes;   /* Σ_t miss bytes (the parity target) */
+    uint64_t h2d_static_fill_bytes;
+    uint64_t h2d_other_bytes;     /* padding/metadata H2D (expected 0) */
+    uint64_t d2h_bytes;           /* run lists + counters read back */
+    uint64_t active_arcs_total;   /* Σ_t Σ_{v∈A_t} deg(v) */
+    uint64_t chunks_total;
+    uint64_t dma_chunks, gather_chunks;
+    double time_run_s;            /* ascetic_run wall time incl. fill, all H2D, all exchange */
+    double time_fill_s;
+    double time_h2d_busy_s;       /* copy-stream busy time (sum of chunk transfers) */
+    double gteps;                 /* active_arcs_total / time_run_s / 1e9 */
+    double gteps_excl_fill;
+    uint64_t vertex_state_bytes;  /* device bytes outside the edge budget */
+} ascetic_stats_t;
+
+typedef struct {
+    uint32_t t;
+    uint32_t rank;
+    uint64_t nA, nH, nM, nruns;
+    uint64_t active_arcs, hit_arcs, miss_bytes;
+    uint64_t digest;              /* Σ_w splitmix64(w ^ word_w * 0x9E3779B97F4A7C15) over A_t's bitmap */
+    uint32_t chunks;
+    uint32_t mode;                /* 1 = zero-copy gather, 2 = DMA */
+    float ms_classify, ms_static, ms_ondemand, ms_h2d, ms_finalize, ms_exchange, ms_total;
+} ascetic_iter_stats_t;
+
+/*
+ * Load a CSR graph ("The graph is presented in the CSR format").
+ *   n       vertices (< 2^32 - 1)
+ *   m       stored arcs (both directions for symmetric graphs)
+ *   off     host uint64[n+1], off[0] = 0, non-decreasing, off[n] = m; copied to the device
+ *   nbr     host uint32[m] neighbour ids, or uint32[2m] (id, weight) pairs with ASCETIC_PAIRS
+ *   wgt     host uint32[m] weights or NULL; if given (without PAIRS) the library builds
+ *           its own interleaved pinned copy
+ *   flags   ASCETIC_* load flags
+ * Ownership: without ASCETIC_COPY the nbr array is pinned IN PLACE (cudaHostRegister,
+ * read-only) and must stay alive and unmodified until ascetic_unload() or the next
+ * load_csr. Memory already page-locked (cudaHostAlloc / torch pin_memory) is used as is.
+ * Errors: EINVAL (off[0] != 0, non-monotone off, off[n] != m, ids >= n with VALIDATE,
+ * wgt with PAIRS), EHOSTMEM (pinning), ENOMEM/ECUDA (device offsets).
+ */
+int ascetic_load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_t* nbr,
+                     const uint32_t* wgt, uint32_t flags);
+
+/*
+ * Split the device edge budget (§3.3):
+ *   bytes            B = Static Region + On-demand Region (vertex state is accounted outside)
+ *   static_fraction  R in [0,1] fixes the split; < 0 selects Eq. 2 with K = 0.10,
+ *                    clamped to [0,1]. NaN or > 1 => EINVAL.
+ * Ms = floor(R*B / 16 KiB) * 16 KiB (<= D), s = max{v : b_e*off[v] <= Ms}, C = B - Ms,
+ * chunk cap = floor(C/2/16)*16. Allocates the static buffer (b_e*off[s] bytes) and two
+ * chunk buffers once. ENOMEM if s < n and the chunk cap is below 16 bytes, or allocation fails.
+ */
+int ascetic_set_budget(uint64_t bytes, double static_fraction);
+
+/* The placement set_budget would choose, computed on the host only (no device, no state):
+ * same arguments as set_budget plus the CSR offsets and payload bytes per arc. */
+typedef struct {
+    double R;
+    uint64_t D, B, Ms, s, static_bytes, C, cap;
+} ascetic_placement_t;
+int ascetic_place(uint64_t n, const uint64_t* off, uint32_t b_e, uint64_t bytes, double static_fraction,
+                  ascetic_placement_t* out);
+
+/* Tuning knob (see ascetic_option). Valid in LOADED or READY state. */
+int ascetic_set_option(int option, int64_t value);
+
+/*
+ * Run one algorithm to completion (SURVEY §8(c) definitions, Jacobi/BSP semantics):
+ *   algo       ascetic_algo. SSSP needs weights (PAIRS or wgt). CC/PR need ASCETIC_SYMMETRIC.
+ *   source     BFS/SSSP source (< n), ignored for CC/PR
+ *   max_iters  0 = until the active set is empty; PR runs exactly max_iters (must be >= 1)
+ * The static fill (one H2D of the front prefix) is part of the run unless KEEP_STATIC
+ * kept it from a previous run. Results stay on the device until ascetic_get_result.
+ */
+int ascetic_run(int algo, uint32_t source, uint32_t max_iters);
+
+/* Statistics of the last run. per_iter may be NULL; up to cap entries are written.
+ * Returns the number of iteration records available (>= 0) or a negative status. */
+int ascetic_stats(ascetic_stats_t* out, ascetic_iter_stats_t* per_iter, uint32_t cap);
+
+/* Copy the last run's result to host_dst: n x uint32 (levels / distances / labels,
+ * UINT32_MAX = unreached) or n x float (PageRank). bytes must be >= 4n. */
+int ascetic_get_result(void* host_dst, uint64_t bytes);
+
+/* Multi-GPU (one process per GPU, §8(e)): fetch a 128-byte unique id on rank 0,
+ * share it out of band (torch.distributed broadcast), then call comm_init on every
+ * rank BEFORE load_csr. Returns EUNSUPPORTED when built without NCCL. */
+int ascetic_get_unique_id(void* out128);
+int ascetic_comm_init(int rank, int world, const void* uid128, int device);
+
+/* Device to use (before load_csr); default = current device. */
+int ascetic_set_device(int device);
+
+/* Release every device buffer and unpin host memory; back to UNLOADED. */
+void ascetic_unload(void);
+
+/* Thread-local message of the last failing call ("" if none). */
+const char* ascetic_last_error(void);
+
+/* Library version string. */
+const char* ascetic_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ASCETIC_H */

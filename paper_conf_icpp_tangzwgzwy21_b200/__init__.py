@@ -1,0 +1,192 @@
+"""ascetic-b200: B200-native hot path of Ascetic (Tang et al., ICPP '21).
+
+Thin ctypes binding over libascetic.so (include/ascetic.h). Argument marshalling only:
+every step of the path (classification, compaction, transfer, edge kernels, finalize)
+runs in the library's sm_100a kernels. There is NO CPU fallback: importing this package
+without the built library raises.
+
+    import paper_conf_icpp_tangzwgzwy21_b200 as asc
+    asc.load_csr(off, nbr, symmetric=True)        # host CSR (uint64 off, uint32 nbr)
+    asc.set_budget(bytes, static_fraction=-1.0)   # Eq. 2 split
+    asc.run("bfs", source=0)                      # or "sssp", "cc", "pr"
+    st, iters = asc.stats()
+    levels = asc.get_result()
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libascetic.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} is not built; run `python -c 'import __graft_entry__ as g; g.build()'` "
+                      "(there is no CPU fallback)")
+
+_lib = ctypes.CDLL(LIB_PATH)
+
+OK, EINVAL, ESTATE, ENOMEM, EHOSTMEM, ECUDA, ENCCL, EUNSUPPORTED = 0, -1, -2, -3, -4, -5, -6, -7
+STATUS = {0: "OK", -1: "EINVAL", -2: "ESTATE", -3: "ENOMEM", -4: "EHOSTMEM", -5: "ECUDA", -6: "ENCCL",
+          -7: "EUNSUPPORTED"}
+ALGOS = {"bfs": 0, "sssp": 1, "cc": 2, "pr": 3}
+SYMMETRIC, COPY, VALIDATE, PAIRS = 1, 2, 4, 8
+OPTIONS = {"chunk_cap": 1, "xfer_mode": 2, "dma_min_run": 3, "overlap": 4, "keep_static": 5,
+           "hub_degree": 6, "timing": 7}
+INF = 0xFFFFFFFF
+
+
+class Stats(ctypes.Structure):
+    _fields_ = [("algo", ctypes.c_int32), ("iterations", ctypes.c_uint32),
+                ("n", ctypes.c_uint64), ("m", ctypes.c_uint64), ("b_e", ctypes.c_uint32),
+                ("rank", ctypes.c_uint32), ("world", ctypes.c_uint32),
+                ("s", ctypes.c_uint64), ("budget_bytes", ctypes.c_uint64), ("static_reserved", ctypes.c_uint64),
+                ("static_bytes", ctypes.c_uint64), ("ondemand_bytes", ctypes.c_uint64),
+                ("chunk_cap", ctypes.c_uint64), ("static_fraction_used", ctypes.c_double),
+                ("h2d_payload_bytes", ctypes.c_uint64), ("h2d_static_fill_bytes", ctypes.c_uint64),
+                ("h2d_other_bytes", ctypes.c_uint64), ("d2h_bytes", ctypes.c_uint64),
+                ("active_arcs_total", ctypes.c_uint64), ("chunks_total", ctypes.c_uint64),
+                ("dma_chunks", ctypes.c_uint64), ("gather_chunks", ctypes.c_uint64),
+                ("time_run_s", ctypes.c_double), ("time_fill_s", ctypes.c_double),
+                ("time_h2d_busy_s", ctypes.c_double), ("gteps", ctypes.c_double),
+                ("gteps_excl_fill", ctypes.c_double), ("vertex_state_bytes", ctypes.c_uint64)]
+
+
+class IterStats(ctypes.Structure):
+    _fields_ = [("t", ctypes.c_uint32), ("rank", ctypes.c_uint32),
+                ("nA", ctypes.c_uint64), ("nH", ctypes.c_uint64), ("nM", ctypes.c_uint64), ("nruns", ctypes.c_uint64),
+                ("active_arcs", ctypes.c_uint64), ("hit_arcs", ctypes.c_uint64), ("miss_bytes", ctypes.c_uint64),
+                ("digest", ctypes.c_uint64), ("chunks", ctypes.c_uint32), ("mode", ctypes.c_uint32),
+                ("ms_classify", ctypes.c_float), ("ms_static", ctypes.c_float), ("ms_ondemand", ctypes.c_float),
+                ("ms_h2d", ctypes.c_float), ("ms_finalize", ctypes.c_float), ("ms_exchange", ctypes.c_float),
+                ("ms_total", ctypes.c_float)]
+
+
+_lib.ascetic_load_csr.argtypes = [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p,
+                                  ctypes.c_void_p, ctypes.c_uint32]
+_lib.ascetic_set_budget.argtypes = [ctypes.c_uint64, ctypes.c_double]
+_lib.ascetic_set_option.argtypes = [ctypes.c_int, ctypes.c_int64]
+_lib.ascetic_run.argtypes = [ctypes.c_int, ctypes.c_uint32, ctypes.c_uint32]
+_lib.ascetic_stats.argtypes = [ctypes.POINTER(Stats), ctypes.POINTER(IterStats), ctypes.c_uint32]
+_lib.ascetic_get_result.argtypes = [ctypes.c_void_p, ctypes.c_uint64]
+_lib.ascetic_get_unique_id.argtypes = [ctypes.c_void_p]
+_lib.ascetic_comm_init.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_int]
+_lib.ascetic_set_device.argtypes = [ctypes.c_int]
+_lib.ascetic_unload.restype = None
+_lib.ascetic_last_error.restype = ctypes.c_char_p
+_lib.ascetic_version.restype = ctypes.c_char_p
+
+EXPORTS = ["ascetic_load_csr", "ascetic_set_budget", "ascetic_set_option", "ascetic_run", "ascetic_stats",
+           "ascetic_get_result", "ascetic_get_unique_id", "ascetic_comm_init", "ascetic_set_device",
+           "ascetic_unload", "ascetic_last_error", "ascetic_version"]
+
+
+class AsceticError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"{STATUS.get(code, code)}: {msg}")
+        self.code = code
+
+
+def _check(rc: int) -> int:
+    if rc < 0:
+        raise AsceticError(rc, _lib.ascetic_last_error().decode())
+    return rc
+
+
+# keep host arrays alive while the library pins them in place
+_keep: dict = {}
+
+
+def version() -> str:
+    return _lib.ascetic_version().decode()
+
+
+def set_device(device: int) -> None:
+    _check(_lib.ascetic_set_device(device))
+
+
+def load_csr(off: np.ndarray, nbr: np.ndarray, wgt: np.ndarray | None = None, *, symmetric: bool = True,
+             pairs: bool = False, copy: bool = False, validate: bool = False) -> None:
+    """off: uint64[n+1]; nbr: uint32[m] (or [2m] (id,w) pairs with pairs=True); wgt: uint32[m] or None."""
+    if off.dtype != np.uint64 or not off.flags.c_contiguous:
+        raise TypeError("off must be a C-contiguous uint64 array")
+    if nbr.dtype != np.uint32 or not nbr.flags.c_contiguous:
+        raise TypeError("nbr must be a C-contiguous uint32 array")
+    n = off.size - 1
+    m = nbr.size // 2 if pairs else nbr.size
+    flags = (SYMMETRIC if symmetric else 0) | (COPY if copy else 0) | (VALIDATE if validate else 0) | \
+            (PAIRS if pairs else 0)
+    wp = None
+    if wgt is not None:
+        if wgt.dtype != np.uint32 or wgt.size != m:
+            raise TypeError("wgt must be uint32[m]")
+        wp = wgt.ctypes.data
+    _check(_lib.ascetic_load_csr(n, m, off.ctypes.data, nbr.ctypes.data if nbr.size else None, wp, flags))
+    _keep["csr"] = (off, nbr, wgt)
+
+
+def set_budget(nbytes: int, static_fraction: float = -1.0) -> None:
+    _check(_lib.ascetic_set_budget(int(nbytes), float(static_fraction)))
+
+
+def set_option(name: str, value: int) -> None:
+    _check(_lib.ascetic_set_option(OPTIONS[name], int(value)))
+
+
+def run(algo: str, source: int = 0, max_iters: int = 0) -> None:
+    _check(_lib.ascetic_run(ALGOS[algo], int(source), int(max_iters)))
+
+
+def _sdict(s: ctypes.Structure) -> dict:
+    return {f: getattr(s, f) for f, _ in s._fields_}
+
+
+def stats(per_iter: bool = True) -> tuple[dict, list[dict]]:
+    st = Stats()
+    k = _check(_lib.ascetic_stats(ctypes.byref(st), None, 0))
+    its = []
+    if per_iter and k:
+        arr = (IterStats * k)()
+        _check(_lib.ascetic_stats(ctypes.byref(st), arr, k))
+        its = [_sdict(arr[i]) for i in range(k)]
+    return _sdict(st), its
+
+
+def get_result(out: np.ndarray | None = None) -> np.ndarray:
+    st = Stats()
+    _check(_lib.ascetic_stats(ctypes.byref(st), None, 0))
+    dt = np.float32 if st.algo == ALGOS["pr"] else np.uint32
+    if out is None:
+        out = np.empty(max(st.n, 1), dtype=dt)[: st.n]
+    _check(_lib.ascetic_get_result(out.ctypes.data, out.nbytes))
+    return out
+
+
+def unload() -> None:
+    _lib.ascetic_unload()
+    _keep.clear()
+
+
+PARITY_FIELDS = ["t", "nA", "nH", "nM", "nruns", "active_arcs", "hit_arcs", "miss_bytes", "digest"]
+
+
+class Placement(ctypes.Structure):
+    _fields_ = [("R", ctypes.c_double), ("D", ctypes.c_uint64), ("B", ctypes.c_uint64), ("Ms", ctypes.c_uint64),
+                ("s", ctypes.c_uint64), ("static_bytes", ctypes.c_uint64), ("C", ctypes.c_uint64),
+                ("cap", ctypes.c_uint64)]
+
+
+_lib.ascetic_place.argtypes = [ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_double,
+                               ctypes.POINTER(Placement)]
+EXPORTS.append("ascetic_place")
+
+
+def place(off: np.ndarray, b_e: int, nbytes: int, static_fraction: float = -1.0) -> dict:
+    """Host-only Eq. 2 placement (what set_budget would choose)."""
+    off = np.ascontiguousarray(off, dtype=np.uint64)
+    p = Placement()
+    _check(_lib.ascetic_place(off.size - 1, off.ctypes.data, b_e, int(nbytes), float(static_fraction),
+                              ctypes.byref(p)))
+    return _sdict(p)

@@ -1,0 +1,114 @@
+// ascetic_internal.h — device data layout and kernel launchers of libascetic.so.
+//
+// Layout in HBM (DESIGN.md §"Data layout"):
+//   resident vertex state (outside the edge budget):
+//     off      uint64[n+1]      CSR offsets
+//     A, S     uint32[nw]       ActiveBitmap / StaticBitmap, nw = ceil(n/32)
+//     next     uint32[nw]       next-frontier bits set by the edge kernels
+//     visited  uint32[nw]       BFS only
+//     val      uint32[n]        level / dist / label;  snap uint32[n] Jacobi snapshot (SSSP, CC)
+//     rank f32[n], contrib f32[n], sum f64[n]  PageRank
+//     hit queues (small / medium / hub) uint32, hub piece prefix uint32,
+//     miss queue uint32 + its arc prefix uint64, miss runs (b,e) uint32 + dst uint64
+//   edge budget B (Eq. 1/2):
+//     static   b_e * off[s] bytes = host nbr bytes [0, b_e*off[s])   (Static Region)
+//     chunk[2] cap bytes each                                        (On-demand Region)
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace ascetic {
+
+constexpr uint32_t kInf = 0xFFFFFFFFu;
+constexpr int kClassifyWarps = 8;                       // words per tile = 8 * 32
+constexpr int kTileWords = kClassifyWarps * 32;         // 256 words = 8192 vertices
+constexpr uint32_t kSmallDeg = 32;                      // hit lists shorter than this: warp-cooperative
+constexpr int kEdgeTile = 2048;                         // arcs per CTA tile in the chunk kernels
+
+// Scan fields of the order-preserving compaction (one decoupled look-back pass).
+struct ScanVal {
+    uint32_t small, med, hub, missq, runs, pieces;
+    unsigned long long miss_arcs;
+};
+
+// Per-iteration totals. Written by the last classify block into device memory AND
+// into mapped pinned host memory (the only device->host traffic per iteration).
+struct IterTotals {
+    unsigned long long nA, nH, nM, active_arcs, hit_arcs, digest;
+    unsigned long long miss_arcs;
+    uint32_t n_small, n_med, n_hub, n_missq, n_runs, n_pieces;
+    uint32_t tile_counter, done_counter;
+    uint32_t ready;          // set to 1 last (host spin target)
+    uint32_t pad;
+};
+
+struct ClassifyArgs {
+    const uint32_t* A;
+    const uint32_t* S;
+    const unsigned long long* off;
+    uint64_t n;
+    uint32_t nwords;
+    uint32_t ntiles;
+    uint32_t hub_deg;
+    uint32_t piece_arcs;
+    uint32_t* hq_small;
+    uint32_t* hq_med;
+    uint32_t* hq_hub;
+    uint32_t* hub_pre;                 // exclusive prefix of pieces per hub
+    uint32_t* mq;                      // miss vertices with deg > 0, ascending
+    unsigned long long* mq_pre;        // exclusive prefix of miss arcs at each mq entry
+    uint32_t* run_b;
+    uint32_t* run_e;
+    unsigned long long* run_dst;       // exclusive prefix of miss arcs at run start
+    ScanVal* tile_agg;
+    ScanVal* tile_incl;
+    uint32_t* tile_flag;
+    uint32_t epoch;
+    IterTotals* tot;                   // device
+    IterTotals* host_tot;              // mapped pinned
+};
+
+// Device state handed to the edge / finalize kernels.
+struct DevState {
+    const unsigned long long* off;
+    uint64_t n;
+    uint32_t nwords;
+    uint32_t* A;
+    uint32_t* S;
+    uint32_t* next;
+    uint32_t* visited;
+    uint32_t* val;
+    uint32_t* snap;
+    float* rank;
+    float* contrib;
+    double* sum;
+    double* dang;          // [0] = current dangling mass, [1] = next
+    uint32_t iter;         // t
+};
+
+struct Queues {
+    const uint32_t* hq_small;
+    const uint32_t* hq_med;
+    const uint32_t* hq_hub;
+    const uint32_t* hub_pre;
+    const uint32_t* mq;
+    const unsigned long long* mq_pre;
+};
+
+// ---- launchers (frontier.cu) ----
+void launch_classify(const ClassifyArgs& a, cudaStream_t s);
+
+// ---- launchers (edges.cu) ----
+void launch_init(int algo, const DevState& d, uint32_t source, cudaStream_t s);
+void launch_static(int algo, const DevState& d, const Queues& q, const void* static_base,
+                   uint32_t n_small, uint32_t n_med, uint32_t n_hub, uint32_t n_pieces,
+                   uint32_t piece_arcs, cudaStream_t s);
+void launch_ondemand(int algo, const DevState& d, const Queues& q, uint32_t n_missq,
+                     const void* chunk, unsigned long long lo, unsigned long long hi, cudaStream_t s);
+void launch_gather(const Queues& q, uint32_t n_missq, const unsigned long long* off,
+                   const void* host_nbr, uint32_t b_e, void* chunk,
+                   unsigned long long lo, unsigned long long hi, cudaStream_t s);
+void launch_finalize(int algo, const DevState& d, cudaStream_t s);
+void launch_set_prefix_bits(uint32_t* bits, uint32_t nwords, uint64_t s_prefix, cudaStream_t s);
+
+}  // namespace ascetic

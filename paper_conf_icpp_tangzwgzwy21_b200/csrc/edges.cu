@@ -1,0 +1,561 @@
+// edges.cu — per-algorithm edge kernels, the zero-copy gather, init and finalize.
+//
+// Paper: Static Computing on the StaticNodes' edges straight from the Static Region
+// (Fig. 4 (3)), On-demand Computing on the edges that landed in the
+// On-demand Region (Fig. 4 (5)), the On-demand Engine's gather of OndemandEdges
+// (P:593-596), and the next active set "generated based on the connected
+// edges". Algorithms: BFS, SSSP, CC (push, Jacobi snapshots, SURVEY §8(c)
+// Q2/Q3) and pull PageRank (d = 0.85).
+//
+// B200 design (DESIGN.md §"Kernels"):
+//  * static hits are degree-bucketed: < 32 arcs -> one warp expands 32 lists with an
+//    in-warp edge-balanced scan; 32..hub -> warp per list with 128-bit ld.global.nc;
+//    >= hub -> the list is cut into fixed pieces, one CTA per piece (multi-CTA hubs).
+//  * chunk kernels are edge-balanced: each CTA owns 2048 consecutive arcs of the
+//    miss stream and maps arcs to sources through a shared-memory tile of the miss
+//    queue's 64-bit prefix (one global binary search per CTA).
+//  * the gather is a zero-copy SM copy: host arcs are read through the mapped pinned
+//    CSR with the same arc->source map, so the host never needs the request list.
+#include "ascetic_internal.h"
+
+namespace ascetic {
+
+namespace {
+
+constexpr unsigned FULL = 0xFFFFFFFFu;
+enum { BFS = 0, SSSP = 1, CC = 2, PR = 3 };
+constexpr double kDamp = 0.85;
+
+// ------------------------------------------------------------------ per-arc ops
+__device__ __forceinline__ void set_next(const DevState& d, uint32_t v) {
+    const uint32_t wi = v >> 5, bit = 1u << (v & 31);
+    if (!(d.next[wi] & bit)) atomicOr(d.next + wi, bit);
+}
+
+__device__ __forceinline__ void bfs_visit(const DevState& d, uint32_t v) {
+    const uint32_t wi = v >> 5, bit = 1u << (v & 31);
+    if (__ldg(d.visited + wi) & bit) return;      // visited changes only in finalize
+    if (d.next[wi] & bit) return;
+    atomicOr(d.next + wi, bit);
+}
+
+__device__ __forceinline__ void relax(const DevState& d, uint32_t v, uint32_t cand) {
+    if (cand >= d.val[v]) return;                 // values only decrease within an iteration
+    const uint32_t old = atomicMin(d.val + v, cand);
+    if (cand < old) set_next(d, v);
+}
+
+__device__ __forceinline__ uint32_t sat_add(uint32_t a, uint32_t w) {
+    const unsigned long long c = (unsigned long long)a + w;
+    return c > (unsigned long long)(kInf - 1) ? kInf - 1 : (uint32_t)c;
+}
+
+// one arc, push algorithms. `arc` points at b_e bytes: id (+ weight).
+template <int ALGO>
+__device__ __forceinline__ void push_arc(const DevState& d, uint32_t sval, uint32_t id, uint32_t w) {
+    if (ALGO == BFS) bfs_visit(d, id);
+    else if (ALGO == SSSP) relax(d, id, sat_add(sval, w));
+    else relax(d, id, sval);
+}
+
+__device__ __forceinline__ double pr_in(const DevState& d, uint32_t id) {
+    return (double)__ldg(d.contrib + id);
+}
+
+__device__ __forceinline__ unsigned long long ub_u64(const unsigned long long* a, uint32_t n,
+                                                     unsigned long long x) {
+    // first index i in [0,n) with a[i] > x (n if none)
+    uint32_t lo = 0, hi = n;
+    while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (__ldg(a + mid) <= x) lo = mid + 1; else hi = mid;
+    }
+    return lo;
+}
+
+__device__ __forceinline__ uint32_t ub_u32(const uint32_t* a, uint32_t n, uint32_t x) {
+    uint32_t lo = 0, hi = n;
+    while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (__ldg(a + mid) <= x) lo = mid + 1; else hi = mid;
+    }
+    return lo;
+}
+
+// contiguous list [a0, a1) of arcs at base (b_e = 4 for ids, 8 for pairs), processed by
+// `nthr` threads with index `tid`, 128-bit loads on the aligned body.
+template <int ALGO>
+__device__ __forceinline__ double expand_list(const DevState& d, const void* base, unsigned long long a0,
+                                              unsigned long long a1, uint32_t sval, int tid, int nthr) {
+    double acc = 0.0;
+    if (ALGO == SSSP) {
+        const uint2* arcs = reinterpret_cast<const uint2*>(base);
+        const unsigned long long h = min(a1, (a0 + 1) & ~1ull);      // 2 arcs per 16 B
+        for (unsigned long long e = a0 + tid; e < h; e += nthr) {
+            const uint2 x = __ldg(arcs + e);
+            push_arc<ALGO>(d, sval, x.x, x.y);
+        }
+        const unsigned long long qb = h >> 1, qe = a1 >> 1;
+        const uint4* q = reinterpret_cast<const uint4*>(base);
+        for (unsigned long long k = qb + tid; k < qe; k += nthr) {
+            const uint4 x = __ldg(q + k);
+            push_arc<ALGO>(d, sval, x.x, x.y);
+            push_arc<ALGO>(d, sval, x.z, x.w);
+        }
+        for (unsigned long long e = max(h, qe << 1) + tid; e < a1; e += nthr) {
+            const uint2 x = __ldg(arcs + e);
+            push_arc<ALGO>(d, sval, x.x, x.y);
+        }
+    } else {
+        const uint32_t* arcs = reinterpret_cast<const uint32_t*>(base);
+        const unsigned long long h = min(a1, (a0 + 3) & ~3ull);      // 4 arcs per 16 B
+        for (unsigned long long e = a0 + tid; e < h; e += nthr) {
+            const uint32_t id = __ldg(arcs + e);
+            if (ALGO == PR) acc += pr_in(d, id); else push_arc<ALGO>(d, sval, id, 0);
+        }
+        const unsigned long long qb = h >> 2, qe = a1 >> 2;
+        const uint4* q = reinterpret_cast<const uint4*>(base);
+        for (unsigned long long k = qb + tid; k < qe; k += nthr) {
+            const uint4 x = __ldg(q + k);
+            if (ALGO == PR) {
+                acc += pr_in(d, x.x) + pr_in(d, x.y) + pr_in(d, x.z) + pr_in(d, x.w);
+            } else {
+                push_arc<ALGO>(d, sval, x.x, 0); push_arc<ALGO>(d, sval, x.y, 0);
+                push_arc<ALGO>(d, sval, x.z, 0); push_arc<ALGO>(d, sval, x.w, 0);
+            }
+        }
+        for (unsigned long long e = max(h, qe << 2) + tid; e < a1; e += nthr) {
+            const uint32_t id = __ldg(arcs + e);
+            if (ALGO == PR) acc += pr_in(d, id); else push_arc<ALGO>(d, sval, id, 0);
+        }
+    }
+    return acc;
+}
+
+__device__ __forceinline__ double warp_sum_d(double x) {
+#pragma unroll
+    for (int o = 16; o; o >>= 1) x += __shfl_xor_sync(FULL, x, o);
+    return x;
+}
+
+// ------------------------------------------------------------------ static: small lists
+template <int ALGO>
+__global__ void __launch_bounds__(256) k_static_small(DevState d, const uint32_t* __restrict__ q, uint32_t nq,
+                                                      const void* __restrict__ sbase) {
+    __shared__ double s_acc[8][32];
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t base = gw * 32;
+    if (base >= nq) return;                                   // warp-uniform
+    const uint32_t idx = base + lane;
+    const bool valid = idx < nq;
+    uint32_t u = 0, deg = 0, sval = 0;
+    unsigned long long start = 0;
+    if (valid) {
+        u = __ldg(q + idx);
+        start = __ldg(d.off + u);
+        deg = (uint32_t)(__ldg(d.off + u + 1) - start);
+        if (ALGO == SSSP || ALGO == CC) sval = __ldg(d.snap + u);
+    }
+    uint32_t incl = deg;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, incl, o);
+        if (lane >= o) incl += y;
+    }
+    const uint32_t excl = incl - deg;
+    const uint32_t total = __shfl_sync(FULL, incl, 31);
+    if (ALGO == PR) s_acc[wib][lane] = 0.0;
+    __syncwarp();
+    for (uint32_t k0 = 0; k0 < total; k0 += 32) {
+        const uint32_t k = k0 + lane;
+        int i = 0;
+#pragma unroll
+        for (int step = 16; step >= 1; step >>= 1) {
+            const uint32_t x = __shfl_sync(FULL, incl, i + step - 1);
+            if (x <= k) i += step;
+        }
+        const unsigned long long ust = __shfl_sync(FULL, start, i);
+        const uint32_t uex = __shfl_sync(FULL, excl, i);
+        const uint32_t usv = __shfl_sync(FULL, sval, i);
+        const bool ok = k < total;
+        const unsigned long long e = ust + (k - uex);
+        if (ALGO == PR) {
+            double x = ok ? pr_in(d, __ldg(reinterpret_cast<const uint32_t*>(sbase) + e)) : 0.0;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const double y = __shfl_up_sync(FULL, x, o);
+                const int oi = __shfl_up_sync(FULL, i, o);
+                if (lane >= o && oi == i) x += y;
+            }
+            const int ni = __shfl_down_sync(FULL, i, 1);
+            const bool nok = __shfl_down_sync(FULL, (int)ok, 1);
+            const bool last = ok && (lane == 31 || !nok || ni != i);
+            if (last) s_acc[wib][i] += x;
+            __syncwarp();
+        } else if (ok) {
+            if (ALGO == SSSP) {
+                const uint2 x = __ldg(reinterpret_cast<const uint2*>(sbase) + e);
+                push_arc<ALGO>(d, usv, x.x, x.y);
+            } else {
+                push_arc<ALGO>(d, usv, __ldg(reinterpret_cast<const uint32_t*>(sbase) + e), 0);
+            }
+        }
+    }
+    if (ALGO == PR && valid) d.sum[u] = s_acc[wib][lane];
+}
+
+// ------------------------------------------------------------------ static: warp per list
+template <int ALGO>
+__global__ void __launch_bounds__(256) k_static_med(DevState d, const uint32_t* __restrict__ q, uint32_t nq,
+                                                    const void* __restrict__ sbase) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (gw >= nq) return;
+    const uint32_t u = __ldg(q + gw);
+    const unsigned long long a0 = __ldg(d.off + u), a1 = __ldg(d.off + u + 1);
+    const uint32_t sval = (ALGO == SSSP || ALGO == CC) ? __ldg(d.snap + u) : 0u;
+    double acc = expand_list<ALGO>(d, sbase, a0, a1, sval, lane, 32);
+    if (ALGO == PR) {
+        acc = warp_sum_d(acc);
+        if (lane == 0) d.sum[u] = acc;
+    }
+}
+
+// ------------------------------------------------------------------ static: hubs, CTA per piece
+template <int ALGO>
+__global__ void __launch_bounds__(256) k_static_hub(DevState d, const uint32_t* __restrict__ hq,
+                                                    const uint32_t* __restrict__ pre, uint32_t nh,
+                                                    uint32_t piece_arcs, const void* __restrict__ sbase) {
+    __shared__ double s_red[8];
+    const uint32_t b = blockIdx.x;
+    const uint32_t h = ub_u32(pre, nh, b) - 1;
+    const uint32_t u = __ldg(hq + h);
+    const uint32_t pidx = b - __ldg(pre + h);
+    const unsigned long long o0 = __ldg(d.off + u), o1 = __ldg(d.off + u + 1);
+    const unsigned long long a0 = o0 + (unsigned long long)pidx * piece_arcs;
+    const unsigned long long a1 = min(o1, a0 + piece_arcs);
+    const uint32_t sval = (ALGO == SSSP || ALGO == CC) ? __ldg(d.snap + u) : 0u;
+    double acc = expand_list<ALGO>(d, sbase, a0, a1, sval, threadIdx.x, blockDim.x);
+    if (ALGO == PR) {
+        acc = warp_sum_d(acc);
+        if ((threadIdx.x & 31) == 0) s_red[threadIdx.x >> 5] = acc;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            double t = 0.0;
+            for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += s_red[w];
+            atomicAdd(d.sum + u, t);
+        }
+    }
+}
+
+// ------------------------------------------------------------------ chunk tile staging
+// CTA tile = arcs [t_lo, t_hi) of the miss stream. Stages the covering miss-queue
+// entries: pre (64-bit exclusive arc prefix), the source id, and an aux word.
+struct TileMap {
+    uint32_t i0, cnt;
+};
+
+__device__ __forceinline__ TileMap stage_tile(const Queues& q, uint32_t nq, unsigned long long t_lo,
+                                              unsigned long long t_hi, unsigned long long* s_pre,
+                                              uint32_t* s_u, uint32_t* s_i) {
+    if (threadIdx.x == 0) {
+        s_i[0] = (uint32_t)ub_u64(q.mq_pre, nq, t_lo) - 1u;
+        s_i[1] = (uint32_t)ub_u64(q.mq_pre, nq, t_hi - 1) - 1u;
+    }
+    __syncthreads();
+    TileMap m;
+    m.i0 = s_i[0];
+    m.cnt = s_i[1] - s_i[0] + 1u;
+    for (uint32_t k = threadIdx.x; k < m.cnt; k += blockDim.x) {
+        s_pre[k] = __ldg(q.mq_pre + m.i0 + k);
+        s_u[k] = __ldg(q.mq + m.i0 + k);
+    }
+    __syncthreads();
+    return m;
+}
+
+// largest k in [lo, cnt) with s_pre[k] <= p (s_pre[lo] <= p guaranteed)
+__device__ __forceinline__ uint32_t find_local(const unsigned long long* s_pre, uint32_t lo, uint32_t cnt,
+                                               unsigned long long p) {
+    uint32_t hi = cnt;
+    while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (s_pre[mid] <= p) lo = mid; else hi = mid;
+    }
+    return lo;
+}
+
+// ------------------------------------------------------------------ on-demand compute
+template <int ALGO>
+__global__ void __launch_bounds__(256) k_ondemand(DevState d, Queues q, uint32_t nq, const void* __restrict__ chunk,
+                                                  unsigned long long lo, unsigned long long hi) {
+    __shared__ unsigned long long s_pre[kEdgeTile];
+    __shared__ uint32_t s_u[kEdgeTile];
+    __shared__ uint32_t s_i[2];
+    const unsigned long long t_lo = lo + (unsigned long long)blockIdx.x * kEdgeTile;
+    const unsigned long long t_hi = min(hi, t_lo + kEdgeTile);
+    const TileMap m = stage_tile(q, nq, t_lo, t_hi, s_pre, s_u, s_i);
+    const int lane = threadIdx.x & 31;
+    uint32_t k = 0;
+    for (unsigned long long p0 = t_lo; p0 < t_hi; p0 += blockDim.x) {
+        const unsigned long long p = p0 + threadIdx.x;
+        const bool ok = p < t_hi;
+        if (ok) k = find_local(s_pre, k, m.cnt, p);
+        const uint32_t u = s_u[k];
+        if (ALGO == PR) {
+            double x = ok ? pr_in(d, __ldg(reinterpret_cast<const uint32_t*>(chunk) + (p - lo))) : 0.0;
+            const int ki = ok ? (int)k : -1 - lane;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const double y = __shfl_up_sync(FULL, x, o);
+                const int oi = __shfl_up_sync(FULL, ki, o);
+                if (lane >= o && oi == ki) x += y;
+            }
+            const int ni = __shfl_down_sync(FULL, ki, 1);
+            if (ok && (lane == 31 || ni != ki)) atomicAdd(d.sum + u, x);
+        } else if (ok) {
+            if (ALGO == SSSP) {
+                const uint2 x = __ldg(reinterpret_cast<const uint2*>(chunk) + (p - lo));
+                push_arc<ALGO>(d, __ldg(d.snap + u), x.x, x.y);
+            } else {
+                push_arc<ALGO>(d, __ldg(d.snap + u), __ldg(reinterpret_cast<const uint32_t*>(chunk) + (p - lo)), 0);
+            }
+        }
+    }
+}
+
+// BFS needs no source: 128-bit loads straight over the chunk.
+__global__ void __launch_bounds__(256) k_ondemand_bfs(DevState d, const uint32_t* __restrict__ chunk,
+                                                      unsigned long long len) {
+    const unsigned long long nq4 = len >> 2;
+    const uint4* c4 = reinterpret_cast<const uint4*>(chunk);
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < nq4; i += stride) {
+        const uint4 x = __ldg(c4 + i);
+        bfs_visit(d, x.x); bfs_visit(d, x.y); bfs_visit(d, x.z); bfs_visit(d, x.w);
+    }
+    const unsigned long long t = (nq4 << 2) + (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t < len) bfs_visit(d, __ldg(chunk + t));
+}
+
+// ------------------------------------------------------------------ zero-copy gather (transfer engine)
+template <int BE>
+__global__ void __launch_bounds__(256) k_gather(Queues q, uint32_t nq, const unsigned long long* __restrict__ off,
+                                                const void* __restrict__ host, void* __restrict__ chunk,
+                                                unsigned long long lo, unsigned long long hi) {
+    __shared__ unsigned long long s_pre[kEdgeTile];
+    __shared__ uint32_t s_u[kEdgeTile];
+    __shared__ uint32_t s_i[2];
+    const unsigned long long t_lo = lo + (unsigned long long)blockIdx.x * kEdgeTile;
+    const unsigned long long t_hi = min(hi, t_lo + kEdgeTile);
+    const TileMap m = stage_tile(q, nq, t_lo, t_hi, s_pre, s_u, s_i);
+    uint32_t k = 0;
+    for (unsigned long long p0 = t_lo; p0 < t_hi; p0 += blockDim.x) {
+        const unsigned long long p = p0 + threadIdx.x;
+        if (p < t_hi) {
+            k = find_local(s_pre, k, m.cnt, p);
+            const unsigned long long src = __ldg(off + s_u[k]) + (p - s_pre[k]);
+            if (BE == 8) {
+                reinterpret_cast<unsigned long long*>(chunk)[p - lo] =
+                    reinterpret_cast<const unsigned long long*>(host)[src];
+            } else {
+                reinterpret_cast<uint32_t*>(chunk)[p - lo] = reinterpret_cast<const uint32_t*>(host)[src];
+            }
+        }
+    }
+}
+
+// ------------------------------------------------------------------ init / finalize
+__global__ void k_fill_u32(uint32_t* p, uint64_t n, uint32_t v) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+        p[i] = v;
+}
+
+__global__ void k_iota_u32(uint32_t* a, uint32_t* b, uint64_t n) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+        a[i] = (uint32_t)i;
+        b[i] = (uint32_t)i;
+    }
+}
+
+__global__ void k_prefix_bits(uint32_t* bits, uint32_t nwords, uint64_t s) {
+    for (uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < nwords; w += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t lo = w * 32;
+        uint32_t x;
+        if (lo + 32 <= s) x = FULL;
+        else if (lo >= s) x = 0u;
+        else x = (1u << (uint32_t)(s - lo)) - 1u;
+        bits[w] = x;
+    }
+}
+
+__global__ void k_set_source(DevState d, uint32_t src, int algo) {
+    d.val[src] = 0;
+    if (algo == SSSP) d.snap[src] = 0;
+    d.A[src >> 5] |= 1u << (src & 31);
+    if (algo == BFS) d.visited[src >> 5] |= 1u << (src & 31);
+}
+
+__global__ void k_pr_init(DevState d) {
+    const double r0 = 1.0 / (double)d.n;
+    double dang = 0.0;
+    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < d.n; v += (uint64_t)gridDim.x * blockDim.x) {
+        const unsigned long long deg = d.off[v + 1] - d.off[v];
+        d.rank[v] = (float)r0;
+        d.contrib[v] = deg ? (float)(r0 / (double)deg) : 0.0f;
+        if (!deg) dang += r0;
+    }
+    dang = warp_sum_d(dang);
+    if ((threadIdx.x & 31) == 0 && dang != 0.0) atomicAdd(d.dang, dang);
+}
+
+__global__ void k_finalize_bfs(DevState d) {
+    for (uint32_t w = blockIdx.x * blockDim.x + threadIdx.x; w < d.nwords; w += gridDim.x * blockDim.x) {
+        const uint32_t nx = d.next[w];
+        const uint32_t vis = d.visited[w];
+        const uint32_t nw = nx & ~vis;
+        d.A[w] = nw;
+        if (nx) d.next[w] = 0;
+        if (nw) {
+            d.visited[w] = vis | nw;
+            uint32_t b = nw;
+            while (b) {
+                const int i = __ffs(b) - 1;
+                b &= b - 1;
+                d.val[(uint64_t)w * 32 + i] = d.iter + 1;
+            }
+        }
+    }
+}
+
+__global__ void k_finalize_minlabel(DevState d) {
+    for (uint32_t w = blockIdx.x * blockDim.x + threadIdx.x; w < d.nwords; w += gridDim.x * blockDim.x) {
+        const uint32_t nx = d.next[w];
+        d.A[w] = nx;
+        if (nx) {
+            d.next[w] = 0;
+            uint32_t b = nx;
+            while (b) {
+                const int i = __ffs(b) - 1;
+                b &= b - 1;
+                const uint64_t v = (uint64_t)w * 32 + i;
+                d.snap[v] = d.val[v];
+            }
+        }
+    }
+}
+
+// r' = (1-d)/n + d (sum + dang/n) in fp64, stored fp32; contrib = fp32(r'/deg);
+// next dangling mass accumulated from the fp64 r'.
+__global__ void k_finalize_pr(DevState d, int cur) {
+    const double inv_n = 1.0 / (double)d.n;
+    const double dc = d.dang[cur];
+    double dn = 0.0;
+    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < d.n; v += (uint64_t)gridDim.x * blockDim.x) {
+        const double r = (1.0 - kDamp) * inv_n + kDamp * (d.sum[v] + dc * inv_n);
+        const unsigned long long deg = __ldg(d.off + v + 1) - __ldg(d.off + v);
+        d.rank[v] = (float)r;
+        d.contrib[v] = deg ? (float)(r / (double)deg) : 0.0f;
+        if (!deg) dn += r;
+    }
+    dn = warp_sum_d(dn);
+    if ((threadIdx.x & 31) == 0 && dn != 0.0) atomicAdd(d.dang + (cur ^ 1), dn);
+}
+
+inline unsigned blocks_for(unsigned long long n, int per_block, unsigned cap = 148u * 16u) {
+    unsigned long long b = (n + per_block - 1) / per_block;
+    if (b < 1) b = 1;
+    return (unsigned)(b > cap ? cap : b);
+}
+
+template <int ALGO>
+void static_launch(const DevState& d, const Queues& q, const void* sbase, uint32_t ns, uint32_t nm, uint32_t nh,
+                   uint32_t npieces, uint32_t piece, cudaStream_t s) {
+    if (ns) k_static_small<ALGO><<<(ns + 255) / 256, 256, 0, s>>>(d, q.hq_small, ns, sbase);
+    if (nm) k_static_med<ALGO><<<(nm + 7) / 8, 256, 0, s>>>(d, q.hq_med, nm, sbase);
+    if (nh) k_static_hub<ALGO><<<npieces, 256, 0, s>>>(d, q.hq_hub, q.hub_pre, nh, piece, sbase);
+}
+
+}  // namespace
+
+void launch_static(int algo, const DevState& d, const Queues& q, const void* sbase, uint32_t ns, uint32_t nm,
+                   uint32_t nh, uint32_t npieces, uint32_t piece, cudaStream_t s) {
+    switch (algo) {
+        case BFS: static_launch<BFS>(d, q, sbase, ns, nm, nh, npieces, piece, s); break;
+        case SSSP: static_launch<SSSP>(d, q, sbase, ns, nm, nh, npieces, piece, s); break;
+        case CC: static_launch<CC>(d, q, sbase, ns, nm, nh, npieces, piece, s); break;
+        default: static_launch<PR>(d, q, sbase, ns, nm, nh, npieces, piece, s); break;
+    }
+}
+
+void launch_ondemand(int algo, const DevState& d, const Queues& q, uint32_t nq, const void* chunk,
+                     unsigned long long lo, unsigned long long hi, cudaStream_t s) {
+    if (hi <= lo) return;
+    const unsigned long long len = hi - lo;
+    if (algo == BFS) {
+        k_ondemand_bfs<<<blocks_for(len, 256 * 4), 256, 0, s>>>(d, reinterpret_cast<const uint32_t*>(chunk), len);
+        return;
+    }
+    const unsigned tiles = (unsigned)((len + kEdgeTile - 1) / kEdgeTile);
+    switch (algo) {
+        case SSSP: k_ondemand<SSSP><<<tiles, 256, 0, s>>>(d, q, nq, chunk, lo, hi); break;
+        case CC: k_ondemand<CC><<<tiles, 256, 0, s>>>(d, q, nq, chunk, lo, hi); break;
+        default: k_ondemand<PR><<<tiles, 256, 0, s>>>(d, q, nq, chunk, lo, hi); break;
+    }
+}
+
+void launch_gather(const Queues& q, uint32_t nq, const unsigned long long* off, const void* host_nbr, uint32_t b_e,
+                   void* chunk, unsigned long long lo, unsigned long long hi, cudaStream_t s) {
+    if (hi <= lo) return;
+    const unsigned tiles = (unsigned)((hi - lo + kEdgeTile - 1) / kEdgeTile);
+    if (b_e == 8) k_gather<8><<<tiles, 256, 0, s>>>(q, nq, off, host_nbr, chunk, lo, hi);
+    else k_gather<4><<<tiles, 256, 0, s>>>(q, nq, off, host_nbr, chunk, lo, hi);
+}
+
+void launch_init(int algo, const DevState& d, uint32_t source, cudaStream_t s) {
+    const unsigned gb = blocks_for(d.n, 256);
+    cudaMemsetAsync(d.A, 0, (size_t)d.nwords * 4, s);
+    cudaMemsetAsync(d.next, 0, (size_t)d.nwords * 4, s);
+    switch (algo) {
+        case BFS:
+            cudaMemsetAsync(d.visited, 0, (size_t)d.nwords * 4, s);
+            k_fill_u32<<<gb, 256, 0, s>>>(d.val, d.n, kInf);
+            k_set_source<<<1, 1, 0, s>>>(d, source, algo);
+            break;
+        case SSSP:
+            k_fill_u32<<<gb, 256, 0, s>>>(d.val, d.n, kInf);
+            k_fill_u32<<<gb, 256, 0, s>>>(d.snap, d.n, kInf);
+            k_set_source<<<1, 1, 0, s>>>(d, source, algo);
+            break;
+        case CC:
+            k_iota_u32<<<gb, 256, 0, s>>>(d.val, d.snap, d.n);
+            k_prefix_bits<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d.A, d.nwords, d.n);
+            break;
+        default:
+            cudaMemsetAsync(d.dang, 0, 2 * sizeof(double), s);
+            k_pr_init<<<gb, 256, 0, s>>>(d);
+            k_prefix_bits<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d.A, d.nwords, d.n);
+            break;
+    }
+}
+
+void launch_finalize(int algo, const DevState& d, cudaStream_t s) {
+    switch (algo) {
+        case BFS: k_finalize_bfs<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d); break;
+        case SSSP:
+        case CC: k_finalize_minlabel<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d); break;
+        default: {
+            const int cur = (int)(d.iter & 1u);
+            cudaMemsetAsync(d.dang + (cur ^ 1), 0, sizeof(double), s);
+            k_finalize_pr<<<blocks_for(d.n, 256), 256, 0, s>>>(d, cur);
+            break;
+        }
+    }
+}
+
+void launch_set_prefix_bits(uint32_t* bits, uint32_t nwords, uint64_t s_prefix, cudaStream_t s) {
+    if (nwords) k_prefix_bits<<<blocks_for(nwords, 256), 256, 0, s>>>(bits, nwords, s_prefix);
+}
+
+}  // namespace ascetic

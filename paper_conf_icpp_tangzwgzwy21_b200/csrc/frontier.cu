@@ -1,0 +1,336 @@
+// frontier.cu — GenDataMap + StaticNodes/On-demandNodes generation in ONE pass.
+//
+// Paper: StaticMap = ActiveBitmap AND StaticBitmap, On-demand Map = StaticMap XOR
+// ActiveBitmap (Fig. 4; §3.1); StaticNodes are
+// generated from StaticMap and handed to the Manager; On-demandNodes
+// with their Degree generate the data request.
+//
+// B200 design (DESIGN.md §"Kernels / classify"): one CTA = 8 warps = 256 bitmap
+// words = 8192 vertices. Each warp owns 32 consecutive words; per word every lane
+// classifies one vertex with register bit ops (AND / AND-NOT, never materialising
+// the maps), reads off[v], off[v+1] only for active vertices (coalesced 8-byte
+// loads), and ballots/popcounts its class. The order-preserving compaction of the
+// hit queues (3 degree buckets), the miss queue (+64-bit arc prefix) and the
+// maximal miss runs (+64-bit destination offsets) is ONE decoupled look-back scan
+// over a 32-byte multi-field value. Run ends are paired with run starts by rank,
+// so a run may span any number of tiles. The last CTA to finish writes the totals
+// straight into mapped pinned host memory: that is the only D2H per iteration.
+#include "ascetic_internal.h"
+
+namespace ascetic {
+
+namespace {
+
+constexpr unsigned FULL = 0xFFFFFFFFu;
+constexpr unsigned long long PHI = 0x9E3779B97F4A7C15ull;
+
+__device__ __forceinline__ unsigned long long mix64(unsigned long long z) {
+    z += 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+__device__ __forceinline__ unsigned long long wsum64(unsigned long long x) {
+#pragma unroll
+    for (int d = 16; d; d >>= 1) x += __shfl_xor_sync(FULL, x, d);
+    return x;
+}
+
+__device__ __forceinline__ unsigned long long wexcl64(unsigned long long x, int lane) {
+    unsigned long long inc = x;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        unsigned long long y = __shfl_up_sync(FULL, inc, d);
+        if (lane >= d) inc += y;
+    }
+    return inc - x;
+}
+
+__device__ __forceinline__ uint32_t wexcl32(uint32_t x, int lane) {
+    uint32_t inc = x;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        uint32_t y = __shfl_up_sync(FULL, inc, d);
+        if (lane >= d) inc += y;
+    }
+    return inc - x;
+}
+
+__device__ __forceinline__ ScanVal sv_zero() {
+    ScanVal z;
+    z.small = z.med = z.hub = z.missq = z.runs = z.pieces = 0;
+    z.miss_arcs = 0;
+    return z;
+}
+
+__device__ __forceinline__ ScanVal sv_add(const ScanVal& a, const ScanVal& b) {
+    ScanVal r;
+    r.small = a.small + b.small;
+    r.med = a.med + b.med;
+    r.hub = a.hub + b.hub;
+    r.missq = a.missq + b.missq;
+    r.runs = a.runs + b.runs;
+    r.pieces = a.pieces + b.pieces;
+    r.miss_arcs = a.miss_arcs + b.miss_arcs;
+    return r;
+}
+
+__device__ __forceinline__ ScanVal sv_warp_sum(ScanVal v) {
+    ScanVal r;
+    r.small = __reduce_add_sync(FULL, v.small);
+    r.med = __reduce_add_sync(FULL, v.med);
+    r.hub = __reduce_add_sync(FULL, v.hub);
+    r.missq = __reduce_add_sync(FULL, v.missq);
+    r.runs = __reduce_add_sync(FULL, v.runs);
+    r.pieces = __reduce_add_sync(FULL, v.pieces);
+    r.miss_arcs = wsum64(v.miss_arcs);
+    return r;
+}
+
+__device__ __forceinline__ void sv_store_volatile(ScanVal* p, const ScanVal& v) {
+    volatile uint32_t* q = reinterpret_cast<volatile uint32_t*>(p);
+    q[0] = v.small; q[1] = v.med; q[2] = v.hub; q[3] = v.missq; q[4] = v.runs; q[5] = v.pieces;
+    *reinterpret_cast<volatile unsigned long long*>(&p->miss_arcs) = v.miss_arcs;
+}
+
+__device__ __forceinline__ ScanVal sv_load_volatile(const ScanVal* p) {
+    const volatile uint32_t* q = reinterpret_cast<const volatile uint32_t*>(p);
+    ScanVal v;
+    v.small = q[0]; v.med = q[1]; v.hub = q[2]; v.missq = q[3]; v.runs = q[4]; v.pieces = q[5];
+    v.miss_arcs = *reinterpret_cast<const volatile unsigned long long*>(&p->miss_arcs);
+    return v;
+}
+
+__global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a) {
+    __shared__ uint32_t s_tile;
+    __shared__ ScanVal s_warp[kClassifyWarps];
+    __shared__ ScanVal s_excl;
+    __shared__ unsigned long long s_ns[kClassifyWarps][6];
+
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint32_t lt = (1u << lane) - 1u;
+    const uint32_t le = lt | (1u << lane);
+    if (threadIdx.x == 0) s_tile = atomicAdd(&a.tot->tile_counter, 1u);
+    __syncthreads();
+    const uint32_t tile = s_tile;
+    const uint32_t w0 = tile * kTileWords + warp * 32;
+    const uint32_t myw = w0 + lane;
+
+    uint32_t myA = 0, myS = 0;
+    if (myw < a.nwords) { myA = __ldg(a.A + myw); myS = __ldg(a.S + myw); }
+    const uint32_t myMiss = myA & ~myS;
+    uint32_t prevMiss = 0, nextMiss = 0;
+    if (w0 > 0 && w0 - 1 < a.nwords) prevMiss = __ldg(a.A + w0 - 1) & ~__ldg(a.S + w0 - 1);
+    if (w0 + 32 < a.nwords) nextMiss = __ldg(a.A + w0 + 32) & ~__ldg(a.S + w0 + 32);
+    const uint32_t anyA = __ballot_sync(FULL, myA != 0);
+    const uint32_t piece = a.piece_arcs;
+
+    // ---------------- phase A: per-warp counts
+    ScanVal mine = sv_zero();
+    unsigned long long aArcs = 0, hArcs = 0;
+    for (int j = 0; j < 32; ++j) {
+        if (!((anyA >> j) & 1u)) continue;                    // warp-uniform
+        const uint32_t aw = __shfl_sync(FULL, myA, j);
+        const uint32_t sw = __shfl_sync(FULL, myS, j);
+        const uint32_t pm = __shfl_sync(FULL, myMiss, (j + 31) & 31);
+        const uint32_t carry_in = (j == 0 ? prevMiss : pm) >> 31;
+        const unsigned long long v = (unsigned long long)(w0 + j) * 32ull + lane;
+        const bool act = (aw >> lane) & 1u;
+        unsigned long long deg = 0;
+        if (act) deg = __ldg(a.off + v + 1) - __ldg(a.off + v);
+        const bool st = (sw >> lane) & 1u;
+        const bool hit = act && st, miss = act && !st;
+        aArcs += deg;
+        if (hit) {
+            hArcs += deg;
+            if (deg > 0) {
+                if (deg < kSmallDeg) mine.small++;
+                else if (deg < a.hub_deg) mine.med++;
+                else { mine.hub++; mine.pieces += (uint32_t)((deg + piece - 1) / piece); }
+            }
+        }
+        if (miss) {
+            mine.miss_arcs += deg;
+            if (deg > 0) mine.missq++;
+        }
+        const uint32_t mw = aw & ~sw;
+        const uint32_t starts = mw & ~((mw << 1) | carry_in);
+        if (lane == 0) mine.runs += __popc(starts);
+    }
+    ScanVal wagg = sv_warp_sum(mine);
+    {
+        unsigned long long nA = __popc(myA), nH = __popc(myA & myS), nM = __popc(myMiss);
+        unsigned long long dg = (myw < a.nwords) ? mix64((unsigned long long)myw ^ ((unsigned long long)myA * PHI)) : 0ull;
+        nA = wsum64(nA); nH = wsum64(nH); nM = wsum64(nM); dg = wsum64(dg);
+        aArcs = wsum64(aArcs); hArcs = wsum64(hArcs);
+        if (lane == 0) {
+            s_warp[warp] = wagg;
+            s_ns[warp][0] = nA; s_ns[warp][1] = nH; s_ns[warp][2] = nM;
+            s_ns[warp][3] = aArcs; s_ns[warp][4] = hArcs; s_ns[warp][5] = dg;
+        }
+    }
+    __syncthreads();
+
+    // ---------------- block aggregate + decoupled look-back (warp 0)
+    if (warp == 0) {
+        ScanVal agg = sv_zero();
+        if (lane == 0) {
+            for (int w = 0; w < kClassifyWarps; ++w) {
+                ScanVal x = s_warp[w];
+                s_warp[w] = agg;            // becomes the warp's exclusive offset in the block
+                agg = sv_add(agg, x);
+            }
+            if (tile == 0) {
+                sv_store_volatile(&a.tile_incl[0], agg);
+                __threadfence();
+                *reinterpret_cast<volatile uint32_t*>(&a.tile_flag[0]) = (a.epoch << 2) | 2u;
+            } else {
+                sv_store_volatile(&a.tile_agg[tile], agg);
+                __threadfence();
+                *reinterpret_cast<volatile uint32_t*>(&a.tile_flag[tile]) = (a.epoch << 2) | 1u;
+            }
+        }
+        ScanVal excl = sv_zero();
+        if (tile > 0) {
+            int base = (int)tile - 1;
+            while (true) {
+                const int idx = base - lane;
+                uint32_t st = 2;
+                ScanVal val = sv_zero();
+                if (idx >= 0) {
+                    uint32_t f;
+                    do {
+                        f = *reinterpret_cast<volatile uint32_t*>(&a.tile_flag[idx]);
+                    } while ((f >> 2) != a.epoch || (f & 3u) == 0u);
+                    __threadfence();
+                    st = f & 3u;
+                    val = sv_load_volatile(st == 2 ? &a.tile_incl[idx] : &a.tile_agg[idx]);
+                }
+                const uint32_t incl_mask = __ballot_sync(FULL, st == 2);
+                const int stop = incl_mask ? (__ffs(incl_mask) - 1) : 31;
+                ScanVal c = (lane <= stop) ? val : sv_zero();
+                excl = sv_add(excl, sv_warp_sum(c));
+                if (incl_mask) break;
+                base -= 32;
+            }
+            if (lane == 0) {
+                sv_store_volatile(&a.tile_incl[tile], sv_add(excl, agg));
+                __threadfence();
+                *reinterpret_cast<volatile uint32_t*>(&a.tile_flag[tile]) = (a.epoch << 2) | 2u;
+            }
+        }
+        if (lane == 0) s_excl = excl;
+    }
+    __syncthreads();
+
+    // ---------------- phase B: scatter with the prefixes
+    const ScanVal wb = sv_add(s_excl, s_warp[warp]);
+    uint32_t bS = wb.small, bM = wb.med, bH = wb.hub, bQ = wb.missq, bR = wb.runs, bP = wb.pieces;
+    unsigned long long bArcs = wb.miss_arcs;
+    for (int j = 0; j < 32; ++j) {
+        if (!((anyA >> j) & 1u)) continue;
+        const uint32_t aw = __shfl_sync(FULL, myA, j);
+        const uint32_t sw = __shfl_sync(FULL, myS, j);
+        const uint32_t pm = __shfl_sync(FULL, myMiss, (j + 31) & 31);
+        const uint32_t nm = __shfl_sync(FULL, myMiss, (j + 1) & 31);
+        const uint32_t carry_in = (j == 0 ? prevMiss : pm) >> 31;
+        const uint32_t carry_out = (j == 31 ? nextMiss : nm) & 1u;
+        const unsigned long long v = (unsigned long long)(w0 + j) * 32ull + lane;
+        const bool act = (aw >> lane) & 1u;
+        unsigned long long deg = 0;
+        if (act) deg = __ldg(a.off + v + 1) - __ldg(a.off + v);
+        const bool st = (sw >> lane) & 1u;
+        const bool hit = act && st, miss = act && !st;
+        const uint32_t hw = aw & sw;
+        if (hw) {
+            const bool isS = hit && deg > 0 && deg < kSmallDeg;
+            const bool isM = hit && deg >= kSmallDeg && deg < a.hub_deg;
+            const bool isH = hit && deg >= a.hub_deg;
+            const uint32_t balS = __ballot_sync(FULL, isS);
+            const uint32_t balM = __ballot_sync(FULL, isM);
+            const uint32_t balH = __ballot_sync(FULL, isH);
+            if (isS) a.hq_small[bS + __popc(balS & lt)] = (uint32_t)v;
+            if (isM) a.hq_med[bM + __popc(balM & lt)] = (uint32_t)v;
+            if (balH) {
+                const uint32_t pc = isH ? (uint32_t)((deg + piece - 1) / piece) : 0u;
+                const uint32_t ex = wexcl32(pc, lane);
+                if (isH) {
+                    const uint32_t k = bH + __popc(balH & lt);
+                    a.hq_hub[k] = (uint32_t)v;
+                    a.hub_pre[k] = bP + ex;
+                }
+                bP += __shfl_sync(FULL, ex + pc, 31);
+            }
+            bS += __popc(balS); bM += __popc(balM); bH += __popc(balH);
+        }
+        const uint32_t mw = aw & ~sw;
+        if (mw) {
+            const unsigned long long md = miss ? deg : 0ull;
+            const unsigned long long ex = wexcl64(md, lane);
+            const unsigned long long tot = __shfl_sync(FULL, ex + md, 31);
+            const bool isQ = miss && deg > 0;
+            const uint32_t balQ = __ballot_sync(FULL, isQ);
+            if (isQ) {
+                const uint32_t k = bQ + __popc(balQ & lt);
+                a.mq[k] = (uint32_t)v;
+                a.mq_pre[k] = bArcs + ex;
+            }
+            const uint32_t starts = mw & ~((mw << 1) | carry_in);
+            const uint32_t ends = mw & ~((mw >> 1) | (carry_out << 31));
+            if ((starts >> lane) & 1u) {
+                const uint32_t r = bR + __popc(starts & lt);
+                a.run_b[r] = (uint32_t)v;
+                a.run_dst[r] = bArcs + ex;
+            }
+            if ((ends >> lane) & 1u) {
+                const uint32_t r = bR + __popc(starts & le) - 1u;
+                a.run_e[r] = (uint32_t)(v + 1);
+            }
+            bQ += __popc(balQ);
+            bR += __popc(starts);
+            bArcs += tot;
+        }
+    }
+
+    // ---------------- non-scan totals, completion, totals to host
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long t[6] = {0, 0, 0, 0, 0, 0};
+        for (int w = 0; w < kClassifyWarps; ++w)
+            for (int k = 0; k < 6; ++k) t[k] += s_ns[w][k];
+        if (t[0]) atomicAdd(&a.tot->nA, t[0]);
+        if (t[1]) atomicAdd(&a.tot->nH, t[1]);
+        if (t[2]) atomicAdd(&a.tot->nM, t[2]);
+        if (t[3]) atomicAdd(&a.tot->active_arcs, t[3]);
+        if (t[4]) atomicAdd(&a.tot->hit_arcs, t[4]);
+        atomicAdd(&a.tot->digest, t[5]);                 // Σ mod 2^64
+        __threadfence();
+        const uint32_t done = atomicAdd(&a.tot->done_counter, 1u);
+        if (done == a.ntiles - 1) {
+            __threadfence();
+            const ScanVal fin = sv_load_volatile(&a.tile_incl[a.ntiles - 1]);
+            volatile IterTotals* vt = a.tot;
+            IterTotals* h = a.host_tot;
+            h->nA = vt->nA; h->nH = vt->nH; h->nM = vt->nM;
+            h->active_arcs = vt->active_arcs; h->hit_arcs = vt->hit_arcs; h->digest = vt->digest;
+            h->miss_arcs = fin.miss_arcs;
+            h->n_small = fin.small; h->n_med = fin.med; h->n_hub = fin.hub;
+            h->n_missq = fin.missq; h->n_runs = fin.runs; h->n_pieces = fin.pieces;
+            a.tot->miss_arcs = fin.miss_arcs;
+            a.tot->n_small = fin.small; a.tot->n_med = fin.med; a.tot->n_hub = fin.hub;
+            a.tot->n_missq = fin.missq; a.tot->n_runs = fin.runs; a.tot->n_pieces = fin.pieces;
+            __threadfence_system();
+            *reinterpret_cast<volatile uint32_t*>(&h->ready) = 1u;
+        }
+    }
+}
+
+}  // namespace
+
+void launch_classify(const ClassifyArgs& a, cudaStream_t s) {
+    if (a.ntiles == 0) return;
+    k_classify<<<a.ntiles, kClassifyWarps * 32, 0, s>>>(a);
+}
+
+}  // namespace ascetic

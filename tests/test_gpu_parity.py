@@ -1,0 +1,185 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle, element by element.
+
+Bit-exact: BFS levels, SSSP distances, CC labels, per-iteration active sets (digest,
+|A|, |H|, |M|, #runs, active/hit arcs) and per-iteration transferred bytes.
+PageRank (fp32 on the GPU vs fp64 oracle): max per-vertex relative error <= 1e-5 and
+L1 <= 1e-6 after the same number of iterations (BASELINE.json north_star).
+"""
+import numpy as np
+import pytest
+
+import graphgen as gg
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+REC = ["nA", "nH", "nM", "nruns", "active_arcs", "hit_arcs", "miss_bytes", "digest"]
+
+
+@pytest.fixture(scope="module")
+def asc():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    import paper_conf_icpp_tangzwgzwy21_b200 as m
+    yield m
+    m.unload()
+
+
+def _oracle(algo, g, src, s_static, max_iters=0):
+    return oracle.run(algo, g.off, g.nbr, src=src, max_iters=max_iters, is_static=oracle.static_prefix(g.n, s_static))
+
+
+def _check_records(its, ref):
+    assert len(its) == len(ref.records)
+    for t, (a, b) in enumerate(zip(its, ref.records)):
+        assert a["t"] == t
+        for f in REC:
+            assert a[f] == b[f], f"iteration {t} field {f}: gpu {a[f]} oracle {b[f]}"
+
+
+def _run(asc, g, algo, src=0, budget=None, frac=-1.0, max_iters=0, chunk_cap=0, xfer=0, hub=2048):
+    asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True)
+    asc.set_option("chunk_cap", chunk_cap)
+    asc.set_option("xfer_mode", xfer)
+    asc.set_option("hub_degree", hub)
+    asc.set_budget(budget if budget is not None else g.csr_bytes // 4, frac)
+    asc.run(algo, src, max_iters)
+    st, its = asc.stats()
+    return st, its, asc.get_result().copy()
+
+
+def _pr_ok(gpu, ref):
+    rel = np.abs(gpu.astype(np.float64) - ref) / np.abs(ref)
+    l1 = np.abs(gpu.astype(np.float64) - ref).sum()
+    assert rel.max() <= 1e-5, rel.max()
+    assert l1 <= 1e-6, l1
+
+
+ALGO_GRAPHS = {
+    "bfs": dict(scale=12, weights=False),
+    "sssp": dict(scale=12, weights=True),
+    "cc": dict(scale=12, weights=False),
+    "pr": dict(scale=12, weights=False),
+}
+
+
+@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pr"])
+@pytest.mark.parametrize("frac", [-1.0, 0.0, 1.0, 0.5])
+@pytest.mark.parametrize("xfer", [1, 2])
+def test_parity_small(asc, algo, frac, xfer):
+    cfg = ALGO_GRAPHS[algo]
+    g = gg.rmat(cfg["scale"], seed=3, weights=cfg["weights"])
+    src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+    iters = 10 if algo == "pr" else 0
+    st, its, res = _run(asc, g, algo, src=src, frac=frac, max_iters=iters, xfer=xfer, chunk_cap=4096)
+    p = oracle.placer(g.off, g.b_e, g.csr_bytes // 4, frac)
+    assert st["s"] == p.s and st["static_bytes"] == p.static_bytes
+    ref = _oracle(algo, g, src, p.s, max_iters=iters)
+    assert st["iterations"] == ref.iterations
+    _check_records(its, ref)
+    assert st["h2d_payload_bytes"] == ref.h2d_payload
+    assert st["active_arcs_total"] == ref.active_arcs_total
+    if algo == "pr":
+        _pr_ok(res, ref.values)
+    else:
+        np.testing.assert_array_equal(res, ref.values)
+
+
+@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc"])
+def test_parity_tiny_chunks_split_hubs(asc, algo):
+    """16-byte chunks force every hub list across many chunks; hub threshold 32 forces multi-CTA hubs."""
+    g = gg.rmat(10, seed=7, weights=(algo == "sssp"))
+    src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+    st, its, res = _run(asc, g, algo, src=src, frac=0.3, chunk_cap=16, xfer=1, hub=32)
+    p = oracle.placer(g.off, g.b_e, g.csr_bytes // 4, 0.3)
+    ref = _oracle(algo, g, src, p.s)
+    np.testing.assert_array_equal(res, ref.values)
+    _check_records(its, ref)
+
+
+def test_parity_pr_tiny_chunks(asc):
+    g = gg.rmat(10, seed=8)
+    st, its, res = _run(asc, g, "pr", frac=0.2, max_iters=7, chunk_cap=48, xfer=1, hub=32)
+    p = oracle.placer(g.off, 4, g.csr_bytes // 4, 0.2)
+    ref = _oracle("pr", g, 0, p.s, max_iters=7)
+    _check_records(its, ref)
+    _pr_ok(res, ref.values)
+
+
+@pytest.mark.parametrize("n", [1, 2, 31, 33, 65, 1000])
+def test_edge_sizes_random(asc, n):
+    """n not a multiple of 32, tiny graphs, isolated vertices."""
+    g = gg.random_graph(n, 2 * n, seed=n)
+    for algo in ["bfs", "cc"]:
+        src = 0
+        st, its, res = _run(asc, g, algo, src=src, budget=max(64, g.csr_bytes // 3), frac=0.5, chunk_cap=32)
+        p = oracle.placer(g.off, 4, max(64, g.csr_bytes // 3), 0.5)
+        ref = _oracle(algo, g, src, p.s)
+        np.testing.assert_array_equal(res, ref.values)
+        _check_records(its, ref)
+
+
+def test_isolated_source(asc):
+    n = 100
+    src = np.array([1, 2, 3], dtype=np.uint32)
+    dst = np.array([2, 3, 4], dtype=np.uint32)
+    g = gg.from_edges(n, src, dst)
+    st, its, res = _run(asc, g, "bfs", src=50, frac=0.5, chunk_cap=16)
+    assert st["iterations"] == 1
+    assert res[50] == 0 and (np.delete(res, 50) == 0xFFFFFFFF).all()
+    assert its[0]["active_arcs"] == 0 and its[0]["miss_bytes"] == 0
+
+
+def test_max_iters_and_repeat_runs(asc):
+    g = gg.rmat(11, seed=4)
+    src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+    _run(asc, g, "bfs", src=src)
+    for k in [1, 2, 3]:
+        asc.run("bfs", src, k)
+        st, its = asc.stats()
+        res = asc.get_result()
+        p = oracle.placer(g.off, 4, g.csr_bytes // 4)
+        ref = _oracle("bfs", g, src, p.s, max_iters=k)
+        np.testing.assert_array_equal(res, ref.values)
+        _check_records(its, ref)
+
+
+def test_c1_config_full(asc):
+    """BASELINE config 1: BFS on RMAT-16 at 25 % of CSR bytes, Eq. 2 split, default chunking."""
+    g = gg.config_graph("c1")
+    budget = gg.config_budget("c1", g)
+    for src in gg.sources(g, 4, seed=1):
+        for xfer in [0, 1, 2]:
+            st, its, res = _run(asc, g, "bfs", src=src, budget=budget, xfer=xfer)
+            p = oracle.placer(g.off, 4, budget)
+            ref = _oracle("bfs", g, src, p.s)
+            np.testing.assert_array_equal(res, ref.values)
+            _check_records(its, ref)
+            assert st["h2d_static_fill_bytes"] == p.static_bytes
+            assert st["h2d_payload_bytes"] == ref.h2d_payload
+
+
+def test_resident_r1_moves_no_payload(asc):
+    g = gg.rmat(12, seed=2)
+    st, its, res = _run(asc, g, "cc", budget=10 * g.csr_bytes)
+    assert st["s"] == g.n and st["h2d_payload_bytes"] == 0
+    ref = _oracle("cc", g, 0, g.n)
+    np.testing.assert_array_equal(res, ref.values)
+
+
+def test_errors_on_gpu(asc):
+    g = gg.rmat(8, seed=1)
+    asc.load_csr(g.off, g.nbr, symmetric=False)
+    asc.set_budget(g.csr_bytes)
+    with pytest.raises(asc.AsceticError):
+        asc.run("cc")                      # CC needs SYMMETRIC
+    with pytest.raises(asc.AsceticError):
+        asc.run("sssp", 0)                 # SSSP needs weights
+    with pytest.raises(asc.AsceticError):
+        asc.run("bfs", g.n)                # source out of range
+    with pytest.raises(asc.AsceticError):
+        asc.run("pr", 0, 0)                # PR needs iterations
+    with pytest.raises(asc.AsceticError) as e:
+        asc.set_budget(10, 0.0)            # on-demand chunk below 16 bytes
+    assert e.value.code == asc.ENOMEM

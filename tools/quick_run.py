@@ -1,0 +1,69 @@
+"""Quick single run of one config on the GPU with per-iteration phase timings (dev tool)."""
+import argparse
+import json
+import os
+import sys
+import time
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import numpy as np  # noqa: E402
+
+import graphgen as gg  # noqa: E402
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--algo", default="sssp")
+    ap.add_argument("--scale", type=int, default=20)
+    ap.add_argument("--frac-budget", type=float, default=0.5)
+    ap.add_argument("--xfer", type=int, default=0)
+    ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--iters", type=int, default=0)
+    ap.add_argument("--config", default="")
+    ap.add_argument("--oracle", action="store_true")
+    a = ap.parse_args()
+    import paper_conf_icpp_tangzwgzwy21_b200 as asc
+    t0 = time.time()
+    if a.config:
+        g = gg.config_graph(a.config)
+        budget = gg.config_budget(a.config, g)
+        algo = gg.CONFIGS[a.config]["algo"]
+        iters = gg.CONFIGS[a.config].get("iters", 0)
+    else:
+        g = gg.rmat(a.scale, seed=2, weights=(a.algo == "sssp"))
+        budget = int(a.frac_budget * g.csr_bytes)
+        algo, iters = a.algo, a.iters
+    print(f"gen {time.time()-t0:.1f}s n={g.n} m={g.m}", flush=True)
+    t0 = time.time()
+    asc.load_csr(g.off, g.nbr, pairs=g.pairs)
+    print(f"load {time.time()-t0:.2f}s", flush=True)
+    asc.set_budget(budget)
+    asc.set_option("xfer_mode", a.xfer)
+    src = gg.sources(g, 1, seed=1)[0]
+    for r in range(a.reps):
+        asc.run(algo, src, iters)
+        st, its = asc.stats()
+        print(json.dumps({k: st[k] for k in ["iterations", "s", "h2d_payload_bytes", "h2d_static_fill_bytes",
+                                              "active_arcs_total", "chunks_total", "dma_chunks", "gather_chunks",
+                                              "time_run_s", "time_fill_s", "time_h2d_busy_s", "gteps",
+                                              "chunk_cap"]}), flush=True)
+    for i in its:
+        print({k: (round(v, 3) if isinstance(v, float) else v) for k, v in i.items() if k != "digest"})
+    if a.oracle:
+        import oracle
+        p = oracle.placer(g.off, g.b_e, budget)
+        t0 = time.time()
+        ref = oracle.run(algo, g.off, g.nbr, src=src, max_iters=iters, is_static=oracle.static_prefix(g.n, p.s))
+        print(f"oracle {time.time()-t0:.2f}s threads={oracle.threads()}")
+        res = asc.get_result()
+        if algo == "pr":
+            print("max rel", float(np.max(np.abs(res - ref.values) / ref.values)))
+        else:
+            print("equal", bool(np.array_equal(res, ref.values)))
+        print("records equal", [ {k: x[k] for k in asc.PARITY_FIELDS} for x in its] ==
+              [{k: x[k] for k in asc.PARITY_FIELDS} for x in ref.records])
+
+
+if __name__ == "__main__":
+    main()
