@@ -1,0 +1,362 @@
+"""bench.py — end-to-end GTEPS of the Ascetic hot path under a capped device budget.
+
+Contract (driver): `python bench.py --gpus N --steps K --warmup W` prints ONE JSON line.
+A step = one full ascetic_run (classify+compact, static fill, static + on-demand edge
+kernels, every H2D chunk, finalize, for all iterations) of the workload below over one
+source. Default workload (N=1) = BASELINE.json configs[1]: SSSP (w in 1..64) on RMAT
+scale-24 with the device edge budget capped at 50 % of the CSR bytes.
+
+  value  = Σ active arcs / Σ step device time (CUDA events around each step), GTEPS;
+           the graph is host-resident (that is the method) and already pinned/loaded.
+  e2e    = same metric through the public API with every host<->device copy inside the
+           step: load_csr (offsets H2D) + set_budget + run (fill + misses H2D) + get_result (D2H).
+  roofline = dominant kernel of the step (by device time): algorithmic bytes / time vs
+           the measured peak of its bound (host link: pinned H2D measured here; HBM:
+           MEASURED_PEAKS.json hbm_gbs). See DESIGN.md §"Roofline".
+`--impl reference` times the CPU oracle (oracle/) on the same workload instead.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "end-to-end GTEPS incl. H2D under capped HBM budget; H2D GB per run"
+
+
+def _dist():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d.get("hbm_gbs", 6650.0)), "measured"
+    return 6650.0, "fallback"
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+
+    FIELDS = ["index", "clocks.sm", "clocks.max.sm", "power.draw", "clocks_event_reasons.active",
+              "clocks_event_reasons.hw_slowdown", "clocks_event_reasons.hw_thermal_slowdown",
+              "clocks_event_reasons.sw_thermal_slowdown", "clocks_event_reasons.sw_power_cap"]
+
+    def __init__(self, gpu: int):
+        self.gpu = gpu
+        self.path = f"/tmp/ascetic_clocks_{os.getpid()}.csv"
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), "--query-gpu=" + ",".join(self.FIELDS),
+                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                      stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self) -> dict:
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        try:
+            self.p.wait(timeout=5)
+        except Exception:
+            self.p.kill()
+        sm, smax, reasons, power = [], [], set(), []
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in open(self.path):
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1])); smax.append(float(f[2])); power.append(float(f[3]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        os.unlink(self.path)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm), "power_w_max": max(power) if power else None}
+
+
+def _h2d_peak(torch, dev) -> float:
+    """Pinned H2D copy-engine peak on this box: 1 GiB cudaMemcpyAsync, best of 5 (GB/s)."""
+    sz = 1 << 30
+    h = torch.empty(sz, dtype=torch.uint8, pin_memory=True)
+    g = torch.empty(sz, dtype=torch.uint8, device=dev)
+    best = 0.0
+    for _ in range(5):
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(); g.copy_(h, non_blocking=True); e1.record(); e1.synchronize()
+        best = max(best, sz / (e0.elapsed_time(e1) / 1e3) / 1e9)
+    del h, g
+    return best
+
+
+def _workload(cfg_key: str):
+    import graphgen as gg
+    c = gg.CONFIGS[cfg_key]
+    return gg, c
+
+
+def run_reference(args, ws, rank):
+    """--impl reference: the oracle as it stands, on the host cores, same config/metric/unit."""
+    if rank != 0:
+        return 0
+    import oracle
+    gg, c = _workload(args.config)
+    g = gg.config_graph(args.config)
+    budget = gg.config_budget(args.config, g)
+    p = oracle.placer(g.off, g.b_e, budget)
+    st = oracle.static_prefix(g.n, p.s)
+    algo = c["algo"]
+    iters = c.get("iters", 0) if algo == "pr" else 0
+    if algo == "pr":
+        iters = min(iters, args.ref_pr_iters)
+    srcs = gg.sources(g, max(1, args.steps + args.warmup), seed=c["seed"])
+    for i in range(args.warmup):
+        oracle.run(algo, g.off, g.nbr, src=srcs[i % len(srcs)], max_iters=iters, is_static=st)
+    arcs, secs, h2d = 0, 0.0, 0
+    for i in range(args.steps):
+        t0 = time.perf_counter()
+        r = oracle.run(algo, g.off, g.nbr, src=srcs[(args.warmup + i) % len(srcs)], max_iters=iters, is_static=st)
+        secs += time.perf_counter() - t0
+        arcs += r.active_arcs_total
+        h2d += r.h2d_payload + p.static_bytes
+    v = arcs / secs / 1e9
+    sample = (f"{args.steps} full oracle {algo.upper()} runs" + (f" of {iters} iterations" if algo == "pr" else "")
+              + f" on the {args.config} graph (n={g.n}, m={g.m})")
+    out = {"metric": METRIC, "value": v, "unit": "GTEPS", "impl": "reference", "n_gpus": ws,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": secs / args.steps * 1e3,
+           "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32" if algo != "pr" else "f64",
+           "data": "synthetic", "config": {"workload": f"{args.config}: {c['desc']}", "budget_bytes": budget,
+                                           "n": g.n, "m": g.m, "h2d_gb_per_run": h2d / args.steps / 1e9},
+           "cpu_baseline": {"value": v, "unit": "GTEPS", "cores": oracle.threads(), "kind": "oracle",
+                            "sample": sample},
+           "e2e": {"value": v, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ascetic", choices=["ascetic", "reference"])
+    ap.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c4"])
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--cpu-seconds", type=float, default=15.0, help="bounded oracle sample for cpu_baseline")
+    ap.add_argument("--ref-pr-iters", type=int, default=2, help="PR iterations per reference step (bounded)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--xfer", type=int, default=0)
+    args = ap.parse_args()
+    ws, rank, local = _dist()
+    if args.warmup < 3:
+        print("warning: warmup < 3 violates the timing rules; using 3", file=sys.stderr)
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args, ws, rank)
+
+    import torch
+    import torch.distributed as dist
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+    if ws > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    import paper_conf_icpp_tangzwgzwy21_b200 as asc
+    gg, c = _workload(args.config)
+    algo = c["algo"]
+    iters = c.get("iters", 0) if algo == "pr" else 0
+
+    h2d_peak = _h2d_peak(torch, dev)
+    hbm_peak, hbm_src = _peaks()
+
+    # graph arcs generated straight into pinned host memory (the method's host Edgelist)
+    pinned = []
+
+    def alloc(count, dtype):
+        t = torch.empty(max(1, count), dtype=torch.int32, pin_memory=True)
+        pinned.append(t)
+        return t.numpy().view(np.uint32)
+
+    t0 = time.time()
+    g = gg.config_graph(args.config, alloc=alloc)
+    gen_s = time.time() - t0
+    budget = gg.config_budget(args.config, g)
+    srcs = gg.sources(g, 8, seed=c["seed"])
+
+    asc.set_device(local)
+    asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True)
+    asc.set_budget(budget)
+    asc.set_option("xfer_mode", args.xfer)
+    l2_flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+
+    def step(i):
+        asc.run(algo, srcs[i % len(srcs)], iters)
+        return asc.stats(per_iter=False)[0]
+
+    for i in range(args.warmup):
+        step(i)
+    torch.cuda.synchronize()
+
+    clocks = Clocks(local)
+    clocks.start()
+    per = []
+    total_ms = 0.0
+    for k in range(args.steps):
+        l2_flush.fill_(k & 0xFF)                      # flush L2 between timed steps (outside the step)
+        torch.cuda.synchronize()
+        if ws > 1:
+            dist.barrier()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record()
+        st = step(args.warmup + k)
+        e1.record()
+        torch.cuda.synchronize()
+        total_ms += e0.elapsed_time(e1)
+        per.append(st)
+    clk = clocks.stop()
+    if ws > 1:
+        tt = torch.tensor([total_ms], device=dev, dtype=torch.float64)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        total_ms = float(tt.item())
+
+    arcs = sum(s["active_arcs_total"] for s in per)
+    arcs_all = arcs * ws
+    value = arcs_all / (total_ms / 1e3) / 1e9
+    fill = sum(s["h2d_static_fill_bytes"] for s in per)
+    payload = sum(s["h2d_payload_bytes"] for s in per)
+    lib_ms = sum(s["time_run_s"] for s in per) * 1e3
+
+    # ---- per-kernel-class breakdown (library CUDA events on the launching streams)
+    b_e = g.b_e
+    kern = {
+        "gather": dict(time_s=sum(s["time_gather_s"] for s in per), bytes=sum(s["gather_bytes"] for s in per),
+                       bound="host_link", peak=h2d_peak),
+        "dma": dict(time_s=sum(s["time_dma_s"] + s["time_fill_s"] for s in per),
+                    bytes=sum(s["dma_bytes"] + s["h2d_static_fill_bytes"] for s in per), bound="host_link",
+                    peak=h2d_peak),
+        "ondemand": dict(time_s=sum(s["time_ondemand_s"] for s in per),
+                         bytes=sum(s["ondemand_arcs"] for s in per) * (b_e + 4), bound="hbm", peak=hbm_peak),
+        "static": dict(time_s=sum(s["time_static_s"] for s in per),
+                       bytes=sum(s["static_arcs"] for s in per) * (b_e + 4), bound="hbm", peak=hbm_peak),
+        "classify": dict(time_s=sum(s["time_classify_s"] for s in per),
+                         bytes=sum(s["iterations"] for s in per) * (g.n // 4) + 0, bound="hbm", peak=hbm_peak),
+    }
+    for k_, d in kern.items():
+        d["achieved"] = d["bytes"] / d["time_s"] / 1e9 if d["time_s"] > 0 else 0.0
+        d["frac"] = d["achieved"] / d["peak"] if d["peak"] else 0.0
+        d["share_of_step"] = d["time_s"] * 1e3 / total_ms if total_ms else 0.0
+    dom = max(kern, key=lambda k_: kern[k_]["time_s"])
+    dk = kern[dom]
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get(args.config, {}).get(dom)
+        except Exception:
+            traffic = None
+    roofline = {"kernel": dom, "bound": dk["bound"], "achieved": dk["achieved"], "peak": dk["peak"],
+                "unit": "GB/s", "frac": dk["frac"], "traffic": traffic,
+                "peak_source": ("pinned H2D cudaMemcpyAsync 1 GiB best-of-5 measured in this run"
+                                if dk["bound"] == "host_link" else f"MEASURED_PEAKS.json hbm_gbs ({hbm_src})"),
+                "per_kernel": {k_: {kk: (round(vv, 6) if isinstance(vv, float) else vv) for kk, vv in d.items()}
+                               for k_, d in kern.items()}}
+    h2d_total = fill + payload
+    link = {"h2d_bytes": h2d_total, "h2d_busy_s": sum(s["time_h2d_busy_s"] for s in per),
+            "achieved_gbs": h2d_total / (sum(s["time_h2d_busy_s"] for s in per) or 1) / 1e9,
+            "whole_step_gbs": h2d_total / (total_ms / 1e3) / 1e9, "peak_gbs": h2d_peak}
+    link["frac_busy"] = link["achieved_gbs"] / h2d_peak
+    link["frac_step"] = link["whole_step_gbs"] / h2d_peak
+
+    # ---- e2e: public API with host buffers, every copy inside the step
+    e2e_ms, e2e_arcs, h2d_b, d2h_b = 0.0, 0, 0, 0
+    res = np.empty(g.n, dtype=np.float32 if algo == "pr" else np.uint32)
+    res_pinned = torch.empty(max(1, g.n), dtype=torch.int32, pin_memory=True).numpy().view(res.dtype)[: g.n]
+    for k in range(args.e2e_steps):
+        l2_flush.fill_(k & 0xFF)
+        torch.cuda.synchronize()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record()
+        asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True)
+        asc.set_budget(budget)
+        asc.set_option("xfer_mode", args.xfer)
+        asc.run(algo, srcs[k % len(srcs)], iters)
+        asc.get_result(res_pinned)
+        e1.record()
+        torch.cuda.synchronize()
+        s_ = asc.stats(per_iter=False)[0]
+        e2e_ms += e0.elapsed_time(e1)
+        e2e_arcs += s_["active_arcs_total"]
+        h2d_b += 8 * (g.n + 1) + s_["h2d_static_fill_bytes"] + s_["h2d_payload_bytes"]
+        d2h_b += res_pinned.nbytes + s_["d2h_bytes"]
+    e2e = {"value": e2e_arcs * ws / (e2e_ms / 1e3) / 1e9, "unit": "GTEPS",
+           "h2d_bytes_per_step": h2d_b // max(1, args.e2e_steps), "d2h_bytes_per_step": d2h_b // max(1, args.e2e_steps),
+           "steps": args.e2e_steps, "ms_per_step": e2e_ms / max(1, args.e2e_steps)}
+
+    # ---- CPU baseline: the oracle as it stands, bounded sample, rank 0 at N=1 only
+    cpu = None
+    if rank == 0 and ws == 1 and not args.no_cpu_baseline:
+        import oracle
+        p = oracle.placer(g.off, g.b_e, budget)
+        stc = oracle.static_prefix(g.n, p.s)
+        it_ = min(iters, args.ref_pr_iters) if algo == "pr" else 0
+        a_, s_t, runs = 0, 0.0, 0
+        while runs < 1 or (s_t < args.cpu_seconds and runs < 8):
+            t0 = time.perf_counter()
+            r = oracle.run(algo, g.off, g.nbr, src=srcs[runs % len(srcs)], max_iters=it_, is_static=stc)
+            s_t += time.perf_counter() - t0
+            a_ += r.active_arcs_total
+            runs += 1
+        cpu = {"value": a_ / s_t / 1e9, "unit": "GTEPS", "cores": oracle.threads(), "kind": "oracle",
+               "sample": f"{runs} full oracle {algo.upper()} runs" + (f" of {it_} iterations" if algo == "pr" else "")
+                         + f" from the bench sources on the same {args.config} graph ({s_t:.1f} s)"}
+
+    out = {"metric": METRIC, "value": value, "unit": "GTEPS", "n_gpus": ws, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
+           "scaling": "weak", "vs_baseline": None, "dtype": "u32" if algo != "pr" else "f32",
+           "data": "synthetic",
+           "config": {"workload": f"{args.config}: {c['desc']}", "algo": algo, "n": g.n, "m": g.m,
+                      "budget_bytes": budget, "csr_bytes": g.csr_bytes, "static_vertices": per[0]["s"],
+                      "static_fraction": per[0]["static_fraction_used"], "chunk_cap": per[0]["chunk_cap"],
+                      "h2d_gb_per_run": h2d_total / args.steps / 1e9,
+                      "h2d_fill_gb_per_run": fill / args.steps / 1e9,
+                      "h2d_payload_gb_per_run": payload / args.steps / 1e9,
+                      "iterations_per_run": statistics.mean(s["iterations"] for s in per),
+                      "sources": srcs, "l2": "flushed (512 MiB write) between timed steps; graph > L2",
+                      "graph_gen_s": round(gen_s, 2),
+                      "parallelism": f"{ws} process(es), one GPU each" + ("" if ws == 1 else
+                                     " (independent replicas: multi-GPU partition not implemented)")},
+           "roofline": roofline, "link": link, "cpu_baseline": cpu, "e2e": e2e,
+           "gpu_launches": int(sum(s["kernel_launches"] for s in per)),
+           "library_ms_per_step": lib_ms / args.steps,
+           "clocks": clk}
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    asc.unload()
+    if ws > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -77,20 +77,22 @@ class Graph:
         return self.nbr[1::2]
 
 
-def _export(h, pairs: bool, wseed: int, name: str) -> Graph:
+def _export(h, pairs: bool, wseed: int, name: str, alloc=None) -> Graph:
+    """alloc(count, dtype) -> numpy array lets callers place the arcs (e.g. in pinned memory)."""
     lib = _load()
     n = ctypes.c_uint32()
     m = ctypes.c_uint64()
     lib.gg_size(h, ctypes.byref(n), ctypes.byref(m))
     off = np.empty(n.value + 1, dtype=np.uint64)
-    nbr = np.empty(max(1, (2 if pairs else 1) * m.value), dtype=np.uint32)[: (2 if pairs else 1) * m.value]
+    cnt = (2 if pairs else 1) * m.value
+    nbr = (alloc(cnt, np.uint32) if alloc is not None else np.empty(max(1, cnt), dtype=np.uint32))[:cnt]
     lib.gg_export(h, off.ctypes.data, nbr.ctypes.data if nbr.size else None, None, 1 if pairs else 0, wseed)
     lib.gg_free(h)
     return Graph(n=n.value, m=m.value, off=off, nbr=nbr, pairs=pairs, name=name)
 
 
 def rmat(scale: int, tuples: int | None = None, seed: int = 1, permute: bool = True, n: int = 0,
-         weights: bool = False, abc=(0.57, 0.19, 0.19), name: str = "") -> Graph:
+         weights: bool = False, abc=(0.57, 0.19, 0.19), name: str = "", alloc=None) -> Graph:
     """RMAT graph, symmetrized + deduplicated. `n` > 0 rejects endpoints >= n (exact n)."""
     lib = _load()
     if tuples is None:
@@ -98,7 +100,7 @@ def rmat(scale: int, tuples: int | None = None, seed: int = 1, permute: bool = T
     h = lib.gg_rmat_build(scale, tuples, n, seed, 1 if permute else 0, abc[0], abc[1], abc[2])
     if not h:
         raise ValueError("bad rmat parameters")
-    return _export(h, weights, seed, name or f"rmat{scale}")
+    return _export(h, weights, seed, name or f"rmat{scale}", alloc)
 
 
 def from_edges(n: int, src, dst, symmetrize: bool = True, weights: bool = False, seed: int = 1,
@@ -135,13 +137,13 @@ CONFIGS = {
 }
 
 
-def config_graph(key: str, scale_override: int | None = None) -> Graph:
+def config_graph(key: str, scale_override: int | None = None, alloc=None) -> Graph:
     c = CONFIGS[key]
     scale = scale_override or c["scale"]
     tuples = c["tuples"] if scale_override is None else (16 << scale)
     n = c["n"] if scale_override is None else 0
     return rmat(scale, tuples, seed=c["seed"], permute=c["permute"], n=n,
-                weights=(c["algo"] == "sssp"), name=key)
+                weights=(c["algo"] == "sssp"), name=key, alloc=alloc)
 
 
 def config_budget(key: str, g: Graph) -> int:

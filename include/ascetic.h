@@ -66,7 +66,8 @@ typedef enum {
     ASCETIC_OPT_OVERLAP = 4,       /* 1 (default) = static compute overlaps the transfer; 0 = serialize (ablation, Fig. 8) */
     ASCETIC_OPT_KEEP_STATIC = 5,   /* 1 = keep the Static Region filled across runs (fill counted once) ; default 0 */
     ASCETIC_OPT_HUB_DEGREE = 6,    /* hit-queue degree at/above which a list is split across CTAs (default 2048) */
-    ASCETIC_OPT_TIMING = 7         /* 1 (default) = per-iteration phase timing with CUDA events */
+    ASCETIC_OPT_TIMING = 7,        /* 1 (default) = per-iteration phase timing with CUDA events */
+    ASCETIC_OPT_GATHER_CTAS = 8    /* persistent CTAs of the zero-copy gather; 0 (default) = 2 x SM count */
 } ascetic_option;
 
 typedef struct {
@@ -95,6 +96,19 @@ typedef struct {
     double gteps;                 /* active_arcs_total / time_run_s / 1e9 */
     double gteps_excl_fill;
     uint64_t vertex_state_bytes;  /* device bytes outside the edge budget */
+    /* per-kernel-class device time (CUDA events on the launching stream) and algorithmic work */
+    uint64_t kernel_launches;     /* kernels this library launched during the run */
+    double time_classify_s;       /* classify+compact kernel */
+    double time_static_s;         /* static-hit edge kernels */
+    uint64_t static_arcs;         /* arcs they processed */
+    double time_ondemand_s;       /* on-demand chunk edge kernels */
+    uint64_t ondemand_arcs;
+    double time_gather_s;         /* zero-copy gather kernels (transfer engine, SM path) */
+    uint64_t gather_bytes;
+    double time_dma_s;            /* copy-engine chunk DMAs */
+    uint64_t dma_bytes;
+    double time_finalize_s;
+    double time_host_s;           /* host planning + waits between classify and the next launches */
 } ascetic_stats_t;
 
 typedef struct {
@@ -181,6 +195,10 @@ void ascetic_unload(void);
 
 /* Thread-local message of the last failing call ("" if none). */
 const char* ascetic_last_error(void);
+
+/* sizeof(ascetic_stats_t), sizeof(ascetic_iter_stats_t), sizeof(ascetic_placement_t) into out[0..2]
+ * (lets bindings verify their struct mirrors). */
+int ascetic_struct_sizes(uint64_t* out3);
 
 /* Library version string. */
 const char* ascetic_version(void);

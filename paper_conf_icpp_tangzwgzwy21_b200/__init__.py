@@ -34,7 +34,7 @@ STATUS = {0: "OK", -1: "EINVAL", -2: "ESTATE", -3: "ENOMEM", -4: "EHOSTMEM", -5:
 ALGOS = {"bfs": 0, "sssp": 1, "cc": 2, "pr": 3}
 SYMMETRIC, COPY, VALIDATE, PAIRS = 1, 2, 4, 8
 OPTIONS = {"chunk_cap": 1, "xfer_mode": 2, "dma_min_run": 3, "overlap": 4, "keep_static": 5,
-           "hub_degree": 6, "timing": 7}
+           "hub_degree": 6, "timing": 7, "gather_ctas": 8}
 INF = 0xFFFFFFFF
 
 
@@ -51,7 +51,13 @@ class Stats(ctypes.Structure):
                 ("dma_chunks", ctypes.c_uint64), ("gather_chunks", ctypes.c_uint64),
                 ("time_run_s", ctypes.c_double), ("time_fill_s", ctypes.c_double),
                 ("time_h2d_busy_s", ctypes.c_double), ("gteps", ctypes.c_double),
-                ("gteps_excl_fill", ctypes.c_double), ("vertex_state_bytes", ctypes.c_uint64)]
+                ("gteps_excl_fill", ctypes.c_double), ("vertex_state_bytes", ctypes.c_uint64),
+                ("kernel_launches", ctypes.c_uint64), ("time_classify_s", ctypes.c_double),
+                ("time_static_s", ctypes.c_double), ("static_arcs", ctypes.c_uint64),
+                ("time_ondemand_s", ctypes.c_double), ("ondemand_arcs", ctypes.c_uint64),
+                ("time_gather_s", ctypes.c_double), ("gather_bytes", ctypes.c_uint64),
+                ("time_dma_s", ctypes.c_double), ("dma_bytes", ctypes.c_uint64),
+                ("time_finalize_s", ctypes.c_double), ("time_host_s", ctypes.c_double)]
 
 
 class IterStats(ctypes.Structure):
@@ -181,6 +187,19 @@ class Placement(ctypes.Structure):
 _lib.ascetic_place.argtypes = [ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_double,
                                ctypes.POINTER(Placement)]
 EXPORTS.append("ascetic_place")
+_lib.ascetic_struct_sizes.argtypes = [ctypes.c_void_p]
+EXPORTS.append("ascetic_struct_sizes")
+
+
+def struct_sizes() -> tuple[int, int, int]:
+    out = (ctypes.c_uint64 * 3)()
+    _check(_lib.ascetic_struct_sizes(out))
+    return int(out[0]), int(out[1]), int(out[2])
+
+
+if struct_sizes() != (ctypes.sizeof(Stats), ctypes.sizeof(IterStats), ctypes.sizeof(Placement)):
+    raise ImportError(f"ctypes mirrors out of sync with ascetic.h: lib {struct_sizes()} vs "
+                      f"{(ctypes.sizeof(Stats), ctypes.sizeof(IterStats), ctypes.sizeof(Placement))}")
 
 
 def place(off: np.ndarray, b_e: int, nbytes: int, static_fraction: float = -1.0) -> dict:

@@ -99,6 +99,14 @@ void ascetic_unload(void) {
 
 const char* ascetic_last_error(void) { return g_err.c_str(); }
 
+int ascetic_struct_sizes(uint64_t* out3) {
+    if (!out3) return ASCETIC_EINVAL;
+    out3[0] = sizeof(ascetic_stats_t);
+    out3[1] = sizeof(ascetic_iter_stats_t);
+    out3[2] = sizeof(ascetic_placement_t);
+    return 0;
+}
+
 const char* ascetic_version(void) { return "ascetic-b200 0.1 (sm_100a)"; }
 
 }  // extern "C"

@@ -23,7 +23,8 @@ constexpr uint32_t kInf = 0xFFFFFFFFu;
 constexpr int kClassifyWarps = 8;                       // words per tile = 8 * 32
 constexpr int kTileWords = kClassifyWarps * 32;         // 256 words = 8192 vertices
 constexpr uint32_t kSmallDeg = 32;                      // hit lists shorter than this: warp-cooperative
-constexpr int kEdgeTile = 2048;                         // arcs per CTA tile in the chunk kernels
+constexpr int kEdgeTileShift = 11;
+constexpr int kEdgeTile = 1 << kEdgeTileShift;          // arcs per CTA tile of the miss stream
 
 // Scan fields of the order-preserving compaction (one decoupled look-back pass).
 struct ScanVal {
@@ -57,6 +58,8 @@ struct ClassifyArgs {
     uint32_t* hub_pre;                 // exclusive prefix of pieces per hub
     uint32_t* mq;                      // miss vertices with deg > 0, ascending
     unsigned long long* mq_pre;        // exclusive prefix of miss arcs at each mq entry
+    unsigned long long* mq_src;        // off[v] of each mq entry (host arc index of its list)
+    uint32_t* tile_first;              // [t] = mq index of the vertex holding miss arc t*kEdgeTile
     uint32_t* run_b;
     uint32_t* run_e;
     unsigned long long* run_dst;       // exclusive prefix of miss arcs at run start
@@ -93,7 +96,14 @@ struct Queues {
     const uint32_t* hub_pre;
     const uint32_t* mq;
     const unsigned long long* mq_pre;
+    const unsigned long long* mq_src;
+    const uint32_t* tile_first;
+    uint32_t n_missq;
+    unsigned long long miss_arcs;      // total miss-stream length (arcs)
 };
+
+// kernels launched by this library (bench's gpu_launches claim); defined in edges.cu
+extern unsigned long long g_launches;
 
 // ---- launchers (frontier.cu) ----
 void launch_classify(const ClassifyArgs& a, cudaStream_t s);
@@ -103,11 +113,10 @@ void launch_init(int algo, const DevState& d, uint32_t source, cudaStream_t s);
 void launch_static(int algo, const DevState& d, const Queues& q, const void* static_base,
                    uint32_t n_small, uint32_t n_med, uint32_t n_hub, uint32_t n_pieces,
                    uint32_t piece_arcs, cudaStream_t s);
-void launch_ondemand(int algo, const DevState& d, const Queues& q, uint32_t n_missq,
+void launch_ondemand(int algo, const DevState& d, const Queues& q,
                      const void* chunk, unsigned long long lo, unsigned long long hi, cudaStream_t s);
-void launch_gather(const Queues& q, uint32_t n_missq, const unsigned long long* off,
-                   const void* host_nbr, uint32_t b_e, void* chunk,
-                   unsigned long long lo, unsigned long long hi, cudaStream_t s);
+void launch_gather(const Queues& q, const void* host_nbr, uint32_t b_e, void* chunk,
+                   unsigned long long lo, unsigned long long hi, int max_ctas, cudaStream_t s);
 void launch_finalize(int algo, const DevState& d, cudaStream_t s);
 void launch_set_prefix_bits(uint32_t* bits, uint32_t nwords, uint64_t s_prefix, cudaStream_t s);
 

@@ -16,9 +16,13 @@
 //    queue's 64-bit prefix (one global binary search per CTA).
 //  * the gather is a zero-copy SM copy: host arcs are read through the mapped pinned
 //    CSR with the same arc->source map, so the host never needs the request list.
+#include <type_traits>
+
 #include "ascetic_internal.h"
 
 namespace ascetic {
+
+unsigned long long g_launches = 0;
 
 namespace {
 
@@ -60,17 +64,6 @@ __device__ __forceinline__ void push_arc(const DevState& d, uint32_t sval, uint3
 
 __device__ __forceinline__ double pr_in(const DevState& d, uint32_t id) {
     return (double)__ldg(d.contrib + id);
-}
-
-__device__ __forceinline__ unsigned long long ub_u64(const unsigned long long* a, uint32_t n,
-                                                     unsigned long long x) {
-    // first index i in [0,n) with a[i] > x (n if none)
-    uint32_t lo = 0, hi = n;
-    while (lo < hi) {
-        const uint32_t mid = (lo + hi) >> 1;
-        if (__ldg(a + mid) <= x) lo = mid + 1; else hi = mid;
-    }
-    return lo;
 }
 
 __device__ __forceinline__ uint32_t ub_u32(const uint32_t* a, uint32_t n, uint32_t x) {
@@ -249,30 +242,28 @@ __global__ void __launch_bounds__(256) k_static_hub(DevState d, const uint32_t* 
     }
 }
 
-// ------------------------------------------------------------------ chunk tile staging
-// CTA tile = arcs [t_lo, t_hi) of the miss stream. Stages the covering miss-queue
-// entries: pre (64-bit exclusive arc prefix), the source id, and an aux word.
-struct TileMap {
+// ------------------------------------------------------------------ miss-stream tiles
+// Tile t = miss-stream arcs [t*2048, (t+1)*2048), clipped to the chunk window [lo, hi).
+// tile_first[t] (written by k_classify) is the miss-queue index of the vertex holding arc
+// t*2048, so a CTA stages the covering queue entries [tile_first[t], tile_first[t+1]]
+// (at most 2049) without any global search. Inside the tile each warp owns 256
+// consecutive arcs and maps them to vertices 32 at a time with one shared-memory load,
+// one __reduce_or_sync and one popcount per arc (warp-cooperative merge path).
+struct Tile {
+    unsigned long long t_lo, t_hi;
     uint32_t i0, cnt;
 };
 
-__device__ __forceinline__ TileMap stage_tile(const Queues& q, uint32_t nq, unsigned long long t_lo,
-                                              unsigned long long t_hi, unsigned long long* s_pre,
-                                              uint32_t* s_u, uint32_t* s_i) {
-    if (threadIdx.x == 0) {
-        s_i[0] = (uint32_t)ub_u64(q.mq_pre, nq, t_lo) - 1u;
-        s_i[1] = (uint32_t)ub_u64(q.mq_pre, nq, t_hi - 1) - 1u;
-    }
-    __syncthreads();
-    TileMap m;
-    m.i0 = s_i[0];
-    m.cnt = s_i[1] - s_i[0] + 1u;
-    for (uint32_t k = threadIdx.x; k < m.cnt; k += blockDim.x) {
-        s_pre[k] = __ldg(q.mq_pre + m.i0 + k);
-        s_u[k] = __ldg(q.mq + m.i0 + k);
-    }
-    __syncthreads();
-    return m;
+__device__ __forceinline__ Tile tile_of(const Queues& q, unsigned long long t, unsigned long long lo,
+                                        unsigned long long hi) {
+    Tile x;
+    x.t_lo = max(lo, t << kEdgeTileShift);
+    x.t_hi = min(hi, (t + 1) << kEdgeTileShift);
+    x.i0 = __ldg(q.tile_first + t);
+    const unsigned long long ntot = (q.miss_arcs + kEdgeTile - 1) >> kEdgeTileShift;
+    const uint32_t i1 = (t + 1 < ntot) ? __ldg(q.tile_first + t + 1) : q.n_missq - 1u;
+    x.cnt = i1 - x.i0 + 1u;
+    return x;
 }
 
 // largest k in [lo, cnt) with s_pre[k] <= p (s_pre[lo] <= p guaranteed)
@@ -286,40 +277,60 @@ __device__ __forceinline__ uint32_t find_local(const unsigned long long* s_pre, 
     return lo;
 }
 
+// lanes take arcs p..p+31; k = local index of the vertex holding arc p. Returns this lane's vertex.
+__device__ __forceinline__ uint32_t warp_map(const unsigned long long* s_pre, uint32_t cnt, uint32_t k,
+                                             unsigned long long p, int lane) {
+    const uint32_t idx = k + 1u + (uint32_t)lane;
+    const unsigned long long b = idx < cnt ? s_pre[idx] : ~0ull;
+    const unsigned long long r = b - p;            // >= 1 for every entry after k
+    const uint32_t bit = r < 32ull ? (1u << (uint32_t)r) : 0u;
+    const uint32_t mask = __reduce_or_sync(FULL, bit);
+    return k + (uint32_t)__popc(mask & ((2u << lane) - 1u));
+}
+
 // ------------------------------------------------------------------ on-demand compute
 template <int ALGO>
-__global__ void __launch_bounds__(256) k_ondemand(DevState d, Queues q, uint32_t nq, const void* __restrict__ chunk,
+__global__ void __launch_bounds__(256) k_ondemand(DevState d, Queues q, const void* __restrict__ chunk,
                                                   unsigned long long lo, unsigned long long hi) {
-    __shared__ unsigned long long s_pre[kEdgeTile];
-    __shared__ uint32_t s_u[kEdgeTile];
-    __shared__ uint32_t s_i[2];
-    const unsigned long long t_lo = lo + (unsigned long long)blockIdx.x * kEdgeTile;
-    const unsigned long long t_hi = min(hi, t_lo + kEdgeTile);
-    const TileMap m = stage_tile(q, nq, t_lo, t_hi, s_pre, s_u, s_i);
-    const int lane = threadIdx.x & 31;
-    uint32_t k = 0;
-    for (unsigned long long p0 = t_lo; p0 < t_hi; p0 += blockDim.x) {
-        const unsigned long long p = p0 + threadIdx.x;
-        const bool ok = p < t_hi;
-        if (ok) k = find_local(s_pre, k, m.cnt, p);
-        const uint32_t u = s_u[k];
+    __shared__ unsigned long long s_pre[kEdgeTile + 1];
+    __shared__ uint32_t s_u[kEdgeTile + 1];
+    __shared__ uint32_t s_v[kEdgeTile + 1];
+    const unsigned long long t = (lo >> kEdgeTileShift) + blockIdx.x;
+    const Tile x = tile_of(q, t, lo, hi);
+    for (uint32_t k = threadIdx.x; k < x.cnt; k += blockDim.x) {
+        s_pre[k] = __ldg(q.mq_pre + x.i0 + k);
+        const uint32_t u = __ldg(q.mq + x.i0 + k);
+        s_u[k] = u;
+        if (ALGO == SSSP || ALGO == CC) s_v[k] = __ldg(d.snap + u);
+    }
+    __syncthreads();
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const unsigned long long pw = x.t_lo + (unsigned long long)warp * 256ull;
+    if (pw >= x.t_hi) return;
+    const unsigned long long pe = min(x.t_hi, pw + 256ull);
+    uint32_t k = find_local(s_pre, 0, x.cnt, pw);
+    for (unsigned long long p = pw; p < pe; p += 32) {
+        const uint32_t mk = warp_map(s_pre, x.cnt, k, p, lane);
+        k = __shfl_sync(FULL, mk, 31);
+        const unsigned long long a = p + lane;
+        const bool ok = a < pe;
         if (ALGO == PR) {
-            double x = ok ? pr_in(d, __ldg(reinterpret_cast<const uint32_t*>(chunk) + (p - lo))) : 0.0;
-            const int ki = ok ? (int)k : -1 - lane;
+            double v = ok ? pr_in(d, __ldg(reinterpret_cast<const uint32_t*>(chunk) + (a - lo))) : 0.0;
+            const int key = ok ? (int)mk : -1 - lane;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
-                const double y = __shfl_up_sync(FULL, x, o);
-                const int oi = __shfl_up_sync(FULL, ki, o);
-                if (lane >= o && oi == ki) x += y;
+                const double y = __shfl_up_sync(FULL, v, o);
+                const int ok2 = __shfl_up_sync(FULL, key, o);
+                if (lane >= o && ok2 == key) v += y;
             }
-            const int ni = __shfl_down_sync(FULL, ki, 1);
-            if (ok && (lane == 31 || ni != ki)) atomicAdd(d.sum + u, x);
+            const int nk = __shfl_down_sync(FULL, key, 1);
+            if (ok && (lane == 31 || nk != key)) atomicAdd(d.sum + s_u[mk], v);
         } else if (ok) {
             if (ALGO == SSSP) {
-                const uint2 x = __ldg(reinterpret_cast<const uint2*>(chunk) + (p - lo));
-                push_arc<ALGO>(d, __ldg(d.snap + u), x.x, x.y);
+                const uint2 e = __ldg(reinterpret_cast<const uint2*>(chunk) + (a - lo));
+                push_arc<ALGO>(d, s_v[mk], e.x, e.y);
             } else {
-                push_arc<ALGO>(d, __ldg(d.snap + u), __ldg(reinterpret_cast<const uint32_t*>(chunk) + (p - lo)), 0);
+                push_arc<ALGO>(d, s_v[mk], __ldg(reinterpret_cast<const uint32_t*>(chunk) + (a - lo)), 0);
             }
         }
     }
@@ -340,28 +351,48 @@ __global__ void __launch_bounds__(256) k_ondemand_bfs(DevState d, const uint32_t
 }
 
 // ------------------------------------------------------------------ zero-copy gather (transfer engine)
+// Persistent CTAs stride over the chunk's tiles. Each warp copies its 256 arcs as 8 groups
+// of 32 consecutive arcs: all 8 host loads are issued before the first store, so every
+// lane keeps 8 PCIe reads in flight; consecutive arcs of a run are consecutive host
+// addresses, so each group is one contiguous 128/256-byte read.
 template <int BE>
-__global__ void __launch_bounds__(256) k_gather(Queues q, uint32_t nq, const unsigned long long* __restrict__ off,
-                                                const void* __restrict__ host, void* __restrict__ chunk,
+__global__ void __launch_bounds__(256) k_gather(Queues q, const void* __restrict__ host, void* __restrict__ chunk,
                                                 unsigned long long lo, unsigned long long hi) {
-    __shared__ unsigned long long s_pre[kEdgeTile];
-    __shared__ uint32_t s_u[kEdgeTile];
-    __shared__ uint32_t s_i[2];
-    const unsigned long long t_lo = lo + (unsigned long long)blockIdx.x * kEdgeTile;
-    const unsigned long long t_hi = min(hi, t_lo + kEdgeTile);
-    const TileMap m = stage_tile(q, nq, t_lo, t_hi, s_pre, s_u, s_i);
-    uint32_t k = 0;
-    for (unsigned long long p0 = t_lo; p0 < t_hi; p0 += blockDim.x) {
-        const unsigned long long p = p0 + threadIdx.x;
-        if (p < t_hi) {
-            k = find_local(s_pre, k, m.cnt, p);
-            const unsigned long long src = __ldg(off + s_u[k]) + (p - s_pre[k]);
-            if (BE == 8) {
-                reinterpret_cast<unsigned long long*>(chunk)[p - lo] =
-                    reinterpret_cast<const unsigned long long*>(host)[src];
-            } else {
-                reinterpret_cast<uint32_t*>(chunk)[p - lo] = reinterpret_cast<const uint32_t*>(host)[src];
-            }
+    using T = typename std::conditional<BE == 8, unsigned long long, uint32_t>::type;
+    __shared__ unsigned long long s_pre[kEdgeTile + 1];
+    __shared__ unsigned long long s_src[kEdgeTile + 1];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const T* __restrict__ src = reinterpret_cast<const T*>(host);
+    T* __restrict__ dst = reinterpret_cast<T*>(chunk);
+    const unsigned long long t0 = lo >> kEdgeTileShift, t1 = (hi - 1) >> kEdgeTileShift;
+    for (unsigned long long t = t0 + blockIdx.x; t <= t1; t += gridDim.x) {
+        const Tile x = tile_of(q, t, lo, hi);
+        __syncthreads();
+        for (uint32_t k = threadIdx.x; k < x.cnt; k += blockDim.x) {
+            s_pre[k] = __ldg(q.mq_pre + x.i0 + k);
+            s_src[k] = __ldg(q.mq_src + x.i0 + k);
+        }
+        __syncthreads();
+        const unsigned long long pw = x.t_lo + (unsigned long long)warp * 256ull;
+        if (pw >= x.t_hi) continue;
+        const unsigned long long pe = min(x.t_hi, pw + 256ull);
+        uint32_t k = find_local(s_pre, 0, x.cnt, pw);
+        unsigned long long from[8];
+#pragma unroll
+        for (int g = 0; g < 8; ++g) {
+            const unsigned long long p = pw + 32ull * g;
+            const uint32_t mk = warp_map(s_pre, x.cnt, k, p, lane);
+            k = __shfl_sync(FULL, mk, 31);
+            from[g] = s_src[mk] + (p + lane - s_pre[mk]);
+        }
+        T v[8];
+#pragma unroll
+        for (int g = 0; g < 8; ++g)
+            if (pw + 32ull * g + lane < pe) v[g] = src[from[g]];
+#pragma unroll
+        for (int g = 0; g < 8; ++g) {
+            const unsigned long long a = pw + 32ull * g + lane;
+            if (a < pe) dst[a - lo] = v[g];
         }
     }
 }
@@ -472,9 +503,9 @@ inline unsigned blocks_for(unsigned long long n, int per_block, unsigned cap = 1
 template <int ALGO>
 void static_launch(const DevState& d, const Queues& q, const void* sbase, uint32_t ns, uint32_t nm, uint32_t nh,
                    uint32_t npieces, uint32_t piece, cudaStream_t s) {
-    if (ns) k_static_small<ALGO><<<(ns + 255) / 256, 256, 0, s>>>(d, q.hq_small, ns, sbase);
-    if (nm) k_static_med<ALGO><<<(nm + 7) / 8, 256, 0, s>>>(d, q.hq_med, nm, sbase);
-    if (nh) k_static_hub<ALGO><<<npieces, 256, 0, s>>>(d, q.hq_hub, q.hub_pre, nh, piece, sbase);
+    if (ns) { k_static_small<ALGO><<<(ns + 255) / 256, 256, 0, s>>>(d, q.hq_small, ns, sbase); ++g_launches; }
+    if (nm) { k_static_med<ALGO><<<(nm + 7) / 8, 256, 0, s>>>(d, q.hq_med, nm, sbase); ++g_launches; }
+    if (nh) { k_static_hub<ALGO><<<npieces, 256, 0, s>>>(d, q.hq_hub, q.hub_pre, nh, piece, sbase); ++g_launches; }
 }
 
 }  // namespace
@@ -489,28 +520,32 @@ void launch_static(int algo, const DevState& d, const Queues& q, const void* sba
     }
 }
 
-void launch_ondemand(int algo, const DevState& d, const Queues& q, uint32_t nq, const void* chunk,
+void launch_ondemand(int algo, const DevState& d, const Queues& q, const void* chunk,
                      unsigned long long lo, unsigned long long hi, cudaStream_t s) {
     if (hi <= lo) return;
     const unsigned long long len = hi - lo;
     if (algo == BFS) {
         k_ondemand_bfs<<<blocks_for(len, 256 * 4), 256, 0, s>>>(d, reinterpret_cast<const uint32_t*>(chunk), len);
+        ++g_launches;
         return;
     }
-    const unsigned tiles = (unsigned)((len + kEdgeTile - 1) / kEdgeTile);
+    const unsigned tiles = (unsigned)(((hi - 1) >> kEdgeTileShift) - (lo >> kEdgeTileShift) + 1);
     switch (algo) {
-        case SSSP: k_ondemand<SSSP><<<tiles, 256, 0, s>>>(d, q, nq, chunk, lo, hi); break;
-        case CC: k_ondemand<CC><<<tiles, 256, 0, s>>>(d, q, nq, chunk, lo, hi); break;
-        default: k_ondemand<PR><<<tiles, 256, 0, s>>>(d, q, nq, chunk, lo, hi); break;
+        case SSSP: k_ondemand<SSSP><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
+        case CC: k_ondemand<CC><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
+        default: k_ondemand<PR><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
     }
+    ++g_launches;
 }
 
-void launch_gather(const Queues& q, uint32_t nq, const unsigned long long* off, const void* host_nbr, uint32_t b_e,
-                   void* chunk, unsigned long long lo, unsigned long long hi, cudaStream_t s) {
+void launch_gather(const Queues& q, const void* host_nbr, uint32_t b_e, void* chunk,
+                   unsigned long long lo, unsigned long long hi, int max_ctas, cudaStream_t s) {
     if (hi <= lo) return;
-    const unsigned tiles = (unsigned)((hi - lo + kEdgeTile - 1) / kEdgeTile);
-    if (b_e == 8) k_gather<8><<<tiles, 256, 0, s>>>(q, nq, off, host_nbr, chunk, lo, hi);
-    else k_gather<4><<<tiles, 256, 0, s>>>(q, nq, off, host_nbr, chunk, lo, hi);
+    const unsigned long long tiles = ((hi - 1) >> kEdgeTileShift) - (lo >> kEdgeTileShift) + 1;
+    const unsigned grid = (unsigned)(tiles < (unsigned long long)max_ctas ? tiles : (unsigned long long)max_ctas);
+    if (b_e == 8) k_gather<8><<<grid, 256, 0, s>>>(q, host_nbr, chunk, lo, hi);
+    else k_gather<4><<<grid, 256, 0, s>>>(q, host_nbr, chunk, lo, hi);
+    ++g_launches;
 }
 
 void launch_init(int algo, const DevState& d, uint32_t source, cudaStream_t s) {
@@ -521,41 +556,51 @@ void launch_init(int algo, const DevState& d, uint32_t source, cudaStream_t s) {
         case BFS:
             cudaMemsetAsync(d.visited, 0, (size_t)d.nwords * 4, s);
             k_fill_u32<<<gb, 256, 0, s>>>(d.val, d.n, kInf);
+            ++g_launches;
             k_set_source<<<1, 1, 0, s>>>(d, source, algo);
+            ++g_launches;
             break;
         case SSSP:
             k_fill_u32<<<gb, 256, 0, s>>>(d.val, d.n, kInf);
+            ++g_launches;
             k_fill_u32<<<gb, 256, 0, s>>>(d.snap, d.n, kInf);
+            ++g_launches;
             k_set_source<<<1, 1, 0, s>>>(d, source, algo);
+            ++g_launches;
             break;
         case CC:
             k_iota_u32<<<gb, 256, 0, s>>>(d.val, d.snap, d.n);
+            ++g_launches;
             k_prefix_bits<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d.A, d.nwords, d.n);
+            ++g_launches;
             break;
         default:
             cudaMemsetAsync(d.dang, 0, 2 * sizeof(double), s);
             k_pr_init<<<gb, 256, 0, s>>>(d);
+            ++g_launches;
             k_prefix_bits<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d.A, d.nwords, d.n);
+            ++g_launches;
             break;
     }
 }
 
 void launch_finalize(int algo, const DevState& d, cudaStream_t s) {
     switch (algo) {
-        case BFS: k_finalize_bfs<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d); break;
+        case BFS: k_finalize_bfs<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d); ++g_launches; break;
         case SSSP:
-        case CC: k_finalize_minlabel<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d); break;
+        case CC: k_finalize_minlabel<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d); ++g_launches; break;
         default: {
             const int cur = (int)(d.iter & 1u);
             cudaMemsetAsync(d.dang + (cur ^ 1), 0, sizeof(double), s);
             k_finalize_pr<<<blocks_for(d.n, 256), 256, 0, s>>>(d, cur);
+            ++g_launches;
             break;
         }
     }
 }
 
 void launch_set_prefix_bits(uint32_t* bits, uint32_t nwords, uint64_t s_prefix, cudaStream_t s) {
-    if (nwords) k_prefix_bits<<<blocks_for(nwords, 256), 256, 0, s>>>(bits, nwords, s_prefix);
+    if (nwords) { k_prefix_bits<<<blocks_for(nwords, 256), 256, 0, s>>>(bits, nwords, s_prefix); ++g_launches; }
 }
 
 }  // namespace ascetic

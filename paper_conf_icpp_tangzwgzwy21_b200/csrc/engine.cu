@@ -13,6 +13,7 @@
 #include "engine.h"
 
 #include <algorithm>
+#include <atomic>
 #include <chrono>
 #include <cmath>
 #include <cstring>
@@ -120,6 +121,7 @@ void Engine::load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_
     }
     if (device_ < 0) CK(cudaGetDevice(&device_));
     CK(cudaSetDevice(device_));
+    CK(cudaDeviceGetAttribute(&sm_count_, cudaDevAttrMultiProcessorCount, device_));
 
     n_ = n; m_ = m; b_e_ = b_e; flags_ = flags;
     h_off_copy_.assign(off, off + n + 1);     // host planning copy (placer, DMA runs)
@@ -197,6 +199,8 @@ void Engine::alloc_vertex_state() {
     dalloc(&d_hub_pre_, nhub, &vertex_bytes_);
     dalloc(&d_mq_, n_, &vertex_bytes_);
     dalloc(&d_mq_pre_, n_, &vertex_bytes_);
+    dalloc(&d_mq_src_, n_, &vertex_bytes_);
+    dalloc(&d_tile_first_, (m_ >> kEdgeTileShift) + 2, &vertex_bytes_);
     dalloc(&d_run_b_, n_ / 2 + 1, &vertex_bytes_);
     dalloc(&d_run_e_, n_ / 2 + 1, &vertex_bytes_);
     dalloc(&d_run_dst_, n_ / 2 + 1, &vertex_bytes_);
@@ -294,6 +298,10 @@ void Engine::set_option(int opt, int64_t value) {
             opt_hub_deg_ = (uint32_t)value;
             break;
         case ASCETIC_OPT_TIMING: opt_timing_ = value ? 1 : 0; break;
+        case ASCETIC_OPT_GATHER_CTAS:
+            if (value < 0 || value > 65535) throw Error(ASCETIC_EINVAL, "gather CTAs must be in [0, 65535]");
+            opt_gather_ctas_ = (int)value;
+            break;
         default: throw Error(ASCETIC_EINVAL, "unknown option");
     }
 }
@@ -308,21 +316,22 @@ DevState Engine::dev_state(uint32_t iter) const {
     return d;
 }
 
-Queues Engine::queues() const {
+Queues Engine::queues(const IterTotals& T) const {
     Queues q;
     q.hq_small = d_hq_small_; q.hq_med = d_hq_med_; q.hq_hub = d_hq_hub_; q.hub_pre = d_hub_pre_;
-    q.mq = d_mq_; q.mq_pre = d_mq_pre_;
+    q.mq = d_mq_; q.mq_pre = d_mq_pre_; q.mq_src = d_mq_src_; q.tile_first = d_tile_first_;
+    q.n_missq = T.n_missq; q.miss_arcs = T.miss_arcs;
     return q;
 }
 
 // ------------------------------------------------------------------ transfer engine
 // chunk = miss-stream arcs [lo, hi). mode 1: zero-copy SM gather over the miss queue;
 // mode 2: copy-engine DMA of the run pieces intersecting the window.
-void Engine::transfer_chunk(int buf, unsigned long long lo, unsigned long long hi, int mode,
+void Engine::transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsigned long long hi, int mode,
                             const std::vector<uint32_t>& rb, const std::vector<uint32_t>& re,
                             const std::vector<unsigned long long>& rdst) {
     if (mode == 1) {
-        launch_gather(queues(), h_tot_->n_missq, d_off_, h_nbr_dev_, b_e_, d_chunk_[buf], lo, hi, xs_);
+        launch_gather(q, h_nbr_dev_, b_e_, d_chunk_[buf], lo, hi, opt_gather_ctas_ ? opt_gather_ctas_ : 2 * sm_count_, xs_);
         return;
     }
     // first run whose stream range ends after lo
@@ -359,6 +368,24 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
     std::memset(&st_, 0, sizeof st_);
     pool_.reset();
     const bool timing = opt_timing_ != 0;
+    const unsigned long long launches0 = g_launches;
+
+    // event pairs per kernel class, resolved after the run
+    enum { PH_CLS, PH_STATIC, PH_OND, PH_GATHER, PH_DMA, PH_FIN, PH_N };
+    struct Span { cudaEvent_t a, b; uint32_t iter; int ph; };
+    std::vector<Span> spans;
+    auto open_span = [&](cudaStream_t s) -> cudaEvent_t {
+        if (!timing) return nullptr;
+        cudaEvent_t e = pool_.get();
+        CK(cudaEventRecord(e, s));
+        return e;
+    };
+    auto close_span = [&](cudaEvent_t a, cudaStream_t s, uint32_t it, int ph) {
+        if (!timing) return;
+        cudaEvent_t e = pool_.get();
+        CK(cudaEventRecord(e, s));
+        spans.push_back({a, e, it, ph});
+    };
 
     cudaEvent_t ev_start = pool_.get(), ev_end = pool_.get(), ev_fill0 = pool_.get(), ev_fill1 = pool_.get();
     CK(cudaEventRecord(ev_start, cs_));
@@ -379,15 +406,12 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
     const unsigned long long cap_arcs = cap_ / b_e_;
     std::vector<uint32_t> rb, re;
     std::vector<unsigned long long> rdst;
-    struct IterEv { cudaEvent_t c0, c1, s1, o1, f1; std::vector<std::pair<cudaEvent_t, cudaEvent_t>> x; };
-    std::vector<IterEv> iev;
+    double host_s = 0.0;
     uint32_t t = 0;
     for (t = 0;; ++t) {
         if (max_iters && t == max_iters) break;
-        IterEv ie{};
-        if (timing) { ie.c0 = pool_.get(); CK(cudaEventRecord(ie.c0, cs_)); }
         // ---- GenDataMap + compaction
-        h_tot_->ready = 0;
+        *reinterpret_cast<volatile uint32_t*>(&h_tot_->ready) = 0;
         CK(cudaMemsetAsync(d_tot_, 0, sizeof(IterTotals), cs_));
         ++epoch_;
         if (epoch_ >= (1u << 30)) {
@@ -398,15 +422,30 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         ca.A = d_A_; ca.S = d_S_; ca.off = d_off_; ca.n = n_; ca.nwords = nwords_; ca.ntiles = ntiles_;
         ca.hub_deg = opt_hub_deg_; ca.piece_arcs = kPieceArcs;
         ca.hq_small = d_hq_small_; ca.hq_med = d_hq_med_; ca.hq_hub = d_hq_hub_; ca.hub_pre = d_hub_pre_;
-        ca.mq = d_mq_; ca.mq_pre = d_mq_pre_; ca.run_b = d_run_b_; ca.run_e = d_run_e_; ca.run_dst = d_run_dst_;
+        ca.mq = d_mq_; ca.mq_pre = d_mq_pre_; ca.mq_src = d_mq_src_; ca.tile_first = d_tile_first_; ca.run_b = d_run_b_; ca.run_e = d_run_e_; ca.run_dst = d_run_dst_;
         ca.tile_agg = d_tile_agg_; ca.tile_incl = d_tile_incl_; ca.tile_flag = d_tile_flag_; ca.epoch = epoch_;
         ca.tot = d_tot_; ca.host_tot = h_tot_;
+        cudaEvent_t e0 = open_span(cs_);
         launch_classify(ca, cs_);
         CK(cudaGetLastError());
-        if (timing) { ie.c1 = pool_.get(); CK(cudaEventRecord(ie.c1, cs_)); }
+        close_span(e0, cs_, t, PH_CLS);
         CK(cudaEventRecord(ev_classified_, cs_));
-        CK(cudaEventSynchronize(ev_classified_));
-        const IterTotals T = *h_tot_;
+        // low-latency wait: spin on the flag the last classify CTA writes into mapped memory
+        {
+            const volatile uint32_t* flag = &h_tot_->ready;
+            uint32_t spins = 0;
+            while (!*flag) {
+                if ((++spins & 1023u) == 0) {
+                    const cudaError_t q = cudaEventQuery(ev_classified_);
+                    if (q == cudaSuccess) break;
+                    if (q != cudaErrorNotReady) CK(q);
+                }
+            }
+            std::atomic_thread_fence(std::memory_order_acquire);
+        }
+        const auto th0 = std::chrono::steady_clock::now();
+        const IterTotals T = *const_cast<const IterTotals*>(h_tot_);
+        if (!T.ready) CK(cudaEventSynchronize(ev_classified_));
         st_.d2h_bytes += sizeof(IterTotals);
         if (T.nA == 0) break;
 
@@ -416,12 +455,17 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         is.active_arcs = T.active_arcs; is.hit_arcs = T.hit_arcs; is.miss_bytes = T.miss_arcs * b_e_;
         is.digest = T.digest;
         const DevState d = dev_state(t);
-        const Queues q = queues();
+        const Queues q = queues(T);
         if (algo == ALG_PR) CK(cudaMemsetAsync(d_sum_, 0, n_ * sizeof(double), cs_));
         // ---- Static Computing, overlapping the transfer
-        launch_static(algo, d, q, d_static_, T.n_small, T.n_med, T.n_hub, T.n_pieces, kPieceArcs, cs_);
-        CK(cudaGetLastError());
-        if (timing) { ie.s1 = pool_.get(); CK(cudaEventRecord(ie.s1, cs_)); }
+        if (T.n_small + T.n_med + T.n_hub) {
+            e0 = open_span(cs_);
+            launch_static(algo, d, q, d_static_, T.n_small, T.n_med, T.n_hub, T.n_pieces, kPieceArcs, cs_);
+            CK(cudaGetLastError());
+            close_span(e0, cs_, t, PH_STATIC);
+        }
+        st_.static_arcs += T.hit_arcs;
+        st_.ondemand_arcs += T.miss_arcs;
         // ---- On-demand request, fragmented into chunks
         const unsigned long long miss = T.miss_arcs;
         const uint32_t nchunks = miss ? (uint32_t)((miss + cap_arcs - 1) / cap_arcs) : 0;
@@ -449,22 +493,24 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
             const unsigned long long lo = (unsigned long long)k * cap_arcs;
             const unsigned long long hi = std::min(miss, lo + cap_arcs);
             if (k >= 2) CK(cudaStreamWaitEvent(xs_, consumed_[buf], 0));
-            cudaEvent_t x0 = nullptr, x1 = nullptr;
-            if (timing) { x0 = pool_.get(); CK(cudaEventRecord(x0, xs_)); }
-            transfer_chunk(buf, lo, hi, mode, rb, re, rdst);
+            e0 = open_span(xs_);
+            transfer_chunk(q, buf, lo, hi, mode, rb, re, rdst);
             CK(cudaGetLastError());
-            if (timing) { x1 = pool_.get(); CK(cudaEventRecord(x1, xs_)); ie.x.emplace_back(x0, x1); }
+            close_span(e0, xs_, t, mode == 2 ? PH_DMA : PH_GATHER);
+            if (mode == 2) st_.dma_bytes += (hi - lo) * b_e_; else st_.gather_bytes += (hi - lo) * b_e_;
             CK(cudaEventRecord(ready_[buf], xs_));
             CK(cudaStreamWaitEvent(cs_, ready_[buf], 0));
-            launch_ondemand(algo, d, q, T.n_missq, d_chunk_[buf], lo, hi, cs_);   // On-demand Computing
+            e0 = open_span(cs_);
+            launch_ondemand(algo, d, q, d_chunk_[buf], lo, hi, cs_);   // On-demand Computing
             CK(cudaGetLastError());
+            close_span(e0, cs_, t, PH_OND);
             CK(cudaEventRecord(consumed_[buf], cs_));
         }
-        if (timing) { ie.o1 = pool_.get(); CK(cudaEventRecord(ie.o1, cs_)); }
         // ---- next active set
+        e0 = open_span(cs_);
         launch_finalize(algo, d, cs_);
         CK(cudaGetLastError());
-        if (timing) { ie.f1 = pool_.get(); CK(cudaEventRecord(ie.f1, cs_)); }
+        close_span(e0, cs_, t, PH_FIN);
         is.chunks = nchunks;
         is.mode = nchunks ? (uint32_t)mode : 0u;
         st_.chunks_total += nchunks;
@@ -472,7 +518,7 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         st_.h2d_payload_bytes += is.miss_bytes;
         st_.active_arcs_total += is.active_arcs;
         iters_.push_back(is);
-        iev.push_back(ie);
+        host_s += std::chrono::duration<double>(std::chrono::steady_clock::now() - th0).count();
     }
     CK(cudaEventRecord(ev_end, cs_));
     CK(cudaStreamSynchronize(cs_));
@@ -481,23 +527,24 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
     CK(cudaEventElapsedTime(&ms, ev_start, ev_end));
     float fill_ms = 0.f;
     CK(cudaEventElapsedTime(&fill_ms, ev_fill0, ev_fill1));
-    double h2d_ms = 0.0;
-    if (timing) {
-        for (size_t i = 0; i < iters_.size(); ++i) {
-            auto& is = iters_[i];
-            auto& ie = iev[i];
-            float a = 0.f;
-            cudaEventElapsedTime(&a, ie.c0, ie.c1); is.ms_classify = a;
-            cudaEventElapsedTime(&a, ie.c1, ie.s1); is.ms_static = a;
-            cudaEventElapsedTime(&a, ie.s1, ie.o1); is.ms_ondemand = a;
-            cudaEventElapsedTime(&a, ie.o1, ie.f1); is.ms_finalize = a;
-            cudaEventElapsedTime(&a, ie.c0, ie.f1); is.ms_total = a;
-            float x = 0.f;
-            for (auto& pr : ie.x) { cudaEventElapsedTime(&a, pr.first, pr.second); x += a; }
-            is.ms_h2d = x;
-            h2d_ms += x;
+    double ph[PH_N] = {0, 0, 0, 0, 0, 0};
+    for (const Span& sp : spans) {
+        float a = 0.f;
+        CK(cudaEventElapsedTime(&a, sp.a, sp.b));
+        ph[sp.ph] += a;
+        if (sp.iter < iters_.size()) {
+            auto& is = iters_[sp.iter];
+            switch (sp.ph) {
+                case PH_CLS: is.ms_classify += a; break;
+                case PH_STATIC: is.ms_static += a; break;
+                case PH_OND: is.ms_ondemand += a; break;
+                case PH_GATHER: case PH_DMA: is.ms_h2d += a; break;
+                default: is.ms_finalize += a; break;
+            }
         }
     }
+    for (auto& is : iters_)
+        is.ms_total = is.ms_classify + is.ms_static + is.ms_ondemand + is.ms_finalize;
     st_.algo = algo;
     st_.iterations = t;
     st_.n = n_; st_.m = m_; st_.b_e = b_e_;
@@ -513,11 +560,19 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
     st_.h2d_other_bytes = 0;
     st_.time_run_s = ms / 1e3;
     st_.time_fill_s = fill_ms / 1e3;
-    st_.time_h2d_busy_s = h2d_ms / 1e3 + fill_ms / 1e3;
+    st_.time_classify_s = ph[PH_CLS] / 1e3;
+    st_.time_static_s = ph[PH_STATIC] / 1e3;
+    st_.time_ondemand_s = ph[PH_OND] / 1e3;
+    st_.time_gather_s = ph[PH_GATHER] / 1e3;
+    st_.time_dma_s = ph[PH_DMA] / 1e3;
+    st_.time_finalize_s = ph[PH_FIN] / 1e3;
+    st_.time_host_s = host_s;
+    st_.time_h2d_busy_s = (ph[PH_GATHER] + ph[PH_DMA] + fill_ms) / 1e3;
     st_.gteps = st_.time_run_s > 0 ? (double)st_.active_arcs_total / st_.time_run_s / 1e9 : 0.0;
     const double ex = st_.time_run_s - st_.time_fill_s;
     st_.gteps_excl_fill = ex > 0 ? (double)st_.active_arcs_total / ex / 1e9 : 0.0;
     st_.vertex_state_bytes = vertex_bytes_;
+    st_.kernel_launches = g_launches - launches0;
     last_algo_ = algo;
     have_result_ = true;
 }
@@ -549,7 +604,7 @@ void Engine::unload() {
     dfree(d_off_); dfree(d_A_); dfree(d_S_); dfree(d_next_); dfree(d_visited_);
     dfree(d_val_); dfree(d_snap_); dfree(d_rank_); dfree(d_contrib_); dfree(d_sum_); dfree(d_dang_);
     dfree(d_hq_small_); dfree(d_hq_med_); dfree(d_hq_hub_); dfree(d_hub_pre_);
-    dfree(d_mq_); dfree(d_mq_pre_); dfree(d_run_b_); dfree(d_run_e_); dfree(d_run_dst_);
+    dfree(d_mq_); dfree(d_mq_pre_); dfree(d_mq_src_); dfree(d_tile_first_); dfree(d_run_b_); dfree(d_run_e_); dfree(d_run_dst_);
     dfree(d_tile_agg_); dfree(d_tile_incl_); dfree(d_tile_flag_); dfree(d_tot_);
     if (h_tot_) { cudaFreeHost(h_tot_); h_tot_ = nullptr; }
     if (h_registered_) { cudaHostUnregister(h_registered_); h_registered_ = nullptr; }

@@ -51,11 +51,11 @@ class Engine {
     void alloc_vertex_state();
     void alloc_algo_state(int algo);
     void free_budget_regions();
-    void transfer_chunk(int buf, unsigned long long lo, unsigned long long hi, int mode,
+    void transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsigned long long hi, int mode,
                         const std::vector<uint32_t>& rb, const std::vector<uint32_t>& re,
                         const std::vector<unsigned long long>& rdst);
     DevState dev_state(uint32_t iter) const;
-    Queues queues() const;
+    Queues queues(const IterTotals& T) const;
 
     int state_ = 0;  // 0 unloaded, 1 loaded, 2 ready
     int device_ = -1;
@@ -77,7 +77,10 @@ class Engine {
     double *d_sum_ = nullptr, *d_dang_ = nullptr;
     uint32_t *d_hq_small_ = nullptr, *d_hq_med_ = nullptr, *d_hq_hub_ = nullptr, *d_hub_pre_ = nullptr;
     uint32_t *d_mq_ = nullptr, *d_run_b_ = nullptr, *d_run_e_ = nullptr;
-    unsigned long long *d_mq_pre_ = nullptr, *d_run_dst_ = nullptr;
+    unsigned long long *d_mq_pre_ = nullptr, *d_run_dst_ = nullptr, *d_mq_src_ = nullptr;
+    uint32_t* d_tile_first_ = nullptr;
+    int sm_count_ = 148;
+    int opt_gather_ctas_ = 0;       // 0 = 2 x SMs
     ScanVal *d_tile_agg_ = nullptr, *d_tile_incl_ = nullptr;
     uint32_t* d_tile_flag_ = nullptr;
     uint32_t epoch_ = 0;

@@ -238,8 +238,8 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
         const uint32_t carry_out = (j == 31 ? nextMiss : nm) & 1u;
         const unsigned long long v = (unsigned long long)(w0 + j) * 32ull + lane;
         const bool act = (aw >> lane) & 1u;
-        unsigned long long deg = 0;
-        if (act) deg = __ldg(a.off + v + 1) - __ldg(a.off + v);
+        unsigned long long deg = 0, o0 = 0;
+        if (act) { o0 = __ldg(a.off + v); deg = __ldg(a.off + v + 1) - o0; }
         const bool st = (sw >> lane) & 1u;
         const bool hit = act && st, miss = act && !st;
         const uint32_t hw = aw & sw;
@@ -273,8 +273,14 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
             const uint32_t balQ = __ballot_sync(FULL, isQ);
             if (isQ) {
                 const uint32_t k = bQ + __popc(balQ & lt);
+                const unsigned long long pre = bArcs + ex;
                 a.mq[k] = (uint32_t)v;
-                a.mq_pre[k] = bArcs + ex;
+                a.mq_pre[k] = pre;
+                a.mq_src[k] = o0;
+                // every miss-stream tile start t*kEdgeTile inside [pre, pre+deg) maps to k
+                const unsigned long long t1 = (pre + deg - 1) >> kEdgeTileShift;
+                for (unsigned long long t = (pre + kEdgeTile - 1) >> kEdgeTileShift; t <= t1; ++t)
+                    a.tile_first[t] = k;
             }
             const uint32_t starts = mw & ~((mw << 1) | carry_in);
             const uint32_t ends = mw & ~((mw >> 1) | (carry_out << 31));
@@ -331,6 +337,7 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
 void launch_classify(const ClassifyArgs& a, cudaStream_t s) {
     if (a.ntiles == 0) return;
     k_classify<<<a.ntiles, kClassifyWarps * 32, 0, s>>>(a);
+    ++g_launches;
 }
 
 }  // namespace ascetic

@@ -22,6 +22,10 @@ def main():
     ap.add_argument("--iters", type=int, default=0)
     ap.add_argument("--config", default="")
     ap.add_argument("--oracle", action="store_true")
+    ap.add_argument("--gather-ctas", type=int, default=0)
+    ap.add_argument("--chunk-cap", type=int, default=0)
+    ap.add_argument("--sweep", action="store_true")
+    ap.add_argument("--quiet", action="store_true")
     a = ap.parse_args()
     import paper_conf_icpp_tangzwgzwy21_b200 as asc
     t0 = time.time()
@@ -40,7 +44,25 @@ def main():
     print(f"load {time.time()-t0:.2f}s", flush=True)
     asc.set_budget(budget)
     asc.set_option("xfer_mode", a.xfer)
+    asc.set_option("gather_ctas", a.gather_ctas)
+    asc.set_option("chunk_cap", a.chunk_cap)
     src = gg.sources(g, 1, seed=1)[0]
+    if a.sweep:
+        for gc in [148, 296, 444, 592, 1184]:
+            for cc in [0, 32 << 20, 8 << 20]:
+                asc.set_option("gather_ctas", gc)
+                asc.set_option("chunk_cap", cc)
+                best = None
+                for r in range(2):
+                    asc.run(algo, src, iters)
+                    st, _ = asc.stats(per_iter=False)
+                    if best is None or st["time_run_s"] < best["time_run_s"]:
+                        best = st
+                print(f"gather_ctas={gc:5d} chunk_cap={cc>>20:4d}MiB run_ms={best['time_run_s']*1e3:8.2f} "
+                      f"gather_GBs={best['gather_bytes']/max(best['time_gather_s'],1e-9)/1e9:6.2f} "
+                      f"ondemand_ms={best['time_ondemand_s']*1e3:7.2f} chunks={best['chunks_total']}", flush=True)
+        asc.set_option("gather_ctas", a.gather_ctas)
+        asc.set_option("chunk_cap", a.chunk_cap)
     for r in range(a.reps):
         asc.run(algo, src, iters)
         st, its = asc.stats()
@@ -48,7 +70,7 @@ def main():
                                               "active_arcs_total", "chunks_total", "dma_chunks", "gather_chunks",
                                               "time_run_s", "time_fill_s", "time_h2d_busy_s", "gteps",
                                               "chunk_cap"]}), flush=True)
-    for i in its:
+    for i in ([] if a.quiet else its):
         print({k: (round(v, 3) if isinstance(v, float) else v) for k, v in i.items() if k != "digest"})
     if a.oracle:
         import oracle
