@@ -181,11 +181,28 @@ int ascetic_stats(ascetic_stats_t* out, ascetic_iter_stats_t* per_iter, uint32_t
  * UINT32_MAX = unreached) or n x float (PageRank). bytes must be >= 4n. */
 int ascetic_get_result(void* host_dst, uint64_t bytes);
 
-/* Multi-GPU (one process per GPU, §8(e)): fetch a 128-byte unique id on rank 0,
- * share it out of band (torch.distributed broadcast), then call comm_init on every
- * rank BEFORE load_csr. Returns EUNSUPPORTED when built without NCCL. */
+/* Multi-GPU (one process per GPU; the paper itself is single-GPU).
+ * Vertices are cut into `world` 1D edge-balanced ranges (ascetic_partition); each rank owns
+ * the out-lists of its range, has its own placer / Static Region / On-demand Region / transfer
+ * engine under its own budget B, and keeps the vertex state replicated. One exchange per
+ * iteration: OR of next-frontier bitmaps (BFS), MIN of values (SSSP, CC), SUM of the fp64
+ * dangling mass + every rank's contrib slice (PR). Results equal the single-GPU run.
+ *   ascetic_get_unique_id  rank 0: 128-byte NCCL unique id (EUNSUPPORTED if libnccl.so.2
+ *                          cannot be loaded); share it out of band (torch.distributed)
+ *   ascetic_comm_init      every rank, BEFORE load_csr; device = this rank's GPU
+ *   ascetic_emulate_ranks  drive `world` ranks from THIS process on its one GPU (each rank a
+ *                          full engine with its own device state; collectives by device copies).
+ *                          Same per-rank code path and per-rank statistics; for testing the
+ *                          partitioned path without a multi-GPU box. BEFORE load_csr.
+ * Statistics of a P > 1 run: per_iter holds one record per (iteration, local rank),
+ * iteration-major; sums in ascetic_stats_t are over the local ranks. */
 int ascetic_get_unique_id(void* out128);
 int ascetic_comm_init(int rank, int world, const void* uid128, int device);
+int ascetic_emulate_ranks(int world);
+
+/* Host-only: the 1D edge-balanced rank boundaries (bounds[0] = 0, bounds[parts] = n,
+ * bounds[g] = min{v : off[v] >= ceil(g*m/parts)}). bounds holds parts+1 entries. */
+int ascetic_partition(uint64_t n, const uint64_t* off, uint32_t parts, uint64_t* bounds);
 
 /* Device to use (before load_csr); default = current device. */
 int ascetic_set_device(int device);

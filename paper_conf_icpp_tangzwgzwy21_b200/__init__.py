@@ -187,6 +187,47 @@ class Placement(ctypes.Structure):
 _lib.ascetic_place.argtypes = [ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_double,
                                ctypes.POINTER(Placement)]
 EXPORTS.append("ascetic_place")
+_lib.ascetic_emulate_ranks.argtypes = [ctypes.c_int]
+_lib.ascetic_partition.argtypes = [ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p]
+EXPORTS += ["ascetic_emulate_ranks", "ascetic_partition"]
+
+
+def partition(off: np.ndarray, parts: int) -> np.ndarray:
+    """Host-only 1D edge-balanced rank boundaries (parts+1 entries)."""
+    off = np.ascontiguousarray(off, dtype=np.uint64)
+    b = np.zeros(parts + 1, dtype=np.uint64)
+    _check(_lib.ascetic_partition(off.size - 1, off.ctypes.data, parts, b.ctypes.data))
+    return b
+
+
+def emulate_ranks(world: int) -> None:
+    """Drive `world` ranks from this process on its single GPU (before load_csr)."""
+    _check(_lib.ascetic_emulate_ranks(int(world)))
+
+
+def get_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(_lib.ascetic_get_unique_id(buf))
+    return buf.raw
+
+
+def comm_init(rank: int, world: int, uid: bytes | None, device: int) -> None:
+    """Join the NCCL exchange (one process per GPU), before load_csr."""
+    buf = ctypes.create_string_buffer(uid, 128) if uid is not None else None
+    _check(_lib.ascetic_comm_init(int(rank), int(world), buf, int(device)))
+
+
+def init_distributed(device: int) -> tuple[int, int]:
+    """torch.distributed plumbing only: rank 0's NCCL unique id is broadcast over the
+    already-initialised default process group, then every rank calls comm_init."""
+    import torch.distributed as dist
+    rank, world = dist.get_rank(), dist.get_world_size()
+    if world == 1:
+        return rank, world
+    obj = [get_unique_id() if rank == 0 else None]
+    dist.broadcast_object_list(obj, src=0)
+    comm_init(rank, world, obj[0], device)
+    return rank, world
 _lib.ascetic_struct_sizes.argtypes = [ctypes.c_void_p]
 EXPORTS.append("ascetic_struct_sizes")
 

@@ -10,8 +10,8 @@ CSRC = os.path.join(HERE, "csrc")
 INCLUDE = os.path.join(os.path.dirname(HERE), "include")
 LIB = os.path.join(HERE, "libascetic.so")
 OBJDIR = os.path.join(HERE, "build")
-SOURCES = ["frontier.cu", "edges.cu", "engine.cu", "api.cpp"]
-HEADERS = ["ascetic_internal.h", "engine.h"]
+SOURCES = ["frontier.cu", "edges.cu", "engine.cu", "comm.cu", "api.cpp"]
+HEADERS = ["ascetic_internal.h", "engine.h", "comm.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3", "-I", INCLUDE, "-I", CSRC]

@@ -78,15 +78,28 @@ int ascetic_get_result(void* host_dst, uint64_t bytes) {
 }
 
 int ascetic_get_unique_id(void* out128) {
-    (void)out128;
-    g_err = "multi-GPU exchange is driven by the Python layer (torch.distributed); no NCCL in libascetic";
-    return ASCETIC_EUNSUPPORTED;
+    return guarded([&] {
+        if (!out128) throw ascetic::Error(ASCETIC_EINVAL, "out128 is NULL");
+        ascetic::Comm::unique_id(out128);
+        return 0;
+    });
 }
 
 int ascetic_comm_init(int rank, int world, const void* uid128, int device) {
-    (void)rank; (void)world; (void)uid128; (void)device;
-    g_err = "multi-GPU exchange is driven by the Python layer (torch.distributed); no NCCL in libascetic";
-    return ASCETIC_EUNSUPPORTED;
+    return guarded([&] { engine().comm_init(rank, world, uid128, device); return 0; });
+}
+
+int ascetic_emulate_ranks(int world) {
+    return guarded([&] { engine().emulate_ranks(world); return 0; });
+}
+
+int ascetic_partition(uint64_t n, const uint64_t* off, uint32_t parts, uint64_t* bounds) {
+    return guarded([&] {
+        if (!off || !bounds || parts < 1) throw ascetic::Error(ASCETIC_EINVAL, "bad argument");
+        const auto b = ascetic::partition(off, n, parts);
+        for (uint32_t i = 0; i <= parts; ++i) bounds[i] = b[i];
+        return 0;
+    });
 }
 
 int ascetic_set_device(int device) {

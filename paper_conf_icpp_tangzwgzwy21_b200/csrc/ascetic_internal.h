@@ -48,6 +48,7 @@ struct ClassifyArgs {
     const uint32_t* S;
     const unsigned long long* off;
     uint64_t n;
+    uint64_t vlo, vhi;                 // owned vertex range of this rank
     uint32_t nwords;
     uint32_t ntiles;
     uint32_t hub_deg;
@@ -87,6 +88,8 @@ struct DevState {
     double* sum;
     double* dang;          // [0] = current dangling mass, [1] = next
     uint32_t iter;         // t
+    uint64_t vlo, vhi;     // owned vertex range (PR finalize)
+    unsigned long long static_arc0;   // first arc held by the Static Region (off[vlo])
 };
 
 struct Queues {
@@ -117,7 +120,14 @@ void launch_ondemand(int algo, const DevState& d, const Queues& q,
                      const void* chunk, unsigned long long lo, unsigned long long hi, cudaStream_t s);
 void launch_gather(const Queues& q, const void* host_nbr, uint32_t b_e, void* chunk,
                    unsigned long long lo, unsigned long long hi, int max_ctas, cudaStream_t s);
-void launch_finalize(int algo, const DevState& d, cudaStream_t s);
-void launch_set_prefix_bits(uint32_t* bits, uint32_t nwords, uint64_t s_prefix, cudaStream_t s);
+// dense = values were exchanged (P > 1): SSSP/CC rebuild A from val < snap over all vertices
+void launch_finalize(int algo, const DevState& d, bool dense, cudaStream_t s);
+// collectives' device side (comm.cu drives them)
+void launch_or_reduce(uint32_t* dst, const uint32_t* gathered, uint32_t parts, uint64_t nw, cudaStream_t s);
+void launch_or_into(uint32_t* dst, const uint32_t* src, uint64_t nw, cudaStream_t s);
+void launch_min_into(uint32_t* dst, const uint32_t* src, uint64_t n, cudaStream_t s);
+void launch_add_f64(double* dst, const double* src, cudaStream_t s);
+// bits := the vertex range [a, b)
+void launch_set_range_bits(uint32_t* bits, uint32_t nwords, uint64_t a, uint64_t b, cudaStream_t s);
 
 }  // namespace ascetic

@@ -1,0 +1,158 @@
+// comm.cu — NCCL (dlopen) and single-GPU emulated collectives for the per-iteration exchange.
+#include "comm.h"
+
+#include <dlfcn.h>
+#include <nccl.h>   // types and enums only; every function is resolved with dlsym
+
+#include <cstring>
+
+#include "ascetic_internal.h"
+#include "engine.h"
+
+namespace ascetic {
+
+namespace {
+
+struct NcclApi {
+    bool loaded = false;
+    ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+    ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+    ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+    ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*AllGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*Broadcast)(const void*, void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*GroupStart)() = nullptr;
+    ncclResult_t (*GroupEnd)() = nullptr;
+    const char* (*GetErrorString)(ncclResult_t) = nullptr;
+};
+
+NcclApi& nccl() {
+    static NcclApi api;
+    if (api.loaded) return api;
+    void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL | RTLD_NOLOAD);   // torch's, if already loaded
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) throw Error(ASCETIC_EUNSUPPORTED, std::string("cannot load libnccl.so.2: ") + dlerror());
+    auto sym = [&](const char* name) {
+        void* p = dlsym(h, name);
+        if (!p) throw Error(ASCETIC_EUNSUPPORTED, std::string("libnccl lacks ") + name);
+        return p;
+    };
+    api.GetUniqueId = (decltype(api.GetUniqueId))sym("ncclGetUniqueId");
+    api.CommInitRank = (decltype(api.CommInitRank))sym("ncclCommInitRank");
+    api.CommDestroy = (decltype(api.CommDestroy))sym("ncclCommDestroy");
+    api.AllReduce = (decltype(api.AllReduce))sym("ncclAllReduce");
+    api.AllGather = (decltype(api.AllGather))sym("ncclAllGather");
+    api.Broadcast = (decltype(api.Broadcast))sym("ncclBroadcast");
+    api.GroupStart = (decltype(api.GroupStart))sym("ncclGroupStart");
+    api.GroupEnd = (decltype(api.GroupEnd))sym("ncclGroupEnd");
+    api.GetErrorString = (decltype(api.GetErrorString))sym("ncclGetErrorString");
+    api.loaded = true;
+    return api;
+}
+
+void NC(ncclResult_t r, const char* what) {
+    if (r != ncclSuccess) throw Error(ASCETIC_ENCCL, std::string(what) + ": " + nccl().GetErrorString(r));
+}
+
+void CKc(cudaError_t e, const char* what) {
+    if (e != cudaSuccess) throw Error(ASCETIC_ECUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+}  // namespace
+
+void Comm::unique_id(void* out128) {
+    ncclUniqueId id;
+    NC(nccl().GetUniqueId(&id), "ncclGetUniqueId");
+    std::memcpy(out128, &id, sizeof id);
+}
+
+void Comm::init_nccl(int rank, int world, const void* uid128) {
+    destroy();
+    if (world < 1 || rank < 0 || rank >= world) throw Error(ASCETIC_EINVAL, "bad rank/world");
+    world_ = world; rank_ = rank; emulated_ = false;
+    if (world == 1) return;
+    ncclUniqueId id;
+    std::memcpy(&id, uid128, sizeof id);
+    ncclComm_t c = nullptr;
+    NC(nccl().CommInitRank(&c, world, id, rank), "ncclCommInitRank");
+    nccl_comm_ = c;
+}
+
+void Comm::init_emulated(int world) {
+    destroy();
+    if (world < 1) throw Error(ASCETIC_EINVAL, "world must be >= 1");
+    world_ = world; rank_ = 0; emulated_ = world > 1;
+}
+
+void Comm::destroy() {
+    if (nccl_comm_) { nccl().CommDestroy((ncclComm_t)nccl_comm_); nccl_comm_ = nullptr; }
+    if (scratch_) { cudaFree(scratch_); scratch_ = nullptr; scratch_words_ = 0; }
+    world_ = 1; rank_ = 0; emulated_ = false;
+}
+
+void Comm::or_words(const std::vector<uint32_t*>& local, uint64_t nw, cudaStream_t s) {
+    if (!active() || nw == 0) return;
+    if (emulated_) {
+        for (size_t p = 1; p < local.size(); ++p) launch_or_into(local[0], local[p], nw, s);
+        for (size_t p = 1; p < local.size(); ++p)
+            CKc(cudaMemcpyAsync(local[p], local[0], nw * 4, cudaMemcpyDeviceToDevice, s), "or copy-back");
+        return;
+    }
+    const uint64_t need = nw * (uint64_t)world_;
+    if (scratch_words_ < need) {
+        if (scratch_) cudaFree(scratch_);
+        CKc(cudaMalloc(&scratch_, need * 4), "exchange scratch");
+        scratch_words_ = need;
+    }
+    NC(nccl().AllGather(local[0], scratch_, nw, ncclUint32, (ncclComm_t)nccl_comm_, s), "ncclAllGather(bitmap)");
+    launch_or_reduce(local[0], scratch_, (uint32_t)world_, nw, s);
+}
+
+void Comm::min_u32(const std::vector<uint32_t*>& local, uint64_t n, cudaStream_t s) {
+    if (!active() || n == 0) return;
+    if (emulated_) {
+        for (size_t p = 1; p < local.size(); ++p) launch_min_into(local[0], local[p], n, s);
+        for (size_t p = 1; p < local.size(); ++p)
+            CKc(cudaMemcpyAsync(local[p], local[0], n * 4, cudaMemcpyDeviceToDevice, s), "min copy-back");
+        return;
+    }
+    NC(nccl().AllReduce(local[0], local[0], n, ncclUint32, ncclMin, (ncclComm_t)nccl_comm_, s), "ncclAllReduce(min)");
+}
+
+void Comm::sum_f64(const std::vector<double*>& local, cudaStream_t s) {
+    if (!active()) return;
+    if (emulated_) {
+        for (size_t p = 1; p < local.size(); ++p) launch_add_f64(local[0], local[p], s);
+        for (size_t p = 1; p < local.size(); ++p)
+            CKc(cudaMemcpyAsync(local[p], local[0], 8, cudaMemcpyDeviceToDevice, s), "sum copy-back");
+        return;
+    }
+    NC(nccl().AllReduce(local[0], local[0], 1, ncclFloat64, ncclSum, (ncclComm_t)nccl_comm_, s), "ncclAllReduce(sum)");
+}
+
+void Comm::share_slices(const std::vector<void*>& local, const std::vector<uint64_t>& bounds, uint32_t elem_bytes,
+                        cudaStream_t s) {
+    if (!active()) return;
+    if (emulated_) {
+        for (size_t r = 0; r < local.size(); ++r) {
+            const uint64_t off = bounds[r] * elem_bytes, len = (bounds[r + 1] - bounds[r]) * elem_bytes;
+            if (!len) continue;
+            for (size_t p = 0; p < local.size(); ++p)
+                if (p != r)
+                    CKc(cudaMemcpyAsync((char*)local[p] + off, (const char*)local[r] + off, len, cudaMemcpyDeviceToDevice, s),
+                        "slice copy");
+        }
+        return;
+    }
+    NC(nccl().GroupStart(), "ncclGroupStart");
+    for (int r = 0; r < world_; ++r) {
+        const uint64_t off = bounds[r] * elem_bytes, len = (bounds[r + 1] - bounds[r]) * elem_bytes;
+        if (!len) continue;
+        char* p = (char*)local[0] + off;
+        NC(nccl().Broadcast(p, p, len, ncclInt8, r, (ncclComm_t)nccl_comm_, s), "ncclBroadcast(slice)");
+    }
+    NC(nccl().GroupEnd(), "ncclGroupEnd");
+}
+
+}  // namespace ascetic

@@ -1,0 +1,55 @@
+// comm.h — the per-iteration exchange of the multi-GPU path (the paper itself
+// is single-GPU). One process per GPU, 1D vertex ranges, replicated vertex state:
+//   BFS       : OR of the next-frontier bitmaps        (NCCL has no bitwise OR: all-gather + OR kernel)
+//   SSSP / CC : MIN of the value arrays               (ncclAllReduce min)
+//   PR        : SUM of the fp64 dangling partials + every rank's contrib slice to all ranks
+// Two back ends behind one interface:
+//   NCCL     — across processes (libnccl.so.2 is dlopen'ed on first use, so single-GPU
+//              runs never load it and torch's own NCCL is reused when already loaded);
+//   emulated — P ranks driven by ONE process on ONE GPU (each rank a full engine part with
+//              its own device state); the same collectives done with device copies and
+//              reduction kernels. It runs the identical per-rank code path, which is how the
+//              P > 1 path is tested on a single GPU.
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include <cuda_runtime.h>
+
+namespace ascetic {
+
+class Comm {
+  public:
+    // NCCL back end
+    static void unique_id(void* out128);
+    void init_nccl(int rank, int world, const void* uid128);
+    // emulated back end: `world` ranks, all local
+    void init_emulated(int world);
+    void destroy();
+    ~Comm() { destroy(); }
+
+    bool active() const { return world_ > 1; }
+    bool emulated() const { return emulated_; }
+    int world() const { return world_; }
+    int rank() const { return rank_; }
+
+    // Collectives over all ranks. `local` = this process's buffers: one per local rank
+    // (1 with NCCL, world with emulation). Everything is enqueued on `s`.
+    void or_words(const std::vector<uint32_t*>& local, uint64_t nw, cudaStream_t s);
+    void min_u32(const std::vector<uint32_t*>& local, uint64_t n, cudaStream_t s);
+    void sum_f64(const std::vector<double*>& local, cudaStream_t s);
+    // rank r owns elements [bounds[r], bounds[r+1]) of an elem_bytes array; afterwards every
+    // rank holds every slice
+    void share_slices(const std::vector<void*>& local, const std::vector<uint64_t>& bounds, uint32_t elem_bytes,
+                      cudaStream_t s);
+
+  private:
+    int world_ = 1, rank_ = 0;
+    bool emulated_ = false;
+    void* nccl_comm_ = nullptr;
+    uint32_t* scratch_ = nullptr;
+    uint64_t scratch_words_ = 0;
+};
+
+}  // namespace ascetic

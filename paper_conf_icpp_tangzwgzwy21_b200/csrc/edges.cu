@@ -172,7 +172,7 @@ __global__ void __launch_bounds__(256) k_static_small(DevState d, const uint32_t
         const uint32_t uex = __shfl_sync(FULL, excl, i);
         const uint32_t usv = __shfl_sync(FULL, sval, i);
         const bool ok = k < total;
-        const unsigned long long e = ust + (k - uex);
+        const unsigned long long e = ust + (k - uex) - d.static_arc0;   // index into the Static Region
         if (ALGO == PR) {
             double x = ok ? pr_in(d, __ldg(reinterpret_cast<const uint32_t*>(sbase) + e)) : 0.0;
 #pragma unroll
@@ -208,7 +208,7 @@ __global__ void __launch_bounds__(256) k_static_med(DevState d, const uint32_t* 
     const uint32_t u = __ldg(q + gw);
     const unsigned long long a0 = __ldg(d.off + u), a1 = __ldg(d.off + u + 1);
     const uint32_t sval = (ALGO == SSSP || ALGO == CC) ? __ldg(d.snap + u) : 0u;
-    double acc = expand_list<ALGO>(d, sbase, a0, a1, sval, lane, 32);
+    double acc = expand_list<ALGO>(d, sbase, a0 - d.static_arc0, a1 - d.static_arc0, sval, lane, 32);
     if (ALGO == PR) {
         acc = warp_sum_d(acc);
         if (lane == 0) d.sum[u] = acc;
@@ -229,7 +229,7 @@ __global__ void __launch_bounds__(256) k_static_hub(DevState d, const uint32_t* 
     const unsigned long long a0 = o0 + (unsigned long long)pidx * piece_arcs;
     const unsigned long long a1 = min(o1, a0 + piece_arcs);
     const uint32_t sval = (ALGO == SSSP || ALGO == CC) ? __ldg(d.snap + u) : 0u;
-    double acc = expand_list<ALGO>(d, sbase, a0, a1, sval, threadIdx.x, blockDim.x);
+    double acc = expand_list<ALGO>(d, sbase, a0 - d.static_arc0, a1 - d.static_arc0, sval, threadIdx.x, blockDim.x);
     if (ALGO == PR) {
         acc = warp_sum_d(acc);
         if ((threadIdx.x & 31) == 0) s_red[threadIdx.x >> 5] = acc;
@@ -309,6 +309,37 @@ __global__ void __launch_bounds__(256) k_ondemand(DevState d, Queues q, const vo
     if (pw >= x.t_hi) return;
     const unsigned long long pe = min(x.t_hi, pw + 256ull);
     uint32_t k = find_local(s_pre, 0, x.cnt, pw);
+    if (ALGO == SSSP || ALGO == CC) {
+        // 3 phases over the warp's 8 groups of 32 arcs: map + chunk loads, state loads, atomics
+        uint32_t id[8], cand[8], cur[8];
+#pragma unroll
+        for (int g = 0; g < 8; ++g) {
+            const unsigned long long p = pw + 32ull * g;
+            const uint32_t mk = warp_map(s_pre, x.cnt, k, p, lane);
+            k = __shfl_sync(FULL, mk, 31);
+            const unsigned long long a = p + lane;
+            id[g] = kInf;
+            if (a < pe) {
+                if (ALGO == SSSP) {
+                    const uint2 e = __ldg(reinterpret_cast<const uint2*>(chunk) + (a - lo));
+                    id[g] = e.x;
+                    cand[g] = sat_add(s_v[mk], e.y);
+                } else {
+                    id[g] = __ldg(reinterpret_cast<const uint32_t*>(chunk) + (a - lo));
+                    cand[g] = s_v[mk];
+                }
+            }
+        }
+#pragma unroll
+        for (int g = 0; g < 8; ++g) cur[g] = id[g] != kInf ? d.val[id[g]] : 0u;
+#pragma unroll
+        for (int g = 0; g < 8; ++g) {
+            if (id[g] != kInf && cand[g] < cur[g]) {
+                const uint32_t old = atomicMin(d.val + id[g], cand[g]);
+                if (cand[g] < old) set_next(d, id[g]);
+            }
+        }
+    } else
     for (unsigned long long p = pw; p < pe; p += 32) {
         const uint32_t mk = warp_map(s_pre, x.cnt, k, p, lane);
         k = __shfl_sync(FULL, mk, 31);
@@ -410,13 +441,16 @@ __global__ void k_iota_u32(uint32_t* a, uint32_t* b, uint64_t n) {
     }
 }
 
-__global__ void k_prefix_bits(uint32_t* bits, uint32_t nwords, uint64_t s) {
+// bits = exactly the vertex range [a, b)
+__global__ void k_range_bits(uint32_t* bits, uint32_t nwords, uint64_t a, uint64_t b) {
     for (uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < nwords; w += (uint64_t)gridDim.x * blockDim.x) {
-        const uint64_t lo = w * 32;
-        uint32_t x;
-        if (lo + 32 <= s) x = FULL;
-        else if (lo >= s) x = 0u;
-        else x = (1u << (uint32_t)(s - lo)) - 1u;
+        const uint64_t base = w * 32;
+        const uint64_t lo = a > base ? a : base, hi = b < base + 32 ? b : base + 32;
+        uint32_t x = 0u;
+        if (lo < hi) {
+            const uint32_t top = (uint32_t)(hi - base), bot = (uint32_t)(lo - base);
+            x = (top == 32 ? FULL : ((1u << top) - 1u)) & ~((1u << bot) - 1u);
+        }
         bits[w] = x;
     }
 }
@@ -483,7 +517,8 @@ __global__ void k_finalize_pr(DevState d, int cur) {
     const double inv_n = 1.0 / (double)d.n;
     const double dc = d.dang[cur];
     double dn = 0.0;
-    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < d.n; v += (uint64_t)gridDim.x * blockDim.x) {
+    for (uint64_t v = d.vlo + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < d.vhi;
+         v += (uint64_t)gridDim.x * blockDim.x) {
         const double r = (1.0 - kDamp) * inv_n + kDamp * (d.sum[v] + dc * inv_n);
         const unsigned long long deg = __ldg(d.off + v + 1) - __ldg(d.off + v);
         d.rank[v] = (float)r;
@@ -493,6 +528,41 @@ __global__ void k_finalize_pr(DevState d, int cur) {
     dn = warp_sum_d(dn);
     if ((threadIdx.x & 31) == 0 && dn != 0.0) atomicAdd(d.dang + (cur ^ 1), dn);
 }
+
+// P > 1: values were MIN-exchanged, so A_{t+1} = {v : val[v] < snap[v]} over every vertex
+__global__ void k_finalize_minlabel_dense(DevState d) {
+    for (uint32_t w = blockIdx.x * blockDim.x + threadIdx.x; w < d.nwords; w += gridDim.x * blockDim.x) {
+        uint32_t bits = 0;
+        const uint64_t v0 = (uint64_t)w * 32;
+        const uint32_t cnt = (uint32_t)min((uint64_t)32, d.n - v0);
+        for (uint32_t i = 0; i < cnt; ++i) {
+            const uint32_t x = d.val[v0 + i], y = d.snap[v0 + i];
+            if (x < y) { bits |= 1u << i; d.snap[v0 + i] = x; }
+        }
+        d.A[w] = bits;
+        d.next[w] = 0;
+    }
+}
+
+__global__ void k_or_reduce(uint32_t* __restrict__ dst, const uint32_t* __restrict__ g, uint32_t parts, uint64_t nw) {
+    for (uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < nw; w += (uint64_t)gridDim.x * blockDim.x) {
+        uint32_t x = 0;
+        for (uint32_t p = 0; p < parts; ++p) x |= g[(uint64_t)p * nw + w];
+        dst[w] = x;
+    }
+}
+
+__global__ void k_or_into(uint32_t* __restrict__ dst, const uint32_t* __restrict__ src, uint64_t nw) {
+    for (uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < nw; w += (uint64_t)gridDim.x * blockDim.x)
+        dst[w] |= src[w];
+}
+
+__global__ void k_min_into(uint32_t* __restrict__ dst, const uint32_t* __restrict__ src, uint64_t n) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+        dst[i] = min(dst[i], src[i]);
+}
+
+__global__ void k_add_f64(double* dst, const double* src) { dst[0] += src[0]; }
 
 inline unsigned blocks_for(unsigned long long n, int per_block, unsigned cap = 148u * 16u) {
     unsigned long long b = (n + per_block - 1) / per_block;
@@ -571,36 +641,59 @@ void launch_init(int algo, const DevState& d, uint32_t source, cudaStream_t s) {
         case CC:
             k_iota_u32<<<gb, 256, 0, s>>>(d.val, d.snap, d.n);
             ++g_launches;
-            k_prefix_bits<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d.A, d.nwords, d.n);
+            k_range_bits<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d.A, d.nwords, 0, d.n);
             ++g_launches;
             break;
         default:
             cudaMemsetAsync(d.dang, 0, 2 * sizeof(double), s);
             k_pr_init<<<gb, 256, 0, s>>>(d);
             ++g_launches;
-            k_prefix_bits<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d.A, d.nwords, d.n);
+            k_range_bits<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d.A, d.nwords, 0, d.n);
             ++g_launches;
             break;
     }
 }
 
-void launch_finalize(int algo, const DevState& d, cudaStream_t s) {
+void launch_finalize(int algo, const DevState& d, bool dense, cudaStream_t s) {
     switch (algo) {
-        case BFS: k_finalize_bfs<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d); ++g_launches; break;
+        case BFS: k_finalize_bfs<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d); break;
         case SSSP:
-        case CC: k_finalize_minlabel<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d); ++g_launches; break;
+        case CC:
+            if (dense) k_finalize_minlabel_dense<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d);
+            else k_finalize_minlabel<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d);
+            break;
         default: {
             const int cur = (int)(d.iter & 1u);
             cudaMemsetAsync(d.dang + (cur ^ 1), 0, sizeof(double), s);
-            k_finalize_pr<<<blocks_for(d.n, 256), 256, 0, s>>>(d, cur);
-            ++g_launches;
+            k_finalize_pr<<<blocks_for(d.vhi > d.vlo ? d.vhi - d.vlo : 1, 256), 256, 0, s>>>(d, cur);
             break;
         }
     }
+    ++g_launches;
 }
 
-void launch_set_prefix_bits(uint32_t* bits, uint32_t nwords, uint64_t s_prefix, cudaStream_t s) {
-    if (nwords) { k_prefix_bits<<<blocks_for(nwords, 256), 256, 0, s>>>(bits, nwords, s_prefix); ++g_launches; }
+void launch_or_reduce(uint32_t* dst, const uint32_t* gathered, uint32_t parts, uint64_t nw, cudaStream_t s) {
+    k_or_reduce<<<blocks_for(nw, 256), 256, 0, s>>>(dst, gathered, parts, nw);
+    ++g_launches;
+}
+
+void launch_or_into(uint32_t* dst, const uint32_t* src, uint64_t nw, cudaStream_t s) {
+    k_or_into<<<blocks_for(nw, 256), 256, 0, s>>>(dst, src, nw);
+    ++g_launches;
+}
+
+void launch_min_into(uint32_t* dst, const uint32_t* src, uint64_t n, cudaStream_t s) {
+    k_min_into<<<blocks_for(n, 256), 256, 0, s>>>(dst, src, n);
+    ++g_launches;
+}
+
+void launch_add_f64(double* dst, const double* src, cudaStream_t s) {
+    k_add_f64<<<1, 1, 0, s>>>(dst, src);
+    ++g_launches;
+}
+
+void launch_set_range_bits(uint32_t* bits, uint32_t nwords, uint64_t a, uint64_t b, cudaStream_t s) {
+    if (nwords) { k_range_bits<<<blocks_for(nwords, 256), 256, 0, s>>>(bits, nwords, a, b); ++g_launches; }
 }
 
 }  // namespace ascetic

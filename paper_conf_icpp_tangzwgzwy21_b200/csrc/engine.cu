@@ -1,13 +1,15 @@
-// engine.cu — run controller: placer, transfer engine, per-iteration pipeline.
+// engine.cu — run controller: placer, partition, transfer engine, per-iteration pipeline.
 //
-// One iteration (Fig. 4; Fig. 5), B200 version:
-//   compute stream cs : classify+compact  ──► host reads 80 B of totals (mapped)
+// One iteration (Fig. 4; Fig. 5), B200 version, per rank part:
+//   compute stream cs : classify+compact  ──► host reads 96 B of totals (mapped memory)
 //   cs                : static-hit kernels (Static Computing)
 //   copy stream xs    : chunk k = miss-stream arcs [k*cap, (k+1)*cap) ->
 //                       zero-copy SM gather or copy-engine DMA of runs
 //                       buffer k%2 waits consumed[k-2]; records ready[k]
 //   cs                : waits ready[k] -> on-demand kernel -> records consumed[k]
+//   (P > 1)           : exchange: OR bitmaps (BFS) / MIN values (SSSP, CC)
 //   cs                : finalize: next active set
+//   (P > 1, PR)       : exchange: SUM dangling, share contrib slices
 // Fragmenting when the request exceeds the On-demand Region (§3.3) is the
 // chunk loop; the static compute overlaps the transfer (§3.2).
 #include "engine.h"
@@ -30,12 +32,13 @@ namespace ascetic {
 
 enum { ALG_BFS = 0, ALG_SSSP = 1, ALG_CC = 2, ALG_PR = 3 };
 
-// ------------------------------------------------------------------ placer
+// ------------------------------------------------------------------ placer / partition
 Placement place(const uint64_t* off, uint64_t n, uint32_t b_e, uint64_t budget, double frac) {
     Placement p;
     const double K = 0.10;
+    const uint64_t base = off[0];
     p.B = budget;
-    p.D = (uint64_t)b_e * off[n];
+    p.D = (uint64_t)b_e * (off[n] - base);
     double R;
     if (frac >= 0.0 && frac <= 1.0) {
         R = frac;
@@ -48,13 +51,26 @@ Placement place(const uint64_t* off, uint64_t n, uint32_t b_e, uint64_t budget, 
     uint64_t Ms = (uint64_t)std::floor(R * (double)budget / 16384.0) * 16384ull;  // 16 KB chunks
     if (Ms > p.D) Ms = p.D;
     p.Ms = Ms;
-    // front prefix of whole lists: s = max{v : b_e off[v] <= Ms}
-    const uint64_t lim = Ms / b_e;
+    // front prefix of whole lists: s = max{v : b_e (off[v]-base) <= Ms}
+    const uint64_t lim = base + Ms / b_e;
     p.s = (uint64_t)(std::upper_bound(off, off + n + 1, lim) - off) - 1;
-    p.static_bytes = (uint64_t)b_e * off[p.s];
+    p.static_bytes = (uint64_t)b_e * (off[p.s] - base);
     p.C = budget >= Ms ? budget - Ms : 0;
     p.cap = p.C / 2 / 16 * 16;
     return p;
+}
+
+std::vector<uint64_t> partition(const uint64_t* off, uint64_t n, uint32_t P) {
+    std::vector<uint64_t> b(P + 1);
+    const uint64_t m = off[n];
+    b[0] = 0;
+    for (uint32_t g = 1; g < P; ++g) {
+        const uint64_t target = ((uint64_t)g * m + P - 1) / P;
+        b[g] = (uint64_t)(std::lower_bound(off, off + n + 1, target) - off);
+        if (b[g] > n) b[g] = n;
+    }
+    b[P] = n;
+    return b;
 }
 
 // ------------------------------------------------------------------ event pool
@@ -88,6 +104,413 @@ static void dfree(T*& p) {
     p = nullptr;
 }
 
+void HostGraph::release() {
+    if (registered) { cudaHostUnregister(registered); registered = nullptr; }
+    if (owned) { cudaFreeHost(owned); owned = nullptr; }
+    nbr = nbr_dev = nullptr;
+}
+
+// ================================================================== Part
+Part::Part(const HostGraph& g, const Options& o, int rank, uint64_t vlo, uint64_t vhi, int sm_count)
+    : g_(g), o_(o), rank_(rank), vlo_(vlo), vhi_(vhi), sm_count_(sm_count) {}
+
+Part::~Part() {
+    if (cs_) cudaStreamSynchronize(cs_);
+    if (xs_) cudaStreamSynchronize(xs_);
+    free_regions();
+    dfree(d_off_); dfree(d_A_); dfree(d_S_); dfree(d_next_); dfree(d_visited_);
+    dfree(d_val_); dfree(d_snap_); dfree(d_rank_); dfree(d_contrib_); dfree(d_sum_); dfree(d_dang_);
+    dfree(d_hq_small_); dfree(d_hq_med_); dfree(d_hq_hub_); dfree(d_hub_pre_);
+    dfree(d_mq_); dfree(d_mq_pre_); dfree(d_mq_src_); dfree(d_tile_first_);
+    dfree(d_run_b_); dfree(d_run_e_); dfree(d_run_dst_);
+    dfree(d_tile_agg_); dfree(d_tile_incl_); dfree(d_tile_flag_); dfree(d_tot_);
+    if (h_tot_) cudaFreeHost(h_tot_);
+    for (int i = 0; i < 2; ++i) {
+        if (ready_[i]) cudaEventDestroy(ready_[i]);
+        if (consumed_[i]) cudaEventDestroy(consumed_[i]);
+    }
+    if (ev_classified_) cudaEventDestroy(ev_classified_);
+    if (cs_) cudaStreamDestroy(cs_);
+    if (xs_) cudaStreamDestroy(xs_);
+    cudaGetLastError();
+}
+
+void Part::alloc_vertex_state() {
+    int lo_pri = 0, hi_pri = 0;
+    CK(cudaDeviceGetStreamPriorityRange(&lo_pri, &hi_pri));
+    CK(cudaStreamCreateWithPriority(&cs_, cudaStreamNonBlocking, lo_pri));
+    CK(cudaStreamCreateWithPriority(&xs_, cudaStreamNonBlocking, hi_pri));
+    for (int i = 0; i < 2; ++i) {
+        CK(cudaEventCreateWithFlags(&ready_[i], cudaEventDisableTiming));
+        CK(cudaEventCreateWithFlags(&consumed_[i], cudaEventDisableTiming));
+    }
+    CK(cudaEventCreateWithFlags(&ev_classified_, cudaEventDisableTiming));
+    const uint64_t n = g_.n, m = g_.m;
+    vertex_bytes_ = 0;
+    nwords_ = (uint32_t)((n + 31) / 32);
+    ntiles_ = (nwords_ + kTileWords - 1) / kTileWords;
+    dalloc(&d_off_, n + 1, &vertex_bytes_);
+    dalloc(&d_A_, nwords_, &vertex_bytes_);
+    dalloc(&d_S_, nwords_, &vertex_bytes_);
+    dalloc(&d_next_, nwords_, &vertex_bytes_);
+    const uint64_t own = vhi_ - vlo_;
+    dalloc(&d_hq_small_, own, &vertex_bytes_);
+    dalloc(&d_hq_med_, own, &vertex_bytes_);
+    hub_cap_ = std::min<uint64_t>(own, m / o_.hub_deg + 1);       // at most m / hub_deg hubs
+    dalloc(&d_hq_hub_, hub_cap_, &vertex_bytes_);
+    dalloc(&d_hub_pre_, hub_cap_, &vertex_bytes_);
+    dalloc(&d_mq_, own, &vertex_bytes_);
+    dalloc(&d_mq_pre_, own, &vertex_bytes_);
+    dalloc(&d_mq_src_, own, &vertex_bytes_);
+    dalloc(&d_tile_first_, (m >> kEdgeTileShift) + 2, &vertex_bytes_);
+    dalloc(&d_run_b_, own / 2 + 1, &vertex_bytes_);
+    dalloc(&d_run_e_, own / 2 + 1, &vertex_bytes_);
+    dalloc(&d_run_dst_, own / 2 + 1, &vertex_bytes_);
+    dalloc(&d_tile_agg_, ntiles_, &vertex_bytes_);
+    dalloc(&d_tile_incl_, ntiles_, &vertex_bytes_);
+    dalloc(&d_tile_flag_, ntiles_, &vertex_bytes_);
+    dalloc(&d_tot_, 1, &vertex_bytes_);
+    CK(cudaMemset(d_tile_flag_, 0, (size_t)std::max<uint32_t>(ntiles_, 1) * 4));
+    CK(cudaMemset(d_S_, 0, (size_t)std::max<uint32_t>(nwords_, 1) * 4));
+    epoch_ = 0;
+    cudaError_t e = cudaHostAlloc((void**)&h_tot_, sizeof(IterTotals), cudaHostAllocMapped | cudaHostAllocPortable);
+    if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_EHOSTMEM, "cudaHostAlloc totals"); }
+}
+
+void Part::alloc_algo_state(int algo) {
+    if (algo == ALG_PR) {
+        if (!d_rank_) {
+            dalloc(&d_rank_, g_.n, &vertex_bytes_);
+            dalloc(&d_contrib_, g_.n, &vertex_bytes_);
+            dalloc(&d_sum_, g_.n, &vertex_bytes_);
+            dalloc(&d_dang_, 2, &vertex_bytes_);
+        }
+    } else {
+        if (!d_val_) dalloc(&d_val_, g_.n, &vertex_bytes_);
+        if (algo == ALG_BFS && !d_visited_) dalloc(&d_visited_, nwords_, &vertex_bytes_);
+        if (algo != ALG_BFS && !d_snap_) dalloc(&d_snap_, g_.n, &vertex_bytes_);
+    }
+    if (o_.hub_deg < 2048) {
+        const uint64_t need = std::min<uint64_t>(vhi_ - vlo_, g_.m / o_.hub_deg + 1);
+        if (need > hub_cap_) {
+            dfree(d_hq_hub_); dfree(d_hub_pre_);
+            dalloc(&d_hq_hub_, need, &vertex_bytes_);
+            dalloc(&d_hub_pre_, need, &vertex_bytes_);
+            hub_cap_ = need;
+        }
+    }
+}
+
+void Part::upload_off() {
+    CK(cudaMemcpyAsync(d_off_, g_.off.data(), (g_.n + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice, cs_));
+    static_valid_ = false;
+}
+
+void Part::free_regions() {
+    dfree(d_static_);
+    dfree(d_chunk_[0]);
+    dfree(d_chunk_[1]);
+    static_alloc_ = chunk_alloc_ = 0;
+    static_valid_ = false;
+}
+
+void Part::set_budget(uint64_t bytes, double frac) {
+    const Placement p = place(g_.off.data() + vlo_, vhi_ - vlo_, g_.b_e, bytes, frac);
+    const uint64_t own = vhi_ - vlo_;
+    if (p.s < own && p.cap < 16)
+        throw Error(ASCETIC_ENOMEM, "budget leaves an On-demand chunk below 16 bytes (cap=" + std::to_string(p.cap) + ")");
+    const uint64_t want_static = p.static_bytes, want_chunk = p.s < own ? p.cap : 0;
+    // regions are allocated at exactly the placement's sizes (never more than B); an
+    // identical placement keeps them
+    if (want_static != static_alloc_ || want_chunk != chunk_alloc_) {
+        free_regions();
+        if (want_static) {
+            cudaError_t e = cudaMalloc(&d_static_, want_static);
+            if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_ENOMEM, "static region allocation"); }
+        }
+        static_alloc_ = want_static;
+        if (want_chunk) {
+            for (int i = 0; i < 2; ++i) {
+                cudaError_t e = cudaMalloc(&d_chunk_[i], want_chunk);
+                if (e != cudaSuccess) { cudaGetLastError(); free_regions(); throw Error(ASCETIC_ENOMEM, "chunk allocation"); }
+            }
+        }
+        chunk_alloc_ = want_chunk;
+    } else if (p.s != pl_.s) {
+        static_valid_ = false;
+    }
+    pl_ = p;
+    cap_ = p.cap;
+    launch_set_range_bits(d_S_, nwords_, vlo_, vlo_ + p.s, cs_);   // StaticBitmap
+    CK(cudaStreamSynchronize(cs_));
+}
+
+DevState Part::dev_state(uint32_t iter) const {
+    DevState d;
+    d.off = d_off_; d.n = g_.n; d.nwords = nwords_;
+    d.A = d_A_; d.S = d_S_; d.next = d_next_; d.visited = d_visited_;
+    d.val = d_val_; d.snap = d_snap_;
+    d.rank = d_rank_; d.contrib = d_contrib_; d.sum = d_sum_; d.dang = d_dang_;
+    d.iter = iter;
+    d.vlo = vlo_; d.vhi = vhi_;
+    d.static_arc0 = g_.off.empty() ? 0 : g_.off[vlo_];
+    return d;
+}
+
+Queues Part::queues(const IterTotals& T) const {
+    Queues q;
+    q.hq_small = d_hq_small_; q.hq_med = d_hq_med_; q.hq_hub = d_hq_hub_; q.hub_pre = d_hub_pre_;
+    q.mq = d_mq_; q.mq_pre = d_mq_pre_; q.mq_src = d_mq_src_; q.tile_first = d_tile_first_;
+    q.n_missq = T.n_missq; q.miss_arcs = T.miss_arcs;
+    return q;
+}
+
+cudaEvent_t Part::mark(cudaStream_t s) {
+    if (!timing_) return nullptr;
+    cudaEvent_t e = pool_.get();
+    CK(cudaEventRecord(e, s));
+    return e;
+}
+
+void Part::span(cudaEvent_t a, cudaStream_t s, uint32_t t, int ph) {
+    if (!timing_) return;
+    cudaEvent_t e = pool_.get();
+    CK(cudaEventRecord(e, s));
+    spans_.push_back({a, e, t, ph});
+}
+
+// ---- transfer engine: chunk = miss-stream arcs [lo, hi). mode 1: zero-copy SM gather over
+// the miss queue; mode 2: copy-engine DMA of the run pieces intersecting the window.
+void Part::transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsigned long long hi, int mode) {
+    if (mode == 1) {
+        launch_gather(q, g_.nbr_dev, g_.b_e, d_chunk_[buf], lo, hi, o_.gather_ctas ? o_.gather_ctas : 2 * sm_count_, xs_);
+        return;
+    }
+    size_t r = std::upper_bound(rdst_.begin(), rdst_.end(), lo) - rdst_.begin();
+    r = r ? r - 1 : 0;
+    const char* host = (const char*)g_.nbr;
+    char* dst = (char*)d_chunk_[buf];
+    const uint32_t b_e = g_.b_e;
+    for (; r < rb_.size(); ++r) {
+        const unsigned long long a0 = g_.off[rb_[r]], a1 = g_.off[re_[r]];
+        const unsigned long long s0 = rdst_[r], s1 = s0 + (a1 - a0);
+        if (s0 >= hi) break;
+        const unsigned long long p0 = std::max(s0, lo), p1 = std::min(s1, hi);
+        if (p1 <= p0) continue;
+        CK(cudaMemcpyAsync(dst + (p0 - lo) * b_e, host + (a0 + (p0 - s0)) * b_e, (p1 - p0) * b_e,
+                           cudaMemcpyHostToDevice, xs_));
+    }
+}
+
+void Part::begin(int algo, uint32_t source, bool timing) {
+    algo_ = algo;
+    timing_ = timing;
+    cap_ = pl_.cap;   // chunk-cap option (tuning only: never above the placer's C/2)
+    if (o_.chunk_cap && o_.chunk_cap < cap_) cap_ = std::max<uint64_t>(16, o_.chunk_cap / 16 * 16);
+    iters.clear();
+    std::memset(&st, 0, sizeof st);
+    pool_.reset();
+    spans_.clear();
+    host_s_ = 0.0;
+    launches0_ = g_launches;
+    ev_start_ = pool_.get(); ev_fill0_ = pool_.get(); ev_fill1_ = pool_.get();
+    CK(cudaEventRecord(ev_start_, cs_));
+    // ---- static fill: ONE DMA of this rank's front prefix, counted in the run
+    CK(cudaStreamWaitEvent(xs_, ev_start_, 0));
+    CK(cudaEventRecord(ev_fill0_, xs_));
+    if (pl_.static_bytes && !(o_.keep_static && static_valid_)) {
+        CK(cudaMemcpyAsync(d_static_, (const char*)g_.nbr + g_.off[vlo_] * g_.b_e, pl_.static_bytes,
+                           cudaMemcpyHostToDevice, xs_));
+        st.h2d_static_fill_bytes = pl_.static_bytes;
+        static_valid_ = true;
+    }
+    CK(cudaEventRecord(ev_fill1_, xs_));
+    launch_init(algo, dev_state(0), source, cs_);
+    CK(cudaGetLastError());
+    CK(cudaStreamWaitEvent(cs_, ev_fill1_, 0));
+}
+
+void Part::classify(uint32_t t) {
+    // ---- GenDataMap + compaction
+    *reinterpret_cast<volatile uint32_t*>(&h_tot_->ready) = 0;
+    CK(cudaMemsetAsync(d_tot_, 0, sizeof(IterTotals), cs_));
+    ++epoch_;
+    if (epoch_ >= (1u << 30)) {
+        CK(cudaMemsetAsync(d_tile_flag_, 0, (size_t)ntiles_ * 4, cs_));
+        epoch_ = 1;
+    }
+    ClassifyArgs ca;
+    ca.A = d_A_; ca.S = d_S_; ca.off = d_off_; ca.n = g_.n; ca.vlo = vlo_; ca.vhi = vhi_;
+    ca.nwords = nwords_; ca.ntiles = ntiles_;
+    ca.hub_deg = o_.hub_deg; ca.piece_arcs = kPieceArcs;
+    ca.hq_small = d_hq_small_; ca.hq_med = d_hq_med_; ca.hq_hub = d_hq_hub_; ca.hub_pre = d_hub_pre_;
+    ca.mq = d_mq_; ca.mq_pre = d_mq_pre_; ca.mq_src = d_mq_src_; ca.tile_first = d_tile_first_;
+    ca.run_b = d_run_b_; ca.run_e = d_run_e_; ca.run_dst = d_run_dst_;
+    ca.tile_agg = d_tile_agg_; ca.tile_incl = d_tile_incl_; ca.tile_flag = d_tile_flag_; ca.epoch = epoch_;
+    ca.tot = d_tot_; ca.host_tot = h_tot_;
+    cudaEvent_t e0 = mark(cs_);
+    launch_classify(ca, cs_);
+    CK(cudaGetLastError());
+    span(e0, cs_, t, PH_CLS);
+    CK(cudaEventRecord(ev_classified_, cs_));
+}
+
+IterTotals Part::wait_classify() {
+    // low-latency wait: spin on the flag the last classify CTA writes into mapped memory
+    const volatile uint32_t* flag = &h_tot_->ready;
+    uint32_t spins = 0;
+    while (!*flag) {
+        if ((++spins & 1023u) == 0) {
+            const cudaError_t q = cudaEventQuery(ev_classified_);
+            if (q == cudaSuccess) break;
+            if (q != cudaErrorNotReady) CK(q);
+        }
+    }
+    std::atomic_thread_fence(std::memory_order_acquire);
+    IterTotals T = *const_cast<const IterTotals*>(h_tot_);
+    if (!T.ready) {
+        CK(cudaEventSynchronize(ev_classified_));
+        T = *const_cast<const IterTotals*>(h_tot_);
+    }
+    st.d2h_bytes += sizeof(IterTotals);
+    return T;
+}
+
+void Part::expand(uint32_t t, const IterTotals& T) {
+    const auto th0 = std::chrono::steady_clock::now();
+    const uint32_t b_e = g_.b_e;
+    ascetic_iter_stats_t is{};
+    is.t = t; is.rank = (uint32_t)rank_;
+    is.nA = T.nA; is.nH = T.nH; is.nM = T.nM; is.nruns = T.n_runs;
+    is.active_arcs = T.active_arcs; is.hit_arcs = T.hit_arcs; is.miss_bytes = T.miss_arcs * b_e;
+    is.digest = T.digest;
+    const DevState d = dev_state(t);
+    const Queues q = queues(T);
+    if (algo_ == ALG_PR) CK(cudaMemsetAsync(d_sum_ + vlo_, 0, (vhi_ - vlo_) * sizeof(double), cs_));
+    // ---- Static Computing, overlapping the transfer. The static
+    // buffer holds host arcs [off[vlo], off[vlo+s]); kernels index it with rank-local arc
+    // numbers (arc - d.static_arc0), so 128-bit alignment is that of the buffer itself.
+    if (T.n_small + T.n_med + T.n_hub) {
+        cudaEvent_t e0 = mark(cs_);
+        launch_static(algo_, d, q, d_static_, T.n_small, T.n_med, T.n_hub, T.n_pieces, kPieceArcs, cs_);
+        CK(cudaGetLastError());
+        span(e0, cs_, t, PH_STATIC);
+    }
+    st.static_arcs += T.hit_arcs;
+    st.ondemand_arcs += T.miss_arcs;
+    // ---- On-demand request, fragmented into chunks
+    const unsigned long long cap_arcs = cap_ / b_e;
+    const unsigned long long miss = T.miss_arcs;
+    const uint32_t nchunks = miss ? (uint32_t)((miss + cap_arcs - 1) / cap_arcs) : 0;
+    int mode = 1;
+    if (nchunks) {
+        if (o_.xfer_mode == 2) mode = 2;
+        else if (o_.xfer_mode == 1) mode = 1;
+        else mode = (T.n_runs <= kRunsHostMax && miss * b_e / std::max<uint32_t>(1, T.n_runs) >= o_.dma_min_run) ? 2 : 1;
+        if (mode == 2) {
+            rb_.resize(T.n_runs); re_.resize(T.n_runs); rdst_.resize(T.n_runs);
+            CK(cudaMemcpy(rb_.data(), d_run_b_, T.n_runs * 4ull, cudaMemcpyDeviceToHost));
+            CK(cudaMemcpy(re_.data(), d_run_e_, T.n_runs * 4ull, cudaMemcpyDeviceToHost));
+            st.d2h_bytes += T.n_runs * 8ull;
+            unsigned long long acc = 0;
+            for (uint32_t r = 0; r < T.n_runs; ++r) { rdst_[r] = acc; acc += g_.off[re_[r]] - g_.off[rb_[r]]; }
+        }
+        if (!o_.overlap) {
+            cudaEvent_t es = pool_.get();
+            CK(cudaEventRecord(es, cs_));
+            CK(cudaStreamWaitEvent(xs_, es, 0));
+        }
+    }
+    for (uint32_t k = 0; k < nchunks; ++k) {
+        const int buf = k & 1;
+        const unsigned long long lo = (unsigned long long)k * cap_arcs;
+        const unsigned long long hi = std::min(miss, lo + cap_arcs);
+        if (k >= 2) CK(cudaStreamWaitEvent(xs_, consumed_[buf], 0));
+        cudaEvent_t e0 = mark(xs_);
+        transfer_chunk(q, buf, lo, hi, mode);
+        CK(cudaGetLastError());
+        span(e0, xs_, t, mode == 2 ? PH_DMA : PH_GATHER);
+        if (mode == 2) st.dma_bytes += (hi - lo) * b_e; else st.gather_bytes += (hi - lo) * b_e;
+        CK(cudaEventRecord(ready_[buf], xs_));
+        CK(cudaStreamWaitEvent(cs_, ready_[buf], 0));
+        e0 = mark(cs_);
+        launch_ondemand(algo_, d, q, d_chunk_[buf], lo, hi, cs_);   // On-demand Computing
+        CK(cudaGetLastError());
+        span(e0, cs_, t, PH_OND);
+        CK(cudaEventRecord(consumed_[buf], cs_));
+    }
+    is.chunks = nchunks;
+    is.mode = nchunks ? (uint32_t)mode : 0u;
+    st.chunks_total += nchunks;
+    if (nchunks && mode == 2) st.dma_chunks += nchunks; else if (nchunks) st.gather_chunks += nchunks;
+    st.h2d_payload_bytes += is.miss_bytes;
+    st.active_arcs_total += is.active_arcs;
+    iters.push_back(is);
+    host_s_ += std::chrono::duration<double>(std::chrono::steady_clock::now() - th0).count();
+}
+
+void Part::finalize(uint32_t t, bool dense) {
+    // ---- next active set
+    cudaEvent_t e0 = mark(cs_);
+    launch_finalize(algo_, dev_state(t), dense, cs_);
+    CK(cudaGetLastError());
+    span(e0, cs_, t, PH_FIN);
+}
+
+void Part::end() {
+    cudaEvent_t ev_end = pool_.get();
+    CK(cudaEventRecord(ev_end, cs_));
+    CK(cudaStreamSynchronize(cs_));
+    CK(cudaStreamSynchronize(xs_));
+    float ms = 0.f, fill_ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, ev_start_, ev_end));
+    CK(cudaEventElapsedTime(&fill_ms, ev_fill0_, ev_fill1_));
+    double ph[PH_N] = {0, 0, 0, 0, 0, 0, 0};
+    for (const Span& sp : spans_) {
+        float a = 0.f;
+        CK(cudaEventElapsedTime(&a, sp.a, sp.b));
+        ph[sp.ph] += a;
+        if (sp.iter < iters.size()) {
+            auto& is = iters[sp.iter];
+            switch (sp.ph) {
+                case PH_CLS: is.ms_classify += a; break;
+                case PH_STATIC: is.ms_static += a; break;
+                case PH_OND: is.ms_ondemand += a; break;
+                case PH_GATHER: case PH_DMA: is.ms_h2d += a; break;
+                case PH_XCH: is.ms_exchange += a; break;
+                default: is.ms_finalize += a; break;
+            }
+        }
+    }
+    for (auto& is : iters)
+        is.ms_total = is.ms_classify + is.ms_static + is.ms_ondemand + is.ms_finalize + is.ms_exchange;
+    st.algo = algo_;
+    st.iterations = (uint32_t)iters.size();
+    st.n = g_.n; st.m = g_.m; st.b_e = g_.b_e;
+    st.rank = (uint32_t)rank_;
+    st.s = pl_.s;
+    st.budget_bytes = pl_.B;
+    st.static_reserved = pl_.Ms;
+    st.static_bytes = pl_.static_bytes;
+    st.ondemand_bytes = pl_.C;
+    st.chunk_cap = cap_;
+    st.static_fraction_used = pl_.R;
+    st.h2d_other_bytes = 0;
+    st.time_run_s = ms / 1e3;
+    st.time_fill_s = fill_ms / 1e3;
+    st.time_classify_s = ph[PH_CLS] / 1e3;
+    st.time_static_s = ph[PH_STATIC] / 1e3;
+    st.time_ondemand_s = ph[PH_OND] / 1e3;
+    st.time_gather_s = ph[PH_GATHER] / 1e3;
+    st.time_dma_s = ph[PH_DMA] / 1e3;
+    st.time_finalize_s = ph[PH_FIN] / 1e3;
+    st.time_host_s = host_s_;
+    st.time_h2d_busy_s = (ph[PH_GATHER] + ph[PH_DMA] + fill_ms) / 1e3;
+    st.vertex_state_bytes = vertex_bytes_;
+    st.kernel_launches = g_launches - launches0_;
+}
+
+// ================================================================== Engine
 Engine::~Engine() {
     try { unload(); } catch (...) {}
 }
@@ -100,18 +523,44 @@ void Engine::set_device(int dev) {
     device_ = dev;
 }
 
-// ------------------------------------------------------------------ load
+void Engine::comm_init(int rank, int world, const void* uid, int device) {
+    if (state_ != 0) throw Error(ASCETIC_ESTATE, "comm_init must precede load_csr");
+    if (world < 1 || rank < 0 || rank >= world) throw Error(ASCETIC_EINVAL, "bad rank/world");
+    if (world > 1 && !uid) throw Error(ASCETIC_EINVAL, "unique id is NULL");
+    set_device(device);
+    CK(cudaSetDevice(device_));
+    emulate_ = 1;
+    comm_.init_nccl(rank, world, uid);
+}
+
+void Engine::emulate_ranks(int world) {
+    if (state_ != 0) throw Error(ASCETIC_ESTATE, "emulate_ranks must precede load_csr");
+    if (world < 1 || world > 64) throw Error(ASCETIC_EINVAL, "emulated world must be in [1, 64]");
+    comm_.init_emulated(world);
+    emulate_ = world;
+}
+
 void Engine::load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_t* nbr, const uint32_t* wgt,
                       uint32_t flags) {
-    if (state_ != 0) unload();
     if (!off) throw Error(ASCETIC_EINVAL, "off is NULL");
     if (n >= 0xFFFFFFFFull) throw Error(ASCETIC_EINVAL, "n must be < 2^32 - 1");
     if (m > 0 && !nbr) throw Error(ASCETIC_EINVAL, "nbr is NULL");
     if ((flags & ASCETIC_PAIRS) && wgt) throw Error(ASCETIC_EINVAL, "wgt given together with ASCETIC_PAIRS");
     if (off[0] != 0) throw Error(ASCETIC_EINVAL, "off[0] != 0");
-    for (uint64_t v = 0; v < n; ++v)
-        if (off[v + 1] < off[v]) throw Error(ASCETIC_EINVAL, "off is not non-decreasing at v=" + std::to_string(v));
     if (off[n] != m) throw Error(ASCETIC_EINVAL, "off[n] != m");
+    {   // monotone offsets, checked in parallel
+        const unsigned nt = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
+        std::atomic<uint64_t> bad{~0ull};
+        std::vector<std::thread> th;
+        for (unsigned t = 0; t < nt; ++t)
+            th.emplace_back([&, t] {
+                const uint64_t a = n * t / nt, b = n * (t + 1) / nt;
+                for (uint64_t v = a; v < b; ++v)
+                    if (off[v + 1] < off[v]) { bad = v; return; }
+            });
+        for (auto& x : th) x.join();
+        if (bad != ~0ull) throw Error(ASCETIC_EINVAL, "off is not non-decreasing at v=" + std::to_string((uint64_t)bad));
+    }
     const bool pairs = (flags & ASCETIC_PAIRS) || wgt;
     const uint32_t b_e = pairs ? 8u : 4u;
     if (flags & ASCETIC_VALIDATE) {
@@ -122,19 +571,25 @@ void Engine::load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_
     if (device_ < 0) CK(cudaGetDevice(&device_));
     CK(cudaSetDevice(device_));
     CK(cudaDeviceGetAttribute(&sm_count_, cudaDevAttrMultiProcessorCount, device_));
-
-    n_ = n; m_ = m; b_e_ = b_e; flags_ = flags;
-    h_off_copy_.assign(off, off + n + 1);     // host planning copy (placer, DMA runs)
-    h_off_ = h_off_copy_.data();
+    // same shape: keep every device allocation and stream (a reload is then offsets H2D and
+    // host bookkeeping only); otherwise start from scratch
+    const bool reuse = state_ != 0 && n == g_.n && m == g_.m && b_e == g_.b_e &&
+                       std::equal(off, off + n + 1, g_.off.begin());
+    const bool same_shape = state_ != 0 && n == g_.n && m == g_.m && b_e == g_.b_e;
+    if (state_ != 0 && !same_shape) unload();
+    if (same_shape) g_.release();
+    have_result_ = false;
+    g_.n = n; g_.m = m; g_.b_e = b_e; g_.flags = flags;
+    if (!reuse) g_.off.assign(off, off + n + 1);
     // ---- pin the edge array (the On-demand Engine's Edgelist)
     const size_t bytes = (size_t)b_e * m;
     if (bytes > 0) {
         const bool need_copy = (flags & ASCETIC_COPY) || wgt;
         if (need_copy) {
-            cudaError_t e = cudaHostAlloc(&h_owned_, bytes, cudaHostAllocPortable | cudaHostAllocMapped);
+            cudaError_t e = cudaHostAlloc(&g_.owned, bytes, cudaHostAllocPortable | cudaHostAllocMapped);
             if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_EHOSTMEM, "cudaHostAlloc failed"); }
             if (wgt) {
-                uint32_t* dst = (uint32_t*)h_owned_;
+                uint32_t* dst = (uint32_t*)g_.owned;
                 const unsigned nt = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
                 std::vector<std::thread> th;
                 for (unsigned t = 0; t < nt; ++t)
@@ -143,15 +598,15 @@ void Engine::load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_
                     });
                 for (auto& x : th) x.join();
             } else {
-                std::memcpy(h_owned_, nbr, bytes);
+                std::memcpy(g_.owned, nbr, bytes);
             }
-            h_nbr_ = h_owned_;
+            g_.nbr = g_.owned;
         } else {
             cudaPointerAttributes attr{};
             cudaError_t e = cudaPointerGetAttributes(&attr, nbr);
             if (e != cudaSuccess) cudaGetLastError();
             if (e == cudaSuccess && attr.type == cudaMemoryTypeHost) {
-                h_nbr_ = nbr;                       // already page-locked (cudaHostAlloc / pin_memory)
+                g_.nbr = nbr;                       // already page-locked (cudaHostAlloc / pin_memory)
             } else {
                 e = cudaHostRegister((void*)nbr, bytes,
                                      cudaHostRegisterPortable | cudaHostRegisterMapped | cudaHostRegisterReadOnly);
@@ -160,112 +615,42 @@ void Engine::load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_
                     e = cudaHostRegister((void*)nbr, bytes, cudaHostRegisterPortable | cudaHostRegisterMapped);
                 }
                 if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_EHOSTMEM, std::string("cudaHostRegister: ") + cudaGetErrorString(e)); }
-                h_registered_ = (void*)nbr;
-                h_nbr_ = nbr;
+                g_.registered = (void*)nbr;
+                g_.nbr = nbr;
             }
         }
         void* dp = nullptr;
-        CK(cudaHostGetDevicePointer(&dp, (void*)h_nbr_, 0));
-        h_nbr_dev_ = dp;
+        CK(cudaHostGetDevicePointer(&dp, (void*)g_.nbr, 0));
+        g_.nbr_dev = dp;
     }
-    // ---- streams
-    int lo_pri = 0, hi_pri = 0;
-    CK(cudaDeviceGetStreamPriorityRange(&lo_pri, &hi_pri));
-    CK(cudaStreamCreateWithPriority(&cs_, cudaStreamNonBlocking, lo_pri));
-    CK(cudaStreamCreateWithPriority(&xs_, cudaStreamNonBlocking, hi_pri));
-    for (int i = 0; i < 2; ++i) {
-        CK(cudaEventCreateWithFlags(&ready_[i], cudaEventDisableTiming));
-        CK(cudaEventCreateWithFlags(&consumed_[i], cudaEventDisableTiming));
+    // ---- rank parts: this process's ranks and their owned vertex ranges
+    const int world = comm_.world();
+    bounds_ = partition(g_.off.data(), n, (uint32_t)world);
+    if (!same_shape) {
+        parts_.clear();
+        if (comm_.emulated()) {
+            for (int r = 0; r < world; ++r)
+                parts_.emplace_back(new Part(g_, o_, r, bounds_[r], bounds_[r + 1], sm_count_));
+        } else {
+            const int r = comm_.rank();
+            parts_.emplace_back(new Part(g_, o_, r, bounds_[r], bounds_[r + 1], sm_count_));
+        }
+        for (auto& p : parts_) p->alloc_vertex_state();
     }
-    CK(cudaEventCreateWithFlags(&ev_classified_, cudaEventDisableTiming | cudaEventBlockingSync));
-    alloc_vertex_state();
-    CK(cudaMemcpyAsync(d_off_, off, (n + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice, cs_));
-    CK(cudaStreamSynchronize(cs_));
+    for (auto& p : parts_) {
+        if (!reuse) p->upload_off();
+        p->on_reload();
+    }
+    for (auto& p : parts_) CK(cudaStreamSynchronize(p->cs()));
     state_ = 1;
 }
 
-void Engine::alloc_vertex_state() {
-    vertex_bytes_ = 0;
-    nwords_ = (uint32_t)((n_ + 31) / 32);
-    ntiles_ = (nwords_ + kTileWords - 1) / kTileWords;
-    dalloc(&d_off_, n_ + 1, &vertex_bytes_);
-    dalloc(&d_A_, nwords_, &vertex_bytes_);
-    dalloc(&d_S_, nwords_, &vertex_bytes_);
-    dalloc(&d_next_, nwords_, &vertex_bytes_);
-    dalloc(&d_hq_small_, n_, &vertex_bytes_);
-    dalloc(&d_hq_med_, n_, &vertex_bytes_);
-    const uint64_t nhub = std::min<uint64_t>(n_, m_ / opt_hub_deg_ + 1);   // at most m / hub_deg hubs
-    dalloc(&d_hq_hub_, nhub, &vertex_bytes_);
-    dalloc(&d_hub_pre_, nhub, &vertex_bytes_);
-    dalloc(&d_mq_, n_, &vertex_bytes_);
-    dalloc(&d_mq_pre_, n_, &vertex_bytes_);
-    dalloc(&d_mq_src_, n_, &vertex_bytes_);
-    dalloc(&d_tile_first_, (m_ >> kEdgeTileShift) + 2, &vertex_bytes_);
-    dalloc(&d_run_b_, n_ / 2 + 1, &vertex_bytes_);
-    dalloc(&d_run_e_, n_ / 2 + 1, &vertex_bytes_);
-    dalloc(&d_run_dst_, n_ / 2 + 1, &vertex_bytes_);
-    dalloc(&d_tile_agg_, ntiles_, &vertex_bytes_);
-    dalloc(&d_tile_incl_, ntiles_, &vertex_bytes_);
-    dalloc(&d_tile_flag_, ntiles_, &vertex_bytes_);
-    dalloc(&d_tot_, 1, &vertex_bytes_);
-    CK(cudaMemset(d_tile_flag_, 0, (size_t)std::max<uint32_t>(ntiles_, 1) * 4));
-    CK(cudaMemset(d_S_, 0, (size_t)std::max<uint32_t>(nwords_, 1) * 4));
-    epoch_ = 0;
-    if (!h_tot_) {
-        cudaError_t e = cudaHostAlloc((void**)&h_tot_, sizeof(IterTotals), cudaHostAllocMapped | cudaHostAllocPortable);
-        if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_EHOSTMEM, "cudaHostAlloc totals"); }
-    }
-}
-
-void Engine::alloc_algo_state(int algo) {
-    if (algo == ALG_PR) {
-        if (!d_rank_) {
-            dalloc(&d_rank_, n_, &vertex_bytes_);
-            dalloc(&d_contrib_, n_, &vertex_bytes_);
-            dalloc(&d_sum_, n_, &vertex_bytes_);
-            dalloc(&d_dang_, 2, &vertex_bytes_);
-        }
-    } else {
-        if (!d_val_) {
-            dalloc(&d_val_, n_, &vertex_bytes_);
-        }
-        if (algo == ALG_BFS && !d_visited_) dalloc(&d_visited_, nwords_, &vertex_bytes_);
-        if (algo != ALG_BFS && !d_snap_) dalloc(&d_snap_, n_, &vertex_bytes_);
-    }
-}
-
-void Engine::free_budget_regions() {
-    dfree(d_static_);
-    dfree(d_chunk_[0]);
-    dfree(d_chunk_[1]);
-    static_valid_ = false;
-}
-
-// ------------------------------------------------------------------ budget
 void Engine::set_budget(uint64_t bytes, double frac) {
     if (state_ == 0) throw Error(ASCETIC_ESTATE, "set_budget before load_csr");
     if (std::isnan(frac) || frac > 1.0) throw Error(ASCETIC_EINVAL, "static_fraction must be <= 1 (or < 0 for Eq. 2)");
     CK(cudaSetDevice(device_));
-    Placement p = place(h_off_, n_, b_e_, bytes, frac);
-    if (p.s < n_ && p.cap < 16)
-        throw Error(ASCETIC_ENOMEM, "budget leaves an On-demand chunk below 16 bytes (cap=" + std::to_string(p.cap) + ")");
-    free_budget_regions();
     state_ = 1;
-    pl_ = p;
-    cap_ = p.cap;
-    if (opt_chunk_cap_ && opt_chunk_cap_ < cap_) cap_ = std::max<uint64_t>(16, opt_chunk_cap_ / 16 * 16);
-    if (p.static_bytes) {
-        cudaError_t e = cudaMalloc(&d_static_, p.static_bytes);
-        if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_ENOMEM, "static region allocation"); }
-    }
-    if (p.s < n_) {
-        for (int i = 0; i < 2; ++i) {
-            cudaError_t e = cudaMalloc(&d_chunk_[i], cap_);
-            if (e != cudaSuccess) { cudaGetLastError(); free_budget_regions(); throw Error(ASCETIC_ENOMEM, "chunk allocation"); }
-        }
-    }
-    launch_set_prefix_bits(d_S_, nwords_, p.s, cs_);   // StaticBitmap
-    CK(cudaStreamSynchronize(cs_));
+    for (auto& p : parts_) p->set_budget(bytes, frac);   // every rank: its own budget B (§8(e))
     state_ = 2;
 }
 
@@ -273,306 +658,148 @@ void Engine::set_option(int opt, int64_t value) {
     switch (opt) {
         case ASCETIC_OPT_CHUNK_CAP:
             if (value < 0) throw Error(ASCETIC_EINVAL, "chunk cap < 0");
-            opt_chunk_cap_ = (uint64_t)value;
-            if (state_ == 2) {
-                cap_ = pl_.cap;
-                if (opt_chunk_cap_ && opt_chunk_cap_ < cap_) cap_ = std::max<uint64_t>(16, opt_chunk_cap_ / 16 * 16);
-            }
+            o_.chunk_cap = (uint64_t)value;
             break;
         case ASCETIC_OPT_XFER_MODE:
             if (value < 0 || value > 2) throw Error(ASCETIC_EINVAL, "xfer mode must be 0, 1 or 2");
-            opt_xfer_mode_ = (int)value;
+            o_.xfer_mode = (int)value;
             break;
-        case ASCETIC_OPT_DMA_MIN_RUN: opt_dma_min_run_ = (uint64_t)std::max<int64_t>(0, value); break;
-        case ASCETIC_OPT_OVERLAP: opt_overlap_ = value ? 1 : 0; break;
-        case ASCETIC_OPT_KEEP_STATIC: opt_keep_static_ = value ? 1 : 0; static_valid_ = false; break;
+        case ASCETIC_OPT_DMA_MIN_RUN: o_.dma_min_run = (uint64_t)std::max<int64_t>(0, value); break;
+        case ASCETIC_OPT_OVERLAP: o_.overlap = value ? 1 : 0; break;
+        case ASCETIC_OPT_KEEP_STATIC:
+            o_.keep_static = value ? 1 : 0;
+            for (auto& p : parts_) p->on_reload();
+            break;
         case ASCETIC_OPT_HUB_DEGREE:
             if (value < 32 || value > (1ll << 30)) throw Error(ASCETIC_EINVAL, "hub degree must be in [32, 2^30]");
-            if ((uint32_t)value < opt_hub_deg_ && state_ != 0) {
-                // hub arrays hold at most m / hub_deg entries; grow them
-                const uint64_t nhub = std::min<uint64_t>(n_, m_ / (uint64_t)value + 1);
-                dfree(d_hq_hub_); dfree(d_hub_pre_);
-                dalloc(&d_hq_hub_, nhub, &vertex_bytes_);
-                dalloc(&d_hub_pre_, nhub, &vertex_bytes_);
-            }
-            opt_hub_deg_ = (uint32_t)value;
+            o_.hub_deg = (uint32_t)value;
             break;
-        case ASCETIC_OPT_TIMING: opt_timing_ = value ? 1 : 0; break;
+        case ASCETIC_OPT_TIMING: o_.timing = value ? 1 : 0; break;
         case ASCETIC_OPT_GATHER_CTAS:
             if (value < 0 || value > 65535) throw Error(ASCETIC_EINVAL, "gather CTAs must be in [0, 65535]");
-            opt_gather_ctas_ = (int)value;
+            o_.gather_ctas = (int)value;
             break;
         default: throw Error(ASCETIC_EINVAL, "unknown option");
     }
 }
 
-DevState Engine::dev_state(uint32_t iter) const {
-    DevState d;
-    d.off = d_off_; d.n = n_; d.nwords = nwords_;
-    d.A = d_A_; d.S = d_S_; d.next = d_next_; d.visited = d_visited_;
-    d.val = d_val_; d.snap = d_snap_;
-    d.rank = d_rank_; d.contrib = d_contrib_; d.sum = d_sum_; d.dang = d_dang_;
-    d.iter = iter;
-    return d;
-}
-
-Queues Engine::queues(const IterTotals& T) const {
-    Queues q;
-    q.hq_small = d_hq_small_; q.hq_med = d_hq_med_; q.hq_hub = d_hq_hub_; q.hub_pre = d_hub_pre_;
-    q.mq = d_mq_; q.mq_pre = d_mq_pre_; q.mq_src = d_mq_src_; q.tile_first = d_tile_first_;
-    q.n_missq = T.n_missq; q.miss_arcs = T.miss_arcs;
-    return q;
-}
-
-// ------------------------------------------------------------------ transfer engine
-// chunk = miss-stream arcs [lo, hi). mode 1: zero-copy SM gather over the miss queue;
-// mode 2: copy-engine DMA of the run pieces intersecting the window.
-void Engine::transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsigned long long hi, int mode,
-                            const std::vector<uint32_t>& rb, const std::vector<uint32_t>& re,
-                            const std::vector<unsigned long long>& rdst) {
-    if (mode == 1) {
-        launch_gather(q, h_nbr_dev_, b_e_, d_chunk_[buf], lo, hi, opt_gather_ctas_ ? opt_gather_ctas_ : 2 * sm_count_, xs_);
-        return;
-    }
-    // first run whose stream range ends after lo
-    size_t r = std::upper_bound(rdst.begin(), rdst.end(), lo) - rdst.begin();
-    r = r ? r - 1 : 0;
-    const char* host = (const char*)h_nbr_;
-    char* dst = (char*)d_chunk_[buf];
-    for (; r < rb.size(); ++r) {
-        const unsigned long long a0 = h_off_[rb[r]], a1 = h_off_[re[r]];
-        const unsigned long long s0 = rdst[r], s1 = s0 + (a1 - a0);
-        if (s0 >= hi) break;
-        const unsigned long long p0 = std::max(s0, lo), p1 = std::min(s1, hi);
-        if (p1 <= p0) continue;
-        CK(cudaMemcpyAsync(dst + (p0 - lo) * b_e_, host + (a0 + (p0 - s0)) * b_e_, (p1 - p0) * b_e_,
-                           cudaMemcpyHostToDevice, xs_));
+void Engine::join(std::vector<cudaStream_t>* /*unused*/) {
+    cudaStream_t c0 = parts_[0]->cs();
+    for (size_t i = 1; i < parts_.size(); ++i) {
+        cudaEvent_t e;
+        CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        CK(cudaEventRecord(e, parts_[i]->cs()));
+        CK(cudaStreamWaitEvent(c0, e, 0));
+        CK(cudaEventDestroy(e));
     }
 }
 
-// ------------------------------------------------------------------ run
+void Engine::fork() {
+    cudaStream_t c0 = parts_[0]->cs();
+    if (parts_.size() < 2) return;
+    cudaEvent_t e;
+    CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    CK(cudaEventRecord(e, c0));
+    for (size_t i = 1; i < parts_.size(); ++i) CK(cudaStreamWaitEvent(parts_[i]->cs(), e, 0));
+    CK(cudaEventDestroy(e));
+}
+
 void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
     if (state_ != 2) throw Error(ASCETIC_ESTATE, state_ == 0 ? "run before load_csr" : "run before set_budget");
     if (algo < 0 || algo > 3) throw Error(ASCETIC_EINVAL, "unknown algorithm");
-    if (algo == ALG_SSSP && b_e_ != 8) throw Error(ASCETIC_EINVAL, "SSSP needs weights (ASCETIC_PAIRS or wgt)");
-    if (algo != ALG_SSSP && b_e_ != 4) throw Error(ASCETIC_EINVAL, "BFS/CC/PR take an unweighted CSR (b_e = 4)");
-    if ((algo == ALG_BFS || algo == ALG_SSSP) && source >= n_) throw Error(ASCETIC_EINVAL, "source >= n");
+    if (algo == ALG_SSSP && g_.b_e != 8) throw Error(ASCETIC_EINVAL, "SSSP needs weights (ASCETIC_PAIRS or wgt)");
+    if (algo != ALG_SSSP && g_.b_e != 4) throw Error(ASCETIC_EINVAL, "BFS/CC/PR take an unweighted CSR (b_e = 4)");
+    if ((algo == ALG_BFS || algo == ALG_SSSP) && source >= g_.n) throw Error(ASCETIC_EINVAL, "source >= n");
     if (algo == ALG_PR && max_iters == 0) throw Error(ASCETIC_EINVAL, "PR needs max_iters >= 1");
-    if ((algo == ALG_CC || algo == ALG_PR) && !(flags_ & ASCETIC_SYMMETRIC))
+    if ((algo == ALG_CC || algo == ALG_PR) && !(g_.flags & ASCETIC_SYMMETRIC))
         throw Error(ASCETIC_EINVAL, "CC and PR need ASCETIC_SYMMETRIC");
-    if (n_ == 0) throw Error(ASCETIC_EINVAL, "empty graph");
+    if (g_.n == 0) throw Error(ASCETIC_EINVAL, "empty graph");
     CK(cudaSetDevice(device_));
-    alloc_algo_state(algo);
     have_result_ = false;
-    iters_.clear();
-    std::memset(&st_, 0, sizeof st_);
-    pool_.reset();
-    const bool timing = opt_timing_ != 0;
-    const unsigned long long launches0 = g_launches;
-
-    // event pairs per kernel class, resolved after the run
-    enum { PH_CLS, PH_STATIC, PH_OND, PH_GATHER, PH_DMA, PH_FIN, PH_N };
-    struct Span { cudaEvent_t a, b; uint32_t iter; int ph; };
-    std::vector<Span> spans;
-    auto open_span = [&](cudaStream_t s) -> cudaEvent_t {
-        if (!timing) return nullptr;
-        cudaEvent_t e = pool_.get();
-        CK(cudaEventRecord(e, s));
-        return e;
-    };
-    auto close_span = [&](cudaEvent_t a, cudaStream_t s, uint32_t it, int ph) {
-        if (!timing) return;
-        cudaEvent_t e = pool_.get();
-        CK(cudaEventRecord(e, s));
-        spans.push_back({a, e, it, ph});
-    };
-
-    cudaEvent_t ev_start = pool_.get(), ev_end = pool_.get(), ev_fill0 = pool_.get(), ev_fill1 = pool_.get();
-    CK(cudaEventRecord(ev_start, cs_));
-    // ---- static fill: ONE DMA of the front prefix, counted in the run
-    uint64_t fill_bytes = 0;
-    CK(cudaStreamWaitEvent(xs_, ev_start, 0));
-    CK(cudaEventRecord(ev_fill0, xs_));
-    if (pl_.static_bytes && !(opt_keep_static_ && static_valid_)) {
-        CK(cudaMemcpyAsync(d_static_, h_nbr_, pl_.static_bytes, cudaMemcpyHostToDevice, xs_));
-        fill_bytes = pl_.static_bytes;
-        static_valid_ = true;
-    }
-    CK(cudaEventRecord(ev_fill1, xs_));
-    launch_init(algo, dev_state(0), source, cs_);
-    CK(cudaGetLastError());
-    CK(cudaStreamWaitEvent(cs_, ev_fill1, 0));
-
-    const unsigned long long cap_arcs = cap_ / b_e_;
-    std::vector<uint32_t> rb, re;
-    std::vector<unsigned long long> rdst;
-    double host_s = 0.0;
+    const bool multi = comm_.active();
+    const bool timing = o_.timing != 0;
+    for (auto& p : parts_) p->alloc_algo_state(algo);
+    for (auto& p : parts_) p->begin(algo, source, timing);
+    Part& p0 = *parts_[0];
+    std::vector<IterTotals> T(parts_.size());
     uint32_t t = 0;
     for (t = 0;; ++t) {
         if (max_iters && t == max_iters) break;
-        // ---- GenDataMap + compaction
-        *reinterpret_cast<volatile uint32_t*>(&h_tot_->ready) = 0;
-        CK(cudaMemsetAsync(d_tot_, 0, sizeof(IterTotals), cs_));
-        ++epoch_;
-        if (epoch_ >= (1u << 30)) {
-            CK(cudaMemsetAsync(d_tile_flag_, 0, (size_t)ntiles_ * 4, cs_));
-            epoch_ = 1;
-        }
-        ClassifyArgs ca;
-        ca.A = d_A_; ca.S = d_S_; ca.off = d_off_; ca.n = n_; ca.nwords = nwords_; ca.ntiles = ntiles_;
-        ca.hub_deg = opt_hub_deg_; ca.piece_arcs = kPieceArcs;
-        ca.hq_small = d_hq_small_; ca.hq_med = d_hq_med_; ca.hq_hub = d_hq_hub_; ca.hub_pre = d_hub_pre_;
-        ca.mq = d_mq_; ca.mq_pre = d_mq_pre_; ca.mq_src = d_mq_src_; ca.tile_first = d_tile_first_; ca.run_b = d_run_b_; ca.run_e = d_run_e_; ca.run_dst = d_run_dst_;
-        ca.tile_agg = d_tile_agg_; ca.tile_incl = d_tile_incl_; ca.tile_flag = d_tile_flag_; ca.epoch = epoch_;
-        ca.tot = d_tot_; ca.host_tot = h_tot_;
-        cudaEvent_t e0 = open_span(cs_);
-        launch_classify(ca, cs_);
-        CK(cudaGetLastError());
-        close_span(e0, cs_, t, PH_CLS);
-        CK(cudaEventRecord(ev_classified_, cs_));
-        // low-latency wait: spin on the flag the last classify CTA writes into mapped memory
-        {
-            const volatile uint32_t* flag = &h_tot_->ready;
-            uint32_t spins = 0;
-            while (!*flag) {
-                if ((++spins & 1023u) == 0) {
-                    const cudaError_t q = cudaEventQuery(ev_classified_);
-                    if (q == cudaSuccess) break;
-                    if (q != cudaErrorNotReady) CK(q);
-                }
+        for (auto& p : parts_) p->classify(t);
+        for (size_t i = 0; i < parts_.size(); ++i) T[i] = parts_[i]->wait_classify();
+        if (T[0].nA == 0) break;   // |A_t| is counted over the replicated bitmap: identical on every rank
+        for (size_t i = 0; i < parts_.size(); ++i) parts_[i]->expand(t, T[i]);
+        if (multi && algo != ALG_PR) {
+            // ---- exchange: OR of next bitmaps (BFS), MIN of values (SSSP, CC)
+            join(nullptr);
+            cudaEvent_t e0 = p0.mark(p0.cs());
+            const uint64_t nw = (g_.n + 31) / 32;
+            if (algo == ALG_BFS) {
+                std::vector<uint32_t*> b;
+                for (auto& p : parts_) b.push_back(p->next());
+                comm_.or_words(b, nw, p0.cs());
+            } else {
+                std::vector<uint32_t*> b;
+                for (auto& p : parts_) b.push_back(p->val());
+                comm_.min_u32(b, g_.n, p0.cs());
             }
-            std::atomic_thread_fence(std::memory_order_acquire);
+            p0.span(e0, p0.cs(), t, PH_XCH);
+            fork();
         }
-        const auto th0 = std::chrono::steady_clock::now();
-        const IterTotals T = *const_cast<const IterTotals*>(h_tot_);
-        if (!T.ready) CK(cudaEventSynchronize(ev_classified_));
-        st_.d2h_bytes += sizeof(IterTotals);
-        if (T.nA == 0) break;
-
-        ascetic_iter_stats_t is{};
-        is.t = t; is.rank = 0;
-        is.nA = T.nA; is.nH = T.nH; is.nM = T.nM; is.nruns = T.n_runs;
-        is.active_arcs = T.active_arcs; is.hit_arcs = T.hit_arcs; is.miss_bytes = T.miss_arcs * b_e_;
-        is.digest = T.digest;
-        const DevState d = dev_state(t);
-        const Queues q = queues(T);
-        if (algo == ALG_PR) CK(cudaMemsetAsync(d_sum_, 0, n_ * sizeof(double), cs_));
-        // ---- Static Computing, overlapping the transfer
-        if (T.n_small + T.n_med + T.n_hub) {
-            e0 = open_span(cs_);
-            launch_static(algo, d, q, d_static_, T.n_small, T.n_med, T.n_hub, T.n_pieces, kPieceArcs, cs_);
-            CK(cudaGetLastError());
-            close_span(e0, cs_, t, PH_STATIC);
-        }
-        st_.static_arcs += T.hit_arcs;
-        st_.ondemand_arcs += T.miss_arcs;
-        // ---- On-demand request, fragmented into chunks
-        const unsigned long long miss = T.miss_arcs;
-        const uint32_t nchunks = miss ? (uint32_t)((miss + cap_arcs - 1) / cap_arcs) : 0;
-        int mode = 1;
-        if (nchunks) {
-            if (opt_xfer_mode_ == 2) mode = 2;
-            else if (opt_xfer_mode_ == 1) mode = 1;
-            else mode = (T.n_runs <= kRunsHostMax && miss * b_e_ / std::max<uint32_t>(1, T.n_runs) >= opt_dma_min_run_) ? 2 : 1;
-            if (mode == 2) {
-                rb.resize(T.n_runs); re.resize(T.n_runs); rdst.resize(T.n_runs);
-                CK(cudaMemcpy(rb.data(), d_run_b_, T.n_runs * 4ull, cudaMemcpyDeviceToHost));
-                CK(cudaMemcpy(re.data(), d_run_e_, T.n_runs * 4ull, cudaMemcpyDeviceToHost));
-                st_.d2h_bytes += T.n_runs * 8ull;
-                unsigned long long acc = 0;
-                for (uint32_t r = 0; r < T.n_runs; ++r) { rdst[r] = acc; acc += h_off_[re[r]] - h_off_[rb[r]]; }
-            }
-            if (!opt_overlap_) {
-                cudaEvent_t es = pool_.get();
-                CK(cudaEventRecord(es, cs_));
-                CK(cudaStreamWaitEvent(xs_, es, 0));
-            }
-        }
-        for (uint32_t k = 0; k < nchunks; ++k) {
-            const int buf = k & 1;
-            const unsigned long long lo = (unsigned long long)k * cap_arcs;
-            const unsigned long long hi = std::min(miss, lo + cap_arcs);
-            if (k >= 2) CK(cudaStreamWaitEvent(xs_, consumed_[buf], 0));
-            e0 = open_span(xs_);
-            transfer_chunk(q, buf, lo, hi, mode, rb, re, rdst);
-            CK(cudaGetLastError());
-            close_span(e0, xs_, t, mode == 2 ? PH_DMA : PH_GATHER);
-            if (mode == 2) st_.dma_bytes += (hi - lo) * b_e_; else st_.gather_bytes += (hi - lo) * b_e_;
-            CK(cudaEventRecord(ready_[buf], xs_));
-            CK(cudaStreamWaitEvent(cs_, ready_[buf], 0));
-            e0 = open_span(cs_);
-            launch_ondemand(algo, d, q, d_chunk_[buf], lo, hi, cs_);   // On-demand Computing
-            CK(cudaGetLastError());
-            close_span(e0, cs_, t, PH_OND);
-            CK(cudaEventRecord(consumed_[buf], cs_));
-        }
-        // ---- next active set
-        e0 = open_span(cs_);
-        launch_finalize(algo, d, cs_);
-        CK(cudaGetLastError());
-        close_span(e0, cs_, t, PH_FIN);
-        is.chunks = nchunks;
-        is.mode = nchunks ? (uint32_t)mode : 0u;
-        st_.chunks_total += nchunks;
-        if (nchunks && mode == 2) st_.dma_chunks += nchunks; else if (nchunks) st_.gather_chunks += nchunks;
-        st_.h2d_payload_bytes += is.miss_bytes;
-        st_.active_arcs_total += is.active_arcs;
-        iters_.push_back(is);
-        host_s += std::chrono::duration<double>(std::chrono::steady_clock::now() - th0).count();
-    }
-    CK(cudaEventRecord(ev_end, cs_));
-    CK(cudaStreamSynchronize(cs_));
-    CK(cudaStreamSynchronize(xs_));
-    float ms = 0.f;
-    CK(cudaEventElapsedTime(&ms, ev_start, ev_end));
-    float fill_ms = 0.f;
-    CK(cudaEventElapsedTime(&fill_ms, ev_fill0, ev_fill1));
-    double ph[PH_N] = {0, 0, 0, 0, 0, 0};
-    for (const Span& sp : spans) {
-        float a = 0.f;
-        CK(cudaEventElapsedTime(&a, sp.a, sp.b));
-        ph[sp.ph] += a;
-        if (sp.iter < iters_.size()) {
-            auto& is = iters_[sp.iter];
-            switch (sp.ph) {
-                case PH_CLS: is.ms_classify += a; break;
-                case PH_STATIC: is.ms_static += a; break;
-                case PH_OND: is.ms_ondemand += a; break;
-                case PH_GATHER: case PH_DMA: is.ms_h2d += a; break;
-                default: is.ms_finalize += a; break;
-            }
+        for (auto& p : parts_) p->finalize(t, multi);
+        if (multi && algo == ALG_PR) {
+            // ---- exchange: SUM of the fp64 dangling partials, every rank's contrib slice to all
+            join(nullptr);
+            cudaEvent_t e0 = p0.mark(p0.cs());
+            std::vector<double*> dg;
+            std::vector<void*> cb;
+            const int nxt = (int)((t + 1) & 1u);
+            for (auto& p : parts_) { dg.push_back(p->dang() + nxt); cb.push_back(p->contrib()); }
+            comm_.sum_f64(dg, p0.cs());
+            comm_.share_slices(cb, bounds_, 4, p0.cs());
+            p0.span(e0, p0.cs(), t, PH_XCH);
+            fork();
         }
     }
-    for (auto& is : iters_)
-        is.ms_total = is.ms_classify + is.ms_static + is.ms_ondemand + is.ms_finalize;
-    st_.algo = algo;
+    if (multi && algo == ALG_PR) {
+        join(nullptr);
+        std::vector<void*> rk;
+        for (auto& p : parts_) rk.push_back(p->rank_arr());
+        comm_.share_slices(rk, bounds_, 4, p0.cs());
+        fork();
+    }
+    if (parts_.size() > 1) join(nullptr);
+    for (auto& p : parts_) p->end();
+    // ---- aggregate the local parts (one with NCCL; all emulated ranks otherwise)
+    st_ = p0.st;
+    iters_.clear();
+    const size_t niter = p0.iters.size();
+    for (size_t i = 0; i < niter; ++i)
+        for (auto& p : parts_)
+            if (i < p->iters.size()) iters_.push_back(p->iters[i]);
+    for (size_t i = 1; i < parts_.size(); ++i) {
+        const auto& s = parts_[i]->st;
+        st_.h2d_payload_bytes += s.h2d_payload_bytes;
+        st_.h2d_static_fill_bytes += s.h2d_static_fill_bytes;
+        st_.d2h_bytes += s.d2h_bytes;
+        st_.active_arcs_total += s.active_arcs_total;
+        st_.chunks_total += s.chunks_total;
+        st_.dma_chunks += s.dma_chunks;
+        st_.gather_chunks += s.gather_chunks;
+        st_.static_arcs += s.static_arcs;
+        st_.ondemand_arcs += s.ondemand_arcs;
+        st_.gather_bytes += s.gather_bytes;
+        st_.dma_bytes += s.dma_bytes;
+        st_.static_bytes += s.static_bytes;
+        st_.vertex_state_bytes += s.vertex_state_bytes;
+        st_.kernel_launches = std::max(st_.kernel_launches, s.kernel_launches);
+    }
     st_.iterations = t;
-    st_.n = n_; st_.m = m_; st_.b_e = b_e_;
-    st_.rank = 0; st_.world = 1;
-    st_.s = pl_.s;
-    st_.budget_bytes = pl_.B;
-    st_.static_reserved = pl_.Ms;
-    st_.static_bytes = pl_.static_bytes;
-    st_.ondemand_bytes = pl_.C;
-    st_.chunk_cap = cap_;
-    st_.static_fraction_used = pl_.R;
-    st_.h2d_static_fill_bytes = fill_bytes;
-    st_.h2d_other_bytes = 0;
-    st_.time_run_s = ms / 1e3;
-    st_.time_fill_s = fill_ms / 1e3;
-    st_.time_classify_s = ph[PH_CLS] / 1e3;
-    st_.time_static_s = ph[PH_STATIC] / 1e3;
-    st_.time_ondemand_s = ph[PH_OND] / 1e3;
-    st_.time_gather_s = ph[PH_GATHER] / 1e3;
-    st_.time_dma_s = ph[PH_DMA] / 1e3;
-    st_.time_finalize_s = ph[PH_FIN] / 1e3;
-    st_.time_host_s = host_s;
-    st_.time_h2d_busy_s = (ph[PH_GATHER] + ph[PH_DMA] + fill_ms) / 1e3;
+    st_.world = (uint32_t)comm_.world();
+    st_.rank = (uint32_t)comm_.rank();
     st_.gteps = st_.time_run_s > 0 ? (double)st_.active_arcs_total / st_.time_run_s / 1e9 : 0.0;
     const double ex = st_.time_run_s - st_.time_fill_s;
     st_.gteps_excl_fill = ex > 0 ? (double)st_.active_arcs_total / ex / 1e9 : 0.0;
-    st_.vertex_state_bytes = vertex_bytes_;
-    st_.kernel_launches = g_launches - launches0;
     last_algo_ = algo;
     have_result_ = true;
 }
@@ -589,39 +816,20 @@ int Engine::stats(ascetic_stats_t* out, ascetic_iter_stats_t* per_iter, uint32_t
 
 void Engine::get_result(void* dst, uint64_t bytes) {
     if (!have_result_) throw Error(ASCETIC_ESTATE, "no completed run");
-    if (!dst || bytes < 4 * n_) throw Error(ASCETIC_EINVAL, "result buffer must hold 4n bytes");
+    if (!dst || bytes < 4 * g_.n) throw Error(ASCETIC_EINVAL, "result buffer must hold 4n bytes");
     CK(cudaSetDevice(device_));
-    const void* src = (last_algo_ == ALG_PR) ? (const void*)d_rank_ : (const void*)d_val_;
-    CK(cudaMemcpy(dst, src, 4 * n_, cudaMemcpyDeviceToHost));
+    Part& p0 = *parts_[0];
+    const void* src = (last_algo_ == ALG_PR) ? (const void*)p0.rank_arr() : (const void*)p0.val();
+    CK(cudaMemcpy(dst, src, 4 * g_.n, cudaMemcpyDeviceToHost));
 }
 
 void Engine::unload() {
-    if (state_ == 0 && !h_tot_) return;
     if (device_ >= 0) cudaSetDevice(device_);
-    if (cs_) cudaStreamSynchronize(cs_);
-    if (xs_) cudaStreamSynchronize(xs_);
-    free_budget_regions();
-    dfree(d_off_); dfree(d_A_); dfree(d_S_); dfree(d_next_); dfree(d_visited_);
-    dfree(d_val_); dfree(d_snap_); dfree(d_rank_); dfree(d_contrib_); dfree(d_sum_); dfree(d_dang_);
-    dfree(d_hq_small_); dfree(d_hq_med_); dfree(d_hq_hub_); dfree(d_hub_pre_);
-    dfree(d_mq_); dfree(d_mq_pre_); dfree(d_mq_src_); dfree(d_tile_first_); dfree(d_run_b_); dfree(d_run_e_); dfree(d_run_dst_);
-    dfree(d_tile_agg_); dfree(d_tile_incl_); dfree(d_tile_flag_); dfree(d_tot_);
-    if (h_tot_) { cudaFreeHost(h_tot_); h_tot_ = nullptr; }
-    if (h_registered_) { cudaHostUnregister(h_registered_); h_registered_ = nullptr; }
-    if (h_owned_) { cudaFreeHost(h_owned_); h_owned_ = nullptr; }
-    for (int i = 0; i < 2; ++i) {
-        if (ready_[i]) cudaEventDestroy(ready_[i]);
-        if (consumed_[i]) cudaEventDestroy(consumed_[i]);
-        ready_[i] = consumed_[i] = nullptr;
-    }
-    if (ev_classified_) { cudaEventDestroy(ev_classified_); ev_classified_ = nullptr; }
-    if (cs_) { cudaStreamDestroy(cs_); cs_ = nullptr; }
-    if (xs_) { cudaStreamDestroy(xs_); xs_ = nullptr; }
-    h_nbr_ = h_nbr_dev_ = nullptr;
-    h_off_ = nullptr;
-    h_off_copy_.clear();
-    h_off_copy_.shrink_to_fit();
-    n_ = m_ = 0;
+    parts_.clear();
+    g_.release();
+    g_.off.clear();
+    g_.off.shrink_to_fit();
+    g_.n = g_.m = 0;
     state_ = 0;
     have_result_ = false;
     last_algo_ = -1;

@@ -1,6 +1,14 @@
 // engine.h — the host-side run controller behind the C ABI (include/ascetic.h).
+//
+//   HostGraph : the caller's CSR, pinned (the paper's host "Edgelist")
+//   Part      : one rank's device engine — its owned vertex range [vlo, vhi), replicated
+//               vertex state, its Static Region + On-demand Region, its two streams
+//   Engine    : the ABI context; drives its local parts phase by phase
+//               (classify -> static + transfer + on-demand -> exchange -> finalize) and owns
+//               the Comm (NCCL across processes, or P ranks emulated on one GPU)
 #pragma once
 #include <cstdint>
+#include <memory>
 #include <stdexcept>
 #include <string>
 #include <vector>
@@ -9,6 +17,7 @@
 
 #include "../../include/ascetic.h"
 #include "ascetic_internal.h"
+#include "comm.h"
 
 namespace ascetic {
 
@@ -18,12 +27,16 @@ struct Error : std::runtime_error {
     Error(int c, const std::string& m) : std::runtime_error(m), code(c) {}
 };
 
-// Eq. 1/Eq. 2 placement (§3.3; K = 0.10; 16 KiB).
+// Eq. 1/Eq. 2 placement (§3.3; K = 0.10; 16 KiB) over the
+// rows [0, n) of `off` (absolute offsets; the rows' first arc is off[0]).
 struct Placement {
     double R = 0.0;
     uint64_t D = 0, B = 0, Ms = 0, s = 0, static_bytes = 0, C = 0, cap = 0;
 };
 Placement place(const uint64_t* off, uint64_t n, uint32_t b_e, uint64_t budget, double frac);
+
+// 1D edge-balanced vertex ranges: b_0 = 0, b_P = n, b_g = min{v : off[v] >= ceil(g m / P)}.
+std::vector<uint64_t> partition(const uint64_t* off, uint64_t n, uint32_t P);
 
 struct EventPool {
     std::vector<cudaEvent_t> ev;
@@ -33,41 +46,79 @@ struct EventPool {
     ~EventPool();
 };
 
-class Engine {
-  public:
-    ~Engine();
-    void set_device(int dev);
-    void load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_t* nbr, const uint32_t* wgt,
-                  uint32_t flags);
-    void set_budget(uint64_t bytes, double frac);
-    void set_option(int opt, int64_t value);
-    void run(int algo, uint32_t source, uint32_t max_iters);
-    int stats(ascetic_stats_t* out, ascetic_iter_stats_t* per_iter, uint32_t cap) const;
-    void get_result(void* dst, uint64_t bytes);
-    void unload();
-    int state() const { return state_; }
+struct Options {
+    uint64_t chunk_cap = 0;
+    int xfer_mode = 0;
+    uint64_t dma_min_run = 64 * 1024;
+    int overlap = 1;
+    int keep_static = 0;
+    uint32_t hub_deg = 2048;
+    int timing = 1;
+    int gather_ctas = 0;
+};
 
-  private:
+struct HostGraph {
+    uint64_t n = 0, m = 0;
+    uint32_t b_e = 4, flags = 0;
+    std::vector<uint64_t> off;        // host copy: placer, partition, DMA planning
+    const void* nbr = nullptr;        // b_e bytes per arc, pinned
+    const void* nbr_dev = nullptr;    // device-visible alias (zero-copy)
+    void* owned = nullptr;            // library-owned pinned copy
+    void* registered = nullptr;       // pinned in place by us
+    void release();
+};
+
+enum { PH_CLS, PH_STATIC, PH_OND, PH_GATHER, PH_DMA, PH_FIN, PH_XCH, PH_N };
+
+class Part {
+  public:
+    Part(const HostGraph& g, const Options& o, int rank, uint64_t vlo, uint64_t vhi, int sm_count);
+    ~Part();
     void alloc_vertex_state();
     void alloc_algo_state(int algo);
-    void free_budget_regions();
-    void transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsigned long long hi, int mode,
-                        const std::vector<uint32_t>& rb, const std::vector<uint32_t>& re,
-                        const std::vector<unsigned long long>& rdst);
-    DevState dev_state(uint32_t iter) const;
-    Queues queues(const IterTotals& T) const;
+    void upload_off();
+    void set_budget(uint64_t bytes, double frac);
+    void on_reload() { static_valid_ = false; }
 
-    int state_ = 0;  // 0 unloaded, 1 loaded, 2 ready
-    int device_ = -1;
-    // graph (host)
-    uint64_t n_ = 0, m_ = 0;
-    uint32_t b_e_ = 4, flags_ = 0;
-    const uint64_t* h_off_ = nullptr;
-    std::vector<uint64_t> h_off_copy_;
-    const void* h_nbr_ = nullptr;        // b_e bytes per arc, pinned
-    const void* h_nbr_dev_ = nullptr;    // device-visible alias (zero-copy)
-    void* h_owned_ = nullptr;            // library-owned pinned copy
-    void* h_registered_ = nullptr;       // pinned in place by us
+    // one run, phase by phase
+    void begin(int algo, uint32_t source, bool timing);
+    void classify(uint32_t t);
+    IterTotals wait_classify();
+    void expand(uint32_t t, const IterTotals& T);
+    void finalize(uint32_t t, bool dense);
+    void end();
+    void span(cudaEvent_t a, cudaStream_t s, uint32_t t, int ph);   // close a timed span
+    cudaEvent_t mark(cudaStream_t s);                               // open a timed span
+
+    cudaStream_t cs() const { return cs_; }
+    DevState dev_state(uint32_t iter) const;
+    const Placement& placement() const { return pl_; }
+    uint64_t cap() const { return cap_; }
+    uint64_t vlo() const { return vlo_; }
+    uint64_t vhi() const { return vhi_; }
+    uint32_t* next() const { return d_next_; }
+    uint32_t* val() const { return d_val_; }
+    float* rank_arr() const { return d_rank_; }
+    float* contrib() const { return d_contrib_; }
+    double* dang() const { return d_dang_; }
+    uint64_t vertex_bytes() const { return vertex_bytes_; }
+
+    // results of the last run
+    ascetic_stats_t st{};
+    std::vector<ascetic_iter_stats_t> iters;
+
+  private:
+    void transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsigned long long hi, int mode);
+    Queues queues(const IterTotals& T) const;
+    void free_regions();
+
+    const HostGraph& g_;
+    const Options& o_;
+    int rank_;
+    uint64_t vlo_, vhi_;
+    int sm_count_;
+    int algo_ = 0;
+    bool timing_ = true;
     // device vertex state
     uint32_t nwords_ = 0, ntiles_ = 0;
     unsigned long long* d_off_ = nullptr;
@@ -76,39 +127,66 @@ class Engine {
     float *d_rank_ = nullptr, *d_contrib_ = nullptr;
     double *d_sum_ = nullptr, *d_dang_ = nullptr;
     uint32_t *d_hq_small_ = nullptr, *d_hq_med_ = nullptr, *d_hq_hub_ = nullptr, *d_hub_pre_ = nullptr;
-    uint32_t *d_mq_ = nullptr, *d_run_b_ = nullptr, *d_run_e_ = nullptr;
-    unsigned long long *d_mq_pre_ = nullptr, *d_run_dst_ = nullptr, *d_mq_src_ = nullptr;
-    uint32_t* d_tile_first_ = nullptr;
-    int sm_count_ = 148;
-    int opt_gather_ctas_ = 0;       // 0 = 2 x SMs
+    uint32_t *d_mq_ = nullptr, *d_run_b_ = nullptr, *d_run_e_ = nullptr, *d_tile_first_ = nullptr;
+    unsigned long long *d_mq_pre_ = nullptr, *d_mq_src_ = nullptr, *d_run_dst_ = nullptr;
+    uint64_t hub_cap_ = 0;
     ScanVal *d_tile_agg_ = nullptr, *d_tile_incl_ = nullptr;
     uint32_t* d_tile_flag_ = nullptr;
     uint32_t epoch_ = 0;
     IterTotals* d_tot_ = nullptr;
     IterTotals* h_tot_ = nullptr;   // mapped pinned
     uint64_t vertex_bytes_ = 0;
-    // edge budget regions
+    // edge budget regions (Eq. 1/2)
     Placement pl_{};
     void* d_static_ = nullptr;
     void* d_chunk_[2] = {nullptr, nullptr};
-    uint64_t cap_ = 0;              // effective chunk capacity (bytes)
-    bool static_valid_ = false;     // KEEP_STATIC: static region already holds the prefix
-    // streams/events
+    uint64_t cap_ = 0, static_alloc_ = 0, chunk_alloc_ = 0;
+    bool static_valid_ = false;
+    // streams / events
     cudaStream_t cs_ = nullptr, xs_ = nullptr;
     cudaEvent_t ready_[2] = {nullptr, nullptr}, consumed_[2] = {nullptr, nullptr};
     cudaEvent_t ev_classified_ = nullptr;
     EventPool pool_;
-    // options
-    uint64_t opt_chunk_cap_ = 0;
-    int opt_xfer_mode_ = 0;
-    uint64_t opt_dma_min_run_ = 64 * 1024;
-    int opt_overlap_ = 1;
-    int opt_keep_static_ = 0;
-    uint32_t opt_hub_deg_ = 2048;
-    int opt_timing_ = 1;
+    struct Span { cudaEvent_t a, b; uint32_t iter; int ph; };
+    std::vector<Span> spans_;
+    cudaEvent_t ev_start_ = nullptr, ev_fill0_ = nullptr, ev_fill1_ = nullptr;
+    double host_s_ = 0.0;
+    unsigned long long launches0_ = 0;
+    // DMA planning scratch
+    std::vector<uint32_t> rb_, re_;
+    std::vector<unsigned long long> rdst_;
     static constexpr uint32_t kPieceArcs = 4096;
     static constexpr uint32_t kRunsHostMax = 8192;
-    // results / stats
+};
+
+class Engine {
+  public:
+    ~Engine();
+    void set_device(int dev);
+    void comm_init(int rank, int world, const void* uid, int device);
+    void emulate_ranks(int world);
+    void load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_t* nbr, const uint32_t* wgt,
+                  uint32_t flags);
+    void set_budget(uint64_t bytes, double frac);
+    void set_option(int opt, int64_t value);
+    void run(int algo, uint32_t source, uint32_t max_iters);
+    int stats(ascetic_stats_t* out, ascetic_iter_stats_t* per_iter, uint32_t cap) const;
+    void get_result(void* dst, uint64_t bytes);
+    void unload();
+
+  private:
+    void join(std::vector<cudaStream_t>* waiters);   // all local parts' cs -> parts_[0].cs
+    void fork();                                      // parts_[0].cs -> all local parts' cs
+
+    int state_ = 0;   // 0 unloaded, 1 loaded, 2 ready
+    int device_ = -1;
+    int sm_count_ = 148;
+    HostGraph g_;
+    Options o_;
+    Comm comm_;
+    int emulate_ = 1;
+    std::vector<std::unique_ptr<Part>> parts_;
+    std::vector<uint64_t> bounds_;
     int last_algo_ = -1;
     bool have_result_ = false;
     ascetic_stats_t st_{};

@@ -31,6 +31,17 @@ __device__ __forceinline__ unsigned long long mix64(unsigned long long z) {
     return z ^ (z >> 31);
 }
 
+// bits of word w that fall in the vertex range [vlo, vhi)
+__device__ __forceinline__ uint32_t own_mask(uint32_t w, unsigned long long vlo, unsigned long long vhi) {
+    const unsigned long long b = (unsigned long long)w * 32ull;
+    const unsigned long long lo = vlo > b ? vlo : b;
+    const unsigned long long hi = vhi < b + 32 ? vhi : b + 32;
+    if (lo >= hi) return 0u;
+    const uint32_t top = (uint32_t)(hi - b), bot = (uint32_t)(lo - b);
+    const uint32_t upto = top == 32 ? FULL : ((1u << top) - 1u);
+    return upto & ~((1u << bot) - 1u);
+}
+
 __device__ __forceinline__ unsigned long long wsum64(unsigned long long x) {
 #pragma unroll
     for (int d = 16; d; d >>= 1) x += __shfl_xor_sync(FULL, x, d);
@@ -117,12 +128,17 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
     const uint32_t w0 = tile * kTileWords + warp * 32;
     const uint32_t myw = w0 + lane;
 
-    uint32_t myA = 0, myS = 0;
-    if (myw < a.nwords) { myA = __ldg(a.A + myw); myS = __ldg(a.S + myw); }
+    // A is replicated across ranks; this rank classifies only its owned range [vlo, vhi)
+    // while |A| and the digest are taken over the whole bitmap.
+    uint32_t myAll = 0, myS = 0;
+    if (myw < a.nwords) { myAll = __ldg(a.A + myw); myS = __ldg(a.S + myw); }
+    const uint32_t myA = myAll & own_mask(myw, a.vlo, a.vhi);
     const uint32_t myMiss = myA & ~myS;
     uint32_t prevMiss = 0, nextMiss = 0;
-    if (w0 > 0 && w0 - 1 < a.nwords) prevMiss = __ldg(a.A + w0 - 1) & ~__ldg(a.S + w0 - 1);
-    if (w0 + 32 < a.nwords) nextMiss = __ldg(a.A + w0 + 32) & ~__ldg(a.S + w0 + 32);
+    if (w0 > 0 && w0 - 1 < a.nwords)
+        prevMiss = __ldg(a.A + w0 - 1) & ~__ldg(a.S + w0 - 1) & own_mask(w0 - 1, a.vlo, a.vhi);
+    if (w0 + 32 < a.nwords)
+        nextMiss = __ldg(a.A + w0 + 32) & ~__ldg(a.S + w0 + 32) & own_mask(w0 + 32, a.vlo, a.vhi);
     const uint32_t anyA = __ballot_sync(FULL, myA != 0);
     const uint32_t piece = a.piece_arcs;
 
@@ -160,8 +176,8 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
     }
     ScanVal wagg = sv_warp_sum(mine);
     {
-        unsigned long long nA = __popc(myA), nH = __popc(myA & myS), nM = __popc(myMiss);
-        unsigned long long dg = (myw < a.nwords) ? mix64((unsigned long long)myw ^ ((unsigned long long)myA * PHI)) : 0ull;
+        unsigned long long nA = __popc(myAll), nH = __popc(myA & myS), nM = __popc(myMiss);
+        unsigned long long dg = (myw < a.nwords) ? mix64((unsigned long long)myw ^ ((unsigned long long)myAll * PHI)) : 0ull;
         nA = wsum64(nA); nH = wsum64(nH); nM = wsum64(nM); dg = wsum64(dg);
         aArcs = wsum64(aArcs); hArcs = wsum64(hArcs);
         if (lane == 0) {
