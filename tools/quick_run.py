@@ -26,14 +26,20 @@ def main():
     ap.add_argument("--chunk-cap", type=int, default=0)
     ap.add_argument("--sweep", action="store_true")
     ap.add_argument("--quiet", action="store_true")
+    ap.add_argument("--budget-mult", type=float, default=0.0, help="budget = mult x CSR bytes (config runs)")
+    ap.add_argument("--algo-override", default="")
+    ap.add_argument("--scale-override", type=int, default=0)
     a = ap.parse_args()
     import paper_conf_icpp_tangzwgzwy21_b200 as asc
     t0 = time.time()
     if a.config:
-        g = gg.config_graph(a.config)
-        budget = gg.config_budget(a.config, g)
-        algo = gg.CONFIGS[a.config]["algo"]
-        iters = gg.CONFIGS[a.config].get("iters", 0)
+        cfg = dict(gg.CONFIGS[a.config])
+        want_w = (a.algo_override or cfg["algo"]) == "sssp"
+        g = gg.rmat(a.scale_override or cfg["scale"], cfg["tuples"] if not a.scale_override else None, seed=cfg["seed"],
+                    permute=cfg["permute"], n=cfg["n"] if not a.scale_override else 0, weights=want_w, name=a.config)
+        budget = gg.config_budget(a.config, g) if a.budget_mult <= 0 else int(a.budget_mult * g.csr_bytes)
+        algo = gg.CONFIGS[a.config]["algo"] if a.algo_override == "" else a.algo_override
+        iters = gg.CONFIGS[a.config].get("iters", 0) if a.iters == 0 else a.iters
     else:
         g = gg.rmat(a.scale, seed=2, weights=(a.algo == "sssp"))
         budget = int(a.frac_budget * g.csr_bytes)
@@ -70,6 +76,14 @@ def main():
                                               "active_arcs_total", "chunks_total", "dma_chunks", "gather_chunks",
                                               "time_run_s", "time_fill_s", "time_h2d_busy_s", "gteps",
                                               "chunk_cap"]}), flush=True)
+        b_e = g.b_e
+        ks = {"static": (st["static_arcs"] * (b_e + 4), st["time_static_s"]),
+              "ondemand": (st["ondemand_arcs"] * (b_e + 4), st["time_ondemand_s"]),
+              "gather": (st["gather_bytes"], st["time_gather_s"]),
+              "classify": (0, st["time_classify_s"]), "finalize": (0, st["time_finalize_s"])}
+        print("  kernels:", {k: (round(t * 1e3, 3), round(b / t / 1e9, 1) if t > 0 else 0) for k, (b, t) in ks.items()},
+              f"GTEPS={st['active_arcs_total'] / st['time_run_s'] / 1e9:.2f} "
+              f"static_Garcs/s={st['static_arcs'] / max(st['time_static_s'], 1e-9) / 1e9:.1f}", flush=True)
     for i in ([] if a.quiet else its):
         print({k: (round(v, 3) if isinstance(v, float) else v) for k, v in i.items() if k != "digest"})
     if a.oracle:
