@@ -67,7 +67,7 @@ typedef enum {
     ASCETIC_OPT_KEEP_STATIC = 5,   /* 1 = keep the Static Region filled across runs (fill counted once) ; default 0 */
     ASCETIC_OPT_HUB_DEGREE = 6,    /* hit-queue degree at/above which a list is split across CTAs (default 2048) */
     ASCETIC_OPT_TIMING = 7,        /* 1 (default) = per-iteration phase timing with CUDA events */
-    ASCETIC_OPT_GATHER_CTAS = 8    /* persistent CTAs of the zero-copy gather; 0 (default) = 2 x SM count */
+    ASCETIC_OPT_GATHER_CTAS = 8    /* persistent CTAs of the zero-copy gather; 0 (default) = 512 / b_e (~1 MiB in flight) */
 } ascetic_option;
 
 typedef struct {
@@ -119,7 +119,12 @@ typedef struct {
     uint64_t digest;              /* Σ_w splitmix64(w ^ word_w * 0x9E3779B97F4A7C15) over A_t's bitmap */
     uint32_t chunks;
     uint32_t mode;                /* 1 = zero-copy gather, 2 = DMA */
+    /* device time of each kernel class in this iteration (CUDA events); ms_total = the
+     * iteration's wall time from its classify launch to the next iteration's */
     float ms_classify, ms_static, ms_ondemand, ms_h2d, ms_finalize, ms_exchange, ms_total;
+    /* host-link idle inside the iteration: before its first chunk transfer, between its
+     * chunk transfers, and after its last one (until the next iteration's classify) */
+    float ms_link_head, ms_link_gaps, ms_link_tail;
 } ascetic_iter_stats_t;
 
 /*

@@ -67,7 +67,8 @@ class IterStats(ctypes.Structure):
                 ("digest", ctypes.c_uint64), ("chunks", ctypes.c_uint32), ("mode", ctypes.c_uint32),
                 ("ms_classify", ctypes.c_float), ("ms_static", ctypes.c_float), ("ms_ondemand", ctypes.c_float),
                 ("ms_h2d", ctypes.c_float), ("ms_finalize", ctypes.c_float), ("ms_exchange", ctypes.c_float),
-                ("ms_total", ctypes.c_float)]
+                ("ms_total", ctypes.c_float), ("ms_link_head", ctypes.c_float), ("ms_link_gaps", ctypes.c_float),
+                ("ms_link_tail", ctypes.c_float)]
 
 
 _lib.ascetic_load_csr.argtypes = [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p,

@@ -30,21 +30,65 @@ constexpr unsigned FULL = 0xFFFFFFFFu;
 enum { BFS = 0, SSSP = 1, CC = 2, PR = 3 };
 constexpr double kDamp = 0.85;
 
+// ------------------------------------------------------------------ L2 policy loads
+// Adjacency lists and chunks are read once: stream them with L2 evict_first so they do not
+// push the randomly accessed vertex state (dist / labels / bitmaps / contrib, the part of
+// the working set with reuse) out of the 126 MB L2; the state is loaded with evict_last.
+__device__ __forceinline__ unsigned long long pol_stream() {
+    unsigned long long p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ unsigned long long pol_keep() {
+    unsigned long long p;
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint4 ld_stream(const uint4* p) {
+    uint4 x;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=r"(x.x), "=r"(x.y), "=r"(x.z), "=r"(x.w) : "l"(p), "l"(pol_stream()));
+    return x;
+}
+__device__ __forceinline__ uint2 ld_stream(const uint2* p) {
+    uint2 x;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u32 {%0,%1}, [%2], %3;"
+                 : "=r"(x.x), "=r"(x.y) : "l"(p), "l"(pol_stream()));
+    return x;
+}
+__device__ __forceinline__ uint32_t ld_stream(const uint32_t* p) {
+    uint32_t x;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(x) : "l"(p), "l"(pol_stream()));
+    return x;
+}
+// state written by atomics during the kernel: coherent load, kept in L2
+__device__ __forceinline__ uint32_t ld_state(const uint32_t* p) {
+    uint32_t x;
+    asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(x) : "l"(p), "l"(pol_keep()));
+    return x;
+}
+// state that is read-only during the kernel (visited bitmap, contrib)
+__device__ __forceinline__ uint32_t ld_state_ro(const uint32_t* p) {
+    uint32_t x;
+    asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(x) : "l"(p), "l"(pol_keep()));
+    return x;
+}
+
 // ------------------------------------------------------------------ per-arc ops
 __device__ __forceinline__ void set_next(const DevState& d, uint32_t v) {
     const uint32_t wi = v >> 5, bit = 1u << (v & 31);
-    if (!(d.next[wi] & bit)) atomicOr(d.next + wi, bit);
+    if (!(ld_state(d.next + wi) & bit)) atomicOr(d.next + wi, bit);
 }
 
 __device__ __forceinline__ void bfs_visit(const DevState& d, uint32_t v) {
     const uint32_t wi = v >> 5, bit = 1u << (v & 31);
-    if (__ldg(d.visited + wi) & bit) return;      // visited changes only in finalize
-    if (d.next[wi] & bit) return;
+    if (ld_state_ro(d.visited + wi) & bit) return;      // visited changes only in finalize
+    if (ld_state(d.next + wi) & bit) return;
     atomicOr(d.next + wi, bit);
 }
 
 __device__ __forceinline__ void relax(const DevState& d, uint32_t v, uint32_t cand) {
-    if (cand >= d.val[v]) return;                 // values only decrease within an iteration
+    if (cand >= ld_state(d.val + v)) return;            // values only decrease within an iteration
     const uint32_t old = atomicMin(d.val + v, cand);
     if (cand < old) set_next(d, v);
 }
@@ -63,7 +107,7 @@ __device__ __forceinline__ void push_arc(const DevState& d, uint32_t sval, uint3
 }
 
 __device__ __forceinline__ double pr_in(const DevState& d, uint32_t id) {
-    return (double)__ldg(d.contrib + id);
+    return (double)__uint_as_float(ld_state_ro(reinterpret_cast<const uint32_t*>(d.contrib) + id));
 }
 
 __device__ __forceinline__ uint32_t ub_u32(const uint32_t* a, uint32_t n, uint32_t x) {
@@ -85,31 +129,31 @@ __device__ __forceinline__ double expand_list(const DevState& d, const void* bas
         const uint2* arcs = reinterpret_cast<const uint2*>(base);
         const unsigned long long h = min(a1, (a0 + 1) & ~1ull);      // 2 arcs per 16 B
         for (unsigned long long e = a0 + tid; e < h; e += nthr) {
-            const uint2 x = __ldg(arcs + e);
+            const uint2 x = ld_stream(arcs + e);
             push_arc<ALGO>(d, sval, x.x, x.y);
         }
         const unsigned long long qb = h >> 1, qe = a1 >> 1;
         const uint4* q = reinterpret_cast<const uint4*>(base);
         for (unsigned long long k = qb + tid; k < qe; k += nthr) {
-            const uint4 x = __ldg(q + k);
+            const uint4 x = ld_stream(q + k);
             push_arc<ALGO>(d, sval, x.x, x.y);
             push_arc<ALGO>(d, sval, x.z, x.w);
         }
         for (unsigned long long e = max(h, qe << 1) + tid; e < a1; e += nthr) {
-            const uint2 x = __ldg(arcs + e);
+            const uint2 x = ld_stream(arcs + e);
             push_arc<ALGO>(d, sval, x.x, x.y);
         }
     } else {
         const uint32_t* arcs = reinterpret_cast<const uint32_t*>(base);
         const unsigned long long h = min(a1, (a0 + 3) & ~3ull);      // 4 arcs per 16 B
         for (unsigned long long e = a0 + tid; e < h; e += nthr) {
-            const uint32_t id = __ldg(arcs + e);
+            const uint32_t id = ld_stream(arcs + e);
             if (ALGO == PR) acc += pr_in(d, id); else push_arc<ALGO>(d, sval, id, 0);
         }
         const unsigned long long qb = h >> 2, qe = a1 >> 2;
         const uint4* q = reinterpret_cast<const uint4*>(base);
         for (unsigned long long k = qb + tid; k < qe; k += nthr) {
-            const uint4 x = __ldg(q + k);
+            const uint4 x = ld_stream(q + k);
             if (ALGO == PR) {
                 acc += pr_in(d, x.x) + pr_in(d, x.y) + pr_in(d, x.z) + pr_in(d, x.w);
             } else {
@@ -118,7 +162,7 @@ __device__ __forceinline__ double expand_list(const DevState& d, const void* bas
             }
         }
         for (unsigned long long e = max(h, qe << 2) + tid; e < a1; e += nthr) {
-            const uint32_t id = __ldg(arcs + e);
+            const uint32_t id = ld_stream(arcs + e);
             if (ALGO == PR) acc += pr_in(d, id); else push_arc<ALGO>(d, sval, id, 0);
         }
     }
@@ -174,7 +218,7 @@ __global__ void __launch_bounds__(256) k_static_small(DevState d, const uint32_t
         const bool ok = k < total;
         const unsigned long long e = ust + (k - uex) - d.static_arc0;   // index into the Static Region
         if (ALGO == PR) {
-            double x = ok ? pr_in(d, __ldg(reinterpret_cast<const uint32_t*>(sbase) + e)) : 0.0;
+            double x = ok ? pr_in(d, ld_stream(reinterpret_cast<const uint32_t*>(sbase) + e)) : 0.0;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
                 const double y = __shfl_up_sync(FULL, x, o);
@@ -188,10 +232,10 @@ __global__ void __launch_bounds__(256) k_static_small(DevState d, const uint32_t
             __syncwarp();
         } else if (ok) {
             if (ALGO == SSSP) {
-                const uint2 x = __ldg(reinterpret_cast<const uint2*>(sbase) + e);
+                const uint2 x = ld_stream(reinterpret_cast<const uint2*>(sbase) + e);
                 push_arc<ALGO>(d, usv, x.x, x.y);
             } else {
-                push_arc<ALGO>(d, usv, __ldg(reinterpret_cast<const uint32_t*>(sbase) + e), 0);
+                push_arc<ALGO>(d, usv, ld_stream(reinterpret_cast<const uint32_t*>(sbase) + e), 0);
             }
         }
     }
@@ -321,17 +365,17 @@ __global__ void __launch_bounds__(256) k_ondemand(DevState d, Queues q, const vo
             id[g] = kInf;
             if (a < pe) {
                 if (ALGO == SSSP) {
-                    const uint2 e = __ldg(reinterpret_cast<const uint2*>(chunk) + (a - lo));
+                    const uint2 e = ld_stream(reinterpret_cast<const uint2*>(chunk) + (a - lo));
                     id[g] = e.x;
                     cand[g] = sat_add(s_v[mk], e.y);
                 } else {
-                    id[g] = __ldg(reinterpret_cast<const uint32_t*>(chunk) + (a - lo));
+                    id[g] = ld_stream(reinterpret_cast<const uint32_t*>(chunk) + (a - lo));
                     cand[g] = s_v[mk];
                 }
             }
         }
 #pragma unroll
-        for (int g = 0; g < 8; ++g) cur[g] = id[g] != kInf ? d.val[id[g]] : 0u;
+        for (int g = 0; g < 8; ++g) cur[g] = id[g] != kInf ? ld_state(d.val + id[g]) : 0u;
 #pragma unroll
         for (int g = 0; g < 8; ++g) {
             if (id[g] != kInf && cand[g] < cur[g]) {
@@ -346,7 +390,7 @@ __global__ void __launch_bounds__(256) k_ondemand(DevState d, Queues q, const vo
         const unsigned long long a = p + lane;
         const bool ok = a < pe;
         if (ALGO == PR) {
-            double v = ok ? pr_in(d, __ldg(reinterpret_cast<const uint32_t*>(chunk) + (a - lo))) : 0.0;
+            double v = ok ? pr_in(d, ld_stream(reinterpret_cast<const uint32_t*>(chunk) + (a - lo))) : 0.0;
             const int key = ok ? (int)mk : -1 - lane;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
@@ -358,10 +402,10 @@ __global__ void __launch_bounds__(256) k_ondemand(DevState d, Queues q, const vo
             if (ok && (lane == 31 || nk != key)) atomicAdd(d.sum + s_u[mk], v);
         } else if (ok) {
             if (ALGO == SSSP) {
-                const uint2 e = __ldg(reinterpret_cast<const uint2*>(chunk) + (a - lo));
+                const uint2 e = ld_stream(reinterpret_cast<const uint2*>(chunk) + (a - lo));
                 push_arc<ALGO>(d, s_v[mk], e.x, e.y);
             } else {
-                push_arc<ALGO>(d, s_v[mk], __ldg(reinterpret_cast<const uint32_t*>(chunk) + (a - lo)), 0);
+                push_arc<ALGO>(d, s_v[mk], ld_stream(reinterpret_cast<const uint32_t*>(chunk) + (a - lo)), 0);
             }
         }
     }
@@ -374,11 +418,11 @@ __global__ void __launch_bounds__(256) k_ondemand_bfs(DevState d, const uint32_t
     const uint4* c4 = reinterpret_cast<const uint4*>(chunk);
     const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
     for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < nq4; i += stride) {
-        const uint4 x = __ldg(c4 + i);
+        const uint4 x = ld_stream(c4 + i);
         bfs_visit(d, x.x); bfs_visit(d, x.y); bfs_visit(d, x.z); bfs_visit(d, x.w);
     }
     const unsigned long long t = (nq4 << 2) + (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x;
-    if (t < len) bfs_visit(d, __ldg(chunk + t));
+    if (t < len) bfs_visit(d, ld_stream(chunk + t));
 }
 
 // ------------------------------------------------------------------ zero-copy gather (transfer engine)

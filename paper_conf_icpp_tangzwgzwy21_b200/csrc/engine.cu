@@ -130,20 +130,30 @@ Part::~Part() {
         if (consumed_[i]) cudaEventDestroy(consumed_[i]);
     }
     if (ev_classified_) cudaEventDestroy(ev_classified_);
+    if (static_go_) cudaEventDestroy(static_go_);
+    if (static_done_) cudaEventDestroy(static_done_);
+    if (ss_) { cudaStreamSynchronize(ss_); cudaStreamDestroy(ss_); }
     if (cs_) cudaStreamDestroy(cs_);
     if (xs_) cudaStreamDestroy(xs_);
     cudaGetLastError();
 }
 
 void Part::alloc_vertex_state() {
+    // priorities (numerically lower = higher): transfer > on-demand/classify/finalize > static
+    // hits. The static-hit kernels have slack (they only need to finish before finalize);
+    // the on-demand kernels gate the reuse of the two chunk buffers, i.e. the link.
     int lo_pri = 0, hi_pri = 0;
     CK(cudaDeviceGetStreamPriorityRange(&lo_pri, &hi_pri));
-    CK(cudaStreamCreateWithPriority(&cs_, cudaStreamNonBlocking, lo_pri));
+    const int mid_pri = hi_pri < lo_pri ? hi_pri + 1 : hi_pri;
+    CK(cudaStreamCreateWithPriority(&cs_, cudaStreamNonBlocking, mid_pri));
     CK(cudaStreamCreateWithPriority(&xs_, cudaStreamNonBlocking, hi_pri));
+    CK(cudaStreamCreateWithPriority(&ss_, cudaStreamNonBlocking, lo_pri));
     for (int i = 0; i < 2; ++i) {
         CK(cudaEventCreateWithFlags(&ready_[i], cudaEventDisableTiming));
         CK(cudaEventCreateWithFlags(&consumed_[i], cudaEventDisableTiming));
     }
+    CK(cudaEventCreateWithFlags(&static_go_, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&static_done_, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&ev_classified_, cudaEventDisableTiming));
     const uint64_t n = g_.n, m = g_.m;
     vertex_bytes_ = 0;
@@ -283,7 +293,12 @@ void Part::span(cudaEvent_t a, cudaStream_t s, uint32_t t, int ph) {
 // the miss queue; mode 2: copy-engine DMA of the run pieces intersecting the window.
 void Part::transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsigned long long hi, int mode) {
     if (mode == 1) {
-        launch_gather(q, g_.nbr_dev, g_.b_e, d_chunk_[buf], lo, hi, o_.gather_ctas ? o_.gather_ctas : 2 * sm_count_, xs_);
+        // default grid keeps ~1 MiB of PCIe reads in flight (CTAs x 256 lanes x 8 loads x b_e):
+        // enough to saturate the link (~20 us of it), while a deeper queue only adds latency
+        // and congests the memory system for the concurrently running edge kernels
+        // (measured: 64 CTAs at b_e = 8 -> same 47 GB/s, 3x faster on-demand kernels than 296)
+        const int ctas = o_.gather_ctas ? o_.gather_ctas : (int)(64u * 8u / g_.b_e);
+        launch_gather(q, g_.nbr_dev, g_.b_e, d_chunk_[buf], lo, hi, ctas, xs_);
         return;
     }
     size_t r = std::upper_bound(rdst_.begin(), rdst_.end(), lo) - rdst_.begin();
@@ -387,14 +402,21 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     const DevState d = dev_state(t);
     const Queues q = queues(T);
     if (algo_ == ALG_PR) CK(cudaMemsetAsync(d_sum_ + vlo_, 0, (vhi_ - vlo_) * sizeof(double), cs_));
-    // ---- Static Computing, overlapping the transfer. The static
-    // buffer holds host arcs [off[vlo], off[vlo+s]); kernels index it with rank-local arc
-    // numbers (arc - d.static_arc0), so 128-bit alignment is that of the buffer itself.
+    // ---- Static Computing, overlapping the transfer, on its own stream so
+    // the on-demand kernels (and through them the chunk buffers' reuse) never queue behind it;
+    // finalize joins it. The static buffer holds host arcs [off[vlo], off[vlo+s]); kernels
+    // index it with rank-local arc numbers (arc - d.static_arc0), so 128-bit alignment is
+    // that of the buffer itself.
+    static_pending_ = false;
     if (T.n_small + T.n_med + T.n_hub) {
-        cudaEvent_t e0 = mark(cs_);
-        launch_static(algo_, d, q, d_static_, T.n_small, T.n_med, T.n_hub, T.n_pieces, kPieceArcs, cs_);
+        CK(cudaEventRecord(static_go_, cs_));
+        CK(cudaStreamWaitEvent(ss_, static_go_, 0));
+        cudaEvent_t e0 = mark(ss_);
+        launch_static(algo_, d, q, d_static_, T.n_small, T.n_med, T.n_hub, T.n_pieces, kPieceArcs, ss_);
         CK(cudaGetLastError());
-        span(e0, cs_, t, PH_STATIC);
+        span(e0, ss_, t, PH_STATIC);
+        CK(cudaEventRecord(static_done_, ss_));
+        static_pending_ = true;
     }
     st.static_arcs += T.hit_arcs;
     st.ondemand_arcs += T.miss_arcs;
@@ -415,11 +437,7 @@ void Part::expand(uint32_t t, const IterTotals& T) {
             unsigned long long acc = 0;
             for (uint32_t r = 0; r < T.n_runs; ++r) { rdst_[r] = acc; acc += g_.off[re_[r]] - g_.off[rb_[r]]; }
         }
-        if (!o_.overlap) {
-            cudaEvent_t es = pool_.get();
-            CK(cudaEventRecord(es, cs_));
-            CK(cudaStreamWaitEvent(xs_, es, 0));
-        }
+        if (!o_.overlap && static_pending_) CK(cudaStreamWaitEvent(xs_, static_done_, 0));   // ablation
     }
     for (uint32_t k = 0; k < nchunks; ++k) {
         const int buf = k & 1;
@@ -449,8 +467,14 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     host_s_ += std::chrono::duration<double>(std::chrono::steady_clock::now() - th0).count();
 }
 
+void Part::join_static() {
+    if (static_pending_) CK(cudaStreamWaitEvent(cs_, static_done_, 0));
+    static_pending_ = false;
+}
+
 void Part::finalize(uint32_t t, bool dense) {
-    // ---- next active set
+    // ---- next active set, after the static-hit kernels
+    join_static();
     cudaEvent_t e0 = mark(cs_);
     launch_finalize(algo_, dev_state(t), dense, cs_);
     CK(cudaGetLastError());
@@ -459,9 +483,11 @@ void Part::finalize(uint32_t t, bool dense) {
 
 void Part::end() {
     cudaEvent_t ev_end = pool_.get();
+    join_static();
     CK(cudaEventRecord(ev_end, cs_));
     CK(cudaStreamSynchronize(cs_));
     CK(cudaStreamSynchronize(xs_));
+    CK(cudaStreamSynchronize(ss_));
     float ms = 0.f, fill_ms = 0.f;
     CK(cudaEventElapsedTime(&ms, ev_start_, ev_end));
     CK(cudaEventElapsedTime(&fill_ms, ev_fill0_, ev_fill1_));
@@ -482,8 +508,32 @@ void Part::end() {
             }
         }
     }
-    for (auto& is : iters)
-        is.ms_total = is.ms_classify + is.ms_static + is.ms_ondemand + is.ms_finalize + is.ms_exchange;
+    // iteration wall time: from its classify launch to the next one (the last: to the run's end)
+    std::vector<cudaEvent_t> cls_start(iters.size() + 1, nullptr);
+    for (const Span& sp : spans_)
+        if (sp.ph == PH_CLS && sp.iter < cls_start.size()) cls_start[sp.iter] = sp.a;
+    std::vector<cudaEvent_t> x_first(iters.size(), nullptr), x_last(iters.size(), nullptr);
+    for (const Span& sp : spans_) {
+        if ((sp.ph == PH_GATHER || sp.ph == PH_DMA) && sp.iter < iters.size()) {
+            if (!x_first[sp.iter]) x_first[sp.iter] = sp.a;
+            x_last[sp.iter] = sp.b;
+        }
+    }
+    for (size_t i = 0; i < iters.size(); ++i) {
+        cudaEvent_t a = cls_start[i], b = cls_start[i + 1] ? cls_start[i + 1] : ev_end;
+        float w = 0.f;
+        if (a) CK(cudaEventElapsedTime(&w, a, b));
+        iters[i].ms_total = w;
+        if (a && x_first[i]) {
+            float h = 0.f, span_ms = 0.f, tl = 0.f;
+            CK(cudaEventElapsedTime(&h, a, x_first[i]));
+            CK(cudaEventElapsedTime(&span_ms, x_first[i], x_last[i]));
+            CK(cudaEventElapsedTime(&tl, x_last[i], b));
+            iters[i].ms_link_head = h;
+            iters[i].ms_link_gaps = span_ms - iters[i].ms_h2d;
+            iters[i].ms_link_tail = tl;
+        }
+    }
     st.algo = algo_;
     st.iterations = (uint32_t)iters.size();
     st.n = g_.n; st.m = g_.m; st.b_e = g_.b_e;
@@ -573,14 +623,22 @@ void Engine::load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_
     CK(cudaDeviceGetAttribute(&sm_count_, cudaDevAttrMultiProcessorCount, device_));
     // same shape: keep every device allocation and stream (a reload is then offsets H2D and
     // host bookkeeping only); otherwise start from scratch
-    const bool reuse = state_ != 0 && n == g_.n && m == g_.m && b_e == g_.b_e &&
-                       std::equal(off, off + n + 1, g_.off.begin());
     const bool same_shape = state_ != 0 && n == g_.n && m == g_.m && b_e == g_.b_e;
     if (state_ != 0 && !same_shape) unload();
     if (same_shape) g_.release();
     have_result_ = false;
     g_.n = n; g_.m = m; g_.b_e = b_e; g_.flags = flags;
-    if (!reuse) g_.off.assign(off, off + n + 1);
+    {   // host planning copy of the offsets (parallel memcpy)
+        g_.off.resize(n + 1);
+        const unsigned nt = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
+        std::vector<std::thread> th;
+        for (unsigned t = 0; t < nt; ++t)
+            th.emplace_back([&, t] {
+                const uint64_t a = (n + 1) * t / nt, b = (n + 1) * (t + 1) / nt;
+                std::memcpy(g_.off.data() + a, off + a, (b - a) * sizeof(uint64_t));
+            });
+        for (auto& x : th) x.join();
+    }
     // ---- pin the edge array (the On-demand Engine's Edgelist)
     const size_t bytes = (size_t)b_e * m;
     if (bytes > 0) {
@@ -637,10 +695,7 @@ void Engine::load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_
         }
         for (auto& p : parts_) p->alloc_vertex_state();
     }
-    for (auto& p : parts_) {
-        if (!reuse) p->upload_off();
-        p->on_reload();
-    }
+    for (auto& p : parts_) p->upload_off();   // offsets H2D on every load (also resets the static region)
     for (auto& p : parts_) CK(cudaStreamSynchronize(p->cs()));
     state_ = 1;
 }
@@ -731,6 +786,7 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         for (size_t i = 0; i < parts_.size(); ++i) parts_[i]->expand(t, T[i]);
         if (multi && algo != ALG_PR) {
             // ---- exchange: OR of next bitmaps (BFS), MIN of values (SSSP, CC)
+            for (auto& p : parts_) p->join_static();
             join(nullptr);
             cudaEvent_t e0 = p0.mark(p0.cs());
             const uint64_t nw = (g_.n + 31) / 32;

@@ -85,6 +85,7 @@ class Part {
     void classify(uint32_t t);
     IterTotals wait_classify();
     void expand(uint32_t t, const IterTotals& T);
+    void join_static();   // cs waits for this iteration's static-hit kernels
     void finalize(uint32_t t, bool dense);
     void end();
     void span(cudaEvent_t a, cudaStream_t s, uint32_t t, int ph);   // close a timed span
@@ -143,8 +144,10 @@ class Part {
     uint64_t cap_ = 0, static_alloc_ = 0, chunk_alloc_ = 0;
     bool static_valid_ = false;
     // streams / events
-    cudaStream_t cs_ = nullptr, xs_ = nullptr;
+    cudaStream_t cs_ = nullptr, xs_ = nullptr, ss_ = nullptr;   // compute, copy, static-hit streams
     cudaEvent_t ready_[2] = {nullptr, nullptr}, consumed_[2] = {nullptr, nullptr};
+    cudaEvent_t static_go_ = nullptr, static_done_ = nullptr;
+    bool static_pending_ = false;
     cudaEvent_t ev_classified_ = nullptr;
     EventPool pool_;
     struct Span { cudaEvent_t a, b; uint32_t iter; int ph; };

@@ -29,6 +29,8 @@ def main():
     ap.add_argument("--budget-mult", type=float, default=0.0, help="budget = mult x CSR bytes (config runs)")
     ap.add_argument("--algo-override", default="")
     ap.add_argument("--scale-override", type=int, default=0)
+    ap.add_argument("--sweep-ctas", default="148,296,444,592,1184")
+    ap.add_argument("--sweep-caps", default="0,32,8")
     a = ap.parse_args()
     import paper_conf_icpp_tangzwgzwy21_b200 as asc
     t0 = time.time()
@@ -54,8 +56,8 @@ def main():
     asc.set_option("chunk_cap", a.chunk_cap)
     src = gg.sources(g, 1, seed=1)[0]
     if a.sweep:
-        for gc in [148, 296, 444, 592, 1184]:
-            for cc in [0, 32 << 20, 8 << 20]:
+        for gc in [int(x) for x in a.sweep_ctas.split(',')]:
+            for cc in [int(x) << 20 for x in a.sweep_caps.split(',')]:
                 asc.set_option("gather_ctas", gc)
                 asc.set_option("chunk_cap", cc)
                 best = None
@@ -66,7 +68,8 @@ def main():
                         best = st
                 print(f"gather_ctas={gc:5d} chunk_cap={cc>>20:4d}MiB run_ms={best['time_run_s']*1e3:8.2f} "
                       f"gather_GBs={best['gather_bytes']/max(best['time_gather_s'],1e-9)/1e9:6.2f} "
-                      f"ondemand_ms={best['time_ondemand_s']*1e3:7.2f} chunks={best['chunks_total']}", flush=True)
+                      f"ondemand_ms={best['time_ondemand_s']*1e3:7.2f} chunks={best['chunks_total']} "
+                      f"GTEPS={best['active_arcs_total']/best['time_run_s']/1e9:.3f}", flush=True)
         asc.set_option("gather_ctas", a.gather_ctas)
         asc.set_option("chunk_cap", a.chunk_cap)
     for r in range(a.reps):
