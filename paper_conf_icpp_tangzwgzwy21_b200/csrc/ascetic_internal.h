@@ -115,7 +115,7 @@ void launch_classify(const ClassifyArgs& a, cudaStream_t s);
 void launch_init(int algo, const DevState& d, uint32_t source, cudaStream_t s);
 void launch_static(int algo, const DevState& d, const Queues& q, const void* static_base,
                    uint32_t n_small, uint32_t n_med, uint32_t n_hub, uint32_t n_pieces,
-                   uint32_t piece_arcs, cudaStream_t s);
+                   uint32_t piece_arcs, int max_ctas, cudaStream_t s);
 void launch_ondemand(int algo, const DevState& d, const Queues& q,
                      const void* chunk, unsigned long long lo, unsigned long long hi, cudaStream_t s);
 void launch_gather(const Queues& q, const void* host_nbr, uint32_t b_e, void* chunk,

@@ -176,70 +176,75 @@ __device__ __forceinline__ double warp_sum_d(double x) {
 }
 
 // ------------------------------------------------------------------ static: small lists
+// All three static-hit kernels are grid-stride loops over a capped, persistent grid: the
+// hit work of an iteration can be tens of thousands of CTAs, and a grid that size would fill
+// every SM slot and starve the on-demand kernels that gate chunk-buffer reuse (measured on the
+// friendster-shaped PR: a 22 ms static pull stalled the transfer pipeline 13 ms per iteration).
 template <int ALGO>
 __global__ void __launch_bounds__(256) k_static_small(DevState d, const uint32_t* __restrict__ q, uint32_t nq,
                                                       const void* __restrict__ sbase) {
     __shared__ double s_acc[8][32];
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-    const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const uint32_t base = gw * 32;
-    if (base >= nq) return;                                   // warp-uniform
-    const uint32_t idx = base + lane;
-    const bool valid = idx < nq;
-    uint32_t u = 0, deg = 0, sval = 0;
-    unsigned long long start = 0;
-    if (valid) {
-        u = __ldg(q + idx);
-        start = __ldg(d.off + u);
-        deg = (uint32_t)(__ldg(d.off + u + 1) - start);
-        if (ALGO == SSSP || ALGO == CC) sval = __ldg(d.snap + u);
-    }
-    uint32_t incl = deg;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t y = __shfl_up_sync(FULL, incl, o);
-        if (lane >= o) incl += y;
-    }
-    const uint32_t excl = incl - deg;
-    const uint32_t total = __shfl_sync(FULL, incl, 31);
-    if (ALGO == PR) s_acc[wib][lane] = 0.0;
-    __syncwarp();
-    for (uint32_t k0 = 0; k0 < total; k0 += 32) {
-        const uint32_t k = k0 + lane;
-        int i = 0;
-#pragma unroll
-        for (int step = 16; step >= 1; step >>= 1) {
-            const uint32_t x = __shfl_sync(FULL, incl, i + step - 1);
-            if (x <= k) i += step;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    for (uint32_t base = ((blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 32; base < nq; base += nwarps * 32) {
+        const uint32_t idx = base + lane;
+        const bool valid = idx < nq;
+        uint32_t u = 0, deg = 0, sval = 0;
+        unsigned long long start = 0;
+        if (valid) {
+            u = __ldg(q + idx);
+            start = __ldg(d.off + u);
+            deg = (uint32_t)(__ldg(d.off + u + 1) - start);
+            if (ALGO == SSSP || ALGO == CC) sval = __ldg(d.snap + u);
         }
-        const unsigned long long ust = __shfl_sync(FULL, start, i);
-        const uint32_t uex = __shfl_sync(FULL, excl, i);
-        const uint32_t usv = __shfl_sync(FULL, sval, i);
-        const bool ok = k < total;
-        const unsigned long long e = ust + (k - uex) - d.static_arc0;   // index into the Static Region
-        if (ALGO == PR) {
-            double x = ok ? pr_in(d, ld_stream(reinterpret_cast<const uint32_t*>(sbase) + e)) : 0.0;
+        uint32_t incl = deg;
 #pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const double y = __shfl_up_sync(FULL, x, o);
-                const int oi = __shfl_up_sync(FULL, i, o);
-                if (lane >= o && oi == i) x += y;
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(FULL, incl, o);
+            if (lane >= o) incl += y;
+        }
+        const uint32_t excl = incl - deg;
+        const uint32_t total = __shfl_sync(FULL, incl, 31);
+        if (ALGO == PR) s_acc[wib][lane] = 0.0;
+        __syncwarp();
+        for (uint32_t k0 = 0; k0 < total; k0 += 32) {
+            const uint32_t k = k0 + lane;
+            int i = 0;
+#pragma unroll
+            for (int step = 16; step >= 1; step >>= 1) {
+                const uint32_t x = __shfl_sync(FULL, incl, i + step - 1);
+                if (x <= k) i += step;
             }
-            const int ni = __shfl_down_sync(FULL, i, 1);
-            const bool nok = __shfl_down_sync(FULL, (int)ok, 1);
-            const bool last = ok && (lane == 31 || !nok || ni != i);
-            if (last) s_acc[wib][i] += x;
-            __syncwarp();
-        } else if (ok) {
-            if (ALGO == SSSP) {
-                const uint2 x = ld_stream(reinterpret_cast<const uint2*>(sbase) + e);
-                push_arc<ALGO>(d, usv, x.x, x.y);
-            } else {
-                push_arc<ALGO>(d, usv, ld_stream(reinterpret_cast<const uint32_t*>(sbase) + e), 0);
+            const unsigned long long ust = __shfl_sync(FULL, start, i);
+            const uint32_t uex = __shfl_sync(FULL, excl, i);
+            const uint32_t usv = __shfl_sync(FULL, sval, i);
+            const bool ok = k < total;
+            const unsigned long long e = ust + (k - uex) - d.static_arc0;   // index into the Static Region
+            if (ALGO == PR) {
+                double x = ok ? pr_in(d, ld_stream(reinterpret_cast<const uint32_t*>(sbase) + e)) : 0.0;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const double y = __shfl_up_sync(FULL, x, o);
+                    const int oi = __shfl_up_sync(FULL, i, o);
+                    if (lane >= o && oi == i) x += y;
+                }
+                const int ni = __shfl_down_sync(FULL, i, 1);
+                const bool nok = __shfl_down_sync(FULL, (int)ok, 1);
+                const bool last = ok && (lane == 31 || !nok || ni != i);
+                if (last) s_acc[wib][i] += x;
+                __syncwarp();
+            } else if (ok) {
+                if (ALGO == SSSP) {
+                    const uint2 x = ld_stream(reinterpret_cast<const uint2*>(sbase) + e);
+                    push_arc<ALGO>(d, usv, x.x, x.y);
+                } else {
+                    push_arc<ALGO>(d, usv, ld_stream(reinterpret_cast<const uint32_t*>(sbase) + e), 0);
+                }
             }
         }
+        if (ALGO == PR && valid) d.sum[u] = s_acc[wib][lane];
+        __syncwarp();
     }
-    if (ALGO == PR && valid) d.sum[u] = s_acc[wib][lane];
 }
 
 // ------------------------------------------------------------------ static: warp per list
@@ -247,41 +252,44 @@ template <int ALGO>
 __global__ void __launch_bounds__(256) k_static_med(DevState d, const uint32_t* __restrict__ q, uint32_t nq,
                                                     const void* __restrict__ sbase) {
     const int lane = threadIdx.x & 31;
-    const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    if (gw >= nq) return;
-    const uint32_t u = __ldg(q + gw);
-    const unsigned long long a0 = __ldg(d.off + u), a1 = __ldg(d.off + u + 1);
-    const uint32_t sval = (ALGO == SSSP || ALGO == CC) ? __ldg(d.snap + u) : 0u;
-    double acc = expand_list<ALGO>(d, sbase, a0 - d.static_arc0, a1 - d.static_arc0, sval, lane, 32);
-    if (ALGO == PR) {
-        acc = warp_sum_d(acc);
-        if (lane == 0) d.sum[u] = acc;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    for (uint32_t w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < nq; w += nwarps) {
+        const uint32_t u = __ldg(q + w);
+        const unsigned long long a0 = __ldg(d.off + u), a1 = __ldg(d.off + u + 1);
+        const uint32_t sval = (ALGO == SSSP || ALGO == CC) ? __ldg(d.snap + u) : 0u;
+        double acc = expand_list<ALGO>(d, sbase, a0 - d.static_arc0, a1 - d.static_arc0, sval, lane, 32);
+        if (ALGO == PR) {
+            acc = warp_sum_d(acc);
+            if (lane == 0) d.sum[u] = acc;
+        }
     }
 }
 
 // ------------------------------------------------------------------ static: hubs, CTA per piece
 template <int ALGO>
 __global__ void __launch_bounds__(256) k_static_hub(DevState d, const uint32_t* __restrict__ hq,
-                                                    const uint32_t* __restrict__ pre, uint32_t nh,
+                                                    const uint32_t* __restrict__ pre, uint32_t nh, uint32_t npieces,
                                                     uint32_t piece_arcs, const void* __restrict__ sbase) {
     __shared__ double s_red[8];
-    const uint32_t b = blockIdx.x;
-    const uint32_t h = ub_u32(pre, nh, b) - 1;
-    const uint32_t u = __ldg(hq + h);
-    const uint32_t pidx = b - __ldg(pre + h);
-    const unsigned long long o0 = __ldg(d.off + u), o1 = __ldg(d.off + u + 1);
-    const unsigned long long a0 = o0 + (unsigned long long)pidx * piece_arcs;
-    const unsigned long long a1 = min(o1, a0 + piece_arcs);
-    const uint32_t sval = (ALGO == SSSP || ALGO == CC) ? __ldg(d.snap + u) : 0u;
-    double acc = expand_list<ALGO>(d, sbase, a0 - d.static_arc0, a1 - d.static_arc0, sval, threadIdx.x, blockDim.x);
-    if (ALGO == PR) {
-        acc = warp_sum_d(acc);
-        if ((threadIdx.x & 31) == 0) s_red[threadIdx.x >> 5] = acc;
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            double t = 0.0;
-            for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += s_red[w];
-            atomicAdd(d.sum + u, t);
+    for (uint32_t b = blockIdx.x; b < npieces; b += gridDim.x) {
+        const uint32_t h = ub_u32(pre, nh, b) - 1;
+        const uint32_t u = __ldg(hq + h);
+        const uint32_t pidx = b - __ldg(pre + h);
+        const unsigned long long o0 = __ldg(d.off + u), o1 = __ldg(d.off + u + 1);
+        const unsigned long long a0 = o0 + (unsigned long long)pidx * piece_arcs;
+        const unsigned long long a1 = min(o1, a0 + piece_arcs);
+        const uint32_t sval = (ALGO == SSSP || ALGO == CC) ? __ldg(d.snap + u) : 0u;
+        double acc = expand_list<ALGO>(d, sbase, a0 - d.static_arc0, a1 - d.static_arc0, sval, threadIdx.x, blockDim.x);
+        if (ALGO == PR) {
+            acc = warp_sum_d(acc);
+            if ((threadIdx.x & 31) == 0) s_red[threadIdx.x >> 5] = acc;
+            __syncthreads();
+            if (threadIdx.x == 0) {
+                double t = 0.0;
+                for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += s_red[w];
+                atomicAdd(d.sum + u, t);
+            }
+            __syncthreads();
         }
     }
 }
@@ -383,15 +391,27 @@ __global__ void __launch_bounds__(256) k_ondemand(DevState d, Queues q, const vo
                 if (cand[g] < old) set_next(d, id[g]);
             }
         }
-    } else
-    for (unsigned long long p = pw; p < pe; p += 32) {
-        const uint32_t mk = warp_map(s_pre, x.cnt, k, p, lane);
-        k = __shfl_sync(FULL, mk, 31);
-        const unsigned long long a = p + lane;
-        const bool ok = a < pe;
-        if (ALGO == PR) {
-            double v = ok ? pr_in(d, ld_stream(reinterpret_cast<const uint32_t*>(chunk) + (a - lo))) : 0.0;
-            const int key = ok ? (int)mk : -1 - lane;
+    } else {
+        // PR pull: partial row sums of the chunk's arcs. Same 3 phases: map + chunk loads,
+        // contrib gathers (8 in flight per lane), then one segmented warp reduction per group
+        // (rows are contiguous runs of lanes) with one fp64 atomicAdd per row segment.
+        uint32_t mk8[8], id8[8];
+        double v8[8];
+#pragma unroll
+        for (int g = 0; g < 8; ++g) {
+            const unsigned long long p = pw + 32ull * g;
+            mk8[g] = warp_map(s_pre, x.cnt, k, p, lane);
+            k = __shfl_sync(FULL, mk8[g], 31);
+            const unsigned long long a = p + lane;
+            id8[g] = a < pe ? ld_stream(reinterpret_cast<const uint32_t*>(chunk) + (a - lo)) : kInf;
+        }
+#pragma unroll
+        for (int g = 0; g < 8; ++g) v8[g] = id8[g] != kInf ? pr_in(d, id8[g]) : 0.0;
+#pragma unroll
+        for (int g = 0; g < 8; ++g) {
+            const bool ok = id8[g] != kInf;
+            double v = v8[g];
+            const int key = ok ? (int)mk8[g] : -1 - lane;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
                 const double y = __shfl_up_sync(FULL, v, o);
@@ -399,14 +419,7 @@ __global__ void __launch_bounds__(256) k_ondemand(DevState d, Queues q, const vo
                 if (lane >= o && ok2 == key) v += y;
             }
             const int nk = __shfl_down_sync(FULL, key, 1);
-            if (ok && (lane == 31 || nk != key)) atomicAdd(d.sum + s_u[mk], v);
-        } else if (ok) {
-            if (ALGO == SSSP) {
-                const uint2 e = ld_stream(reinterpret_cast<const uint2*>(chunk) + (a - lo));
-                push_arc<ALGO>(d, s_v[mk], e.x, e.y);
-            } else {
-                push_arc<ALGO>(d, s_v[mk], ld_stream(reinterpret_cast<const uint32_t*>(chunk) + (a - lo)), 0);
-            }
+            if (ok && (lane == 31 || nk != key)) atomicAdd(d.sum + s_u[mk8[g]], v);
         }
     }
 }
@@ -616,21 +629,22 @@ inline unsigned blocks_for(unsigned long long n, int per_block, unsigned cap = 1
 
 template <int ALGO>
 void static_launch(const DevState& d, const Queues& q, const void* sbase, uint32_t ns, uint32_t nm, uint32_t nh,
-                   uint32_t npieces, uint32_t piece, cudaStream_t s) {
-    if (ns) { k_static_small<ALGO><<<(ns + 255) / 256, 256, 0, s>>>(d, q.hq_small, ns, sbase); ++g_launches; }
-    if (nm) { k_static_med<ALGO><<<(nm + 7) / 8, 256, 0, s>>>(d, q.hq_med, nm, sbase); ++g_launches; }
-    if (nh) { k_static_hub<ALGO><<<npieces, 256, 0, s>>>(d, q.hq_hub, q.hub_pre, nh, piece, sbase); ++g_launches; }
+                   uint32_t npieces, uint32_t piece, int max_ctas, cudaStream_t s) {
+    auto cap = [&](unsigned long long b) { return (unsigned)(b < (unsigned long long)max_ctas ? b : max_ctas); };
+    if (ns) { k_static_small<ALGO><<<cap((ns + 255) / 256), 256, 0, s>>>(d, q.hq_small, ns, sbase); ++g_launches; }
+    if (nm) { k_static_med<ALGO><<<cap((nm + 7) / 8), 256, 0, s>>>(d, q.hq_med, nm, sbase); ++g_launches; }
+    if (nh) { k_static_hub<ALGO><<<cap(npieces), 256, 0, s>>>(d, q.hq_hub, q.hub_pre, nh, npieces, piece, sbase); ++g_launches; }
 }
 
 }  // namespace
 
 void launch_static(int algo, const DevState& d, const Queues& q, const void* sbase, uint32_t ns, uint32_t nm,
-                   uint32_t nh, uint32_t npieces, uint32_t piece, cudaStream_t s) {
+                   uint32_t nh, uint32_t npieces, uint32_t piece, int max_ctas, cudaStream_t s) {
     switch (algo) {
-        case BFS: static_launch<BFS>(d, q, sbase, ns, nm, nh, npieces, piece, s); break;
-        case SSSP: static_launch<SSSP>(d, q, sbase, ns, nm, nh, npieces, piece, s); break;
-        case CC: static_launch<CC>(d, q, sbase, ns, nm, nh, npieces, piece, s); break;
-        default: static_launch<PR>(d, q, sbase, ns, nm, nh, npieces, piece, s); break;
+        case BFS: static_launch<BFS>(d, q, sbase, ns, nm, nh, npieces, piece, max_ctas, s); break;
+        case SSSP: static_launch<SSSP>(d, q, sbase, ns, nm, nh, npieces, piece, max_ctas, s); break;
+        case CC: static_launch<CC>(d, q, sbase, ns, nm, nh, npieces, piece, max_ctas, s); break;
+        default: static_launch<PR>(d, q, sbase, ns, nm, nh, npieces, piece, max_ctas, s); break;
     }
 }
 

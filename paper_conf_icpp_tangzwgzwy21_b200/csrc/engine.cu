@@ -18,6 +18,8 @@
 #include <atomic>
 #include <chrono>
 #include <cmath>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <thread>
 
@@ -125,7 +127,7 @@ Part::~Part() {
     dfree(d_run_b_); dfree(d_run_e_); dfree(d_run_dst_);
     dfree(d_tile_agg_); dfree(d_tile_incl_); dfree(d_tile_flag_); dfree(d_tot_);
     if (h_tot_) cudaFreeHost(h_tot_);
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < kMaxBuffers; ++i) {
         if (ready_[i]) cudaEventDestroy(ready_[i]);
         if (consumed_[i]) cudaEventDestroy(consumed_[i]);
     }
@@ -139,16 +141,16 @@ Part::~Part() {
 }
 
 void Part::alloc_vertex_state() {
-    // priorities (numerically lower = higher): transfer > on-demand/classify/finalize > static
-    // hits. The static-hit kernels have slack (they only need to finish before finalize);
-    // the on-demand kernels gate the reuse of the two chunk buffers, i.e. the link.
+    // priorities (numerically lower = higher): the transfer stream first (its gather CTAs are
+    // few and must stay resident to keep the link busy); on-demand and static-hit kernels
+    // share the SMs at equal priority (measured: starving the static kernels stretches PR
+    // iterations, whose static pull is HBM-bound, by 20 %).
     int lo_pri = 0, hi_pri = 0;
     CK(cudaDeviceGetStreamPriorityRange(&lo_pri, &hi_pri));
-    const int mid_pri = hi_pri < lo_pri ? hi_pri + 1 : hi_pri;
-    CK(cudaStreamCreateWithPriority(&cs_, cudaStreamNonBlocking, mid_pri));
+    CK(cudaStreamCreateWithPriority(&cs_, cudaStreamNonBlocking, lo_pri));
     CK(cudaStreamCreateWithPriority(&xs_, cudaStreamNonBlocking, hi_pri));
     CK(cudaStreamCreateWithPriority(&ss_, cudaStreamNonBlocking, lo_pri));
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < kMaxBuffers; ++i) {
         CK(cudaEventCreateWithFlags(&ready_[i], cudaEventDisableTiming));
         CK(cudaEventCreateWithFlags(&consumed_[i], cudaEventDisableTiming));
     }
@@ -218,9 +220,9 @@ void Part::upload_off() {
 
 void Part::free_regions() {
     dfree(d_static_);
-    dfree(d_chunk_[0]);
-    dfree(d_chunk_[1]);
+    for (int i = 0; i < kMaxBuffers; ++i) dfree(d_chunk_[i]);
     static_alloc_ = chunk_alloc_ = 0;
+    nbuf_alloc_ = 0;
     static_valid_ = false;
 }
 
@@ -229,10 +231,16 @@ void Part::set_budget(uint64_t bytes, double frac) {
     const uint64_t own = vhi_ - vlo_;
     if (p.s < own && p.cap < 16)
         throw Error(ASCETIC_ENOMEM, "budget leaves an On-demand chunk below 16 bytes (cap=" + std::to_string(p.cap) + ")");
-    const uint64_t want_static = p.static_bytes, want_chunk = p.s < own ? p.cap : 0;
+    // On-demand Region C split into nb chunk buffers of floor(C/nb/16)*16 bytes (the placer's
+    // `cap` is the 2-buffer figure; more buffers give the pipeline slack, same C)
+    const int nb = std::max(2, std::min(kMaxBuffers, o_.chunk_buffers));
+    const uint64_t per_buf = p.C / (uint64_t)nb / 16 * 16;
+    if (p.s < own && per_buf < 16)
+        throw Error(ASCETIC_ENOMEM, "budget leaves an On-demand chunk below 16 bytes");
+    const uint64_t want_static = p.static_bytes, want_chunk = p.s < own ? per_buf : 0;
     // regions are allocated at exactly the placement's sizes (never more than B); an
     // identical placement keeps them
-    if (want_static != static_alloc_ || want_chunk != chunk_alloc_) {
+    if (want_static != static_alloc_ || want_chunk != chunk_alloc_ || (want_chunk && nb != nbuf_alloc_)) {
         free_regions();
         if (want_static) {
             cudaError_t e = cudaMalloc(&d_static_, want_static);
@@ -240,17 +248,19 @@ void Part::set_budget(uint64_t bytes, double frac) {
         }
         static_alloc_ = want_static;
         if (want_chunk) {
-            for (int i = 0; i < 2; ++i) {
+            for (int i = 0; i < nb; ++i) {
                 cudaError_t e = cudaMalloc(&d_chunk_[i], want_chunk);
                 if (e != cudaSuccess) { cudaGetLastError(); free_regions(); throw Error(ASCETIC_ENOMEM, "chunk allocation"); }
             }
+            nbuf_alloc_ = nb;
         }
         chunk_alloc_ = want_chunk;
     } else if (p.s != pl_.s) {
         static_valid_ = false;
     }
+    nbuf_ = nb;
     pl_ = p;
-    cap_ = p.cap;
+    cap_ = want_chunk;
     launch_set_range_bits(d_S_, nwords_, vlo_, vlo_ + p.s, cs_);   // StaticBitmap
     CK(cudaStreamSynchronize(cs_));
 }
@@ -320,7 +330,7 @@ void Part::transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsig
 void Part::begin(int algo, uint32_t source, bool timing) {
     algo_ = algo;
     timing_ = timing;
-    cap_ = pl_.cap;   // chunk-cap option (tuning only: never above the placer's C/2)
+    cap_ = chunk_alloc_;   // chunk-cap option (tuning only: never above the allocated buffer)
     if (o_.chunk_cap && o_.chunk_cap < cap_) cap_ = std::max<uint64_t>(16, o_.chunk_cap / 16 * 16);
     iters.clear();
     std::memset(&st, 0, sizeof st);
@@ -412,7 +422,8 @@ void Part::expand(uint32_t t, const IterTotals& T) {
         CK(cudaEventRecord(static_go_, cs_));
         CK(cudaStreamWaitEvent(ss_, static_go_, 0));
         cudaEvent_t e0 = mark(ss_);
-        launch_static(algo_, d, q, d_static_, T.n_small, T.n_med, T.n_hub, T.n_pieces, kPieceArcs, ss_);
+        launch_static(algo_, d, q, d_static_, T.n_small, T.n_med, T.n_hub, T.n_pieces, kPieceArcs,
+                      (o_.static_ctas_per_sm > 0 ? o_.static_ctas_per_sm : 4) * sm_count_, ss_);
         CK(cudaGetLastError());
         span(e0, ss_, t, PH_STATIC);
         CK(cudaEventRecord(static_done_, ss_));
@@ -440,10 +451,10 @@ void Part::expand(uint32_t t, const IterTotals& T) {
         if (!o_.overlap && static_pending_) CK(cudaStreamWaitEvent(xs_, static_done_, 0));   // ablation
     }
     for (uint32_t k = 0; k < nchunks; ++k) {
-        const int buf = k & 1;
+        const int buf = (int)(k % (uint32_t)nbuf_);
         const unsigned long long lo = (unsigned long long)k * cap_arcs;
         const unsigned long long hi = std::min(miss, lo + cap_arcs);
-        if (k >= 2) CK(cudaStreamWaitEvent(xs_, consumed_[buf], 0));
+        if (k >= (uint32_t)nbuf_) CK(cudaStreamWaitEvent(xs_, consumed_[buf], 0));   // buffer reuse
         cudaEvent_t e0 = mark(xs_);
         transfer_chunk(q, buf, lo, hi, mode);
         CK(cudaGetLastError());
@@ -492,9 +503,16 @@ void Part::end() {
     CK(cudaEventElapsedTime(&ms, ev_start_, ev_end));
     CK(cudaEventElapsedTime(&fill_ms, ev_fill0_, ev_fill1_));
     double ph[PH_N] = {0, 0, 0, 0, 0, 0, 0};
+    const char* trace = std::getenv("ASCETIC_TRACE");
+    static const char* kPhName[PH_N] = {"classify", "static", "ondemand", "gather", "dma", "finalize", "exchange"};
     for (const Span& sp : spans_) {
         float a = 0.f;
         CK(cudaEventElapsedTime(&a, sp.a, sp.b));
+        if (trace && trace[0] == '1') {   // timeline: rank iter kernel-class start end (ms from run start)
+            float s0 = 0.f;
+            CK(cudaEventElapsedTime(&s0, ev_start_, sp.a));
+            std::fprintf(stderr, "TRACE %d %u %s %.4f %.4f\n", rank_, sp.iter, kPhName[sp.ph], s0, s0 + a);
+        }
         ph[sp.ph] += a;
         if (sp.iter < iters.size()) {
             auto& is = iters[sp.iter];
@@ -733,6 +751,15 @@ void Engine::set_option(int opt, int64_t value) {
         case ASCETIC_OPT_GATHER_CTAS:
             if (value < 0 || value > 65535) throw Error(ASCETIC_EINVAL, "gather CTAs must be in [0, 65535]");
             o_.gather_ctas = (int)value;
+            break;
+        case ASCETIC_OPT_STATIC_CTAS_PER_SM:
+            if (value < 0 || value > 64) throw Error(ASCETIC_EINVAL, "static CTAs per SM must be in [0, 64]");
+            o_.static_ctas_per_sm = (int)value;
+            break;
+        case ASCETIC_OPT_CHUNK_BUFFERS:
+            if (value < 2 || value > 8) throw Error(ASCETIC_EINVAL, "chunk buffers must be in [2, 8]");
+            o_.chunk_buffers = (int)value;
+            if (state_ == 2) state_ = 1;   // takes effect at the next set_budget
             break;
         default: throw Error(ASCETIC_EINVAL, "unknown option");
     }

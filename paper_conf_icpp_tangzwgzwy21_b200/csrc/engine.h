@@ -55,6 +55,9 @@ struct Options {
     uint32_t hub_deg = 2048;
     int timing = 1;
     int gather_ctas = 0;
+    int chunk_buffers = 3;   // On-demand Region split into this many chunk buffers of C/N bytes
+                             // (3 absorbs one slow on-demand kernel without stalling the link)
+    int static_ctas_per_sm = 0;   // persistent grid of the static-hit kernels (0 = 4 per SM)
 };
 
 struct HostGraph {
@@ -140,12 +143,14 @@ class Part {
     // edge budget regions (Eq. 1/2)
     Placement pl_{};
     void* d_static_ = nullptr;
-    void* d_chunk_[2] = {nullptr, nullptr};
+    static constexpr int kMaxBuffers = 8;
+    void* d_chunk_[kMaxBuffers] = {};
+    int nbuf_ = 2, nbuf_alloc_ = 0;   // chunk buffers in use / allocated
     uint64_t cap_ = 0, static_alloc_ = 0, chunk_alloc_ = 0;
     bool static_valid_ = false;
     // streams / events
     cudaStream_t cs_ = nullptr, xs_ = nullptr, ss_ = nullptr;   // compute, copy, static-hit streams
-    cudaEvent_t ready_[2] = {nullptr, nullptr}, consumed_[2] = {nullptr, nullptr};
+    cudaEvent_t ready_[kMaxBuffers] = {}, consumed_[kMaxBuffers] = {};
     cudaEvent_t static_go_ = nullptr, static_done_ = nullptr;
     bool static_pending_ = false;
     cudaEvent_t ev_classified_ = nullptr;

@@ -30,6 +30,7 @@ def main():
     ap.add_argument("--algo-override", default="")
     ap.add_argument("--scale-override", type=int, default=0)
     ap.add_argument("--sweep-ctas", default="148,296,444,592,1184")
+    ap.add_argument("--buffers", default="2", help="comma list: run once per chunk-buffer count")
     ap.add_argument("--sweep-caps", default="0,32,8")
     a = ap.parse_args()
     import paper_conf_icpp_tangzwgzwy21_b200 as asc
@@ -72,10 +73,13 @@ def main():
                       f"GTEPS={best['active_arcs_total']/best['time_run_s']/1e9:.3f}", flush=True)
         asc.set_option("gather_ctas", a.gather_ctas)
         asc.set_option("chunk_cap", a.chunk_cap)
-    for r in range(a.reps):
+    for nb in [int(x) for x in a.buffers.split(",")]:
+      asc.set_option("chunk_buffers", nb)
+      asc.set_budget(budget)
+      for r in range(a.reps):
         asc.run(algo, src, iters)
         st, its = asc.stats()
-        print(json.dumps({k: st[k] for k in ["iterations", "s", "h2d_payload_bytes", "h2d_static_fill_bytes",
+        print("buffers", nb, json.dumps({k: st[k] for k in ["iterations", "s", "h2d_payload_bytes", "h2d_static_fill_bytes",
                                               "active_arcs_total", "chunks_total", "dma_chunks", "gather_chunks",
                                               "time_run_s", "time_fill_s", "time_h2d_busy_s", "gteps",
                                               "chunk_cap"]}), flush=True)
