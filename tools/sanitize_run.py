@@ -1,0 +1,51 @@
+"""Small end-to-end runs of every algorithm for compute-sanitizer (memcheck / racecheck /
+synccheck): tiny chunks (many chunk windows, lists split across chunks), hub splitting,
+gather and DMA transfer modes, and 2 emulated ranks. Checks results against the oracle."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import numpy as np  # noqa: E402
+
+import graphgen as gg  # noqa: E402
+import oracle  # noqa: E402
+
+
+def main():
+    import paper_conf_icpp_tangzwgzwy21_b200 as asc
+    bad = 0
+    for world in (1, 2):
+        asc.unload()
+        asc.emulate_ranks(world)
+        for algo in ["bfs", "sssp", "cc", "pr"]:
+            g = gg.rmat(9, seed=5, weights=(algo == "sssp"))
+            src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+            it = 4 if algo == "pr" else 0
+            for xfer, cap, hub in [(1, 64, 32), (2, 0, 2048), (0, 1024, 64)]:
+                asc.unload()
+                asc.load_csr(g.off, g.nbr, pairs=g.pairs)
+                asc.set_option("xfer_mode", xfer)
+                asc.set_option("chunk_cap", cap)
+                asc.set_option("hub_degree", hub)
+                asc.set_budget(g.csr_bytes // (3 * world), 0.4)
+                asc.run(algo, src, it)
+                res = asc.get_result()
+                bounds = oracle.partition(g.off, world)
+                st = np.zeros(g.n, dtype=np.uint8)
+                for k in range(world):
+                    lo, hi = int(bounds[k]), int(bounds[k + 1])
+                    p = oracle.placer(g.off[lo:hi + 1] - g.off[lo], g.b_e, g.csr_bytes // (3 * world), 0.4)
+                    st[lo:lo + p.s] = 1
+                ref = oracle.run(algo, g.off, g.nbr, src=src, max_iters=it, is_static=st)
+                ok = (np.max(np.abs(res - ref.values) / ref.values) < 1e-5) if algo == "pr" else np.array_equal(res, ref.values)
+                bad += 0 if ok else 1
+                print(f"world={world} {algo} xfer={xfer} cap={cap} hub={hub}: {'ok' if ok else 'MISMATCH'}", flush=True)
+    asc.unload()
+    asc.emulate_ranks(1)
+    print("mismatches:", bad)
+    sys.exit(1 if bad else 0)
+
+
+if __name__ == "__main__":
+    main()
