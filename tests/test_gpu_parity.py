@@ -183,3 +183,63 @@ def test_errors_on_gpu(asc):
     with pytest.raises(asc.AsceticError) as e:
         asc.set_budget(10, 0.0)            # on-demand chunk below 16 bytes
     assert e.value.code == asc.ENOMEM
+
+
+def test_load_variants_copy_wgt_validate(asc):
+    """COPY (library-owned pinned copy), separate weight array (interleaved by the library),
+    VALIDATE, and duplicate arcs / self-loops kept in the CSR (degree counts multiplicity)."""
+    g = gg.rmat(11, seed=12, weights=True)
+    ids, w = g.ids().copy(), g.weights().copy()
+    src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+    p = oracle.placer(g.off, 8, g.csr_bytes // 3)
+    ref = _oracle("sssp", g, src, p.s)
+    for kw in [dict(copy=True), dict(validate=True)]:
+        asc.load_csr(g.off, g.nbr, pairs=True, **kw)
+        asc.set_budget(g.csr_bytes // 3)
+        asc.run("sssp", src)
+        np.testing.assert_array_equal(asc.get_result(), ref.values)
+    asc.load_csr(g.off, ids, wgt=w)                       # separate weights
+    asc.set_budget(g.csr_bytes // 3)
+    asc.run("sssp", src)
+    np.testing.assert_array_equal(asc.get_result(), ref.values)
+    st, its = asc.stats()
+    _check_records(its, ref)
+    # multigraph with self-loops: the oracle and the engine both count multiplicity
+    n = 300
+    rng = np.random.default_rng(5)
+    s_ = rng.integers(0, n, 2000).astype(np.uint32)
+    d_ = rng.integers(0, n, 2000).astype(np.uint32)
+    gm = gg.from_edges(n, s_, d_, keep_dups=True)
+    for algo in ["bfs", "cc"]:
+        st, its, res = _run(asc, gm, algo, src=0, budget=gm.csr_bytes // 2, frac=0.5, chunk_cap=64)
+        pm = oracle.placer(gm.off, 4, gm.csr_bytes // 2, 0.5)
+        refm = _oracle(algo, gm, 0, pm.s)
+        np.testing.assert_array_equal(res, refm.values)
+        _check_records(its, refm)
+
+
+@pytest.mark.parametrize("opt,val", [("overlap", 0), ("keep_static", 1), ("chunk_buffers", 2),
+                                     ("chunk_buffers", 8), ("gather_ctas", 1), ("static_ctas_per_sm", 1),
+                                     ("timing", 0)])
+def test_options_do_not_change_results(asc, opt, val):
+    """Tuning knobs change scheduling only: results, records and bytes stay bit-exact."""
+    g = gg.rmat(12, seed=14, weights=True)
+    src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+    asc.load_csr(g.off, g.nbr, pairs=True)
+    asc.set_option(opt, val)
+    asc.set_budget(g.csr_bytes // 4)
+    p = oracle.placer(g.off, 8, g.csr_bytes // 4)
+    ref = _oracle("sssp", g, src, p.s)
+    for rep in range(2):                                   # keep_static: 2nd run skips the fill
+        asc.run("sssp", src)
+        st, its = asc.stats()
+        np.testing.assert_array_equal(asc.get_result(), ref.values)
+        _check_records(its, ref)
+        assert st["h2d_payload_bytes"] == ref.h2d_payload
+        if opt == "keep_static" and rep == 1:
+            assert st["h2d_static_fill_bytes"] == 0
+        else:
+            assert st["h2d_static_fill_bytes"] == p.static_bytes
+    defaults = {"overlap": 1, "keep_static": 0, "chunk_buffers": 3, "gather_ctas": 0, "static_ctas_per_sm": 0,
+                "timing": 1}
+    asc.set_option(opt, defaults[opt])
