@@ -306,6 +306,7 @@ def main():
 
     # ---- e2e: public API with host buffers, every copy inside the step
     e2e_ms, e2e_arcs, h2d_b, d2h_b = 0.0, 0, 0, 0
+    e2e_parts = {}
     res = np.empty(g.n, dtype=np.float32 if algo == "pr" else np.uint32)
     res_pinned = torch.empty(max(1, g.n), dtype=torch.int32, pin_memory=True).numpy().view(res.dtype)[: g.n]
     for k in range(args.e2e_steps):
@@ -314,14 +315,21 @@ def main():
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record()
+        h0 = time.perf_counter()
         asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True)
+        h1 = time.perf_counter()
         asc.set_budget(budget)
         asc.set_option("xfer_mode", args.xfer)
+        h2 = time.perf_counter()
         asc.run(algo, srcs[k % len(srcs)], iters)
+        h3 = time.perf_counter()
         asc.get_result(res_pinned)
+        h4 = time.perf_counter()
         e1.record()
         torch.cuda.synchronize()
         s_ = asc.stats(per_iter=False)[0]
+        for key, v in (("load_csr", h1 - h0), ("set_budget", h2 - h1), ("run", h3 - h2), ("get_result", h4 - h3)):
+            e2e_parts[key] = e2e_parts.get(key, 0.0) + v * 1e3 / max(1, args.e2e_steps)
         e2e_ms += e0.elapsed_time(e1)
         e2e_arcs += s_["active_arcs_total"]
         h2d_b += 8 * (g.n + 1) + s_["h2d_static_fill_bytes"] + s_["h2d_payload_bytes"]
@@ -333,7 +341,8 @@ def main():
         e2e_arcs, h2d_b, d2h_b = _sum_ranks(e2e_arcs), _sum_ranks(h2d_b), _sum_ranks(d2h_b)
     e2e = {"value": e2e_arcs / (e2e_ms / 1e3) / 1e9, "unit": "GTEPS",
            "h2d_bytes_per_step": h2d_b // max(1, args.e2e_steps), "d2h_bytes_per_step": d2h_b // max(1, args.e2e_steps),
-           "steps": args.e2e_steps, "ms_per_step": e2e_ms / max(1, args.e2e_steps)}
+           "steps": args.e2e_steps, "ms_per_step": e2e_ms / max(1, args.e2e_steps),
+           "host_ms_per_call": {k: round(v, 3) for k, v in e2e_parts.items()}}
 
     # ---- CPU baseline: the oracle as it stands, bounded sample, rank 0 at N=1 only
     cpu = None

@@ -327,8 +327,11 @@ void Part::transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsig
     }
 }
 
-void Part::begin(int algo, uint32_t source, bool timing) {
+void Part::begin(int algo, uint32_t source, uint32_t max_iters, bool timing) {
     algo_ = algo;
+    max_iters_ = max_iters;
+    gchunk_ = 0;
+    prefetched_ = 0;
     timing_ = timing;
     cap_ = chunk_alloc_;   // chunk-cap option (tuning only: never above the allocated buffer)
     if (o_.chunk_cap && o_.chunk_cap < cap_) cap_ = std::max<uint64_t>(16, o_.chunk_cap / 16 * 16);
@@ -450,23 +453,56 @@ void Part::expand(uint32_t t, const IterTotals& T) {
         }
         if (!o_.overlap && static_pending_) CK(cudaStreamWaitEvent(xs_, static_done_, 0));   // ablation
     }
+    // chunks already transferred at the end of the previous iteration (PR prefetch) must be
+    // exactly this iteration's first windows
+    if (prefetched_ && (mode != 2 || miss != prefetch_miss_ || T.n_runs != prefetch_runs_))
+        throw Error(ASCETIC_ECUDA, "internal: prefetched chunks do not match the iteration's miss stream");
+    const uint64_t g0 = gchunk_;   // global chunk number of this iteration's chunk 0
     for (uint32_t k = 0; k < nchunks; ++k) {
-        const int buf = (int)(k % (uint32_t)nbuf_);
+        const uint64_t gk = g0 + k;
+        const int buf = (int)(gk % (uint64_t)nbuf_);
         const unsigned long long lo = (unsigned long long)k * cap_arcs;
         const unsigned long long hi = std::min(miss, lo + cap_arcs);
-        if (k >= (uint32_t)nbuf_) CK(cudaStreamWaitEvent(xs_, consumed_[buf], 0));   // buffer reuse
-        cudaEvent_t e0 = mark(xs_);
-        transfer_chunk(q, buf, lo, hi, mode);
-        CK(cudaGetLastError());
-        span(e0, xs_, t, mode == 2 ? PH_DMA : PH_GATHER);
+        if (k >= prefetched_) {
+            if (gk >= (uint64_t)nbuf_) CK(cudaStreamWaitEvent(xs_, consumed_[buf], 0));   // buffer reuse
+            cudaEvent_t e0 = mark(xs_);
+            transfer_chunk(q, buf, lo, hi, mode);
+            CK(cudaGetLastError());
+            span(e0, xs_, t, mode == 2 ? PH_DMA : PH_GATHER);
+            CK(cudaEventRecord(ready_[buf], xs_));
+        }
         if (mode == 2) st.dma_bytes += (hi - lo) * b_e; else st.gather_bytes += (hi - lo) * b_e;
-        CK(cudaEventRecord(ready_[buf], xs_));
+        cudaEvent_t e0 = nullptr;
         CK(cudaStreamWaitEvent(cs_, ready_[buf], 0));
         e0 = mark(cs_);
         launch_ondemand(algo_, d, q, d_chunk_[buf], lo, hi, cs_);   // On-demand Computing
         CK(cudaGetLastError());
         span(e0, cs_, t, PH_OND);
         CK(cudaEventRecord(consumed_[buf], cs_));
+    }
+    gchunk_ = g0 + nchunks;
+    prefetched_ = 0;
+    // ---- PR: A_t = V every iteration, so the next iteration's miss stream is this one and its
+    // transfer does not depend on this iteration's values. Issue the next iteration's first
+    // chunks now (each still waits for its buffer's consumer): the link keeps streaming
+    // through this iteration's tail, finalize and the next classify.
+    if (algo_ == ALG_PR && mode == 2 && nchunks && o_.prefetch && t + 1 < max_iters_) {
+        const uint32_t np = std::min<uint32_t>(nchunks, (uint32_t)nbuf_);
+        for (uint32_t k = 0; k < np; ++k) {
+            const uint64_t gk = gchunk_ + k;
+            const int buf = (int)(gk % (uint64_t)nbuf_);
+            const unsigned long long lo = (unsigned long long)k * cap_arcs;
+            const unsigned long long hi = std::min(miss, lo + cap_arcs);
+            if (gk >= (uint64_t)nbuf_) CK(cudaStreamWaitEvent(xs_, consumed_[buf], 0));
+            cudaEvent_t e0 = mark(xs_);
+            transfer_chunk(q, buf, lo, hi, mode);
+            CK(cudaGetLastError());
+            span(e0, xs_, t + 1, PH_DMA);
+            CK(cudaEventRecord(ready_[buf], xs_));
+        }
+        prefetched_ = np;
+        prefetch_miss_ = miss;
+        prefetch_runs_ = T.n_runs;
     }
     is.chunks = nchunks;
     is.mode = nchunks ? (uint32_t)mode : 0u;
@@ -752,6 +788,7 @@ void Engine::set_option(int opt, int64_t value) {
             if (value < 0 || value > 65535) throw Error(ASCETIC_EINVAL, "gather CTAs must be in [0, 65535]");
             o_.gather_ctas = (int)value;
             break;
+        case ASCETIC_OPT_PREFETCH: o_.prefetch = value ? 1 : 0; break;
         case ASCETIC_OPT_STATIC_CTAS_PER_SM:
             if (value < 0 || value > 64) throw Error(ASCETIC_EINVAL, "static CTAs per SM must be in [0, 64]");
             o_.static_ctas_per_sm = (int)value;
@@ -801,7 +838,7 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
     const bool multi = comm_.active();
     const bool timing = o_.timing != 0;
     for (auto& p : parts_) p->alloc_algo_state(algo);
-    for (auto& p : parts_) p->begin(algo, source, timing);
+    for (auto& p : parts_) p->begin(algo, source, max_iters, timing);
     Part& p0 = *parts_[0];
     std::vector<IterTotals> T(parts_.size());
     uint32_t t = 0;

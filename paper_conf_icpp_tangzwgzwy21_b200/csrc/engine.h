@@ -58,6 +58,7 @@ struct Options {
     int chunk_buffers = 3;   // On-demand Region split into this many chunk buffers of C/N bytes
                              // (3 absorbs one slow on-demand kernel without stalling the link)
     int static_ctas_per_sm = 0;   // persistent grid of the static-hit kernels (0 = 4 per SM)
+    int prefetch = 1;             // PR: issue the next iteration's first chunk transfers early
 };
 
 struct HostGraph {
@@ -84,7 +85,7 @@ class Part {
     void on_reload() { static_valid_ = false; }
 
     // one run, phase by phase
-    void begin(int algo, uint32_t source, bool timing);
+    void begin(int algo, uint32_t source, uint32_t max_iters, bool timing);
     void classify(uint32_t t);
     IterTotals wait_classify();
     void expand(uint32_t t, const IterTotals& T);
@@ -153,6 +154,11 @@ class Part {
     cudaEvent_t ready_[kMaxBuffers] = {}, consumed_[kMaxBuffers] = {};
     cudaEvent_t static_go_ = nullptr, static_done_ = nullptr;
     bool static_pending_ = false;
+    uint64_t gchunk_ = 0;            // chunks issued so far in this run (buffer = gchunk % nbuf)
+    uint32_t prefetched_ = 0;        // next iteration's chunks already issued (PR prefetch)
+    unsigned long long prefetch_miss_ = 0;
+    uint32_t prefetch_runs_ = 0;
+    uint32_t max_iters_ = 0;
     cudaEvent_t ev_classified_ = nullptr;
     EventPool pool_;
     struct Span { cudaEvent_t a, b; uint32_t iter; int ph; };

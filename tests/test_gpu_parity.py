@@ -243,3 +243,30 @@ def test_options_do_not_change_results(asc, opt, val):
     defaults = {"overlap": 1, "keep_static": 0, "chunk_buffers": 3, "gather_ctas": 0, "static_ctas_per_sm": 0,
                 "timing": 1}
     asc.set_option(opt, defaults[opt])
+
+
+@pytest.mark.parametrize("prefetch", [0, 1])
+@pytest.mark.parametrize("nbuf", [2, 3, 5])
+def test_pr_cross_iteration_prefetch(asc, prefetch, nbuf):
+    """PR with copy-engine DMA chunks and the next-iteration prefetch: many small chunks per
+    iteration so prefetched buffers wrap around; results and per-iteration bytes unchanged."""
+    g = gg.rmat(12, seed=21)
+    asc.load_csr(g.off, g.nbr)
+    asc.set_option("prefetch", prefetch)
+    asc.set_option("chunk_buffers", nbuf)
+    asc.set_option("xfer_mode", 2)
+    asc.set_option("chunk_cap", 4096)
+    asc.set_budget(g.csr_bytes // 3, 0.5)
+    asc.run("pr", 0, 9)
+    st, its = asc.stats()
+    res = asc.get_result().copy()
+    asc.set_option("prefetch", 1)
+    asc.set_option("chunk_buffers", 3)
+    asc.set_option("xfer_mode", 0)
+    asc.set_option("chunk_cap", 0)
+    p = oracle.placer(g.off, 4, g.csr_bytes // 3, 0.5)
+    ref = _oracle("pr", g, 0, p.s, max_iters=9)
+    _check_records(its, ref)
+    _pr_ok(res, ref.values)
+    assert st["dma_chunks"] == st["chunks_total"] > 9 * nbuf
+    assert st["dma_bytes"] == st["h2d_payload_bytes"] == ref.h2d_payload
