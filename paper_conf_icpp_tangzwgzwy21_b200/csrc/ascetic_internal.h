@@ -70,6 +70,8 @@ struct ClassifyArgs {
     uint32_t epoch;
     IterTotals* tot;                   // device
     IterTotals* host_tot;              // mapped pinned
+    uint32_t* host_runs;               // mapped pinned: (b, e) of the first host_runs_cap runs
+    uint32_t host_runs_cap;
 };
 
 // Device state handed to the edge / finalize kernels.

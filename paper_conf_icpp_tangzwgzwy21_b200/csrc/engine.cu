@@ -127,6 +127,7 @@ Part::~Part() {
     dfree(d_run_b_); dfree(d_run_e_); dfree(d_run_dst_);
     dfree(d_tile_agg_); dfree(d_tile_incl_); dfree(d_tile_flag_); dfree(d_tot_);
     if (h_tot_) cudaFreeHost(h_tot_);
+    if (h_runs_) cudaFreeHost(h_runs_);
     for (int i = 0; i < kMaxBuffers; ++i) {
         if (ready_[i]) cudaEventDestroy(ready_[i]);
         if (consumed_[i]) cudaEventDestroy(consumed_[i]);
@@ -187,6 +188,8 @@ void Part::alloc_vertex_state() {
     epoch_ = 0;
     cudaError_t e = cudaHostAlloc((void**)&h_tot_, sizeof(IterTotals), cudaHostAllocMapped | cudaHostAllocPortable);
     if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_EHOSTMEM, "cudaHostAlloc totals"); }
+    e = cudaHostAlloc((void**)&h_runs_, 2ull * kRunsHostMax * sizeof(uint32_t), cudaHostAllocMapped | cudaHostAllocPortable);
+    if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_EHOSTMEM, "cudaHostAlloc run list"); }
 }
 
 void Part::alloc_algo_state(int algo) {
@@ -376,6 +379,7 @@ void Part::classify(uint32_t t) {
     ca.run_b = d_run_b_; ca.run_e = d_run_e_; ca.run_dst = d_run_dst_;
     ca.tile_agg = d_tile_agg_; ca.tile_incl = d_tile_incl_; ca.tile_flag = d_tile_flag_; ca.epoch = epoch_;
     ca.tot = d_tot_; ca.host_tot = h_tot_;
+    ca.host_runs = h_runs_; ca.host_runs_cap = kRunsHostMax;
     cudaEvent_t e0 = mark(cs_);
     launch_classify(ca, cs_);
     CK(cudaGetLastError());
@@ -444,9 +448,16 @@ void Part::expand(uint32_t t, const IterTotals& T) {
         else if (o_.xfer_mode == 1) mode = 1;
         else mode = (T.n_runs <= kRunsHostMax && miss * b_e / std::max<uint32_t>(1, T.n_runs) >= o_.dma_min_run) ? 2 : 1;
         if (mode == 2) {
+            // the run list is already in mapped host memory (classify writes the first
+            // kRunsHostMax runs there): no device round trip before the DMAs can be planned
             rb_.resize(T.n_runs); re_.resize(T.n_runs); rdst_.resize(T.n_runs);
-            CK(cudaMemcpy(rb_.data(), d_run_b_, T.n_runs * 4ull, cudaMemcpyDeviceToHost));
-            CK(cudaMemcpy(re_.data(), d_run_e_, T.n_runs * 4ull, cudaMemcpyDeviceToHost));
+            const volatile uint32_t* hr = h_runs_;
+            const uint32_t nh = std::min<uint32_t>(T.n_runs, kRunsHostMax);
+            for (uint32_t r = 0; r < nh; ++r) { rb_[r] = hr[2 * r]; re_[r] = hr[2 * r + 1]; }
+            if (T.n_runs > nh) {   // forced DMA mode with a long run list: fetch the rest
+                CK(cudaMemcpy(rb_.data() + nh, d_run_b_ + nh, (T.n_runs - nh) * 4ull, cudaMemcpyDeviceToHost));
+                CK(cudaMemcpy(re_.data() + nh, d_run_e_ + nh, (T.n_runs - nh) * 4ull, cudaMemcpyDeviceToHost));
+            }
             st.d2h_bytes += T.n_runs * 8ull;
             unsigned long long acc = 0;
             for (uint32_t r = 0; r < T.n_runs; ++r) { rdst_[r] = acc; acc += g_.off[re_[r]] - g_.off[rb_[r]]; }

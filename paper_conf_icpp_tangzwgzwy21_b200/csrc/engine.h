@@ -140,6 +140,7 @@ class Part {
     uint32_t epoch_ = 0;
     IterTotals* d_tot_ = nullptr;
     IterTotals* h_tot_ = nullptr;   // mapped pinned
+    uint32_t* h_runs_ = nullptr;    // mapped pinned (b, e) pairs of the first kRunsHostMax runs
     uint64_t vertex_bytes_ = 0;
     // edge budget regions (Eq. 1/2)
     Placement pl_{};

@@ -304,10 +304,12 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
                 const uint32_t r = bR + __popc(starts & lt);
                 a.run_b[r] = (uint32_t)v;
                 a.run_dst[r] = bArcs + ex;
+                if (r < a.host_runs_cap) a.host_runs[2 * r] = (uint32_t)v;        // DMA planning copy
             }
             if ((ends >> lane) & 1u) {
                 const uint32_t r = bR + __popc(starts & le) - 1u;
                 a.run_e[r] = (uint32_t)(v + 1);
+                if (r < a.host_runs_cap) a.host_runs[2 * r + 1] = (uint32_t)(v + 1);
             }
             bQ += __popc(balQ);
             bR += __popc(starts);
@@ -327,7 +329,7 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
         if (t[3]) atomicAdd(&a.tot->active_arcs, t[3]);
         if (t[4]) atomicAdd(&a.tot->hit_arcs, t[4]);
         atomicAdd(&a.tot->digest, t[5]);                 // Σ mod 2^64
-        __threadfence();
+        __threadfence_system();   // this CTA's mapped-memory run writes before its completion count
         const uint32_t done = atomicAdd(&a.tot->done_counter, 1u);
         if (done == a.ntiles - 1) {
             __threadfence();

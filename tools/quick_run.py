@@ -30,7 +30,8 @@ def main():
     ap.add_argument("--algo-override", default="")
     ap.add_argument("--scale-override", type=int, default=0)
     ap.add_argument("--sweep-ctas", default="148,296,444,592,1184")
-    ap.add_argument("--buffers", default="2", help="comma list: run once per chunk-buffer count")
+    ap.add_argument("--buffers", default="3", help="comma list: run once per chunk-buffer count")
+    ap.add_argument("--static-ctas", default="0", help="comma list of static CTAs per SM (0 = default)")
     ap.add_argument("--sweep-caps", default="0,32,8")
     a = ap.parse_args()
     import paper_conf_icpp_tangzwgzwy21_b200 as asc
@@ -73,8 +74,10 @@ def main():
                       f"GTEPS={best['active_arcs_total']/best['time_run_s']/1e9:.3f}", flush=True)
         asc.set_option("gather_ctas", a.gather_ctas)
         asc.set_option("chunk_cap", a.chunk_cap)
-    for nb in [int(x) for x in a.buffers.split(",")]:
+    for nb, sc in [(int(x), int(y)) for x in a.buffers.split(",") for y in a.static_ctas.split(",")]:
       asc.set_option("chunk_buffers", nb)
+      asc.set_option("static_ctas_per_sm", sc)
+      print("static_ctas_per_sm", sc, end=" ")
       asc.set_budget(budget)
       for r in range(a.reps):
         asc.run(algo, src, iters)
