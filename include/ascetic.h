@@ -222,6 +222,24 @@ void ascetic_unload(void);
 /* Thread-local message of the last failing call ("" if none). */
 const char* ascetic_last_error(void);
 
+/* Test/diagnostic entry point: run ONE GenDataMap + compaction (the classify kernel) of rank
+ * `rank` (0 unless emulating ranks) on the active set given as host bitmap words (bit v%32 of
+ * word v/32, nwords = ceil(n/32)) against the current StaticBitmap (READY state), and copy its
+ * outputs to the caller's host arrays (each `cap` entries; counts are returned even when an
+ * array is too small, in which case it is left unwritten). run_dst / missq_pre are in ARCS
+ * (multiply by b_e for bytes). Overwrites the engine's active set. */
+typedef struct {
+    uint32_t *hit_small, *hit_med, *hit_hub, *hub_pre;    /* hit queues by degree bucket, ascending ids */
+    uint32_t *missq;                                      /* missed vertices with deg > 0, ascending */
+    uint64_t *missq_pre, *missq_src;                      /* exclusive miss-arc prefix; off[v] */
+    uint32_t *run_b, *run_e;                              /* maximal runs [b, e) of the missed set */
+    uint64_t *run_dst;                                    /* exclusive miss-arc prefix at each run start */
+    uint64_t cap;
+    uint64_t n_small, n_med, n_hub, n_pieces, n_missq, n_runs, miss_arcs;
+    uint64_t nA, nH, nM, active_arcs, hit_arcs, digest;
+} ascetic_classify_out_t;
+int ascetic_debug_classify(int rank, const uint32_t* active_words, uint64_t nwords, ascetic_classify_out_t* out);
+
 /* sizeof(ascetic_stats_t), sizeof(ascetic_iter_stats_t), sizeof(ascetic_placement_t) into out[0..2]
  * (lets bindings verify their struct mirrors). */
 int ascetic_struct_sizes(uint64_t* out3);

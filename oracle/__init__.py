@@ -67,6 +67,9 @@ def _load():
                                ctypes.c_void_p, ctypes.c_void_p, ctypes.POINTER(_Iter), ctypes.c_uint32,
                                ctypes.POINTER(_Summary)]
         lib.or_threads.restype = ctypes.c_int
+        lib.or_classify.argtypes = [ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p,
+                                    ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                    ctypes.c_void_p, ctypes.c_void_p]
         _lib = lib
     return _lib
 
@@ -101,6 +104,26 @@ def partition(off: np.ndarray, P: int) -> np.ndarray:
     b = np.zeros(P + 1, dtype=np.uint64)
     lib.or_partition(off.size - 1, off.ctypes.data, P, b.ctypes.data)
     return b
+
+
+def classify(off: np.ndarray, b_e: int, active: np.ndarray, is_static: np.ndarray) -> dict:
+    """StaticNodes, On-demandNodes and the on-demand request's runs + byte offsets (Fig. 4)."""
+    lib = _load()
+    off = np.ascontiguousarray(off, dtype=np.uint64)
+    n = off.size - 1
+    a = np.ascontiguousarray(active, dtype=np.uint8)
+    s = np.ascontiguousarray(is_static, dtype=np.uint8)
+    hits = np.zeros(max(n, 1), dtype=np.uint32)
+    misses = np.zeros(max(n, 1), dtype=np.uint32)
+    rb = np.zeros(max(n, 1), dtype=np.uint32)
+    re = np.zeros(max(n, 1), dtype=np.uint32)
+    rd = np.zeros(max(n, 1), dtype=np.uint64)
+    out = np.zeros(3, dtype=np.uint64)
+    lib.or_classify(n, off.ctypes.data, b_e, a.ctypes.data, s.ctypes.data, hits.ctypes.data, misses.ctypes.data,
+                    rb.ctypes.data, re.ctypes.data, rd.ctypes.data, out.ctypes.data)
+    nh, nm, nr = (int(x) for x in out)
+    return dict(hits=hits[:nh].copy(), misses=misses[:nm].copy(), run_b=rb[:nr].copy(), run_e=re[:nr].copy(),
+                run_dst=rd[:nr].copy())
 
 
 def digest(active: np.ndarray) -> int:

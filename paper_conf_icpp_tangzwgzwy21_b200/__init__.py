@@ -194,6 +194,40 @@ _lib.ascetic_partition.argtypes = [ctypes.c_uint64, ctypes.c_void_p, ctypes.c_ui
 EXPORTS += ["ascetic_emulate_ranks", "ascetic_partition"]
 
 
+class ClassifyOut(ctypes.Structure):
+    _fields_ = [(f, ctypes.c_void_p) for f in ["hit_small", "hit_med", "hit_hub", "hub_pre", "missq", "missq_pre",
+                                               "missq_src", "run_b", "run_e", "run_dst"]] + \
+               [(f, ctypes.c_uint64) for f in ["cap", "n_small", "n_med", "n_hub", "n_pieces", "n_missq", "n_runs",
+                                               "miss_arcs", "nA", "nH", "nM", "active_arcs", "hit_arcs", "digest"]]
+
+
+_lib.ascetic_debug_classify.argtypes = [ctypes.c_int, ctypes.c_void_p, ctypes.c_uint64, ctypes.POINTER(ClassifyOut)]
+EXPORTS.append("ascetic_debug_classify")
+
+
+def debug_classify(active: np.ndarray, rank: int = 0) -> dict:
+    """One classify+compaction of `active` (bool[n]) against the current StaticBitmap (test use)."""
+    a = np.ascontiguousarray(active, dtype=bool)
+    n = a.size
+    words = np.packbits(np.concatenate([a, np.zeros((-n) % 32, bool)]).reshape(-1, 32)[:, ::-1], axis=1)
+    words = np.ascontiguousarray(words[:, ::-1]).view(np.uint32).reshape(-1) if n else np.zeros(0, np.uint32)
+    cap = max(n, 1)
+    arr = {k: np.zeros(cap, dtype=np.uint32) for k in ["hit_small", "hit_med", "hit_hub", "hub_pre", "missq",
+                                                      "run_b", "run_e"]}
+    arr.update({k: np.zeros(cap, dtype=np.uint64) for k in ["missq_pre", "missq_src", "run_dst"]})
+    o = ClassifyOut()
+    for k, v in arr.items():
+        setattr(o, k, v.ctypes.data)
+    o.cap = cap
+    _check(_lib.ascetic_debug_classify(rank, words.ctypes.data if words.size else None, words.size, ctypes.byref(o)))
+    cnt = {"hit_small": o.n_small, "hit_med": o.n_med, "hit_hub": o.n_hub, "hub_pre": o.n_hub, "missq": o.n_missq,
+           "missq_pre": o.n_missq, "missq_src": o.n_missq, "run_b": o.n_runs, "run_e": o.n_runs, "run_dst": o.n_runs}
+    res = {k: v[:cnt[k]].copy() for k, v in arr.items()}
+    res.update({f: getattr(o, f) for f in ["n_pieces", "miss_arcs", "nA", "nH", "nM", "active_arcs", "hit_arcs",
+                                           "digest"]})
+    return res
+
+
 def partition(off: np.ndarray, parts: int) -> np.ndarray:
     """Host-only 1D edge-balanced rank boundaries (parts+1 entries)."""
     off = np.ascontiguousarray(off, dtype=np.uint64)

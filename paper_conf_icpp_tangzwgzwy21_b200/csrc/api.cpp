@@ -61,6 +61,10 @@ int ascetic_place(uint64_t n, const uint64_t* off, uint32_t b_e, uint64_t bytes,
     });
 }
 
+int ascetic_debug_classify(int rank, const uint32_t* active_words, uint64_t nwords, ascetic_classify_out_t* out) {
+    return guarded([&] { engine().debug_classify(rank, active_words, nwords, out); return 0; });
+}
+
 int ascetic_set_option(int option, int64_t value) {
     return guarded([&] { engine().set_option(option, value); return 0; });
 }

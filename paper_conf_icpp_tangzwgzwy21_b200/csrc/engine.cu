@@ -525,6 +525,39 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     host_s_ += std::chrono::duration<double>(std::chrono::steady_clock::now() - th0).count();
 }
 
+void Part::debug_classify(const uint32_t* active_words, uint64_t nwords, ascetic_classify_out_t* out) {
+    if (nwords != nwords_) throw Error(ASCETIC_EINVAL, "active bitmap must have ceil(n/32) words");
+    for (uint64_t w = 0; w < nwords; ++w) {   // bits beyond n must be clear
+        const uint64_t lo = w * 32;
+        if (lo + 32 > g_.n && (active_words[w] >> (g_.n - lo)) != 0 && g_.n - lo < 32)
+            throw Error(ASCETIC_EINVAL, "active bitmap has bits set beyond n");
+    }
+    CK(cudaMemcpyAsync(d_A_, active_words, nwords * 4, cudaMemcpyHostToDevice, cs_));
+    const bool timing = timing_;
+    timing_ = false;
+    classify(0);
+    timing_ = timing;
+    const IterTotals T = wait_classify();
+    CK(cudaStreamSynchronize(cs_));
+    out->n_small = T.n_small; out->n_med = T.n_med; out->n_hub = T.n_hub; out->n_pieces = T.n_pieces;
+    out->n_missq = T.n_missq; out->n_runs = T.n_runs; out->miss_arcs = T.miss_arcs;
+    out->nA = T.nA; out->nH = T.nH; out->nM = T.nM; out->active_arcs = T.active_arcs; out->hit_arcs = T.hit_arcs;
+    out->digest = T.digest;
+    auto get = [&](void* dst, const void* src, uint64_t count, size_t elem) {
+        if (dst && count && count <= out->cap) CK(cudaMemcpy(dst, src, count * elem, cudaMemcpyDeviceToHost));
+    };
+    get(out->hit_small, d_hq_small_, T.n_small, 4);
+    get(out->hit_med, d_hq_med_, T.n_med, 4);
+    get(out->hit_hub, d_hq_hub_, T.n_hub, 4);
+    get(out->hub_pre, d_hub_pre_, T.n_hub, 4);
+    get(out->missq, d_mq_, T.n_missq, 4);
+    get(out->missq_pre, d_mq_pre_, T.n_missq, 8);
+    get(out->missq_src, d_mq_src_, T.n_missq, 8);
+    get(out->run_b, d_run_b_, T.n_runs, 4);
+    get(out->run_e, d_run_e_, T.n_runs, 4);
+    get(out->run_dst, d_run_dst_, T.n_runs, 8);
+}
+
 void Part::join_static() {
     if (static_pending_) CK(cudaStreamWaitEvent(cs_, static_done_, 0));
     static_pending_ = false;
@@ -811,6 +844,15 @@ void Engine::set_option(int opt, int64_t value) {
             break;
         default: throw Error(ASCETIC_EINVAL, "unknown option");
     }
+}
+
+void Engine::debug_classify(int rank, const uint32_t* active_words, uint64_t nwords, ascetic_classify_out_t* out) {
+    if (state_ != 2) throw Error(ASCETIC_ESTATE, "debug_classify needs a loaded graph and a budget");
+    if (!active_words || !out) throw Error(ASCETIC_EINVAL, "NULL argument");
+    if (rank < 0 || rank >= (int)parts_.size()) throw Error(ASCETIC_EINVAL, "rank is not a local rank");
+    CK(cudaSetDevice(device_));
+    have_result_ = false;
+    parts_[rank]->debug_classify(active_words, nwords, out);
 }
 
 void Engine::join(std::vector<cudaStream_t>* /*unused*/) {

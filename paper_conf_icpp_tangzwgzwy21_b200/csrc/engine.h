@@ -89,6 +89,7 @@ class Part {
     void classify(uint32_t t);
     IterTotals wait_classify();
     void expand(uint32_t t, const IterTotals& T);
+    void debug_classify(const uint32_t* active_words, uint64_t nwords, ascetic_classify_out_t* out);
     void join_static();   // cs waits for this iteration's static-hit kernels
     void finalize(uint32_t t, bool dense);
     void end();
@@ -184,6 +185,7 @@ class Engine {
                   uint32_t flags);
     void set_budget(uint64_t bytes, double frac);
     void set_option(int opt, int64_t value);
+    void debug_classify(int rank, const uint32_t* active_words, uint64_t nwords, ascetic_classify_out_t* out);
     void run(int algo, uint32_t source, uint32_t max_iters);
     int stats(ascetic_stats_t* out, ascetic_iter_stats_t* per_iter, uint32_t cap) const;
     void get_result(void* dst, uint64_t bytes);

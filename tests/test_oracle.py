@@ -382,3 +382,25 @@ def test_oracle_zero_budget_r0_moves_every_reached_list_once():
     assert r.h2d_payload == 4 * int(deg[r.values != pins.INF].sum())
     r1 = oracle.run("bfs", g.off, g.nbr, src=src, is_static=np.ones(g.n, dtype=np.uint8))
     assert r1.h2d_payload == 0
+
+
+@pytest.mark.parametrize("n,p_active,p_static", [(1, 1.0, 0.0), (37, 0.5, 0.3), (1000, 0.3, 0.5), (5000, 0.9, 0.1),
+                                                 (64, 1.0, 1.0), (64, 0.0, 0.5)])
+def test_classify_vs_vectorized(n, p_active, p_static):
+    """or_classify (plain loop) vs a vectorised numpy construction of the same sets/runs/offsets."""
+    rng = np.random.default_rng(n)
+    deg = rng.integers(0, 9, n)
+    off = np.concatenate([[0], np.cumsum(deg)]).astype(np.uint64)
+    a = rng.random(n) < p_active
+    s = rng.random(n) < p_static
+    for b_e in (4, 8):
+        c = oracle.classify(off, b_e, a, s)
+        np.testing.assert_array_equal(c["hits"], np.nonzero(a & s)[0])
+        miss = a & ~s
+        np.testing.assert_array_equal(c["misses"], np.nonzero(miss)[0])
+        edges = np.diff(np.concatenate([[0], miss.astype(np.int8), [0]]))
+        np.testing.assert_array_equal(c["run_b"], np.nonzero(edges == 1)[0])
+        np.testing.assert_array_equal(c["run_e"], np.nonzero(edges == -1)[0])
+        mbytes = np.where(miss, deg * b_e, 0)
+        cum = np.concatenate([[0], np.cumsum(mbytes)])
+        np.testing.assert_array_equal(c["run_dst"], cum[c["run_b"]])
