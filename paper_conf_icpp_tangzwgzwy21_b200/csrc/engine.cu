@@ -135,6 +135,7 @@ Part::~Part() {
     if (ev_classified_) cudaEventDestroy(ev_classified_);
     if (static_go_) cudaEventDestroy(static_go_);
     if (static_done_) cudaEventDestroy(static_done_);
+    if (sync_ev_) cudaEventDestroy(sync_ev_);
     if (ss_) { cudaStreamSynchronize(ss_); cudaStreamDestroy(ss_); }
     if (cs_) cudaStreamDestroy(cs_);
     if (xs_) cudaStreamDestroy(xs_);
@@ -157,6 +158,7 @@ void Part::alloc_vertex_state() {
     }
     CK(cudaEventCreateWithFlags(&static_go_, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&static_done_, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&sync_ev_, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&ev_classified_, cudaEventDisableTiming));
     const uint64_t n = g_.n, m = g_.m;
     vertex_bytes_ = 0;
@@ -855,25 +857,21 @@ void Engine::debug_classify(int rank, const uint32_t* active_words, uint64_t nwo
     parts_[rank]->debug_classify(active_words, nwords, out);
 }
 
-void Engine::join(std::vector<cudaStream_t>* /*unused*/) {
+// emulated ranks: every part's compute stream -> part 0's (the collectives run there) and back.
+// Each part's sync event is re-recorded per use (a wait binds to the record enqueued before it).
+void Engine::join() {
     cudaStream_t c0 = parts_[0]->cs();
     for (size_t i = 1; i < parts_.size(); ++i) {
-        cudaEvent_t e;
-        CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-        CK(cudaEventRecord(e, parts_[i]->cs()));
-        CK(cudaStreamWaitEvent(c0, e, 0));
-        CK(cudaEventDestroy(e));
+        CK(cudaEventRecord(parts_[i]->sync_event(), parts_[i]->cs()));
+        CK(cudaStreamWaitEvent(c0, parts_[i]->sync_event(), 0));
     }
 }
 
 void Engine::fork() {
-    cudaStream_t c0 = parts_[0]->cs();
     if (parts_.size() < 2) return;
-    cudaEvent_t e;
-    CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-    CK(cudaEventRecord(e, c0));
+    cudaEvent_t e = parts_[0]->sync_event();
+    CK(cudaEventRecord(e, parts_[0]->cs()));
     for (size_t i = 1; i < parts_.size(); ++i) CK(cudaStreamWaitEvent(parts_[i]->cs(), e, 0));
-    CK(cudaEventDestroy(e));
 }
 
 void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
@@ -904,7 +902,7 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         if (multi && algo != ALG_PR) {
             // ---- exchange: OR of next bitmaps (BFS), MIN of values (SSSP, CC)
             for (auto& p : parts_) p->join_static();
-            join(nullptr);
+            join();
             cudaEvent_t e0 = p0.mark(p0.cs());
             const uint64_t nw = (g_.n + 31) / 32;
             if (algo == ALG_BFS) {
@@ -922,7 +920,7 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         for (auto& p : parts_) p->finalize(t, multi);
         if (multi && algo == ALG_PR) {
             // ---- exchange: SUM of the fp64 dangling partials, every rank's contrib slice to all
-            join(nullptr);
+            join();
             cudaEvent_t e0 = p0.mark(p0.cs());
             std::vector<double*> dg;
             std::vector<void*> cb;
@@ -935,13 +933,13 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         }
     }
     if (multi && algo == ALG_PR) {
-        join(nullptr);
+        join();
         std::vector<void*> rk;
         for (auto& p : parts_) rk.push_back(p->rank_arr());
         comm_.share_slices(rk, bounds_, 4, p0.cs());
         fork();
     }
-    if (parts_.size() > 1) join(nullptr);
+    if (parts_.size() > 1) join();
     for (auto& p : parts_) p->end();
     // ---- aggregate the local parts (one with NCCL; all emulated ranks otherwise)
     st_ = p0.st;

@@ -97,6 +97,7 @@ class Part {
     cudaEvent_t mark(cudaStream_t s);                               // open a timed span
 
     cudaStream_t cs() const { return cs_; }
+    cudaEvent_t sync_event() const { return sync_ev_; }
     DevState dev_state(uint32_t iter) const;
     const Placement& placement() const { return pl_; }
     uint64_t cap() const { return cap_; }
@@ -154,7 +155,7 @@ class Part {
     // streams / events
     cudaStream_t cs_ = nullptr, xs_ = nullptr, ss_ = nullptr;   // compute, copy, static-hit streams
     cudaEvent_t ready_[kMaxBuffers] = {}, consumed_[kMaxBuffers] = {};
-    cudaEvent_t static_go_ = nullptr, static_done_ = nullptr;
+    cudaEvent_t static_go_ = nullptr, static_done_ = nullptr, sync_ev_ = nullptr;
     bool static_pending_ = false;
     uint64_t gchunk_ = 0;            // chunks issued so far in this run (buffer = gchunk % nbuf)
     uint32_t prefetched_ = 0;        // next iteration's chunks already issued (PR prefetch)
@@ -192,7 +193,7 @@ class Engine {
     void unload();
 
   private:
-    void join(std::vector<cudaStream_t>* waiters);   // all local parts' cs -> parts_[0].cs
+    void join();                                      // all local parts' cs -> parts_[0].cs
     void fork();                                      // parts_[0].cs -> all local parts' cs
 
     int state_ = 0;   // 0 unloaded, 1 loaded, 2 ready
