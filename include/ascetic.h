@@ -70,8 +70,12 @@ typedef enum {
     ASCETIC_OPT_GATHER_CTAS = 8,   /* persistent CTAs of the zero-copy gather; 0 (default) = 512 / b_e (~1 MiB in flight) */
     ASCETIC_OPT_CHUNK_BUFFERS = 9, /* On-demand Region C split into N buffers of C/N (2..8, default 3); set before set_budget */
     ASCETIC_OPT_STATIC_CTAS_PER_SM = 10, /* persistent grid of the static-hit kernels, CTAs per SM (0 = default 4) */
-    ASCETIC_OPT_PREFETCH = 11      /* 1 (default): PR issues the next iteration's first chunk DMAs at the end of the
+    ASCETIC_OPT_PREFETCH = 11,     /* 1 (default): PR issues the next iteration's first chunk DMAs at the end of the
                                       current one (A_t = V, so the miss stream repeats); 0 = off */
+    ASCETIC_OPT_REPARTITION = 12   /* 1: Eq. 3 adaptive re-partition (§3.3) after each data map:
+                                      if V_ondemand > C and V_static/M_static < 0.5 V/D, shrink the Static Region
+                                      by M_static*V/D (floored to 16 KiB) and re-generate the map. Default 0, as
+                                      in the paper's evaluation. Changes per-iteration bytes. */
 } ascetic_option;
 
 typedef struct {
@@ -113,6 +117,7 @@ typedef struct {
     uint64_t dma_bytes;
     double time_finalize_s;
     double time_host_s;           /* host planning + waits between classify and the next launches */
+    uint64_t repartitions;        /* Eq. 3 re-partitions performed (ASCETIC_OPT_REPARTITION) */
 } ascetic_stats_t;
 
 typedef struct {
@@ -129,6 +134,7 @@ typedef struct {
     /* host-link idle inside the iteration: before its first chunk transfer, between its
      * chunk transfers, and after its last one (until the next iteration's classify) */
     float ms_link_head, ms_link_gaps, ms_link_tail;
+    uint64_t s_static;            /* static vertices of this rank in this iteration (front prefix length) */
 } ascetic_iter_stats_t;
 
 /*

@@ -34,7 +34,7 @@ class _Iter(ctypes.Structure):
     _fields_ = [("t", ctypes.c_uint32), ("rank", ctypes.c_uint32), ("nA", ctypes.c_uint64),
                 ("nH", ctypes.c_uint64), ("nM", ctypes.c_uint64), ("nruns", ctypes.c_uint64),
                 ("active_arcs", ctypes.c_uint64), ("hit_arcs", ctypes.c_uint64),
-                ("miss_bytes", ctypes.c_uint64), ("digest", ctypes.c_uint64)]
+                ("miss_bytes", ctypes.c_uint64), ("digest", ctypes.c_uint64), ("s", ctypes.c_uint64)]
 
 
 class _Summary(ctypes.Structure):
@@ -42,7 +42,7 @@ class _Summary(ctypes.Structure):
                 ("h2d_payload", ctypes.c_uint64), ("active_arcs_total", ctypes.c_uint64)]
 
 
-ITER_FIELDS = ["t", "rank", "nA", "nH", "nM", "nruns", "active_arcs", "hit_arcs", "miss_bytes", "digest"]
+ITER_FIELDS = ["t", "rank", "nA", "nH", "nM", "nruns", "active_arcs", "hit_arcs", "miss_bytes", "digest", "s"]
 
 
 def build(force: bool = False) -> str:
@@ -62,10 +62,11 @@ def _load():
         lib.or_partition.argtypes = [ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p]
         lib.or_digest.restype = ctypes.c_uint64
         lib.or_digest.argtypes = [ctypes.c_uint64, ctypes.c_void_p]
-        lib.or_run.argtypes = [ctypes.c_int, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint32,
-                               ctypes.c_uint32, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p,
-                               ctypes.c_void_p, ctypes.c_void_p, ctypes.POINTER(_Iter), ctypes.c_uint32,
-                               ctypes.POINTER(_Summary)]
+        lib.or_run_ex.argtypes = [ctypes.c_int, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint32,
+                                  ctypes.c_uint32, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p,
+                                  ctypes.c_void_p, ctypes.c_void_p, ctypes.POINTER(_Iter), ctypes.c_uint32,
+                                  ctypes.POINTER(_Summary), ctypes.c_int, ctypes.c_uint64, ctypes.c_uint64,
+                                  ctypes.POINTER(ctypes.c_uint64)]
         lib.or_threads.restype = ctypes.c_int
         lib.or_classify.argtypes = [ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p,
                                     ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
@@ -138,6 +139,7 @@ class Result:
     records: list[dict]
     h2d_payload: int
     active_arcs_total: int
+    repartitions: int = 0
 
 
 def static_prefix(n: int, s: int) -> np.ndarray:
@@ -147,8 +149,11 @@ def static_prefix(n: int, s: int) -> np.ndarray:
 
 
 def run(algo: str | int, off: np.ndarray, nbr: np.ndarray, src: int = 0, max_iters: int = 0,
-        is_static: np.ndarray | None = None, bounds: np.ndarray | None = None) -> Result:
-    """Run the oracle. nbr = ids (bfs/cc/pr) or interleaved (id,w) pairs (sssp)."""
+        is_static: np.ndarray | None = None, bounds: np.ndarray | None = None,
+        eq3_budget: int = 0, eq3_ms: int = 0) -> Result:
+    """Run the oracle. nbr = ids (bfs/cc/pr) or interleaved (id,w) pairs (sssp).
+    eq3_budget > 0 applies the Eq. 3 re-partition (one rank; is_static = the front prefix placed
+    in eq3_ms bytes of the budget)."""
     lib = _load()
     a = ALGOS[algo] if isinstance(algo, str) else algo
     off = np.ascontiguousarray(off, dtype=np.uint64)
@@ -162,11 +167,14 @@ def run(algo: str | int, off: np.ndarray, nbr: np.ndarray, src: int = 0, max_ite
     cap = (min(n + 2, 1 << 16) if a != PR else max(1, max_iters)) * P
     recs = (_Iter * cap)()
     s = _Summary()
-    rc = lib.or_run(a, n, off.ctypes.data, nbr.ctypes.data if nbr.size else None, src, max_iters,
-                    st.ctypes.data if n else None, P, b.ctypes.data if b is not None else None,
-                    res_u.ctypes.data if n else None, res_f.ctypes.data if n else None, recs, cap, ctypes.byref(s))
+    reparts = ctypes.c_uint64(0)
+    rc = lib.or_run_ex(a, n, off.ctypes.data, nbr.ctypes.data if nbr.size else None, src, max_iters,
+                       st.ctypes.data if n else None, P, b.ctypes.data if b is not None else None,
+                       res_u.ctypes.data if n else None, res_f.ctypes.data if n else None, recs, cap, ctypes.byref(s),
+                       1 if eq3_budget > 0 else 0, eq3_budget, eq3_ms, ctypes.byref(reparts))
     if rc != 0:
         raise ValueError(f"oracle rejected arguments (rc={rc})")
     records = [{f: int(getattr(recs[i], f)) for f in ITER_FIELDS} for i in range(s.nrec)]
     vals = res_f.copy() if a == PR else res_u.copy()
-    return Result(vals, int(s.iterations), records, int(s.h2d_payload), int(s.active_arcs_total))
+    return Result(vals, int(s.iterations), records, int(s.h2d_payload), int(s.active_arcs_total),
+                  int(reparts.value))

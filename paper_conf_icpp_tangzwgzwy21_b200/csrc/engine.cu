@@ -224,11 +224,25 @@ void Part::upload_off() {
 }
 
 void Part::free_regions() {
-    dfree(d_static_);
-    for (int i = 0; i < kMaxBuffers; ++i) dfree(d_chunk_[i]);
+    dfree(arena_);
+    arena_bytes_ = 0;
+    d_static_ = nullptr;
+    for (int i = 0; i < kMaxBuffers; ++i) d_chunk_[i] = nullptr;
     static_alloc_ = chunk_alloc_ = 0;
     nbuf_alloc_ = 0;
     static_valid_ = false;
+}
+
+// The edge budget is ONE arena of at most B bytes: the Static Region is its front
+// [0, static_bytes) ⊆ [0, Ms), the On-demand Region [Ms, arena) is cut into nbuf_ chunk buffers.
+// Moving Ms (Eq. 3 re-partition) keeps the static prefix in place and re-cuts the rest.
+void Part::layout_regions(uint64_t Ms) {
+    d_static_ = arena_;
+    const uint64_t per = arena_bytes_ > Ms ? (arena_bytes_ - Ms) / (uint64_t)nbuf_ / 16 * 16 : 0;
+    for (int i = 0; i < kMaxBuffers; ++i) d_chunk_[i] = (per && i < nbuf_) ? arena_ + Ms + (uint64_t)i * per : nullptr;
+    chunk_alloc_ = per;
+    cap_ = per;   // chunk-cap option (tuning only): never above the buffer
+    if (o_.chunk_cap && o_.chunk_cap < cap_) cap_ = std::max<uint64_t>(16, o_.chunk_cap / 16 * 16);
 }
 
 void Part::set_budget(uint64_t bytes, double frac) {
@@ -239,35 +253,56 @@ void Part::set_budget(uint64_t bytes, double frac) {
     // On-demand Region C split into nb chunk buffers of floor(C/nb/16)*16 bytes (the placer's
     // `cap` is the 2-buffer figure; more buffers give the pipeline slack, same C)
     const int nb = std::max(2, std::min(kMaxBuffers, o_.chunk_buffers));
-    const uint64_t per_buf = p.C / (uint64_t)nb / 16 * 16;
+    // chunk buffers never need more than the rank's whole payload D
+    const uint64_t per_buf = std::min<uint64_t>(p.C / (uint64_t)nb, std::max<uint64_t>(p.D, 16)) / 16 * 16;
     if (p.s < own && per_buf < 16)
         throw Error(ASCETIC_ENOMEM, "budget leaves an On-demand chunk below 16 bytes");
-    const uint64_t want_static = p.static_bytes, want_chunk = p.s < own ? per_buf : 0;
-    // regions are allocated at exactly the placement's sizes (never more than B); an
-    // identical placement keeps them
-    if (want_static != static_alloc_ || want_chunk != chunk_alloc_ || (want_chunk && nb != nbuf_alloc_)) {
+    // arena = Ms + nb chunk buffers (<= B); just the static prefix when everything is static
+    const uint64_t want = std::max<uint64_t>(16, p.s < own ? p.Ms + (uint64_t)nb * per_buf : p.static_bytes);
+    if (want != arena_bytes_ || nb != nbuf_alloc_) {
         free_regions();
-        if (want_static) {
-            cudaError_t e = cudaMalloc(&d_static_, want_static);
-            if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_ENOMEM, "static region allocation"); }
-        }
-        static_alloc_ = want_static;
-        if (want_chunk) {
-            for (int i = 0; i < nb; ++i) {
-                cudaError_t e = cudaMalloc(&d_chunk_[i], want_chunk);
-                if (e != cudaSuccess) { cudaGetLastError(); free_regions(); throw Error(ASCETIC_ENOMEM, "chunk allocation"); }
-            }
-            nbuf_alloc_ = nb;
-        }
-        chunk_alloc_ = want_chunk;
+        cudaError_t e = cudaMalloc((void**)&arena_, want);
+        if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_ENOMEM, "edge-budget arena allocation"); }
+        arena_bytes_ = want;
+        nbuf_alloc_ = nb;
     } else if (p.s != pl_.s) {
         static_valid_ = false;
     }
+    static_alloc_ = p.static_bytes;
     nbuf_ = nb;
     pl_ = p;
-    cap_ = want_chunk;
+    ms_cur_ = p.Ms;
+    s_cur_ = p.s;
+    layout_regions(p.Ms);
     launch_set_range_bits(d_S_, nwords_, vlo_, vlo_ + p.s, cs_);   // StaticBitmap
     CK(cudaStreamSynchronize(cs_));
+}
+
+// Eq. 3 (§3.3): after the data map of an iteration is generated, if the on-demand
+// data exceed the On-demand Region and the Static Region is under-used (V_static / M_static <
+// 0.5 V / D), shrink the Static Region by M_static * V / D (floored to 16 KiB) and
+// hand that memory to the On-demand Region; the caller re-generates the data map.
+bool Part::maybe_repartition(const IterTotals& T) {
+    if (ms_cur_ == 0 || pl_.D == 0) return false;
+    const double b_e = g_.b_e;
+    const double V = b_e * (double)T.active_arcs, Vs = b_e * (double)T.hit_arcs, Vo = b_e * (double)T.miss_arcs;
+    const double D = (double)pl_.D, Ms = (double)ms_cur_;
+    const double C = (double)(pl_.B > ms_cur_ ? pl_.B - ms_cur_ : 0);
+    if (!(Vo > C && Vs / Ms < 0.5 * V / D)) return false;
+    const uint64_t delta = (uint64_t)std::floor(Ms * V / D);
+    const uint64_t ms_new = (ms_cur_ - std::min(delta, ms_cur_)) / 16384ull * 16384ull;
+    if (ms_new >= ms_cur_) return false;
+    const uint64_t* off = g_.off.data() + vlo_;
+    const uint64_t lim = off[0] + ms_new / g_.b_e;
+    const uint64_t s_new = (uint64_t)(std::upper_bound(off, off + (vhi_ - vlo_) + 1, lim) - off) - 1;
+    CK(cudaStreamSynchronize(xs_));   // no transfer may still target the old chunk layout
+    static_valid_ = false;            // chunk buffers now overlay the old static tail
+    ms_cur_ = ms_new;
+    s_cur_ = s_new;
+    layout_regions(ms_new);
+    launch_set_range_bits(d_S_, nwords_, vlo_, vlo_ + s_new, cs_);
+    st.repartitions += 1;
+    return true;
 }
 
 DevState Part::dev_state(uint32_t iter) const {
@@ -338,8 +373,13 @@ void Part::begin(int algo, uint32_t source, uint32_t max_iters, bool timing) {
     gchunk_ = 0;
     prefetched_ = 0;
     timing_ = timing;
-    cap_ = chunk_alloc_;   // chunk-cap option (tuning only: never above the allocated buffer)
-    if (o_.chunk_cap && o_.chunk_cap < cap_) cap_ = std::max<uint64_t>(16, o_.chunk_cap / 16 * 16);
+    // every run starts from the placer's split (an Eq. 3 shrink lasts for the run it happened in)
+    if (ms_cur_ != pl_.Ms || s_cur_ != pl_.s) {
+        ms_cur_ = pl_.Ms;
+        s_cur_ = pl_.s;
+        launch_set_range_bits(d_S_, nwords_, vlo_, vlo_ + pl_.s, cs_);
+    }
+    layout_regions(ms_cur_);
     iters.clear();
     std::memset(&st, 0, sizeof st);
     pool_.reset();
@@ -418,6 +458,7 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     is.nA = T.nA; is.nH = T.nH; is.nM = T.nM; is.nruns = T.n_runs;
     is.active_arcs = T.active_arcs; is.hit_arcs = T.hit_arcs; is.miss_bytes = T.miss_arcs * b_e;
     is.digest = T.digest;
+    is.s_static = s_cur_;
     const DevState d = dev_state(t);
     const Queues q = queues(T);
     if (algo_ == ALG_PR) CK(cudaMemsetAsync(d_sum_ + vlo_, 0, (vhi_ - vlo_) * sizeof(double), cs_));
@@ -499,7 +540,7 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     // transfer does not depend on this iteration's values. Issue the next iteration's first
     // chunks now (each still waits for its buffer's consumer): the link keeps streaming
     // through this iteration's tail, finalize and the next classify.
-    if (algo_ == ALG_PR && mode == 2 && nchunks && o_.prefetch && t + 1 < max_iters_) {
+    if (algo_ == ALG_PR && mode == 2 && nchunks && o_.prefetch && !o_.repartition && t + 1 < max_iters_) {
         const uint32_t np = std::min<uint32_t>(nchunks, (uint32_t)nbuf_);
         for (uint32_t k = 0; k < np; ++k) {
             const uint64_t gk = gchunk_ + k;
@@ -835,6 +876,7 @@ void Engine::set_option(int opt, int64_t value) {
             o_.gather_ctas = (int)value;
             break;
         case ASCETIC_OPT_PREFETCH: o_.prefetch = value ? 1 : 0; break;
+        case ASCETIC_OPT_REPARTITION: o_.repartition = value ? 1 : 0; break;
         case ASCETIC_OPT_STATIC_CTAS_PER_SM:
             if (value < 0 || value > 64) throw Error(ASCETIC_EINVAL, "static CTAs per SM must be in [0, 64]");
             o_.static_ctas_per_sm = (int)value;
@@ -898,6 +940,14 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         for (auto& p : parts_) p->classify(t);
         for (size_t i = 0; i < parts_.size(); ++i) T[i] = parts_[i]->wait_classify();
         if (T[0].nA == 0) break;   // |A_t| is counted over the replicated bitmap: identical on every rank
+        if (o_.repartition) {      // Eq. 3, then re-generate the data map
+            for (size_t i = 0; i < parts_.size(); ++i) {
+                if (parts_[i]->maybe_repartition(T[i])) {
+                    parts_[i]->classify(t);
+                    T[i] = parts_[i]->wait_classify();
+                }
+            }
+        }
         for (size_t i = 0; i < parts_.size(); ++i) parts_[i]->expand(t, T[i]);
         if (multi && algo != ALG_PR) {
             // ---- exchange: OR of next bitmaps (BFS), MIN of values (SSSP, CC)
@@ -963,6 +1013,7 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         st_.dma_bytes += s.dma_bytes;
         st_.static_bytes += s.static_bytes;
         st_.vertex_state_bytes += s.vertex_state_bytes;
+        st_.repartitions += s.repartitions;
         st_.kernel_launches = std::max(st_.kernel_launches, s.kernel_launches);
     }
     st_.iterations = t;

@@ -59,6 +59,7 @@ struct Options {
                              // (3 absorbs one slow on-demand kernel without stalling the link)
     int static_ctas_per_sm = 0;   // persistent grid of the static-hit kernels (0 = 4 per SM)
     int prefetch = 1;             // PR: issue the next iteration's first chunk transfers early
+    int repartition = 0;          // Eq. 3 adaptive re-partition (off, as in the paper's evaluation)
 };
 
 struct HostGraph {
@@ -90,6 +91,7 @@ class Part {
     IterTotals wait_classify();
     void expand(uint32_t t, const IterTotals& T);
     void debug_classify(const uint32_t* active_words, uint64_t nwords, ascetic_classify_out_t* out);
+    bool maybe_repartition(const IterTotals& T);   // Eq. 3; true = re-generate the data map
     void join_static();   // cs waits for this iteration's static-hit kernels
     void finalize(uint32_t t, bool dense);
     void end();
@@ -118,6 +120,7 @@ class Part {
     void transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsigned long long hi, int mode);
     Queues queues(const IterTotals& T) const;
     void free_regions();
+    void layout_regions(uint64_t Ms);
 
     const HostGraph& g_;
     const Options& o_;
@@ -146,9 +149,12 @@ class Part {
     uint64_t vertex_bytes_ = 0;
     // edge budget regions (Eq. 1/2)
     Placement pl_{};
+    char* arena_ = nullptr;          // the edge budget: Static Region + On-demand Region
+    uint64_t arena_bytes_ = 0;
+    uint64_t ms_cur_ = 0, s_cur_ = 0; // current split (Eq. 3 may shrink it during a run)
     void* d_static_ = nullptr;
     static constexpr int kMaxBuffers = 8;
-    void* d_chunk_[kMaxBuffers] = {};
+    char* d_chunk_[kMaxBuffers] = {};
     int nbuf_ = 2, nbuf_alloc_ = 0;   // chunk buffers in use / allocated
     uint64_t cap_ = 0, static_alloc_ = 0, chunk_alloc_ = 0;
     bool static_valid_ = false;

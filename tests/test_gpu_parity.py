@@ -270,3 +270,34 @@ def test_pr_cross_iteration_prefetch(asc, prefetch, nbuf):
     _pr_ok(res, ref.values)
     assert st["dma_chunks"] == st["chunks_total"] > 9 * nbuf
     assert st["dma_bytes"] == st["h2d_payload_bytes"] == ref.h2d_payload
+
+
+@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc"])
+def test_eq3_repartition_parity(asc, algo):
+    """Eq. 3 adaptive re-partition (ASCETIC_OPT_REPARTITION): the shrink decisions, the static
+    prefix per iteration, every record and the results match the oracle's Eq. 3."""
+    from tests.test_oracle import two_communities
+    g = two_communities()
+    if algo == "sssp":
+        s_, d_ = np.repeat(np.arange(g.n), np.diff(g.off.astype(np.int64))).astype(np.uint32), g.nbr
+        g = gg.from_edges(g.n, s_, d_, weights=True)
+    budget = g.csr_bytes // 2
+    asc.load_csr(g.off, g.nbr, pairs=g.pairs)
+    asc.set_option("repartition", 1)
+    asc.set_budget(budget)
+    src = 900
+    for rep in range(2):                                   # the split resets for every run
+        asc.run(algo, src)
+        st, its = asc.stats()
+        res = asc.get_result().copy()
+        p = oracle.placer(g.off, g.b_e, budget)
+        ref = oracle.run(algo, g.off, g.nbr, src=src, is_static=oracle.static_prefix(g.n, p.s),
+                         eq3_budget=budget, eq3_ms=p.Ms)
+        np.testing.assert_array_equal(res, ref.values)
+        _check_records(its, ref)
+        assert [i["s_static"] for i in its] == [r["s"] for r in ref.records]
+        assert st["repartitions"] == ref.repartitions
+        assert st["h2d_payload_bytes"] == ref.h2d_payload
+    if algo == "bfs":
+        assert ref.repartitions >= 1
+    asc.set_option("repartition", 0)

@@ -384,6 +384,48 @@ def test_oracle_zero_budget_r0_moves_every_reached_list_once():
     assert r1.h2d_payload == 0
 
 
+def two_communities(half=600, seed=3):
+    """Two random communities [0, half) and [half, 2 half) joined by one bridge: a BFS from the
+    second one keeps its early frontiers out of the static front prefix (Eq. 3 fires)."""
+    rng = np.random.default_rng(seed)
+    a = rng.integers(0, half, (4 * half, 2))
+    b = rng.integers(half, 2 * half, (4 * half, 2))
+    e = np.concatenate([a, b, [[half - 1, half]]]).astype(np.uint32)
+    return gg.from_edges(2 * half, e[:, 0], e[:, 1])
+
+
+def test_eq3_repartition_vs_restatement():
+    """Eq. 3 restated over scipy BFS level sets: when V_ondemand > C and
+    V_static/M_static < 0.5 V/D, M_static -= M_static V/D (16 KiB floor), prefix recomputed."""
+    g = two_communities()
+    deg = np.diff(g.off.astype(np.int64))
+    A = sp.csr_matrix((np.ones(g.m), g.nbr.astype(np.int64), g.off.astype(np.int64)), shape=(g.n, g.n))
+    src = 900
+    lev = csgraph.shortest_path(A, unweighted=True, indices=src)
+    L = int(lev[np.isfinite(lev)].max())
+    budget = g.csr_bytes // 2
+    p = oracle.placer(g.off, 4, budget)
+    D = 4.0 * g.m
+    Ms, s = p.Ms, p.s
+    recs = []
+    for t in range(L + 1):
+        act = lev == t
+        V, Vs, Vo = 4.0 * deg[act].sum(), 4.0 * deg[act & (np.arange(g.n) < s)].sum(), 4.0 * deg[act & (np.arange(g.n) >= s)].sum()
+        if Ms > 0 and Vo > budget - Ms and Vs / Ms < 0.5 * V / D:
+            new = (Ms - min(int(np.floor(Ms * V / D)), Ms)) // 16384 * 16384
+            if new < Ms:
+                Ms = new
+                s = int(np.searchsorted(4 * g.off.astype(np.int64), Ms, side="right")) - 1
+        recs.append(pins.records_from_sets([act], g.off, 4, s)[0] | {"t": t})
+    got = oracle.run("bfs", g.off, g.nbr, src=src, is_static=oracle.static_prefix(g.n, p.s),
+                     eq3_budget=budget, eq3_ms=p.Ms)
+    assert got.repartitions >= 1
+    assert got.records == recs
+    plain = oracle.run("bfs", g.off, g.nbr, src=src, is_static=oracle.static_prefix(g.n, p.s))
+    np.testing.assert_array_equal(got.values, plain.values)        # Eq. 3 moves bytes, never results
+    assert got.h2d_payload != plain.h2d_payload
+
+
 @pytest.mark.parametrize("n,p_active,p_static", [(1, 1.0, 0.0), (37, 0.5, 0.3), (1000, 0.3, 0.5), (5000, 0.9, 0.1),
                                                  (64, 1.0, 1.0), (64, 0.0, 0.5)])
 def test_classify_vs_vectorized(n, p_active, p_static):
