@@ -72,10 +72,12 @@ typedef enum {
     ASCETIC_OPT_STATIC_CTAS_PER_SM = 10, /* persistent grid of the static-hit kernels, CTAs per SM (0 = default 4) */
     ASCETIC_OPT_PREFETCH = 11,     /* 1 (default): PR issues the next iteration's first chunk DMAs at the end of the
                                       current one (A_t = V, so the miss stream repeats); 0 = off */
-    ASCETIC_OPT_REPARTITION = 12   /* 1: Eq. 3 adaptive re-partition (§3.3) after each data map:
+    ASCETIC_OPT_REPARTITION = 12,  /* 1: Eq. 3 adaptive re-partition (§3.3) after each data map:
                                       if V_ondemand > C and V_static/M_static < 0.5 V/D, shrink the Static Region
                                       by M_static*V/D (floored to 16 KiB) and re-generate the map. Default 0, as
                                       in the paper's evaluation. Changes per-iteration bytes. */
+    ASCETIC_OPT_STATIC_PLACEMENT = 13 /* initial static content (§5): 0 = front prefix (default),
+                                      1 = rear suffix of whole lists fitting in Ms. Set before set_budget. */
 } ascetic_option;
 
 typedef struct {

@@ -99,6 +99,21 @@ def placer(off: np.ndarray, b_e: int, budget: int, frac: float = -1.0) -> Placem
     return Placement(p.R, p.D, p.B, p.Ms, p.s, p.static_bytes, p.C, p.cap)
 
 
+def rear_start(off: np.ndarray, b_e: int, Ms: int) -> int:
+    """First vertex of the rear (suffix) static set placed in Ms bytes."""
+    lib = _load()
+    lib.or_rear_start.restype = ctypes.c_uint64
+    lib.or_rear_start.argtypes = [ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64]
+    off = np.ascontiguousarray(off, dtype=np.uint64)
+    return int(lib.or_rear_start(off.size - 1, off.ctypes.data, b_e, Ms))
+
+
+def static_rear(n: int, s_lo: int) -> np.ndarray:
+    st = np.zeros(n, dtype=np.uint8)
+    st[s_lo:] = 1
+    return st
+
+
 def partition(off: np.ndarray, P: int) -> np.ndarray:
     lib = _load()
     off = np.ascontiguousarray(off, dtype=np.uint64)

@@ -246,8 +246,18 @@ void Part::layout_regions(uint64_t Ms) {
 }
 
 void Part::set_budget(uint64_t bytes, double frac) {
-    const Placement p = place(g_.off.data() + vlo_, vhi_ - vlo_, g_.b_e, bytes, frac);
+    Placement p = place(g_.off.data() + vlo_, vhi_ - vlo_, g_.b_e, bytes, frac);
     const uint64_t own = vhi_ - vlo_;
+    stat_lo_ = vlo_;
+    if (o_.static_rear) {
+        // rear initial content (§5): the suffix of whole lists that fits in Ms,
+        // s_lo = min{v : b_e (off[vhi] - off[v]) <= Ms}
+        const uint64_t* off = g_.off.data();
+        const uint64_t lim = off[vhi_] - std::min<uint64_t>(p.Ms / g_.b_e, off[vhi_]);
+        stat_lo_ = (uint64_t)(std::lower_bound(off + vlo_, off + vhi_ + 1, lim) - off);
+        p.s = vhi_ - stat_lo_;
+        p.static_bytes = (uint64_t)g_.b_e * (off[vhi_] - off[stat_lo_]);
+    }
     if (p.s < own && p.cap < 16)
         throw Error(ASCETIC_ENOMEM, "budget leaves an On-demand chunk below 16 bytes (cap=" + std::to_string(p.cap) + ")");
     // On-demand Region C split into nb chunk buffers of floor(C/nb/16)*16 bytes (the placer's
@@ -274,7 +284,7 @@ void Part::set_budget(uint64_t bytes, double frac) {
     ms_cur_ = p.Ms;
     s_cur_ = p.s;
     layout_regions(p.Ms);
-    launch_set_range_bits(d_S_, nwords_, vlo_, vlo_ + p.s, cs_);   // StaticBitmap
+    launch_set_range_bits(d_S_, nwords_, stat_lo_, stat_lo_ + p.s, cs_);   // StaticBitmap
     CK(cudaStreamSynchronize(cs_));
 }
 
@@ -283,7 +293,7 @@ void Part::set_budget(uint64_t bytes, double frac) {
 // 0.5 V / D), shrink the Static Region by M_static * V / D (floored to 16 KiB) and
 // hand that memory to the On-demand Region; the caller re-generates the data map.
 bool Part::maybe_repartition(const IterTotals& T) {
-    if (ms_cur_ == 0 || pl_.D == 0) return false;
+    if (ms_cur_ == 0 || pl_.D == 0 || o_.static_rear) return false;   // Eq. 3 shrinks a front prefix
     const double b_e = g_.b_e;
     const double V = b_e * (double)T.active_arcs, Vs = b_e * (double)T.hit_arcs, Vo = b_e * (double)T.miss_arcs;
     const double D = (double)pl_.D, Ms = (double)ms_cur_;
@@ -313,7 +323,7 @@ DevState Part::dev_state(uint32_t iter) const {
     d.rank = d_rank_; d.contrib = d_contrib_; d.sum = d_sum_; d.dang = d_dang_;
     d.iter = iter;
     d.vlo = vlo_; d.vhi = vhi_;
-    d.static_arc0 = g_.off.empty() ? 0 : g_.off[vlo_];
+    d.static_arc0 = g_.off.empty() ? 0 : g_.off[stat_lo_];
     return d;
 }
 
@@ -377,7 +387,7 @@ void Part::begin(int algo, uint32_t source, uint32_t max_iters, bool timing) {
     if (ms_cur_ != pl_.Ms || s_cur_ != pl_.s) {
         ms_cur_ = pl_.Ms;
         s_cur_ = pl_.s;
-        launch_set_range_bits(d_S_, nwords_, vlo_, vlo_ + pl_.s, cs_);
+        launch_set_range_bits(d_S_, nwords_, stat_lo_, stat_lo_ + pl_.s, cs_);
     }
     layout_regions(ms_cur_);
     iters.clear();
@@ -392,7 +402,7 @@ void Part::begin(int algo, uint32_t source, uint32_t max_iters, bool timing) {
     CK(cudaStreamWaitEvent(xs_, ev_start_, 0));
     CK(cudaEventRecord(ev_fill0_, xs_));
     if (pl_.static_bytes && !(o_.keep_static && static_valid_)) {
-        CK(cudaMemcpyAsync(d_static_, (const char*)g_.nbr + g_.off[vlo_] * g_.b_e, pl_.static_bytes,
+        CK(cudaMemcpyAsync(d_static_, (const char*)g_.nbr + g_.off[stat_lo_] * g_.b_e, pl_.static_bytes,
                            cudaMemcpyHostToDevice, xs_));
         st.h2d_static_fill_bytes = pl_.static_bytes;
         static_valid_ = true;
@@ -877,6 +887,11 @@ void Engine::set_option(int opt, int64_t value) {
             break;
         case ASCETIC_OPT_PREFETCH: o_.prefetch = value ? 1 : 0; break;
         case ASCETIC_OPT_REPARTITION: o_.repartition = value ? 1 : 0; break;
+        case ASCETIC_OPT_STATIC_PLACEMENT:
+            if (value < 0 || value > 1) throw Error(ASCETIC_EINVAL, "static placement: 0 = front, 1 = rear");
+            o_.static_rear = (int)value;
+            if (state_ == 2) state_ = 1;   // takes effect at the next set_budget
+            break;
         case ASCETIC_OPT_STATIC_CTAS_PER_SM:
             if (value < 0 || value > 64) throw Error(ASCETIC_EINVAL, "static CTAs per SM must be in [0, 64]");
             o_.static_ctas_per_sm = (int)value;

@@ -60,6 +60,7 @@ struct Options {
     int static_ctas_per_sm = 0;   // persistent grid of the static-hit kernels (0 = 4 per SM)
     int prefetch = 1;             // PR: issue the next iteration's first chunk transfers early
     int repartition = 0;          // Eq. 3 adaptive re-partition (off, as in the paper's evaluation)
+    int static_rear = 0;          // initial static content: 0 = front prefix, 1 = rear suffix
 };
 
 struct HostGraph {
@@ -152,6 +153,7 @@ class Part {
     char* arena_ = nullptr;          // the edge budget: Static Region + On-demand Region
     uint64_t arena_bytes_ = 0;
     uint64_t ms_cur_ = 0, s_cur_ = 0; // current split (Eq. 3 may shrink it during a run)
+    uint64_t stat_lo_ = 0;            // first static vertex: vlo (front) or the rear suffix start
     void* d_static_ = nullptr;
     static constexpr int kMaxBuffers = 8;
     char* d_chunk_[kMaxBuffers] = {};

@@ -272,6 +272,35 @@ def test_pr_cross_iteration_prefetch(asc, prefetch, nbuf):
     assert st["dma_bytes"] == st["h2d_payload_bytes"] == ref.h2d_payload
 
 
+@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pr"])
+def test_rear_static_placement(asc, algo):
+    """Rear initial content (§5): the static set is the suffix of whole lists
+    that fits in Ms; records, bytes and results vs the oracle on that set."""
+    g = gg.rmat(12, seed=17, weights=(algo == "sssp"))
+    src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+    iters = 6 if algo == "pr" else 0
+    budget = g.csr_bytes // 3
+    asc.load_csr(g.off, g.nbr, pairs=g.pairs)
+    asc.set_option("static_placement", 1)
+    asc.set_option("chunk_cap", 8192)
+    asc.set_budget(budget)
+    asc.run(algo, src, iters)
+    st, its = asc.stats()
+    res = asc.get_result().copy()
+    asc.set_option("static_placement", 0)
+    asc.set_option("chunk_cap", 0)
+    p = oracle.placer(g.off, g.b_e, budget)
+    s_lo = oracle.rear_start(g.off, g.b_e, p.Ms)
+    ref = oracle.run(algo, g.off, g.nbr, src=src, max_iters=iters, is_static=oracle.static_rear(g.n, s_lo))
+    assert st["s"] == g.n - s_lo
+    assert st["h2d_static_fill_bytes"] == g.b_e * (int(g.off[-1]) - int(g.off[s_lo]))
+    _check_records(its, ref)
+    if algo == "pr":
+        _pr_ok(res, ref.values)
+    else:
+        np.testing.assert_array_equal(res, ref.values)
+
+
 @pytest.mark.parametrize("algo", ["bfs", "sssp", "cc"])
 def test_eq3_repartition_parity(asc, algo):
     """Eq. 3 adaptive re-partition (ASCETIC_OPT_REPARTITION): the shrink decisions, the static

@@ -76,6 +76,15 @@ def test_placer_nan_and_negative_clamp():
     assert p.R == 0.0 and p.Ms == 0 and p.s == 0
 
 
+def test_rear_start_is_smallest_fitting_suffix():
+    g = gg.rmat(11, seed=9)
+    o = g.off.astype(np.int64)
+    for Ms in [0, 100, 16384, 4 * g.m // 3, 4 * g.m, 10 * g.m]:
+        s_lo = oracle.rear_start(g.off, 4, Ms)
+        assert 4 * (o[-1] - o[s_lo]) <= Ms
+        assert s_lo == 0 or 4 * (o[-1] - o[s_lo - 1]) > Ms
+
+
 def test_partition_edge_balanced():
     g = gg.rmat(12, seed=3)
     for P in [1, 2, 3, 4, 8]:
