@@ -28,8 +28,10 @@ def main():
         src = gg.sources(g, 1, seed=c["seed"])[0]
         asc.load_csr(g.off, g.nbr, pairs=g.pairs)
 
-        def one(label, nbytes, frac, overlap=1):
+        def one(label, nbytes, frac, overlap=1, rear=0, eq3=0):
             asc.set_option("overlap", overlap)
+            asc.set_option("static_placement", rear)
+            asc.set_option("repartition", eq3)
             asc.set_budget(nbytes, frac)
             best = None
             for _ in range(2):
@@ -37,7 +39,8 @@ def main():
                 st, _ = asc.stats(per_iter=False)
                 if best is None or st["time_run_s"] < best["time_run_s"]:
                     best = st
-            r = dict(config=key, study=label, budget_frac_of_csr=round(nbytes / g.csr_bytes, 3),
+            r = dict(config=key, study=label, repartitions=best["repartitions"],
+                     budget_frac_of_csr=round(nbytes / g.csr_bytes, 3),
                      R=round(best["static_fraction_used"], 4), overlap=overlap, run_ms=round(best["time_run_s"] * 1e3, 2),
                      gteps=round(best["active_arcs_total"] / best["time_run_s"] / 1e9, 3),
                      fill_gb=round(best["h2d_static_fill_bytes"] / 1e9, 3),
@@ -47,12 +50,17 @@ def main():
             print(json.dumps(r), flush=True)
 
         one("eq2", budget, -1.0)
-        for R in [0.0, 0.2, 0.4, 0.6, 0.8, 0.9, 0.95, 1.0]:
-            one("R-sweep", budget, R)
-        one("overlap-off", budget, -1.0, overlap=0)
-        for f in [0.25, 0.5, 0.75, 1.0]:
-            one("budget-sweep", int(f * g.csr_bytes), -1.0)
+        if os.environ.get("ABLATION_QUICK") != "1":
+            for R in [0.0, 0.2, 0.4, 0.6, 0.8, 0.9, 0.95, 1.0]:
+                one("R-sweep", budget, R)
+            one("overlap-off", budget, -1.0, overlap=0)
+            for f in [0.25, 0.5, 0.75, 1.0]:
+                one("budget-sweep", int(f * g.csr_bytes), -1.0)
+        one("rear-fill", budget, -1.0, rear=1)
+        one("eq3-repartition", budget, -1.0, eq3=1)
         asc.set_option("overlap", 1)
+        asc.set_option("static_placement", 0)
+        asc.set_option("repartition", 0)
         asc.unload()
         del g
     out = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "gpurun_out", "ablation.md")
