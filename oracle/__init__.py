@@ -34,15 +34,18 @@ class _Iter(ctypes.Structure):
     _fields_ = [("t", ctypes.c_uint32), ("rank", ctypes.c_uint32), ("nA", ctypes.c_uint64),
                 ("nH", ctypes.c_uint64), ("nM", ctypes.c_uint64), ("nruns", ctypes.c_uint64),
                 ("active_arcs", ctypes.c_uint64), ("hit_arcs", ctypes.c_uint64),
-                ("miss_bytes", ctypes.c_uint64), ("digest", ctypes.c_uint64), ("s", ctypes.c_uint64)]
+                ("miss_bytes", ctypes.c_uint64), ("digest", ctypes.c_uint64), ("s", ctypes.c_uint64),
+                ("swaps", ctypes.c_uint64), ("replace_bytes", ctypes.c_uint64)]
 
 
 class _Summary(ctypes.Structure):
     _fields_ = [("iterations", ctypes.c_uint32), ("nrec", ctypes.c_uint32),
-                ("h2d_payload", ctypes.c_uint64), ("active_arcs_total", ctypes.c_uint64)]
+                ("h2d_payload", ctypes.c_uint64), ("active_arcs_total", ctypes.c_uint64),
+                ("h2d_replace", ctypes.c_uint64)]
 
 
-ITER_FIELDS = ["t", "rank", "nA", "nH", "nM", "nruns", "active_arcs", "hit_arcs", "miss_bytes", "digest", "s"]
+ITER_FIELDS = ["t", "rank", "nA", "nH", "nM", "nruns", "active_arcs", "hit_arcs", "miss_bytes", "digest", "s",
+               "swaps", "replace_bytes"]
 
 
 def build(force: bool = False) -> str:
@@ -67,6 +70,10 @@ def _load():
                                   ctypes.c_void_p, ctypes.c_void_p, ctypes.POINTER(_Iter), ctypes.c_uint32,
                                   ctypes.POINTER(_Summary), ctypes.c_int, ctypes.c_uint64, ctypes.c_uint64,
                                   ctypes.POINTER(ctypes.c_uint64)]
+        lib.or_run_hot.argtypes = [ctypes.c_int, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint32,
+                                   ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                   ctypes.POINTER(_Iter), ctypes.c_uint32, ctypes.POINTER(_Summary), ctypes.c_void_p,
+                                   ctypes.c_uint32, ctypes.c_int]
         lib.or_threads.restype = ctypes.c_int
         lib.or_classify.argtypes = [ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p,
                                     ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
@@ -155,6 +162,7 @@ class Result:
     h2d_payload: int
     active_arcs_total: int
     repartitions: int = 0
+    replace_bytes: int = 0      # §3.4 swap bytes (run_hot)
 
 
 def static_prefix(n: int, s: int) -> np.ndarray:
@@ -193,3 +201,37 @@ def run(algo: str | int, off: np.ndarray, nbr: np.ndarray, src: int = 0, max_ite
     vals = res_f.copy() if a == PR else res_u.copy()
     return Result(vals, int(s.iterations), records, int(s.h2d_payload), int(s.active_arcs_total),
                   int(reparts.value))
+
+
+def run_hot(algo: str | int, off: np.ndarray, nbr: np.ndarray, static_bytes, src: int = 0, max_iters: int = 0,
+            kswap: int = 0, policy: str | None = None, bounds: np.ndarray | None = None) -> Result:
+    """Run with the §3.4 data replacement: 16 KiB chunks, hotness counters, up to
+    `kswap` chunk swaps per iteration and rank. static_bytes = Ms (int, or one per rank).
+    policy: "cumulative" (default for bfs/sssp/cc) or "last" (default for pr), P:946-950."""
+    lib = _load()
+    a = ALGOS[algo] if isinstance(algo, str) else algo
+    if policy is None:
+        policy = "last" if a == PR else "cumulative"
+    if policy not in ("cumulative", "last"):
+        raise ValueError(policy)
+    off = np.ascontiguousarray(off, dtype=np.uint64)
+    nbr = np.ascontiguousarray(nbr, dtype=np.uint32)
+    n = off.size - 1
+    P = 1 if bounds is None else len(bounds) - 1
+    b = None if bounds is None else np.ascontiguousarray(bounds, dtype=np.uint64)
+    ms = np.ascontiguousarray(np.broadcast_to(np.asarray(static_bytes, dtype=np.uint64), (P,)), dtype=np.uint64)
+    res_u = np.zeros(max(n, 1), dtype=np.uint32)[:n]
+    res_f = np.zeros(max(n, 1), dtype=np.float64)[:n]
+    cap = (min(n + 2, 1 << 16) if a != PR else max(1, max_iters)) * P
+    recs = (_Iter * cap)()
+    s = _Summary()
+    rc = lib.or_run_hot(a, n, off.ctypes.data, nbr.ctypes.data if nbr.size else None, src, max_iters, P,
+                        b.ctypes.data if b is not None else None, res_u.ctypes.data if n else None,
+                        res_f.ctypes.data if n else None, recs, cap, ctypes.byref(s), ms.ctypes.data, kswap,
+                        1 if policy == "cumulative" else 0)
+    if rc != 0:
+        raise ValueError(f"oracle rejected arguments (rc={rc})")
+    records = [{f: int(getattr(recs[i], f)) for f in ITER_FIELDS} for i in range(s.nrec)]
+    vals = res_f.copy() if a == PR else res_u.copy()
+    return Result(vals, int(s.iterations), records, int(s.h2d_payload), int(s.active_arcs_total), 0,
+                  int(s.h2d_replace))

@@ -11,3 +11,12 @@ if ROOT not in sys.path:
 def pytest_configure(config):
     config.addinivalue_line("markers", "gpu: needs a B200 (run under gpurun)")
     config.addinivalue_line("markers", "slow: larger CPU cases")
+
+
+def pytest_sessionstart(session):
+    # a fresh checkout has no built artefacts (they are git-ignored): build them once here so
+    # the CPU suite runs from a clean tree; nvcc cross-compiles sm_100a without a GPU
+    need = [os.path.join(ROOT, "paper_conf_icpp_tangzwgzwy21_b200", "libascetic.so")]
+    if any(not os.path.exists(p) for p in need):
+        import __graft_entry__
+        __graft_entry__.build()

@@ -127,5 +127,5 @@ def records_from_sets(sets, off, b_e, s_static, rank_bounds=None):
             out.append(dict(t=t, rank=g, nA=int(A.sum()), nH=int(h.sum()), nM=int(mm.sum()),
                             nruns=runs_of(mm), active_arcs=int(deg[lo:hi][a].sum()),
                             hit_arcs=int(deg[lo:hi][h].sum()), miss_bytes=int(b_e * deg[lo:hi][mm].sum()),
-                            digest=digest(A), s=int(st[lo:hi].sum())))
+                            digest=digest(A), s=int(st[lo:hi].sum()), swaps=0, replace_bytes=0))
     return out
