@@ -76,8 +76,19 @@ typedef enum {
                                       if V_ondemand > C and V_static/M_static < 0.5 V/D, shrink the Static Region
                                       by M_static*V/D (floored to 16 KiB) and re-generate the map. Default 0, as
                                       in the paper's evaluation. Changes per-iteration bytes. */
-    ASCETIC_OPT_STATIC_PLACEMENT = 13 /* initial static content (§5): 0 = front prefix (default),
+    ASCETIC_OPT_STATIC_PLACEMENT = 13, /* initial static content (§5): 0 = front prefix (default),
                                       1 = rear suffix of whole lists fitting in Ms. Set before set_budget. */
+    ASCETIC_OPT_REPLACE_CHUNKS = 14, /* §3.4 data replacement (Fig. 6): K = 16 KiB chunk swaps
+                                      examined per iteration and rank (0 = off, the default; max 65536).
+                                      The Static Region becomes Ms/16 KiB chunk slots (initially the front
+                                      chunks, filled whole); after each iteration's data map, per-chunk access
+                                      counters (active arcs read) update the hotness table; during on-demand
+                                      computing the K hottest non-resident chunks replace the K coldest
+                                      resident ones while strictly hotter, effective next iteration. A vertex
+                                      is static iff every chunk its list touches is resident. Front placement
+                                      only; exclusive with Eq. 3. Set before set_budget. Changes bytes. */
+    ASCETIC_OPT_REPLACE_POLICY = 15 /* hotness counter: 0 = by algorithm (default: cumulative for
+                                      BFS/SSSP/CC, last iteration for PR), 1 = cumulative, 2 = last iteration */
 } ascetic_option;
 
 typedef struct {
@@ -86,7 +97,7 @@ typedef struct {
     uint64_t n, m;                /* vertices, stored arcs */
     uint32_t b_e;                 /* payload bytes per arc: 4, or 8 with ASCETIC_PAIRS */
     uint32_t rank, world;
-    uint64_t s;                   /* static vertices are [0, s) (front prefix) */
+    uint64_t s;                   /* static vertices are [0, s) (front prefix) at the start of the run */
     uint64_t budget_bytes;        /* B: Static + On-demand edge regions */
     uint64_t static_reserved;     /* Ms = R*B floored to 16 KiB */
     uint64_t static_bytes;        /* b_e * off[s] actually resident */
@@ -120,6 +131,9 @@ typedef struct {
     double time_finalize_s;
     double time_host_s;           /* host planning + waits between classify and the next launches */
     uint64_t repartitions;        /* Eq. 3 re-partitions performed (ASCETIC_OPT_REPARTITION) */
+    uint64_t h2d_replace_bytes;   /* §3.4 swapped-in chunk bytes (ASCETIC_OPT_REPLACE_CHUNKS) */
+    uint64_t swaps_total;         /* §3.4 chunk swaps performed */
+    double time_replace_s;        /* copy-stream time of the swap DMAs */
 } ascetic_stats_t;
 
 typedef struct {
@@ -136,7 +150,9 @@ typedef struct {
     /* host-link idle inside the iteration: before its first chunk transfer, between its
      * chunk transfers, and after its last one (until the next iteration's classify) */
     float ms_link_head, ms_link_gaps, ms_link_tail;
-    uint64_t s_static;            /* static vertices of this rank in this iteration (front prefix length) */
+    uint64_t s_static;            /* static vertices of this rank in this iteration (|S ∩ rank|) */
+    uint64_t swaps;               /* §3.4: chunks swapped in during this iteration (effective at t+1) */
+    uint64_t replace_bytes;       /* bytes of those chunks (16 KiB each; the rank's last chunk may be short) */
 } ascetic_iter_stats_t;
 
 /*

@@ -35,7 +35,8 @@ ALGOS = {"bfs": 0, "sssp": 1, "cc": 2, "pr": 3}
 SYMMETRIC, COPY, VALIDATE, PAIRS = 1, 2, 4, 8
 OPTIONS = {"chunk_cap": 1, "xfer_mode": 2, "dma_min_run": 3, "overlap": 4, "keep_static": 5,
            "hub_degree": 6, "timing": 7, "gather_ctas": 8, "chunk_buffers": 9, "static_ctas_per_sm": 10,
-           "prefetch": 11, "repartition": 12, "static_placement": 13}
+           "prefetch": 11, "repartition": 12, "static_placement": 13, "replace_chunks": 14,
+           "replace_policy": 15}
 INF = 0xFFFFFFFF
 
 
@@ -59,7 +60,8 @@ class Stats(ctypes.Structure):
                 ("time_gather_s", ctypes.c_double), ("gather_bytes", ctypes.c_uint64),
                 ("time_dma_s", ctypes.c_double), ("dma_bytes", ctypes.c_uint64),
                 ("time_finalize_s", ctypes.c_double), ("time_host_s", ctypes.c_double),
-                ("repartitions", ctypes.c_uint64)]
+                ("repartitions", ctypes.c_uint64), ("h2d_replace_bytes", ctypes.c_uint64),
+                ("swaps_total", ctypes.c_uint64), ("time_replace_s", ctypes.c_double)]
 
 
 class IterStats(ctypes.Structure):
@@ -70,7 +72,8 @@ class IterStats(ctypes.Structure):
                 ("ms_classify", ctypes.c_float), ("ms_static", ctypes.c_float), ("ms_ondemand", ctypes.c_float),
                 ("ms_h2d", ctypes.c_float), ("ms_finalize", ctypes.c_float), ("ms_exchange", ctypes.c_float),
                 ("ms_total", ctypes.c_float), ("ms_link_head", ctypes.c_float), ("ms_link_gaps", ctypes.c_float),
-                ("ms_link_tail", ctypes.c_float), ("s_static", ctypes.c_uint64)]
+                ("ms_link_tail", ctypes.c_float), ("s_static", ctypes.c_uint64), ("swaps", ctypes.c_uint64),
+                ("replace_bytes", ctypes.c_uint64)]
 
 
 _lib.ascetic_load_csr.argtypes = [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p,

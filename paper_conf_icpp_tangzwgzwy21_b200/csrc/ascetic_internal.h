@@ -41,6 +41,7 @@ struct IterTotals {
     uint32_t tile_counter, done_counter;
     uint32_t ready;          // set to 1 last (host spin target)
     uint32_t pad;
+    unsigned long long nS;   // |S ∩ owned range| (static vertices of this rank in this iteration)
 };
 
 struct ClassifyArgs {
@@ -92,7 +93,14 @@ struct DevState {
     uint32_t iter;         // t
     uint64_t vlo, vhi;     // owned vertex range (PR finalize)
     unsigned long long static_arc0;   // first arc held by the Static Region (off[vlo])
+    // §3.4 replacement: Static Region = 16 KiB slots; slot_of[c] = slot of rank-local chunk c
+    // (kNoSlot if not resident). nullptr = contiguous prefix (no remapping).
+    const uint32_t* slot_of;
 };
+
+constexpr uint32_t kNoSlot = 0xFFFFFFFFu;
+constexpr int kChunkShift = 14;                          // §3.4 16 KB chunks
+constexpr uint64_t kChunkBytes = 1ull << kChunkShift;
 
 struct Queues {
     const uint32_t* hq_small;
@@ -122,6 +130,12 @@ void launch_ondemand(int algo, const DevState& d, const Queues& q,
                      const void* chunk, unsigned long long lo, unsigned long long hi, cudaStream_t s);
 void launch_gather(const Queues& q, const void* host_nbr, uint32_t b_e, void* chunk,
                    unsigned long long lo, unsigned long long hi, int max_ctas, cudaStream_t s);
+// §3.4: per-chunk accesses (active arcs) of this iteration's hit + miss queues into acc
+void launch_chunk_access(const DevState& d, const Queues& q, uint32_t n_small, uint32_t n_med, uint32_t n_hub,
+                         uint32_t b_e, uint32_t* acc, cudaStream_t s);
+// §3.4: apply swaps (in[i] gets out[i]'s slot) and recompute S for the vertices touching the changed chunks
+void launch_apply_swaps(const DevState& d, uint32_t* slot_of, const uint32_t* swaps /* in[k], out[k], slot[k] */,
+                        uint32_t k, uint32_t b_e, cudaStream_t s);
 // dense = values were exchanged (P > 1): SSSP/CC rebuild A from val < snap over all vertices
 void launch_finalize(int algo, const DevState& d, bool dense, cudaStream_t s);
 // collectives' device side (comm.cu drives them)

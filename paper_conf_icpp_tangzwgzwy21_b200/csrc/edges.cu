@@ -119,9 +119,20 @@ __device__ __forceinline__ uint32_t ub_u32(const uint32_t* a, uint32_t n, uint32
     return lo;
 }
 
+// §3.4 replacement: the Static Region is a set of 16 KiB slots; unit i (U-byte units) of the
+// rank's payload lives at slot_of[chunk] * (16 KiB / U) + i mod (16 KiB / U). Without
+// replacement the region is the contiguous front prefix (identity). An aligned 16-byte load
+// never straddles a chunk, so the 128-bit body loop stays vectorised.
+template <bool REMAP, int U>
+__device__ __forceinline__ unsigned long long sidx(const DevState& d, unsigned long long i) {
+    if (!REMAP) return i;
+    constexpr unsigned long long per = kChunkBytes / U;
+    return (unsigned long long)__ldg(d.slot_of + i / per) * per + (i % per);
+}
+
 // contiguous list [a0, a1) of arcs at base (b_e = 4 for ids, 8 for pairs), processed by
 // `nthr` threads with index `tid`, 128-bit loads on the aligned body.
-template <int ALGO>
+template <int ALGO, bool REMAP = false>
 __device__ __forceinline__ double expand_list(const DevState& d, const void* base, unsigned long long a0,
                                               unsigned long long a1, uint32_t sval, int tid, int nthr) {
     double acc = 0.0;
@@ -129,31 +140,31 @@ __device__ __forceinline__ double expand_list(const DevState& d, const void* bas
         const uint2* arcs = reinterpret_cast<const uint2*>(base);
         const unsigned long long h = min(a1, (a0 + 1) & ~1ull);      // 2 arcs per 16 B
         for (unsigned long long e = a0 + tid; e < h; e += nthr) {
-            const uint2 x = ld_stream(arcs + e);
+            const uint2 x = ld_stream(arcs + sidx<REMAP, 8>(d, e));
             push_arc<ALGO>(d, sval, x.x, x.y);
         }
         const unsigned long long qb = h >> 1, qe = a1 >> 1;
         const uint4* q = reinterpret_cast<const uint4*>(base);
         for (unsigned long long k = qb + tid; k < qe; k += nthr) {
-            const uint4 x = ld_stream(q + k);
+            const uint4 x = ld_stream(q + sidx<REMAP, 16>(d, k));
             push_arc<ALGO>(d, sval, x.x, x.y);
             push_arc<ALGO>(d, sval, x.z, x.w);
         }
         for (unsigned long long e = max(h, qe << 1) + tid; e < a1; e += nthr) {
-            const uint2 x = ld_stream(arcs + e);
+            const uint2 x = ld_stream(arcs + sidx<REMAP, 8>(d, e));
             push_arc<ALGO>(d, sval, x.x, x.y);
         }
     } else {
         const uint32_t* arcs = reinterpret_cast<const uint32_t*>(base);
         const unsigned long long h = min(a1, (a0 + 3) & ~3ull);      // 4 arcs per 16 B
         for (unsigned long long e = a0 + tid; e < h; e += nthr) {
-            const uint32_t id = ld_stream(arcs + e);
+            const uint32_t id = ld_stream(arcs + sidx<REMAP, 4>(d, e));
             if (ALGO == PR) acc += pr_in(d, id); else push_arc<ALGO>(d, sval, id, 0);
         }
         const unsigned long long qb = h >> 2, qe = a1 >> 2;
         const uint4* q = reinterpret_cast<const uint4*>(base);
         for (unsigned long long k = qb + tid; k < qe; k += nthr) {
-            const uint4 x = ld_stream(q + k);
+            const uint4 x = ld_stream(q + sidx<REMAP, 16>(d, k));
             if (ALGO == PR) {
                 acc += pr_in(d, x.x) + pr_in(d, x.y) + pr_in(d, x.z) + pr_in(d, x.w);
             } else {
@@ -162,7 +173,7 @@ __device__ __forceinline__ double expand_list(const DevState& d, const void* bas
             }
         }
         for (unsigned long long e = max(h, qe << 2) + tid; e < a1; e += nthr) {
-            const uint32_t id = ld_stream(arcs + e);
+            const uint32_t id = ld_stream(arcs + sidx<REMAP, 4>(d, e));
             if (ALGO == PR) acc += pr_in(d, id); else push_arc<ALGO>(d, sval, id, 0);
         }
     }
@@ -180,7 +191,7 @@ __device__ __forceinline__ double warp_sum_d(double x) {
 // hit work of an iteration can be tens of thousands of CTAs, and a grid that size would fill
 // every SM slot and starve the on-demand kernels that gate chunk-buffer reuse (measured on the
 // friendster-shaped PR: a 22 ms static pull stalled the transfer pipeline 13 ms per iteration).
-template <int ALGO>
+template <int ALGO, bool REMAP>
 __global__ void __launch_bounds__(256) k_static_small(DevState d, const uint32_t* __restrict__ q, uint32_t nq,
                                                       const void* __restrict__ sbase) {
     __shared__ double s_acc[8][32];
@@ -221,7 +232,7 @@ __global__ void __launch_bounds__(256) k_static_small(DevState d, const uint32_t
             const bool ok = k < total;
             const unsigned long long e = ust + (k - uex) - d.static_arc0;   // index into the Static Region
             if (ALGO == PR) {
-                double x = ok ? pr_in(d, ld_stream(reinterpret_cast<const uint32_t*>(sbase) + e)) : 0.0;
+                double x = ok ? pr_in(d, ld_stream(reinterpret_cast<const uint32_t*>(sbase) + sidx<REMAP, 4>(d, e))) : 0.0;
 #pragma unroll
                 for (int o = 1; o < 32; o <<= 1) {
                     const double y = __shfl_up_sync(FULL, x, o);
@@ -235,10 +246,10 @@ __global__ void __launch_bounds__(256) k_static_small(DevState d, const uint32_t
                 __syncwarp();
             } else if (ok) {
                 if (ALGO == SSSP) {
-                    const uint2 x = ld_stream(reinterpret_cast<const uint2*>(sbase) + e);
+                    const uint2 x = ld_stream(reinterpret_cast<const uint2*>(sbase) + sidx<REMAP, 8>(d, e));
                     push_arc<ALGO>(d, usv, x.x, x.y);
                 } else {
-                    push_arc<ALGO>(d, usv, ld_stream(reinterpret_cast<const uint32_t*>(sbase) + e), 0);
+                    push_arc<ALGO>(d, usv, ld_stream(reinterpret_cast<const uint32_t*>(sbase) + sidx<REMAP, 4>(d, e)), 0);
                 }
             }
         }
@@ -248,7 +259,7 @@ __global__ void __launch_bounds__(256) k_static_small(DevState d, const uint32_t
 }
 
 // ------------------------------------------------------------------ static: warp per list
-template <int ALGO>
+template <int ALGO, bool REMAP>
 __global__ void __launch_bounds__(256) k_static_med(DevState d, const uint32_t* __restrict__ q, uint32_t nq,
                                                     const void* __restrict__ sbase) {
     const int lane = threadIdx.x & 31;
@@ -257,7 +268,7 @@ __global__ void __launch_bounds__(256) k_static_med(DevState d, const uint32_t* 
         const uint32_t u = __ldg(q + w);
         const unsigned long long a0 = __ldg(d.off + u), a1 = __ldg(d.off + u + 1);
         const uint32_t sval = (ALGO == SSSP || ALGO == CC) ? __ldg(d.snap + u) : 0u;
-        double acc = expand_list<ALGO>(d, sbase, a0 - d.static_arc0, a1 - d.static_arc0, sval, lane, 32);
+        double acc = expand_list<ALGO, REMAP>(d, sbase, a0 - d.static_arc0, a1 - d.static_arc0, sval, lane, 32);
         if (ALGO == PR) {
             acc = warp_sum_d(acc);
             if (lane == 0) d.sum[u] = acc;
@@ -266,7 +277,7 @@ __global__ void __launch_bounds__(256) k_static_med(DevState d, const uint32_t* 
 }
 
 // ------------------------------------------------------------------ static: hubs, CTA per piece
-template <int ALGO>
+template <int ALGO, bool REMAP>
 __global__ void __launch_bounds__(256) k_static_hub(DevState d, const uint32_t* __restrict__ hq,
                                                     const uint32_t* __restrict__ pre, uint32_t nh, uint32_t npieces,
                                                     uint32_t piece_arcs, const void* __restrict__ sbase) {
@@ -279,7 +290,8 @@ __global__ void __launch_bounds__(256) k_static_hub(DevState d, const uint32_t* 
         const unsigned long long a0 = o0 + (unsigned long long)pidx * piece_arcs;
         const unsigned long long a1 = min(o1, a0 + piece_arcs);
         const uint32_t sval = (ALGO == SSSP || ALGO == CC) ? __ldg(d.snap + u) : 0u;
-        double acc = expand_list<ALGO>(d, sbase, a0 - d.static_arc0, a1 - d.static_arc0, sval, threadIdx.x, blockDim.x);
+        double acc = expand_list<ALGO, REMAP>(d, sbase, a0 - d.static_arc0, a1 - d.static_arc0, sval, threadIdx.x,
+                                              blockDim.x);
         if (ALGO == PR) {
             acc = warp_sum_d(acc);
             if ((threadIdx.x & 31) == 0) s_red[threadIdx.x >> 5] = acc;
@@ -621,19 +633,119 @@ __global__ void k_min_into(uint32_t* __restrict__ dst, const uint32_t* __restric
 
 __global__ void k_add_f64(double* dst, const double* src) { dst[0] += src[0]; }
 
+// ------------------------------------------------------------------ §3.4 data replacement
+// Accesses of this iteration per 16 KiB chunk: every active list with deg > 0 is
+// in exactly one of the hit queues or the miss queue; its arcs [a, e) (rank-local) add their
+// overlap with each chunk they touch. Consecutive queue entries are ascending vertex ids, so
+// neighbouring lanes mostly hit the same chunk: single-chunk lists are combined per warp
+// (match + reduce) before the atomic.
+__global__ void __launch_bounds__(256) k_chunk_access(DevState d, Queues q, uint32_t n_small, uint32_t n_med,
+                                                      uint32_t n_hub, uint32_t epc_shift, uint32_t* __restrict__ acc) {
+    const unsigned long long total = (unsigned long long)n_small + n_med + n_hub + q.n_missq;
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    const unsigned long long x0 = d.static_arc0;
+    for (unsigned long long i0 = (unsigned long long)blockIdx.x * blockDim.x; i0 < total; i0 += stride) {
+        const unsigned long long i = i0 + threadIdx.x;
+        uint32_t key = 0xFFFFFFFFu, val = 0;
+        if (i < total) {
+            unsigned long long j = i;
+            uint32_t v;
+            if (j < n_small) v = __ldg(q.hq_small + j);
+            else if ((j -= n_small) < n_med) v = __ldg(q.hq_med + j);
+            else if ((j -= n_med) < n_hub) v = __ldg(q.hq_hub + j);
+            else v = __ldg(q.mq + (j - n_hub));
+            const unsigned long long a = __ldg(d.off + v) - x0, e = __ldg(d.off + v + 1) - x0;
+            const unsigned long long c0 = a >> epc_shift, c1 = (e - 1) >> epc_shift;
+            if (c0 == c1) {
+                key = (uint32_t)c0;
+                val = (uint32_t)(e - a);
+            } else {
+                for (unsigned long long c = c0; c <= c1; ++c) {
+                    const unsigned long long lo = max(a, c << epc_shift), hi = min(e, (c + 1) << epc_shift);
+                    atomicAdd(acc + c, (uint32_t)(hi - lo));
+                }
+            }
+        }
+        const uint32_t peers = __match_any_sync(FULL, key);
+        const uint32_t sum = __reduce_add_sync(peers, val);
+        if (key != 0xFFFFFFFFu && (threadIdx.x & 31) == __ffs(peers) - 1) atomicAdd(acc + key, sum);
+    }
+}
+
+// Swap i: chunk in[i] takes the slot of chunk out[i] (the swap DMAs already landed). Then the
+// StaticBitmap is recomputed for every vertex touching a changed chunk: v is static iff all
+// chunks of its list are resident; a degree-0 vertex at arc x belongs to chunk (x-1)/epc.
+__global__ void k_apply_swaps(uint32_t* __restrict__ slot_of, const uint32_t* __restrict__ sw, uint32_t k) {
+    // sw = [in[0..k), out[0..k), slot[0..k)]: in and out are disjoint chunk sets
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < k; i += gridDim.x * blockDim.x) {
+        slot_of[sw[i]] = sw[2 * k + i];
+        slot_of[sw[k + i]] = kNoSlot;
+    }
+}
+
+__device__ __forceinline__ bool chunks_resident(const uint32_t* slot_of, unsigned long long a, unsigned long long e,
+                                                uint32_t epc_shift) {
+    if (e == a) return a == 0 || slot_of[(a - 1) >> epc_shift] != kNoSlot;
+    for (unsigned long long c = a >> epc_shift; c <= (e - 1) >> epc_shift; ++c)
+        if (slot_of[c] == kNoSlot) return false;
+    return true;
+}
+
+// one warp per changed chunk (2k of them: the swapped-in and the evicted)
+__global__ void __launch_bounds__(256) k_static_rebits(DevState d, const uint32_t* __restrict__ slot_of,
+                                                       const uint32_t* __restrict__ sw, uint32_t nchg,
+                                                       uint32_t epc_shift) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (w >= nchg) return;
+    const unsigned long long x0 = d.static_arc0;
+    const unsigned long long c = sw[w];
+    const unsigned long long lo = x0 + (c << epc_shift), hi = x0 + ((c + 1) << epc_shift);
+    // first v in [vlo, vhi) with off[v+1] > lo (its list ends after the chunk starts)
+    unsigned long long L = d.vlo, R = d.vhi;
+    while (L < R) {
+        const unsigned long long mid = (L + R) >> 1;
+        if (d.off[mid + 1] > lo) R = mid; else L = mid + 1;
+    }
+    for (unsigned long long v0 = L;; v0 += 32) {
+        const unsigned long long v = v0 + lane;
+        bool in = false;
+        if (v < d.vhi) {
+            const unsigned long long a = d.off[v], e = d.off[v + 1];
+            in = a <= hi;
+            if (in) {
+                const uint32_t bit = 1u << (v & 31);
+                if (chunks_resident(slot_of, a - x0, e - x0, epc_shift)) atomicOr(d.S + (v >> 5), bit);
+                else atomicAnd(d.S + (v >> 5), ~bit);
+            }
+        }
+        if (!__any_sync(FULL, in)) break;
+    }
+}
+
 inline unsigned blocks_for(unsigned long long n, int per_block, unsigned cap = 148u * 16u) {
     unsigned long long b = (n + per_block - 1) / per_block;
     if (b < 1) b = 1;
     return (unsigned)(b > cap ? cap : b);
 }
 
+template <int ALGO, bool REMAP>
+void static_launch_t(const DevState& d, const Queues& q, const void* sbase, uint32_t ns, uint32_t nm, uint32_t nh,
+                     uint32_t npieces, uint32_t piece, int max_ctas, cudaStream_t s) {
+    auto cap = [&](unsigned long long b) { return (unsigned)(b < (unsigned long long)max_ctas ? b : max_ctas); };
+    if (ns) { k_static_small<ALGO, REMAP><<<cap((ns + 255) / 256), 256, 0, s>>>(d, q.hq_small, ns, sbase); ++g_launches; }
+    if (nm) { k_static_med<ALGO, REMAP><<<cap((nm + 7) / 8), 256, 0, s>>>(d, q.hq_med, nm, sbase); ++g_launches; }
+    if (nh) {
+        k_static_hub<ALGO, REMAP><<<cap(npieces), 256, 0, s>>>(d, q.hq_hub, q.hub_pre, nh, npieces, piece, sbase);
+        ++g_launches;
+    }
+}
+
 template <int ALGO>
 void static_launch(const DevState& d, const Queues& q, const void* sbase, uint32_t ns, uint32_t nm, uint32_t nh,
                    uint32_t npieces, uint32_t piece, int max_ctas, cudaStream_t s) {
-    auto cap = [&](unsigned long long b) { return (unsigned)(b < (unsigned long long)max_ctas ? b : max_ctas); };
-    if (ns) { k_static_small<ALGO><<<cap((ns + 255) / 256), 256, 0, s>>>(d, q.hq_small, ns, sbase); ++g_launches; }
-    if (nm) { k_static_med<ALGO><<<cap((nm + 7) / 8), 256, 0, s>>>(d, q.hq_med, nm, sbase); ++g_launches; }
-    if (nh) { k_static_hub<ALGO><<<cap(npieces), 256, 0, s>>>(d, q.hq_hub, q.hub_pre, nh, npieces, piece, sbase); ++g_launches; }
+    if (d.slot_of) static_launch_t<ALGO, true>(d, q, sbase, ns, nm, nh, npieces, piece, max_ctas, s);
+    else static_launch_t<ALGO, false>(d, q, sbase, ns, nm, nh, npieces, piece, max_ctas, s);
 }
 
 }  // namespace
@@ -646,6 +758,24 @@ void launch_static(int algo, const DevState& d, const Queues& q, const void* sba
         case CC: static_launch<CC>(d, q, sbase, ns, nm, nh, npieces, piece, max_ctas, s); break;
         default: static_launch<PR>(d, q, sbase, ns, nm, nh, npieces, piece, max_ctas, s); break;
     }
+}
+
+void launch_chunk_access(const DevState& d, const Queues& q, uint32_t n_small, uint32_t n_med, uint32_t n_hub,
+                         uint32_t b_e, uint32_t* acc, cudaStream_t s) {
+    const unsigned long long total = (unsigned long long)n_small + n_med + n_hub + q.n_missq;
+    if (!total) return;
+    const uint32_t epc_shift = kChunkShift - (b_e == 8 ? 3 : 2);
+    k_chunk_access<<<blocks_for(total, 256), 256, 0, s>>>(d, q, n_small, n_med, n_hub, epc_shift, acc);
+    ++g_launches;
+}
+
+void launch_apply_swaps(const DevState& d, uint32_t* slot_of, const uint32_t* sw, uint32_t k, uint32_t b_e,
+                        cudaStream_t s) {
+    if (!k) return;
+    const uint32_t epc_shift = kChunkShift - (b_e == 8 ? 3 : 2);
+    k_apply_swaps<<<blocks_for(k, 256), 256, 0, s>>>(slot_of, sw, k);
+    k_static_rebits<<<(2 * k + 7) / 8, 256, 0, s>>>(d, slot_of, sw, 2 * k, epc_shift);
+    g_launches += 2;
 }
 
 void launch_ondemand(int algo, const DevState& d, const Queues& q, const void* chunk,

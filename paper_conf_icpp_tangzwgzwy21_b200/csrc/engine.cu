@@ -133,6 +133,9 @@ Part::~Part() {
         if (consumed_[i]) cudaEventDestroy(consumed_[i]);
     }
     if (ev_classified_) cudaEventDestroy(ev_classified_);
+    free_hot();
+    if (ev_acc_) cudaEventDestroy(ev_acc_);
+    if (ev_swapped_) cudaEventDestroy(ev_swapped_);
     if (static_go_) cudaEventDestroy(static_go_);
     if (static_done_) cudaEventDestroy(static_done_);
     if (sync_ev_) cudaEventDestroy(sync_ev_);
@@ -160,6 +163,8 @@ void Part::alloc_vertex_state() {
     CK(cudaEventCreateWithFlags(&static_done_, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&sync_ev_, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&ev_classified_, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&ev_acc_, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&ev_swapped_, cudaEventDisableTiming));
     const uint64_t n = g_.n, m = g_.m;
     vertex_bytes_ = 0;
     nwords_ = (uint32_t)((n + 31) / 32);
@@ -285,7 +290,37 @@ void Part::set_budget(uint64_t bytes, double frac) {
     s_cur_ = p.s;
     layout_regions(p.Ms);
     launch_set_range_bits(d_S_, nwords_, stat_lo_, stat_lo_ + p.s, cs_);   // StaticBitmap
+    // §3.4 data replacement: the Static Region becomes ceil(Ms / 16 KiB) chunk slots, initially the
+    // front chunks (filled whole); only meaningful when some lists stay outside it
+    hot_ = o_.replace_k > 0 && p.s < own && p.Ms > 0;
+    if (hot_) {
+        if (o_.static_rear) throw Error(ASCETIC_EINVAL, "replacement needs the front initial placement");
+        hNC_ = (p.D + kChunkBytes - 1) / kChunkBytes;
+        hNS_ = (p.Ms + kChunkBytes - 1) / kChunkBytes;
+        if (hNC_ > 0xFFFFFFF0ull) throw Error(ASCETIC_EINVAL, "too many 16 KiB chunks for replacement");
+        if (hNC_ != hot_alloc_nc_ || o_.replace_k != hot_alloc_k_) {
+            free_hot();
+            dalloc(&d_slot_of_, hNC_, nullptr);
+            dalloc(&d_acc_, hNC_, nullptr);
+            dalloc(&d_swap_, 3ull * o_.replace_k, nullptr);
+            cudaError_t e = cudaHostAlloc((void**)&h_acc_, hNC_ * 4, cudaHostAllocPortable);
+            if (e == cudaSuccess) e = cudaHostAlloc((void**)&h_swap_, 12ull * o_.replace_k, cudaHostAllocPortable);
+            if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_EHOSTMEM, "cudaHostAlloc (replacement tables)"); }
+            hot_alloc_nc_ = hNC_;
+            hot_alloc_k_ = o_.replace_k;
+        }
+        hot_dirty_ = true;   // begin() installs the initial slots
+    }
     CK(cudaStreamSynchronize(cs_));
+}
+
+void Part::free_hot() {
+    dfree(d_slot_of_); dfree(d_acc_); dfree(d_swap_);
+    if (h_acc_) cudaFreeHost(h_acc_);
+    if (h_swap_) cudaFreeHost(h_swap_);
+    h_acc_ = h_swap_ = nullptr;
+    hot_alloc_nc_ = 0;
+    hot_alloc_k_ = 0;
 }
 
 // Eq. 3 (§3.3): after the data map of an iteration is generated, if the on-demand
@@ -324,6 +359,7 @@ DevState Part::dev_state(uint32_t iter) const {
     d.iter = iter;
     d.vlo = vlo_; d.vhi = vhi_;
     d.static_arc0 = g_.off.empty() ? 0 : g_.off[stat_lo_];
+    d.slot_of = hot_ ? d_slot_of_ : nullptr;
     return d;
 }
 
@@ -390,6 +426,21 @@ void Part::begin(int algo, uint32_t source, uint32_t max_iters, bool timing) {
         launch_set_range_bits(d_S_, nwords_, stat_lo_, stat_lo_ + pl_.s, cs_);
     }
     layout_regions(ms_cur_);
+    if (hot_) {
+        // every run starts from the front chunks [0, hNS_) in slots [0, hNS_) and a zero hotness table
+        if (hot_dirty_) {
+            slot_of_.assign(hNC_, kNoSlot);
+            slot_chunk_.resize(hNS_);
+            for (uint64_t c = 0; c < hNS_; ++c) { slot_of_[c] = (uint32_t)c; slot_chunk_[c] = (uint32_t)c; }
+            CK(cudaMemcpyAsync(d_slot_of_, slot_of_.data(), hNC_ * 4, cudaMemcpyHostToDevice, cs_));
+            CK(cudaStreamSynchronize(cs_));
+            launch_set_range_bits(d_S_, nwords_, stat_lo_, stat_lo_ + pl_.s, cs_);
+            static_valid_ = false;
+            hot_dirty_ = false;
+        }
+        hot_h_.assign(hNC_, 0);
+    }
+    acc_pending_ = false;
     iters.clear();
     std::memset(&st, 0, sizeof st);
     pool_.reset();
@@ -401,10 +452,12 @@ void Part::begin(int algo, uint32_t source, uint32_t max_iters, bool timing) {
     // ---- static fill: ONE DMA of this rank's front prefix, counted in the run
     CK(cudaStreamWaitEvent(xs_, ev_start_, 0));
     CK(cudaEventRecord(ev_fill0_, xs_));
-    if (pl_.static_bytes && !(o_.keep_static && static_valid_)) {
-        CK(cudaMemcpyAsync(d_static_, (const char*)g_.nbr + g_.off[stat_lo_] * g_.b_e, pl_.static_bytes,
+    // with replacement the slots are filled whole: Ms bytes (the chunk holding the prefix end too)
+    const uint64_t fill = hot_ ? pl_.Ms : pl_.static_bytes;
+    if (fill && !(o_.keep_static && static_valid_)) {
+        CK(cudaMemcpyAsync(d_static_, (const char*)g_.nbr + g_.off[stat_lo_] * g_.b_e, fill,
                            cudaMemcpyHostToDevice, xs_));
-        st.h2d_static_fill_bytes = pl_.static_bytes;
+        st.h2d_static_fill_bytes = fill;
         static_valid_ = true;
     }
     CK(cudaEventRecord(ev_fill1_, xs_));
@@ -468,7 +521,7 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     is.nA = T.nA; is.nH = T.nH; is.nM = T.nM; is.nruns = T.n_runs;
     is.active_arcs = T.active_arcs; is.hit_arcs = T.hit_arcs; is.miss_bytes = T.miss_arcs * b_e;
     is.digest = T.digest;
-    is.s_static = s_cur_;
+    is.s_static = T.nS;
     const DevState d = dev_state(t);
     const Queues q = queues(T);
     if (algo_ == ALG_PR) CK(cudaMemsetAsync(d_sum_ + vlo_, 0, (vhi_ - vlo_) * sizeof(double), cs_));
@@ -478,6 +531,18 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     // index it with rank-local arc numbers (arc - d.static_arc0), so 128-bit alignment is
     // that of the buffer itself.
     static_pending_ = false;
+    static_launched_ = false;
+    // §3.4: this iteration's accesses per 16 KiB chunk -> pinned host table, read by
+    // replace() while the on-demand chunks stream (the server thread of Fig. 6)
+    if (hot_ && !(max_iters_ && t + 1 == max_iters_)) {
+        CK(cudaMemsetAsync(d_acc_, 0, hNC_ * 4, cs_));
+        launch_chunk_access(d, q, T.n_small, T.n_med, T.n_hub, b_e, d_acc_, cs_);
+        CK(cudaGetLastError());
+        CK(cudaMemcpyAsync(h_acc_, d_acc_, hNC_ * 4, cudaMemcpyDeviceToHost, cs_));
+        CK(cudaEventRecord(ev_acc_, cs_));
+        acc_pending_ = true;
+        st.d2h_bytes += hNC_ * 4;
+    }
     if (T.n_small + T.n_med + T.n_hub) {
         CK(cudaEventRecord(static_go_, cs_));
         CK(cudaStreamWaitEvent(ss_, static_go_, 0));
@@ -488,6 +553,7 @@ void Part::expand(uint32_t t, const IterTotals& T) {
         span(e0, ss_, t, PH_STATIC);
         CK(cudaEventRecord(static_done_, ss_));
         static_pending_ = true;
+        static_launched_ = true;
     }
     st.static_arcs += T.hit_arcs;
     st.ondemand_arcs += T.miss_arcs;
@@ -550,7 +616,7 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     // transfer does not depend on this iteration's values. Issue the next iteration's first
     // chunks now (each still waits for its buffer's consumer): the link keeps streaming
     // through this iteration's tail, finalize and the next classify.
-    if (algo_ == ALG_PR && mode == 2 && nchunks && o_.prefetch && !o_.repartition && t + 1 < max_iters_) {
+    if (algo_ == ALG_PR && mode == 2 && nchunks && o_.prefetch && !o_.repartition && !hot_ && t + 1 < max_iters_) {
         const uint32_t np = std::min<uint32_t>(nchunks, (uint32_t)nbuf_);
         for (uint32_t k = 0; k < np; ++k) {
             const uint64_t gk = gchunk_ + k;
@@ -616,6 +682,79 @@ void Part::join_static() {
     static_pending_ = false;
 }
 
+// §3.4 (Fig. 6; swaps "when GPU is processing the On-demand Region"):
+// update the HotnessTable with this iteration's chunk accesses (cumulative for BFS/SSSP/CC, last
+// iteration for PR), then swap the K hottest non-resident chunks (h desc, id asc)
+// with the K coldest resident ones (h asc, id asc) while strictly hotter. The swap DMAs run on
+// the copy stream after this iteration's miss chunks and static-hit kernels; slot table and
+// StaticBitmap are updated on the compute stream before the next GenDataMap.
+void Part::replace(uint32_t t) {
+    if (!acc_pending_) return;
+    acc_pending_ = false;
+    const auto th0 = std::chrono::steady_clock::now();
+    CK(cudaEventSynchronize(ev_acc_));
+    const bool cum = o_.replace_policy == 1 || (o_.replace_policy == 0 && algo_ != ALG_PR);
+    const uint32_t K = o_.replace_k;
+    uint64_t* h = hot_h_.data();
+    const uint32_t* acc = h_acc_;
+    if (cum) for (uint64_t c = 0; c < hNC_; ++c) h[c] += acc[c];
+    else for (uint64_t c = 0; c < hNC_; ++c) h[c] = acc[c];
+    // K hottest non-resident chunks: bounded heap ordered by `better`, so its top is the worst kept
+    auto better = [&](uint32_t a, uint32_t b) { return h[a] != h[b] ? h[a] > h[b] : a < b; };  // min-heap
+    std::vector<uint32_t> hot;
+    hot.reserve(K + 1);
+    for (uint64_t c = 0; c < hNC_; ++c) {
+        if (slot_of_[c] != kNoSlot) continue;
+        if (hot.size() == K) {
+            if (h[c] <= h[hot.front()]) continue;   // ascending ids: a tie never displaces
+            std::pop_heap(hot.begin(), hot.end(), better);
+            hot.back() = (uint32_t)c;
+        } else {
+            hot.push_back((uint32_t)c);
+        }
+        std::push_heap(hot.begin(), hot.end(), better);
+    }
+    std::sort(hot.begin(), hot.end(), better);
+    // K coldest resident chunks (there are hNS_ of them: scan the slots)
+    std::vector<uint32_t> cold(slot_chunk_);
+    auto colder = [&](uint32_t a, uint32_t b) { return h[a] != h[b] ? h[a] < h[b] : a < b; };
+    const size_t kc = std::min<size_t>(K, cold.size());
+    std::partial_sort(cold.begin(), cold.begin() + kc, cold.end(), colder);
+    uint32_t k = 0;
+    uint64_t bytes = 0;
+    while (k < hot.size() && k < kc && h[hot[k]] > h[cold[k]]) ++k;
+    if (k) {
+        const uint64_t x0 = g_.off[vlo_] * (uint64_t)g_.b_e;
+        if (static_launched_) CK(cudaStreamWaitEvent(xs_, static_done_, 0));   // evicted slots no longer read
+        cudaEvent_t e0 = mark(xs_);
+        for (uint32_t i = 0; i < k; ++i) {
+            const uint32_t cin = hot[i], cout = cold[i], slot = slot_of_[cout];
+            slot_of_[cin] = slot;
+            slot_of_[cout] = kNoSlot;
+            slot_chunk_[slot] = cin;
+            const uint64_t sz = std::min<uint64_t>(kChunkBytes, pl_.D - (uint64_t)cin * kChunkBytes);
+            CK(cudaMemcpyAsync((char*)d_static_ + (uint64_t)slot * kChunkBytes,
+                               (const char*)g_.nbr + x0 + (uint64_t)cin * kChunkBytes, sz, cudaMemcpyHostToDevice, xs_));
+            bytes += sz;
+            h_swap_[i] = cin;
+            h_swap_[k + i] = cout;
+            h_swap_[2 * k + i] = slot;
+        }
+        CK(cudaMemcpyAsync(d_swap_, h_swap_, 12ull * k, cudaMemcpyHostToDevice, xs_));
+        span(e0, xs_, t, PH_REPL);
+        CK(cudaEventRecord(ev_swapped_, xs_));
+        CK(cudaStreamWaitEvent(cs_, ev_swapped_, 0));
+        launch_apply_swaps(dev_state(t), d_slot_of_, d_swap_, k, g_.b_e, cs_);
+        CK(cudaGetLastError());
+        hot_dirty_ = true;
+        static_valid_ = false;   // the region no longer holds the front prefix (keep_static)
+    }
+    if (!iters.empty()) { iters.back().swaps = k; iters.back().replace_bytes = bytes; }
+    st.h2d_replace_bytes += bytes;
+    st.swaps_total += k;
+    host_s_ += std::chrono::duration<double>(std::chrono::steady_clock::now() - th0).count();
+}
+
 void Part::finalize(uint32_t t, bool dense) {
     // ---- next active set, after the static-hit kernels
     join_static();
@@ -635,9 +774,10 @@ void Part::end() {
     float ms = 0.f, fill_ms = 0.f;
     CK(cudaEventElapsedTime(&ms, ev_start_, ev_end));
     CK(cudaEventElapsedTime(&fill_ms, ev_fill0_, ev_fill1_));
-    double ph[PH_N] = {0, 0, 0, 0, 0, 0, 0};
+    double ph[PH_N] = {};
     const char* trace = std::getenv("ASCETIC_TRACE");
-    static const char* kPhName[PH_N] = {"classify", "static", "ondemand", "gather", "dma", "finalize", "exchange"};
+    static const char* kPhName[PH_N] = {"classify", "static", "ondemand", "gather", "dma", "finalize", "exchange",
+                                        "replace"};
     for (const Span& sp : spans_) {
         float a = 0.f;
         CK(cudaEventElapsedTime(&a, sp.a, sp.b));
@@ -655,6 +795,7 @@ void Part::end() {
                 case PH_OND: is.ms_ondemand += a; break;
                 case PH_GATHER: case PH_DMA: is.ms_h2d += a; break;
                 case PH_XCH: is.ms_exchange += a; break;
+                case PH_REPL: is.ms_h2d += a; break;
                 default: is.ms_finalize += a; break;
             }
         }
@@ -706,7 +847,8 @@ void Part::end() {
     st.time_dma_s = ph[PH_DMA] / 1e3;
     st.time_finalize_s = ph[PH_FIN] / 1e3;
     st.time_host_s = host_s_;
-    st.time_h2d_busy_s = (ph[PH_GATHER] + ph[PH_DMA] + fill_ms) / 1e3;
+    st.time_h2d_busy_s = (ph[PH_GATHER] + ph[PH_DMA] + ph[PH_REPL] + fill_ms) / 1e3;
+    st.time_replace_s = ph[PH_REPL] / 1e3;
     st.vertex_state_bytes = vertex_bytes_;
     st.kernel_launches = g_launches - launches0_;
 }
@@ -892,6 +1034,15 @@ void Engine::set_option(int opt, int64_t value) {
             o_.static_rear = (int)value;
             if (state_ == 2) state_ = 1;   // takes effect at the next set_budget
             break;
+        case ASCETIC_OPT_REPLACE_CHUNKS:
+            if (value < 0 || value > 65536) throw Error(ASCETIC_EINVAL, "replace chunks must be in [0, 65536]");
+            o_.replace_k = (uint32_t)value;
+            if (state_ == 2) state_ = 1;   // takes effect at the next set_budget
+            break;
+        case ASCETIC_OPT_REPLACE_POLICY:
+            if (value < 0 || value > 2) throw Error(ASCETIC_EINVAL, "replace policy: 0 = by algorithm, 1 = cumulative, 2 = last");
+            o_.replace_policy = (int)value;
+            break;
         case ASCETIC_OPT_STATIC_CTAS_PER_SM:
             if (value < 0 || value > 64) throw Error(ASCETIC_EINVAL, "static CTAs per SM must be in [0, 64]");
             o_.static_ctas_per_sm = (int)value;
@@ -941,6 +1092,7 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
     if ((algo == ALG_CC || algo == ALG_PR) && !(g_.flags & ASCETIC_SYMMETRIC))
         throw Error(ASCETIC_EINVAL, "CC and PR need ASCETIC_SYMMETRIC");
     if (g_.n == 0) throw Error(ASCETIC_EINVAL, "empty graph");
+    if (o_.replace_k && o_.repartition) throw Error(ASCETIC_EINVAL, "replacement (§3.4) and Eq. 3 re-partition are exclusive");
     CK(cudaSetDevice(device_));
     have_result_ = false;
     const bool multi = comm_.active();
@@ -996,6 +1148,7 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
             p0.span(e0, p0.cs(), t, PH_XCH);
             fork();
         }
+        for (auto& p : parts_) p->replace(t);   // §3.4 swaps, effective at t+1
     }
     if (multi && algo == ALG_PR) {
         join();
@@ -1029,6 +1182,9 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         st_.static_bytes += s.static_bytes;
         st_.vertex_state_bytes += s.vertex_state_bytes;
         st_.repartitions += s.repartitions;
+        st_.h2d_replace_bytes += s.h2d_replace_bytes;
+        st_.swaps_total += s.swaps_total;
+        st_.time_replace_s = std::max(st_.time_replace_s, s.time_replace_s);
         st_.kernel_launches = std::max(st_.kernel_launches, s.kernel_launches);
     }
     st_.iterations = t;

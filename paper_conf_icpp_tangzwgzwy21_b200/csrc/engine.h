@@ -61,6 +61,8 @@ struct Options {
     int prefetch = 1;             // PR: issue the next iteration's first chunk transfers early
     int repartition = 0;          // Eq. 3 adaptive re-partition (off, as in the paper's evaluation)
     int static_rear = 0;          // initial static content: 0 = front prefix, 1 = rear suffix
+    uint32_t replace_k = 0;       // §3.4 data replacement: chunk swaps examined per iteration (0 = off)
+    int replace_policy = 0;       // hotness counter: 0 = by algorithm, 1 = cumulative, 2 = last iteration
 };
 
 struct HostGraph {
@@ -74,7 +76,7 @@ struct HostGraph {
     void release();
 };
 
-enum { PH_CLS, PH_STATIC, PH_OND, PH_GATHER, PH_DMA, PH_FIN, PH_XCH, PH_N };
+enum { PH_CLS, PH_STATIC, PH_OND, PH_GATHER, PH_DMA, PH_FIN, PH_XCH, PH_REPL, PH_N };
 
 class Part {
   public:
@@ -93,6 +95,7 @@ class Part {
     void expand(uint32_t t, const IterTotals& T);
     void debug_classify(const uint32_t* active_words, uint64_t nwords, ascetic_classify_out_t* out);
     bool maybe_repartition(const IterTotals& T);   // Eq. 3; true = re-generate the data map
+    void replace(uint32_t t);                      // §3.4: hotness update + chunk swaps (effective at t+1)
     void join_static();   // cs waits for this iteration's static-hit kernels
     void finalize(uint32_t t, bool dense);
     void end();
@@ -177,6 +180,16 @@ class Part {
     cudaEvent_t ev_start_ = nullptr, ev_fill0_ = nullptr, ev_fill1_ = nullptr;
     double host_s_ = 0.0;
     unsigned long long launches0_ = 0;
+    // §3.4 data replacement: the Static Region as hNS_ slots of 16 KiB over the rank's hNC_ chunks
+    bool hot_ = false, hot_dirty_ = false, acc_pending_ = false, static_launched_ = false;
+    uint64_t hNC_ = 0, hNS_ = 0, hot_alloc_nc_ = 0;
+    uint32_t hot_alloc_k_ = 0;
+    uint32_t *d_slot_of_ = nullptr, *d_acc_ = nullptr, *d_swap_ = nullptr;
+    uint32_t *h_acc_ = nullptr, *h_swap_ = nullptr;     // pinned
+    std::vector<uint32_t> slot_of_, slot_chunk_;       // host mirror: chunk -> slot, slot -> chunk
+    std::vector<uint64_t> hot_h_;                      // HotnessTable (Fig. 6)
+    cudaEvent_t ev_acc_ = nullptr, ev_swapped_ = nullptr;
+    void free_hot();
     // DMA planning scratch
     std::vector<uint32_t> rb_, re_;
     std::vector<unsigned long long> rdst_;

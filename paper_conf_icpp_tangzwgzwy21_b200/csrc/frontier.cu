@@ -177,6 +177,8 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
     ScanVal wagg = sv_warp_sum(mine);
     {
         unsigned long long nA = __popc(myAll), nH = __popc(myA & myS), nM = __popc(myMiss);
+        unsigned long long nS = wsum64((unsigned long long)__popc(myS & own_mask(myw, a.vlo, a.vhi)));
+        if (lane == 0 && nS) atomicAdd(&a.tot->nS, nS);
         unsigned long long dg = (myw < a.nwords) ? mix64((unsigned long long)myw ^ ((unsigned long long)myAll * PHI)) : 0ull;
         nA = wsum64(nA); nH = wsum64(nH); nM = wsum64(nM); dg = wsum64(dg);
         aArcs = wsum64(aArcs); hArcs = wsum64(hArcs);
@@ -336,7 +338,7 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
             const ScanVal fin = sv_load_volatile(&a.tile_incl[a.ntiles - 1]);
             volatile IterTotals* vt = a.tot;
             IterTotals* h = a.host_tot;
-            h->nA = vt->nA; h->nH = vt->nH; h->nM = vt->nM;
+            h->nA = vt->nA; h->nH = vt->nH; h->nM = vt->nM; h->nS = vt->nS;
             h->active_arcs = vt->active_arcs; h->hit_arcs = vt->hit_arcs; h->digest = vt->digest;
             h->miss_arcs = fin.miss_arcs;
             h->n_small = fin.small; h->n_med = fin.med; h->n_hub = fin.hub;

@@ -41,7 +41,7 @@ def _record(t, rank, A, stat, lo, hi, deg, b_e, digest):
     d = deg[lo:hi]
     return dict(t=t, rank=rank, nA=int(A.sum()), nH=int(h.sum()), nM=int(m.sum()), nruns=_runs(m),
                 active_arcs=int(d[a].sum()), hit_arcs=int(d[h].sum()), miss_bytes=int(b_e * d[m].sum()),
-                digest=digest, s=int(stat[lo:hi].sum()))
+                digest=digest, s=int(stat[lo:hi].sum()), swaps=0, replace_bytes=0)
 
 
 def _or_allgather(mask):
