@@ -73,7 +73,8 @@ def _load():
         lib.or_run_hot.argtypes = [ctypes.c_int, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint32,
                                    ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
                                    ctypes.POINTER(_Iter), ctypes.c_uint32, ctypes.POINTER(_Summary), ctypes.c_void_p,
-                                   ctypes.c_uint32, ctypes.c_int]
+                                   ctypes.c_uint32, ctypes.c_int, ctypes.c_int, ctypes.c_uint64]
+        lib.or_random_chunks.argtypes = [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_void_p]
         lib.or_threads.restype = ctypes.c_int
         lib.or_classify.argtypes = [ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p,
                                     ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
@@ -204,10 +205,12 @@ def run(algo: str | int, off: np.ndarray, nbr: np.ndarray, src: int = 0, max_ite
 
 
 def run_hot(algo: str | int, off: np.ndarray, nbr: np.ndarray, static_bytes, src: int = 0, max_iters: int = 0,
-            kswap: int = 0, policy: str | None = None, bounds: np.ndarray | None = None) -> Result:
+            kswap: int = 0, policy: str | None = None, bounds: np.ndarray | None = None,
+            random_seed: int | None = None) -> Result:
     """Run with the §3.4 data replacement: 16 KiB chunks, hotness counters, up to
     `kswap` chunk swaps per iteration and rank. static_bytes = Ms (int, or one per rank).
-    policy: "cumulative" (default for bfs/sssp/cc) or "last" (default for pr), P:946-950."""
+    policy: "cumulative" (default for bfs/sssp/cc) or "last" (default for pr), P:946-950.
+    random_seed: start from the seeded random chunk set (§5 random initial content) instead of the front."""
     lib = _load()
     a = ALGOS[algo] if isinstance(algo, str) else algo
     if policy is None:
@@ -228,10 +231,18 @@ def run_hot(algo: str | int, off: np.ndarray, nbr: np.ndarray, static_bytes, src
     rc = lib.or_run_hot(a, n, off.ctypes.data, nbr.ctypes.data if nbr.size else None, src, max_iters, P,
                         b.ctypes.data if b is not None else None, res_u.ctypes.data if n else None,
                         res_f.ctypes.data if n else None, recs, cap, ctypes.byref(s), ms.ctypes.data, kswap,
-                        1 if policy == "cumulative" else 0)
+                        1 if policy == "cumulative" else 0, 0 if random_seed is None else 1,
+                        0 if random_seed is None else int(random_seed))
     if rc != 0:
         raise ValueError(f"oracle rejected arguments (rc={rc})")
     records = [{f: int(getattr(recs[i], f)) for f in ITER_FIELDS} for i in range(s.nrec)]
     vals = res_f.copy() if a == PR else res_u.copy()
     return Result(vals, int(s.iterations), records, int(s.h2d_payload), int(s.active_arcs_total), 0,
                   int(s.h2d_replace))
+
+
+def random_chunks(nc: int, ns: int, seed: int) -> np.ndarray:
+    """Resident flags of the seeded random initial Static Region (ns of nc 16 KiB chunks)."""
+    res = np.zeros(max(nc, 1), dtype=np.uint8)
+    _load().or_random_chunks(nc, ns, seed, res.ctypes.data)
+    return res[:nc].astype(bool)

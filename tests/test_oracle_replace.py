@@ -72,7 +72,7 @@ def test_replace_pr_last_iteration_counter_never_swaps():
     assert r2.replace_bytes == 0
 
 
-def restated_bfs_replacement(off, nbr, src, Ms, K):
+def restated_bfs_replacement(off, nbr, src, Ms, K, res0=None):
     """§3.4 restated with numpy over scipy's BFS level sets (independent of oracle.c's loops)."""
     n = off.size - 1
     A = sp.csr_matrix((np.ones(nbr.size), nbr.astype(np.int64), off.astype(np.int64)), shape=(n, n))
@@ -83,6 +83,8 @@ def restated_bfs_replacement(off, nbr, src, Ms, K):
     NC = (D + CHUNK - 1) // CHUNK
     res = np.zeros(NC, dtype=bool)
     res[:(Ms + CHUNK - 1) // CHUNK] = True
+    if res0 is not None:
+        res = np.array(res0, dtype=bool)
     h = np.zeros(NC, dtype=np.int64)
     a_byte, e_byte = 4 * o[:-1], 4 * o[1:]
     deg = o[1:] - o[:-1]
@@ -168,3 +170,28 @@ def test_replace_multi_rank_k0_matches_front_and_splits():
     k8 = oracle.run_hot("bfs", g.off, g.nbr, static_bytes=ms, src=src, kswap=8, bounds=b)
     np.testing.assert_array_equal(front.values, k8.values)
     assert [r["rank"] for r in k8.records[:P]] == list(range(P))
+
+
+@pytest.mark.parametrize("nc,ns,seed", [(1, 1, 1), (10, 3, 1), (1000, 250, 7), (5000, 4999, 3), (64, 0, 2)])
+def test_random_chunks_are_the_smallest_keys(nc, ns, seed):
+    """§5 random initial content: the ns chunks with the smallest
+    splitmix64((seed << 32) ^ c) keys (the digest's splitmix, pinned in tests/pins.py)."""
+    res = oracle.random_chunks(nc, ns, seed)
+    assert res.sum() == min(ns, nc)
+    keys = np.array([pins.splitmix(((seed << 32) ^ c) & pins.M64) for c in range(nc)], dtype=object)
+    if 0 < ns < nc:
+        assert max(keys[res]) < min(keys[~res])
+
+
+@pytest.mark.parametrize("seed,K", [(1, 0), (5, 0), (2, 8)])
+def test_random_initial_content_vs_restatement(seed, K):
+    g = gg.rmat(12, seed=12)
+    src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+    p = oracle.placer(g.off, 4, g.csr_bytes, frac=0.35)
+    nc = (4 * g.m + CHUNK - 1) // CHUNK
+    res0 = oracle.random_chunks(nc, (p.Ms + CHUNK - 1) // CHUNK, seed)
+    got = oracle.run_hot("bfs", g.off, g.nbr, static_bytes=p.Ms, src=src, kswap=K, random_seed=seed)
+    assert got.records == restated_bfs_replacement(g.off, g.nbr, src, p.Ms, K, res0=res0)
+    front = oracle.run_hot("bfs", g.off, g.nbr, static_bytes=p.Ms, src=src, kswap=K)
+    np.testing.assert_array_equal(got.values, front.values)
+    assert got.records[0]["s"] != front.records[0]["s"]      # a different static set

@@ -28,10 +28,11 @@ def main():
         src = gg.sources(g, 1, seed=c["seed"])[0]
         asc.load_csr(g.off, g.nbr, pairs=g.pairs)
 
-        def one(label, nbytes, frac, overlap=1, rear=0, eq3=0):
+        def one(label, nbytes, frac, overlap=1, rear=0, eq3=0, replace=0):
             asc.set_option("overlap", overlap)
             asc.set_option("static_placement", rear)
             asc.set_option("repartition", eq3)
+            asc.set_option("replace_chunks", replace)
             asc.set_budget(nbytes, frac)
             best = None
             for _ in range(2):
@@ -45,31 +46,43 @@ def main():
                      gteps=round(best["active_arcs_total"] / best["time_run_s"] / 1e9, 3),
                      fill_gb=round(best["h2d_static_fill_bytes"] / 1e9, 3),
                      miss_gb=round(best["h2d_payload_bytes"] / 1e9, 3),
-                     h2d_gb=round((best["h2d_static_fill_bytes"] + best["h2d_payload_bytes"]) / 1e9, 3))
+                     replace_k=replace, swaps=best["swaps_total"], replace_gb=round(best["h2d_replace_bytes"] / 1e9, 3),
+                     replace_ms=round(best["time_replace_s"] * 1e3, 2), host_ms=round(best["time_host_s"] * 1e3, 2),
+                     h2d_gb=round((best["h2d_static_fill_bytes"] + best["h2d_payload_bytes"]
+                                   + best["h2d_replace_bytes"]) / 1e9, 3))
             rows.append(r)
             print(json.dumps(r), flush=True)
 
+        only = os.environ.get("ABLATION_ONLY", "")
         one("eq2", budget, -1.0)
-        if os.environ.get("ABLATION_QUICK") != "1":
+        if only == "replace":
+            # §3.4 data replacement: K chunk swaps per iteration, counter by algorithm
+            for K in [16, 256, 4096, 65536]:
+                one("replace", budget, -1.0, replace=K)
+        elif os.environ.get("ABLATION_QUICK") != "1":
             for R in [0.0, 0.2, 0.4, 0.6, 0.8, 0.9, 0.95, 1.0]:
                 one("R-sweep", budget, R)
             one("overlap-off", budget, -1.0, overlap=0)
             for f in [0.25, 0.5, 0.75, 1.0]:
                 one("budget-sweep", int(f * g.csr_bytes), -1.0)
-        one("rear-fill", budget, -1.0, rear=1)
-        one("eq3-repartition", budget, -1.0, eq3=1)
+        if only != "replace":
+            one("rear-fill", budget, -1.0, rear=1)
+            one("eq3-repartition", budget, -1.0, eq3=1)
         asc.set_option("overlap", 1)
+        asc.set_option("replace_chunks", 0)
         asc.set_option("static_placement", 0)
         asc.set_option("repartition", 0)
         asc.unload()
         del g
     out = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "gpurun_out", "ablation.md")
     with open(out, "w") as f:
-        f.write("| config | study | budget/CSR | R | overlap | run ms | GTEPS | fill GB | miss GB | H2D GB |\n")
-        f.write("|---|---|---|---|---|---|---|---|---|---|\n")
+        f.write("| config | study | budget/CSR | R | overlap | K | run ms | GTEPS | fill GB | miss GB | swaps | "
+                "replace GB | replace ms | host ms | H2D GB |\n")
+        f.write("|---|---|---|---|---|---|---|---|---|---|---|---|---|---|---|\n")
         for r in rows:
             f.write(f"| {r['config']} | {r['study']} | {r['budget_frac_of_csr']} | {r['R']} | {r['overlap']} | "
-                    f"{r['run_ms']} | {r['gteps']} | {r['fill_gb']} | {r['miss_gb']} | {r['h2d_gb']} |\n")
+                    f"{r['replace_k']} | {r['run_ms']} | {r['gteps']} | {r['fill_gb']} | {r['miss_gb']} | "
+                    f"{r['swaps']} | {r['replace_gb']} | {r['replace_ms']} | {r['host_ms']} | {r['h2d_gb']} |\n")
     print(open(out).read())
 
 
