@@ -77,7 +77,10 @@ typedef enum {
                                       by M_static*V/D (floored to 16 KiB) and re-generate the map. Default 0, as
                                       in the paper's evaluation. Changes per-iteration bytes. */
     ASCETIC_OPT_STATIC_PLACEMENT = 13, /* initial static content (§5): 0 = front prefix (default),
-                                      1 = rear suffix of whole lists fitting in Ms. Set before set_budget. */
+                                      1 = rear suffix of whole lists fitting in Ms, 2 = random: the
+                                      ceil(Ms/16 KiB) chunks with the smallest splitmix64((seed<<32) ^ c)
+                                      (Static Region as 16 KiB slots, as with REPLACE_CHUNKS). Set before
+                                      set_budget. */
     ASCETIC_OPT_REPLACE_CHUNKS = 14, /* §3.4 data replacement (Fig. 6): K = 16 KiB chunk swaps
                                       examined per iteration and rank (0 = off, the default; max 65536).
                                       The Static Region becomes Ms/16 KiB chunk slots (initially the front
@@ -85,10 +88,12 @@ typedef enum {
                                       counters (active arcs read) update the hotness table; during on-demand
                                       computing the K hottest non-resident chunks replace the K coldest
                                       resident ones while strictly hotter, effective next iteration. A vertex
-                                      is static iff every chunk its list touches is resident. Front placement
-                                      only; exclusive with Eq. 3. Set before set_budget. Changes bytes. */
-    ASCETIC_OPT_REPLACE_POLICY = 15 /* hotness counter: 0 = by algorithm (default: cumulative for
+                                      is static iff every chunk its list touches is resident. Front
+                                      or random placement; exclusive with Eq. 3. Set before set_budget.
+                                      Changes bytes. */
+    ASCETIC_OPT_REPLACE_POLICY = 15, /* hotness counter: 0 = by algorithm (default: cumulative for
                                       BFS/SSSP/CC, last iteration for PR), 1 = cumulative, 2 = last iteration */
+    ASCETIC_OPT_PLACEMENT_SEED = 16  /* seed of the random initial content (default 1). Set before set_budget. */
 } ascetic_option;
 
 typedef struct {

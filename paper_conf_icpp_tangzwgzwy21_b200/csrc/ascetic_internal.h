@@ -136,6 +136,12 @@ void launch_chunk_access(const DevState& d, const Queues& q, uint32_t n_small, u
 // §3.4: apply swaps (in[i] gets out[i]'s slot) and recompute S for the vertices touching the changed chunks
 void launch_apply_swaps(const DevState& d, uint32_t* slot_of, const uint32_t* swaps /* in[k], out[k], slot[k] */,
                         uint32_t k, uint32_t b_e, cudaStream_t s);
+// copy `count` 16 KiB chunks ids[i] of the rank's payload (host bytes x0 + 16 KiB * id, the last
+// chunk clipped at D) from the mapped host CSR into slot slots[i] (or i) of the Static Region
+void launch_copy_chunks(const void* host_dev, uint64_t x0, uint64_t D, const uint32_t* ids, const uint32_t* slots,
+                        uint32_t count, void* dst, cudaStream_t s);
+// S := {v in [vlo, vhi) : every chunk of v's list is resident} (full rebuild)
+void launch_static_bits(const DevState& d, const uint32_t* slot_of, uint32_t b_e, cudaStream_t s);
 // dense = values were exchanged (P > 1): SSSP/CC rebuild A from val < snap over all vertices
 void launch_finalize(int algo, const DevState& d, bool dense, cudaStream_t s);
 // collectives' device side (comm.cu drives them)

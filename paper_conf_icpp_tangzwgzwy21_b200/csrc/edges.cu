@@ -723,6 +723,53 @@ __global__ void __launch_bounds__(256) k_static_rebits(DevState d, const uint32_
     }
 }
 
+// S over the owned range from the chunk residency (random initial content): one warp per
+// 32-vertex word, the word written whole (a part's S holds only its own range's bits)
+__global__ void __launch_bounds__(256) k_static_bits_all(DevState d, const uint32_t* __restrict__ slot_of,
+                                                         uint32_t epc_shift) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t w0 = d.vlo >> 5, w1 = (d.vhi + 31) >> 5;
+    const uint64_t nw = (uint64_t)gridDim.x * blockDim.x >> 5;
+    for (uint64_t w = w0 + ((blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5); w < w1; w += nw) {
+        const uint64_t v = w * 32 + lane;
+        bool st = false;
+        if (v >= d.vlo && v < d.vhi)
+            st = chunks_resident(slot_of, __ldg(d.off + v) - d.static_arc0, __ldg(d.off + v + 1) - d.static_arc0,
+                                 epc_shift);
+        const uint32_t word = __ballot_sync(FULL, st);
+        if (lane == 0) d.S[w] = word;
+    }
+}
+
+// Chunk copy (random fill, §3.4 swaps): CTA i copies chunk ids[i] (16 KiB, clipped at D) from the
+// mapped host CSR to its slot; 16 B loads when the rank's payload start is 16-byte aligned,
+// 4 B otherwise; all of a thread's loads are issued before its stores.
+__global__ void __launch_bounds__(256) k_copy_chunks(const char* __restrict__ host, unsigned long long x0,
+                                                     unsigned long long D, const uint32_t* __restrict__ ids,
+                                                     const uint32_t* __restrict__ slots, uint32_t count,
+                                                     char* __restrict__ dst) {
+    for (uint32_t i = blockIdx.x; i < count; i += gridDim.x) {
+        const unsigned long long c = ids[i], slot = slots ? slots[i] : i;
+        const unsigned long long o = c << kChunkShift;
+        const unsigned long long len = min((unsigned long long)kChunkBytes, D - o);
+        const char* src = host + x0 + o;
+        char* out = dst + (slot << kChunkShift);
+        if ((x0 & 15ull) == 0 && len == kChunkBytes) {
+            const uint4* s4 = reinterpret_cast<const uint4*>(src);
+            uint4* d4 = reinterpret_cast<uint4*>(out);
+            uint4 v[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) v[j] = s4[threadIdx.x + 256 * j];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) d4[threadIdx.x + 256 * j] = v[j];
+        } else {
+            const uint32_t* s1 = reinterpret_cast<const uint32_t*>(src);
+            uint32_t* d1 = reinterpret_cast<uint32_t*>(out);
+            for (unsigned long long j = threadIdx.x; j < len / 4; j += blockDim.x) d1[j] = s1[j];
+        }
+    }
+}
+
 inline unsigned blocks_for(unsigned long long n, int per_block, unsigned cap = 148u * 16u) {
     unsigned long long b = (n + per_block - 1) / per_block;
     if (b < 1) b = 1;
@@ -776,6 +823,23 @@ void launch_apply_swaps(const DevState& d, uint32_t* slot_of, const uint32_t* sw
     k_apply_swaps<<<blocks_for(k, 256), 256, 0, s>>>(slot_of, sw, k);
     k_static_rebits<<<(2 * k + 7) / 8, 256, 0, s>>>(d, slot_of, sw, 2 * k, epc_shift);
     g_launches += 2;
+}
+
+void launch_copy_chunks(const void* host_dev, uint64_t x0, uint64_t D, const uint32_t* ids, const uint32_t* slots,
+                        uint32_t count, void* dst, cudaStream_t s) {
+    if (!count) return;
+    // 64 CTAs x 16 KiB = 1 MiB of host reads in flight (the transfer engine's sizing)
+    k_copy_chunks<<<count < 64u ? count : 64u, 256, 0, s>>>(reinterpret_cast<const char*>(host_dev), x0, D, ids, slots,
+                                                          count, reinterpret_cast<char*>(dst));
+    ++g_launches;
+}
+
+void launch_static_bits(const DevState& d, const uint32_t* slot_of, uint32_t b_e, cudaStream_t s) {
+    const uint32_t epc_shift = kChunkShift - (b_e == 8 ? 3 : 2);
+    const unsigned long long words = ((d.vhi + 31) >> 5) - (d.vlo >> 5);
+    if (!words) return;
+    k_static_bits_all<<<blocks_for(words, 8), 256, 0, s>>>(d, slot_of, epc_shift);
+    ++g_launches;
 }
 
 void launch_ondemand(int algo, const DevState& d, const Queues& q, const void* chunk,

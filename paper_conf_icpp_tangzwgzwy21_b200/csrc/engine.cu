@@ -254,7 +254,7 @@ void Part::set_budget(uint64_t bytes, double frac) {
     Placement p = place(g_.off.data() + vlo_, vhi_ - vlo_, g_.b_e, bytes, frac);
     const uint64_t own = vhi_ - vlo_;
     stat_lo_ = vlo_;
-    if (o_.static_rear) {
+    if (o_.placement == 1) {
         // rear initial content (§5): the suffix of whole lists that fits in Ms,
         // s_lo = min{v : b_e (off[vhi] - off[v]) <= Ms}
         const uint64_t* off = g_.off.data();
@@ -290,32 +290,55 @@ void Part::set_budget(uint64_t bytes, double frac) {
     s_cur_ = p.s;
     layout_regions(p.Ms);
     launch_set_range_bits(d_S_, nwords_, stat_lo_, stat_lo_ + p.s, cs_);   // StaticBitmap
-    // §3.4 data replacement: the Static Region becomes ceil(Ms / 16 KiB) chunk slots, initially the
-    // front chunks (filled whole); only meaningful when some lists stay outside it
-    hot_ = o_.replace_k > 0 && p.s < own && p.Ms > 0;
+    // §3.4 data replacement and the random initial content (§5): the Static Region
+    // becomes ceil(Ms / 16 KiB) chunk slots, filled whole; only meaningful when some lists stay
+    // outside it
+    if (o_.replace_k > 0 && o_.placement == 1) throw Error(ASCETIC_EINVAL, "replacement needs the front or random placement");
+    hot_ = (o_.replace_k > 0 || o_.placement == 2) && p.s < own && p.Ms > 0;
     if (hot_) {
-        if (o_.static_rear) throw Error(ASCETIC_EINVAL, "replacement needs the front initial placement");
         hNC_ = (p.D + kChunkBytes - 1) / kChunkBytes;
         hNS_ = (p.Ms + kChunkBytes - 1) / kChunkBytes;
         if (hNC_ > 0xFFFFFFF0ull) throw Error(ASCETIC_EINVAL, "too many 16 KiB chunks for replacement");
+        init_chunks_.resize(hNS_);
+        if (o_.placement == 2) {
+            // the hNS_ chunks with the smallest splitmix64((seed << 32) ^ c), ties by c (DESIGN R27)
+            std::vector<std::pair<uint64_t, uint32_t>> key(hNC_);
+            for (uint64_t c = 0; c < hNC_; ++c) {
+                uint64_t z = (o_.placement_seed << 32) ^ c;
+                z += 0x9E3779B97F4A7C15ull;
+                z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+                z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+                key[c] = {z ^ (z >> 31), (uint32_t)c};
+            }
+            std::nth_element(key.begin(), key.begin() + (hNS_ - 1), key.end());
+            for (uint64_t i = 0; i < hNS_; ++i) init_chunks_[i] = key[i].second;
+            std::sort(init_chunks_.begin(), init_chunks_.end());
+        } else {
+            for (uint64_t i = 0; i < hNS_; ++i) init_chunks_[i] = (uint32_t)i;
+        }
+        init_fill_bytes_ = 0;
+        for (uint32_t c : init_chunks_) init_fill_bytes_ += std::min<uint64_t>(kChunkBytes, p.D - (uint64_t)c * kChunkBytes);
         if (hNC_ != hot_alloc_nc_ || o_.replace_k != hot_alloc_k_) {
             free_hot();
             dalloc(&d_slot_of_, hNC_, nullptr);
             dalloc(&d_acc_, hNC_, nullptr);
-            dalloc(&d_swap_, 3ull * o_.replace_k, nullptr);
+            dalloc(&d_init_, hNC_, nullptr);
+            dalloc(&d_swap_, 3ull * std::max<uint32_t>(o_.replace_k, 1), nullptr);
             cudaError_t e = cudaHostAlloc((void**)&h_acc_, hNC_ * 4, cudaHostAllocPortable);
-            if (e == cudaSuccess) e = cudaHostAlloc((void**)&h_swap_, 12ull * o_.replace_k, cudaHostAllocPortable);
+            if (e == cudaSuccess)
+                e = cudaHostAlloc((void**)&h_swap_, 12ull * std::max<uint32_t>(o_.replace_k, 1), cudaHostAllocPortable);
             if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_EHOSTMEM, "cudaHostAlloc (replacement tables)"); }
             hot_alloc_nc_ = hNC_;
             hot_alloc_k_ = o_.replace_k;
         }
+        CK(cudaMemcpyAsync(d_init_, init_chunks_.data(), hNS_ * 4, cudaMemcpyHostToDevice, cs_));
         hot_dirty_ = true;   // begin() installs the initial slots
     }
     CK(cudaStreamSynchronize(cs_));
 }
 
 void Part::free_hot() {
-    dfree(d_slot_of_); dfree(d_acc_); dfree(d_swap_);
+    dfree(d_slot_of_); dfree(d_acc_); dfree(d_swap_); dfree(d_init_);
     if (h_acc_) cudaFreeHost(h_acc_);
     if (h_swap_) cudaFreeHost(h_swap_);
     h_acc_ = h_swap_ = nullptr;
@@ -328,7 +351,7 @@ void Part::free_hot() {
 // 0.5 V / D), shrink the Static Region by M_static * V / D (floored to 16 KiB) and
 // hand that memory to the On-demand Region; the caller re-generates the data map.
 bool Part::maybe_repartition(const IterTotals& T) {
-    if (ms_cur_ == 0 || pl_.D == 0 || o_.static_rear) return false;   // Eq. 3 shrinks a front prefix
+    if (ms_cur_ == 0 || pl_.D == 0 || o_.placement != 0) return false;   // Eq. 3 shrinks a front prefix
     const double b_e = g_.b_e;
     const double V = b_e * (double)T.active_arcs, Vs = b_e * (double)T.hit_arcs, Vo = b_e * (double)T.miss_arcs;
     const double D = (double)pl_.D, Ms = (double)ms_cur_;
@@ -430,11 +453,12 @@ void Part::begin(int algo, uint32_t source, uint32_t max_iters, bool timing) {
         // every run starts from the front chunks [0, hNS_) in slots [0, hNS_) and a zero hotness table
         if (hot_dirty_) {
             slot_of_.assign(hNC_, kNoSlot);
-            slot_chunk_.resize(hNS_);
-            for (uint64_t c = 0; c < hNS_; ++c) { slot_of_[c] = (uint32_t)c; slot_chunk_[c] = (uint32_t)c; }
+            slot_chunk_ = init_chunks_;
+            for (uint64_t i = 0; i < hNS_; ++i) slot_of_[init_chunks_[i]] = (uint32_t)i;
             CK(cudaMemcpyAsync(d_slot_of_, slot_of_.data(), hNC_ * 4, cudaMemcpyHostToDevice, cs_));
             CK(cudaStreamSynchronize(cs_));
-            launch_set_range_bits(d_S_, nwords_, stat_lo_, stat_lo_ + pl_.s, cs_);
+            if (o_.placement == 2) launch_static_bits(dev_state(0), d_slot_of_, g_.b_e, cs_);
+            else launch_set_range_bits(d_S_, nwords_, stat_lo_, stat_lo_ + pl_.s, cs_);
             static_valid_ = false;
             hot_dirty_ = false;
         }
@@ -452,11 +476,18 @@ void Part::begin(int algo, uint32_t source, uint32_t max_iters, bool timing) {
     // ---- static fill: ONE DMA of this rank's front prefix, counted in the run
     CK(cudaStreamWaitEvent(xs_, ev_start_, 0));
     CK(cudaEventRecord(ev_fill0_, xs_));
-    // with replacement the slots are filled whole: Ms bytes (the chunk holding the prefix end too)
-    const uint64_t fill = hot_ ? pl_.Ms : pl_.static_bytes;
+    // with slots the chunks are filled whole: Ms bytes for the front chunks (one DMA), the chosen
+    // chunks for the random content (one zero-copy chunk-copy kernel)
+    const uint64_t fill = hot_ ? init_fill_bytes_ : pl_.static_bytes;
     if (fill && !(o_.keep_static && static_valid_)) {
-        CK(cudaMemcpyAsync(d_static_, (const char*)g_.nbr + g_.off[stat_lo_] * g_.b_e, fill,
-                           cudaMemcpyHostToDevice, xs_));
+        if (hot_ && o_.placement == 2) {
+            launch_copy_chunks(g_.nbr_dev, g_.off[vlo_] * (uint64_t)g_.b_e, pl_.D, d_init_, nullptr, (uint32_t)hNS_,
+                               d_static_, xs_);
+            CK(cudaGetLastError());
+        } else {
+            CK(cudaMemcpyAsync(d_static_, (const char*)g_.nbr + g_.off[stat_lo_] * g_.b_e, fill,
+                               cudaMemcpyHostToDevice, xs_));
+        }
         st.h2d_static_fill_bytes = fill;
         static_valid_ = true;
     }
@@ -534,7 +565,7 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     static_launched_ = false;
     // §3.4: this iteration's accesses per 16 KiB chunk -> pinned host table, read by
     // replace() while the on-demand chunks stream (the server thread of Fig. 6)
-    if (hot_ && !(max_iters_ && t + 1 == max_iters_)) {
+    if (hot_ && o_.replace_k > 0 && !(max_iters_ && t + 1 == max_iters_)) {
         CK(cudaMemsetAsync(d_acc_, 0, hNC_ * 4, cs_));
         launch_chunk_access(d, q, T.n_small, T.n_med, T.n_hub, b_e, d_acc_, cs_);
         CK(cudaGetLastError());
@@ -689,7 +720,7 @@ void Part::join_static() {
 // the copy stream after this iteration's miss chunks and static-hit kernels; slot table and
 // StaticBitmap are updated on the compute stream before the next GenDataMap.
 void Part::replace(uint32_t t) {
-    if (!acc_pending_) return;
+    if (!acc_pending_ || o_.replace_k == 0) return;
     acc_pending_ = false;
     const auto th0 = std::chrono::steady_clock::now();
     CK(cudaEventSynchronize(ev_acc_));
@@ -732,15 +763,16 @@ void Part::replace(uint32_t t) {
             slot_of_[cin] = slot;
             slot_of_[cout] = kNoSlot;
             slot_chunk_[slot] = cin;
-            const uint64_t sz = std::min<uint64_t>(kChunkBytes, pl_.D - (uint64_t)cin * kChunkBytes);
-            CK(cudaMemcpyAsync((char*)d_static_ + (uint64_t)slot * kChunkBytes,
-                               (const char*)g_.nbr + x0 + (uint64_t)cin * kChunkBytes, sz, cudaMemcpyHostToDevice, xs_));
-            bytes += sz;
+            bytes += std::min<uint64_t>(kChunkBytes, pl_.D - (uint64_t)cin * kChunkBytes);
             h_swap_[i] = cin;
             h_swap_[k + i] = cout;
             h_swap_[2 * k + i] = slot;
         }
+        // the swap list, then one zero-copy kernel copying the K incoming 16 KiB chunks from the
+        // pinned host CSR into their slots (16 KiB contiguous reads run at the link's rate)
         CK(cudaMemcpyAsync(d_swap_, h_swap_, 12ull * k, cudaMemcpyHostToDevice, xs_));
+        launch_copy_chunks(g_.nbr_dev, x0, pl_.D, d_swap_, d_swap_ + 2 * k, k, d_static_, xs_);
+        CK(cudaGetLastError());
         span(e0, xs_, t, PH_REPL);
         CK(cudaEventRecord(ev_swapped_, xs_));
         CK(cudaStreamWaitEvent(cs_, ev_swapped_, 0));
@@ -830,7 +862,7 @@ void Part::end() {
     st.iterations = (uint32_t)iters.size();
     st.n = g_.n; st.m = g_.m; st.b_e = g_.b_e;
     st.rank = (uint32_t)rank_;
-    st.s = pl_.s;
+    st.s = iters.empty() ? pl_.s : iters[0].s_static;   // static vertices at the start of the run
     st.budget_bytes = pl_.B;
     st.static_reserved = pl_.Ms;
     st.static_bytes = pl_.static_bytes;
@@ -1030,14 +1062,18 @@ void Engine::set_option(int opt, int64_t value) {
         case ASCETIC_OPT_PREFETCH: o_.prefetch = value ? 1 : 0; break;
         case ASCETIC_OPT_REPARTITION: o_.repartition = value ? 1 : 0; break;
         case ASCETIC_OPT_STATIC_PLACEMENT:
-            if (value < 0 || value > 1) throw Error(ASCETIC_EINVAL, "static placement: 0 = front, 1 = rear");
-            o_.static_rear = (int)value;
+            if (value < 0 || value > 2) throw Error(ASCETIC_EINVAL, "static placement: 0 = front, 1 = rear, 2 = random");
+            o_.placement = (int)value;
             if (state_ == 2) state_ = 1;   // takes effect at the next set_budget
             break;
         case ASCETIC_OPT_REPLACE_CHUNKS:
             if (value < 0 || value > 65536) throw Error(ASCETIC_EINVAL, "replace chunks must be in [0, 65536]");
             o_.replace_k = (uint32_t)value;
             if (state_ == 2) state_ = 1;   // takes effect at the next set_budget
+            break;
+        case ASCETIC_OPT_PLACEMENT_SEED:
+            o_.placement_seed = (uint64_t)value;
+            if (state_ == 2) state_ = 1;
             break;
         case ASCETIC_OPT_REPLACE_POLICY:
             if (value < 0 || value > 2) throw Error(ASCETIC_EINVAL, "replace policy: 0 = by algorithm, 1 = cumulative, 2 = last");
@@ -1093,6 +1129,7 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         throw Error(ASCETIC_EINVAL, "CC and PR need ASCETIC_SYMMETRIC");
     if (g_.n == 0) throw Error(ASCETIC_EINVAL, "empty graph");
     if (o_.replace_k && o_.repartition) throw Error(ASCETIC_EINVAL, "replacement (§3.4) and Eq. 3 re-partition are exclusive");
+    if (o_.repartition && o_.placement != 0) throw Error(ASCETIC_EINVAL, "Eq. 3 re-partition shrinks a front prefix");
     CK(cudaSetDevice(device_));
     have_result_ = false;
     const bool multi = comm_.active();

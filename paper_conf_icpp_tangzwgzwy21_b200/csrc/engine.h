@@ -60,7 +60,8 @@ struct Options {
     int static_ctas_per_sm = 0;   // persistent grid of the static-hit kernels (0 = 4 per SM)
     int prefetch = 1;             // PR: issue the next iteration's first chunk transfers early
     int repartition = 0;          // Eq. 3 adaptive re-partition (off, as in the paper's evaluation)
-    int static_rear = 0;          // initial static content: 0 = front prefix, 1 = rear suffix
+    int placement = 0;            // initial static content: 0 = front prefix, 1 = rear suffix, 2 = random chunks
+    uint64_t placement_seed = 1;  // seed of the random initial chunk set
     uint32_t replace_k = 0;       // §3.4 data replacement: chunk swaps examined per iteration (0 = off)
     int replace_policy = 0;       // hotness counter: 0 = by algorithm, 1 = cumulative, 2 = last iteration
 };
@@ -187,6 +188,9 @@ class Part {
     uint32_t *d_slot_of_ = nullptr, *d_acc_ = nullptr, *d_swap_ = nullptr;
     uint32_t *h_acc_ = nullptr, *h_swap_ = nullptr;     // pinned
     std::vector<uint32_t> slot_of_, slot_chunk_;       // host mirror: chunk -> slot, slot -> chunk
+    std::vector<uint32_t> init_chunks_;                // initial resident chunks, ascending (slot i = init_chunks_[i])
+    uint32_t* d_init_ = nullptr;                       // device copy of init_chunks_ (fill list)
+    uint64_t init_fill_bytes_ = 0;
     std::vector<uint64_t> hot_h_;                      // HotnessTable (Fig. 6)
     cudaEvent_t ev_acc_ = nullptr, ev_swapped_ = nullptr;
     void free_hot();

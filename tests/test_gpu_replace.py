@@ -22,7 +22,7 @@ def asc():
     m.unload()
     yield m
     for k, v in [("replace_chunks", 0), ("replace_policy", 0), ("chunk_cap", 0), ("xfer_mode", 0),
-                 ("hub_degree", 2048)]:
+                 ("hub_degree", 2048), ("static_placement", 0), ("placement_seed", 1)]:
         m.set_option(k, v)
     m.unload()
     m.emulate_ranks(1)
@@ -160,3 +160,49 @@ def test_replace_rejects_rear_and_eq3(asc):
     with pytest.raises(asc.AsceticError):
         asc.run("bfs", 0)
     asc.set_option("repartition", 0)
+
+
+@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pr"])
+@pytest.mark.parametrize("seed,K", [(1, 0), (7, 0), (3, 32)])
+def test_random_initial_content(asc, algo, seed, K):
+    """§5 random initial content: the seeded chunk set is filled by the chunk-copy
+    kernel, S is rebuilt from the residency; with and without §3.4 swaps on top."""
+    g = gg.rmat(14, seed=47, weights=(algo == "sssp"))
+    src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+    iters = 5 if algo == "pr" else 0
+    budget = g.csr_bytes // 3
+    asc.load_csr(g.off, g.nbr, pairs=g.pairs)
+    asc.set_option("static_placement", 2)
+    asc.set_option("placement_seed", seed)
+    asc.set_option("replace_chunks", K)
+    asc.set_budget(budget)
+    p = oracle.placer(g.off, g.b_e, budget)
+    ref = oracle.run_hot(algo, g.off, g.nbr, static_bytes=p.Ms, src=src, max_iters=iters, kswap=K, random_seed=seed)
+    for rep in range(2):
+        asc.run(algo, src, iters)
+        st, its = asc.stats()
+        _values_ok(algo, asc.get_result().copy(), ref)
+        _check(its, ref)
+        assert st["s"] == ref.records[0]["s"]
+        assert st["h2d_payload_bytes"] == ref.h2d_payload
+        assert st["h2d_replace_bytes"] == ref.replace_bytes
+
+
+@pytest.mark.parametrize("P", [2, 3])
+def test_random_initial_content_ranks(asc, P):
+    """Per-rank random chunk sets; rank payload starts are not 16-byte aligned (4-byte copy path)."""
+    g = gg.rmat(13, seed=48)
+    src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+    budget = g.csr_bytes // (3 * P)
+    asc.emulate_ranks(P)
+    asc.load_csr(g.off, g.nbr)
+    asc.set_option("static_placement", 2)
+    asc.set_option("placement_seed", 5)
+    asc.set_budget(budget)
+    asc.run("cc", src)
+    st, its = asc.stats()
+    b = oracle.partition(g.off, P)
+    ms = [oracle.placer(g.off[int(b[k]):int(b[k + 1]) + 1] - g.off[int(b[k])], 4, budget).Ms for k in range(P)]
+    ref = oracle.run_hot("cc", g.off, g.nbr, static_bytes=ms, src=src, kswap=0, bounds=b, random_seed=5)
+    np.testing.assert_array_equal(asc.get_result(), ref.values)
+    _check(its, ref)
