@@ -19,8 +19,8 @@ _SRC = os.path.join(_HERE, "oracle.c")
 _LIB = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
-BFS, SSSP, CC, PR = 0, 1, 2, 3
-ALGOS = {"bfs": BFS, "sssp": SSSP, "cc": CC, "pr": PR}
+BFS, SSSP, CC, PR, PRD = 0, 1, 2, 3, 4
+ALGOS = {"bfs": BFS, "sssp": SSSP, "cc": CC, "pr": PR, "prd": PRD}
 INF = 0xFFFFFFFF
 
 
@@ -75,6 +75,7 @@ def _load():
                                    ctypes.POINTER(_Iter), ctypes.c_uint32, ctypes.POINTER(_Summary), ctypes.c_void_p,
                                    ctypes.c_uint32, ctypes.c_int, ctypes.c_int, ctypes.c_uint64]
         lib.or_random_chunks.argtypes = [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_void_p]
+        lib.or_set_prd_tol.argtypes = [ctypes.c_uint64]
         lib.or_threads.restype = ctypes.c_int
         lib.or_classify.argtypes = [ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p,
                                     ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
@@ -199,7 +200,7 @@ def run(algo: str | int, off: np.ndarray, nbr: np.ndarray, src: int = 0, max_ite
     if rc != 0:
         raise ValueError(f"oracle rejected arguments (rc={rc})")
     records = [{f: int(getattr(recs[i], f)) for f in ITER_FIELDS} for i in range(s.nrec)]
-    vals = res_f.copy() if a == PR else res_u.copy()
+    vals = res_f.copy() if a in (PR, PRD) else res_u.copy()
     return Result(vals, int(s.iterations), records, int(s.h2d_payload), int(s.active_arcs_total),
                   int(reparts.value))
 
@@ -236,7 +237,7 @@ def run_hot(algo: str | int, off: np.ndarray, nbr: np.ndarray, static_bytes, src
     if rc != 0:
         raise ValueError(f"oracle rejected arguments (rc={rc})")
     records = [{f: int(getattr(recs[i], f)) for f in ITER_FIELDS} for i in range(s.nrec)]
-    vals = res_f.copy() if a == PR else res_u.copy()
+    vals = res_f.copy() if a in (PR, PRD) else res_u.copy()
     return Result(vals, int(s.iterations), records, int(s.h2d_payload), int(s.active_arcs_total), 0,
                   int(s.h2d_replace))
 
@@ -246,3 +247,8 @@ def random_chunks(nc: int, ns: int, seed: int) -> np.ndarray:
     res = np.zeros(max(nc, 1), dtype=np.uint8)
     _load().or_random_chunks(nc, ns, seed, res.ctypes.data)
     return res[:nc].astype(bool)
+
+
+def set_prd_tol(ppm: int) -> None:
+    """PageRank-delta threshold tau = floor(res0 * ppm / 1e6), res0 = floor(3 * 2^56 / (20 n))."""
+    _load().or_set_prd_tol(int(ppm))
