@@ -47,7 +47,9 @@ typedef enum {
     ASCETIC_EUNSUPPORTED = -7  /* feature not built */
 } ascetic_status;
 
-typedef enum { ASCETIC_BFS = 0, ASCETIC_SSSP = 1, ASCETIC_CC = 2, ASCETIC_PR = 3 } ascetic_algo;
+typedef enum { ASCETIC_BFS = 0, ASCETIC_SSSP = 1, ASCETIC_CC = 2, ASCETIC_PR = 3,
+               ASCETIC_PRD = 4  /* PageRank-delta: Subway's frontier-driven PR, see run() */
+} ascetic_algo;
 
 /* load_csr flags */
 enum {
@@ -93,7 +95,9 @@ typedef enum {
                                       Changes bytes. */
     ASCETIC_OPT_REPLACE_POLICY = 15, /* hotness counter: 0 = by algorithm (default: cumulative for
                                       BFS/SSSP/CC, last iteration for PR), 1 = cumulative, 2 = last iteration */
-    ASCETIC_OPT_PLACEMENT_SEED = 16  /* seed of the random initial content (default 1). Set before set_budget. */
+    ASCETIC_OPT_PLACEMENT_SEED = 16, /* seed of the random initial content (default 1). Set before set_budget. */
+    ASCETIC_OPT_PRD_TOL_PPM = 17     /* PageRank-delta activation threshold tau in ppm of the initial residual
+                                      (1-d)/n (default 10000 = 1 %) */
 } ascetic_option;
 
 typedef struct {
@@ -206,6 +210,11 @@ int ascetic_set_option(int option, int64_t value);
  *   algo       ascetic_algo. SSSP needs weights (PAIRS or wgt). CC/PR need ASCETIC_SYMMETRIC.
  *   source     BFS/SSSP source (< n), ignored for CC/PR
  *   max_iters  0 = until the active set is empty; PR runs exactly max_iters (must be >= 1)
+ * ASCETIC_PRD (PageRank-delta, frontier-driven) is computed in 2^-56 fixed
+ * point with integer atomics, d = 17/20: res_0 = floor(3*2^56/(20n)), A_t = {v : res[v] > tau};
+ * each active u moves res[u] into r[u] and pushes floor(17 res[u] / (20 deg u)) along its
+ * out-arcs; the result is fp32((r + res) 2^-56). Bit-exact against the oracle; one rank only
+ * (EUNSUPPORTED under comm_init / emulate_ranks > 1); no ASCETIC_SYMMETRIC needed.
  * The static fill (one H2D of the front prefix) is part of the run unless KEEP_STATIC
  * kept it from a previous run. Results stay on the device until ascetic_get_result.
  */
@@ -216,7 +225,7 @@ int ascetic_run(int algo, uint32_t source, uint32_t max_iters);
 int ascetic_stats(ascetic_stats_t* out, ascetic_iter_stats_t* per_iter, uint32_t cap);
 
 /* Copy the last run's result to host_dst: n x uint32 (levels / distances / labels,
- * UINT32_MAX = unreached) or n x float (PageRank). bytes must be >= 4n. */
+ * UINT32_MAX = unreached) or n x float (PageRank, PageRank-delta). bytes must be >= 4n. */
 int ascetic_get_result(void* host_dst, uint64_t bytes);
 
 /* Multi-GPU (one process per GPU; the paper itself is single-GPU).

@@ -31,12 +31,12 @@ _lib = ctypes.CDLL(LIB_PATH)
 OK, EINVAL, ESTATE, ENOMEM, EHOSTMEM, ECUDA, ENCCL, EUNSUPPORTED = 0, -1, -2, -3, -4, -5, -6, -7
 STATUS = {0: "OK", -1: "EINVAL", -2: "ESTATE", -3: "ENOMEM", -4: "EHOSTMEM", -5: "ECUDA", -6: "ENCCL",
           -7: "EUNSUPPORTED"}
-ALGOS = {"bfs": 0, "sssp": 1, "cc": 2, "pr": 3}
+ALGOS = {"bfs": 0, "sssp": 1, "cc": 2, "pr": 3, "prd": 4}
 SYMMETRIC, COPY, VALIDATE, PAIRS = 1, 2, 4, 8
 OPTIONS = {"chunk_cap": 1, "xfer_mode": 2, "dma_min_run": 3, "overlap": 4, "keep_static": 5,
            "hub_degree": 6, "timing": 7, "gather_ctas": 8, "chunk_buffers": 9, "static_ctas_per_sm": 10,
            "prefetch": 11, "repartition": 12, "static_placement": 13, "replace_chunks": 14,
-           "replace_policy": 15, "placement_seed": 16}
+           "replace_policy": 15, "placement_seed": 16, "prd_tol_ppm": 17}
 INF = 0xFFFFFFFF
 
 
@@ -169,7 +169,7 @@ def stats(per_iter: bool = True) -> tuple[dict, list[dict]]:
 def get_result(out: np.ndarray | None = None) -> np.ndarray:
     st = Stats()
     _check(_lib.ascetic_stats(ctypes.byref(st), None, 0))
-    dt = np.float32 if st.algo == ALGOS["pr"] else np.uint32
+    dt = np.float32 if st.algo in (ALGOS["pr"], ALGOS["prd"]) else np.uint32
     if out is None:
         out = np.empty(max(st.n, 1), dtype=dt)[: st.n]
     _check(_lib.ascetic_get_result(out.ctypes.data, out.nbytes))

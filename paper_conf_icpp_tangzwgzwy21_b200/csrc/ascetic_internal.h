@@ -96,6 +96,9 @@ struct DevState {
     // §3.4 replacement: Static Region = 16 KiB slots; slot_of[c] = slot of rank-local chunk c
     // (kNoSlot if not resident). nullptr = contiguous prefix (no remapping).
     const uint32_t* slot_of;
+    // PageRank-delta (fixed point 2^-56): rank, residual, push value; tau = activation threshold
+    unsigned long long *pr_r, *pr_res, *pr_c;
+    unsigned long long tau;
 };
 
 constexpr uint32_t kNoSlot = 0xFFFFFFFFu;
@@ -144,6 +147,8 @@ void launch_copy_chunks(const void* host_dev, uint64_t x0, uint64_t D, const uin
 void launch_static_bits(const DevState& d, const uint32_t* slot_of, uint32_t b_e, cudaStream_t s);
 // dense = values were exchanged (P > 1): SSSP/CC rebuild A from val < snap over all vertices
 void launch_finalize(int algo, const DevState& d, bool dense, cudaStream_t s);
+// PRD: rank[v] = fp32((r + res) 2^-56)
+void launch_prd_output(const DevState& d, cudaStream_t s);
 // collectives' device side (comm.cu drives them)
 void launch_or_reduce(uint32_t* dst, const uint32_t* gathered, uint32_t parts, uint64_t nw, cudaStream_t s);
 void launch_or_into(uint32_t* dst, const uint32_t* src, uint64_t nw, cudaStream_t s);

@@ -27,7 +27,18 @@ unsigned long long g_launches = 0;
 namespace {
 
 constexpr unsigned FULL = 0xFFFFFFFFu;
-enum { BFS = 0, SSSP = 1, CC = 2, PR = 3 };
+enum { BFS = 0, SSSP = 1, CC = 2, PR = 3, PRD = 4 };
+
+// per-source value pushed along each arc: snapshot dist/label (u32), or PRD's fixed-point push c[u] (u64)
+template <int ALGO>
+using SrcVal = typename std::conditional<ALGO == PRD, unsigned long long, uint32_t>::type;
+
+template <int ALGO>
+__device__ __forceinline__ SrcVal<ALGO> src_val(const DevState& d, uint32_t u) {
+    if constexpr (ALGO == PRD) return __ldg(d.pr_c + u);
+    else if constexpr (ALGO == SSSP || ALGO == CC) return __ldg(d.snap + u);
+    else return 0u;
+}
 constexpr double kDamp = 0.85;
 
 // ------------------------------------------------------------------ L2 policy loads
@@ -98,11 +109,20 @@ __device__ __forceinline__ uint32_t sat_add(uint32_t a, uint32_t w) {
     return c > (unsigned long long)(kInf - 1) ? kInf - 1 : (uint32_t)c;
 }
 
+// PageRank-delta push (DESIGN R28-R30): res[v] += c[u] in 2^-56 fixed point (integer atomics,
+// order-independent); the one thread whose add crosses tau marks v for the next active set.
+__device__ __forceinline__ void prd_push(const DevState& d, uint32_t v, unsigned long long c) {
+    if (c == 0) return;
+    const unsigned long long old = atomicAdd(d.pr_res + v, c);
+    if (old <= d.tau && old + c > d.tau) set_next(d, v);
+}
+
 // one arc, push algorithms. `arc` points at b_e bytes: id (+ weight).
 template <int ALGO>
-__device__ __forceinline__ void push_arc(const DevState& d, uint32_t sval, uint32_t id, uint32_t w) {
-    if (ALGO == BFS) bfs_visit(d, id);
-    else if (ALGO == SSSP) relax(d, id, sat_add(sval, w));
+__device__ __forceinline__ void push_arc(const DevState& d, SrcVal<ALGO> sval, uint32_t id, uint32_t w) {
+    if constexpr (ALGO == BFS) bfs_visit(d, id);
+    else if constexpr (ALGO == SSSP) relax(d, id, sat_add(sval, w));
+    else if constexpr (ALGO == PRD) prd_push(d, id, sval);
     else relax(d, id, sval);
 }
 
@@ -134,7 +154,7 @@ __device__ __forceinline__ unsigned long long sidx(const DevState& d, unsigned l
 // `nthr` threads with index `tid`, 128-bit loads on the aligned body.
 template <int ALGO, bool REMAP = false>
 __device__ __forceinline__ double expand_list(const DevState& d, const void* base, unsigned long long a0,
-                                              unsigned long long a1, uint32_t sval, int tid, int nthr) {
+                                              unsigned long long a1, SrcVal<ALGO> sval, int tid, int nthr) {
     double acc = 0.0;
     if (ALGO == SSSP) {
         const uint2* arcs = reinterpret_cast<const uint2*>(base);
@@ -200,13 +220,14 @@ __global__ void __launch_bounds__(256) k_static_small(DevState d, const uint32_t
     for (uint32_t base = ((blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 32; base < nq; base += nwarps * 32) {
         const uint32_t idx = base + lane;
         const bool valid = idx < nq;
-        uint32_t u = 0, deg = 0, sval = 0;
+        uint32_t u = 0, deg = 0;
+        SrcVal<ALGO> sval = 0;
         unsigned long long start = 0;
         if (valid) {
             u = __ldg(q + idx);
             start = __ldg(d.off + u);
             deg = (uint32_t)(__ldg(d.off + u + 1) - start);
-            if (ALGO == SSSP || ALGO == CC) sval = __ldg(d.snap + u);
+            sval = src_val<ALGO>(d, u);
         }
         uint32_t incl = deg;
 #pragma unroll
@@ -228,7 +249,7 @@ __global__ void __launch_bounds__(256) k_static_small(DevState d, const uint32_t
             }
             const unsigned long long ust = __shfl_sync(FULL, start, i);
             const uint32_t uex = __shfl_sync(FULL, excl, i);
-            const uint32_t usv = __shfl_sync(FULL, sval, i);
+            const SrcVal<ALGO> usv = __shfl_sync(FULL, sval, i);
             const bool ok = k < total;
             const unsigned long long e = ust + (k - uex) - d.static_arc0;   // index into the Static Region
             if (ALGO == PR) {
@@ -267,7 +288,7 @@ __global__ void __launch_bounds__(256) k_static_med(DevState d, const uint32_t* 
     for (uint32_t w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < nq; w += nwarps) {
         const uint32_t u = __ldg(q + w);
         const unsigned long long a0 = __ldg(d.off + u), a1 = __ldg(d.off + u + 1);
-        const uint32_t sval = (ALGO == SSSP || ALGO == CC) ? __ldg(d.snap + u) : 0u;
+        const SrcVal<ALGO> sval = src_val<ALGO>(d, u);
         double acc = expand_list<ALGO, REMAP>(d, sbase, a0 - d.static_arc0, a1 - d.static_arc0, sval, lane, 32);
         if (ALGO == PR) {
             acc = warp_sum_d(acc);
@@ -289,7 +310,7 @@ __global__ void __launch_bounds__(256) k_static_hub(DevState d, const uint32_t* 
         const unsigned long long o0 = __ldg(d.off + u), o1 = __ldg(d.off + u + 1);
         const unsigned long long a0 = o0 + (unsigned long long)pidx * piece_arcs;
         const unsigned long long a1 = min(o1, a0 + piece_arcs);
-        const uint32_t sval = (ALGO == SSSP || ALGO == CC) ? __ldg(d.snap + u) : 0u;
+        const SrcVal<ALGO> sval = src_val<ALGO>(d, u);
         double acc = expand_list<ALGO, REMAP>(d, sbase, a0 - d.static_arc0, a1 - d.static_arc0, sval, threadIdx.x,
                                               blockDim.x);
         if (ALGO == PR) {
@@ -358,14 +379,14 @@ __global__ void __launch_bounds__(256) k_ondemand(DevState d, Queues q, const vo
                                                   unsigned long long lo, unsigned long long hi) {
     __shared__ unsigned long long s_pre[kEdgeTile + 1];
     __shared__ uint32_t s_u[kEdgeTile + 1];
-    __shared__ uint32_t s_v[kEdgeTile + 1];
+    __shared__ SrcVal<ALGO> s_v[kEdgeTile + 1];
     const unsigned long long t = (lo >> kEdgeTileShift) + blockIdx.x;
     const Tile x = tile_of(q, t, lo, hi);
     for (uint32_t k = threadIdx.x; k < x.cnt; k += blockDim.x) {
         s_pre[k] = __ldg(q.mq_pre + x.i0 + k);
         const uint32_t u = __ldg(q.mq + x.i0 + k);
         s_u[k] = u;
-        if (ALGO == SSSP || ALGO == CC) s_v[k] = __ldg(d.snap + u);
+        if (ALGO != PR) s_v[k] = src_val<ALGO>(d, u);
     }
     __syncthreads();
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -373,7 +394,24 @@ __global__ void __launch_bounds__(256) k_ondemand(DevState d, Queues q, const vo
     if (pw >= x.t_hi) return;
     const unsigned long long pe = min(x.t_hi, pw + 256ull);
     uint32_t k = find_local(s_pre, 0, x.cnt, pw);
-    if (ALGO == SSSP || ALGO == CC) {
+    if constexpr (ALGO == PRD) {
+        // 2 phases: map + chunk loads for the warp's 8 groups of 32 arcs, then the residual atomics
+        uint32_t id[8];
+        unsigned long long c[8];
+#pragma unroll
+        for (int g = 0; g < 8; ++g) {
+            const unsigned long long p = pw + 32ull * g;
+            const uint32_t mk = warp_map(s_pre, x.cnt, k, p, lane);
+            k = __shfl_sync(FULL, mk, 31);
+            const unsigned long long a = p + lane;
+            id[g] = kInf;
+            c[g] = s_v[mk];
+            if (a < pe) id[g] = ld_stream(reinterpret_cast<const uint32_t*>(chunk) + (a - lo));
+        }
+#pragma unroll
+        for (int g = 0; g < 8; ++g)
+            if (id[g] != kInf) prd_push(d, id[g], c[g]);
+    } else if constexpr (ALGO == SSSP || ALGO == CC) {
         // 3 phases over the warp's 8 groups of 32 arcs: map + chunk loads, state loads, atomics
         uint32_t id[8], cand[8], cur[8];
 #pragma unroll
@@ -542,6 +580,51 @@ __global__ void k_pr_init(DevState d) {
     }
     dang = warp_sum_d(dang);
     if ((threadIdx.x & 31) == 0 && dang != 0.0) atomicAdd(d.dang, dang);
+}
+
+// PRD (DESIGN R28-R30): r = 0, res = res0; A_0 = {v : res0 > tau} absorbs at once
+__global__ void k_prd_init(DevState d, unsigned long long res0) {
+    const bool act = res0 > d.tau;
+    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < d.n; v += (uint64_t)gridDim.x * blockDim.x) {
+        const unsigned long long deg = d.off[v + 1] - d.off[v];
+        d.pr_r[v] = act ? res0 : 0ull;
+        d.pr_res[v] = act ? 0ull : res0;
+        d.pr_c[v] = act && deg ? (17ull * res0) / (20ull * deg) : 0ull;
+    }
+    if (act)
+        for (uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < d.nwords; w += (uint64_t)gridDim.x * blockDim.x) {
+            const uint64_t base = w * 32;
+            const uint32_t cnt = (uint32_t)min((uint64_t)32, d.n - base);
+            d.A[w] = cnt == 32 ? FULL : ((1u << cnt) - 1u);
+        }
+}
+
+// PRD finalize: A_{t+1} = the vertices whose residual crossed tau this iteration; each absorbs
+// r += res, c = floor(17 res / (20 deg)), res = 0 (the push value of iteration t+1)
+__global__ void k_finalize_prd(DevState d) {
+    for (uint32_t w = blockIdx.x * blockDim.x + threadIdx.x; w < d.nwords; w += gridDim.x * blockDim.x) {
+        const uint32_t nx = d.next[w];
+        d.A[w] = nx;
+        if (nx) {
+            d.next[w] = 0;
+            uint32_t b = nx;
+            while (b) {
+                const int i = __ffs(b) - 1;
+                b &= b - 1;
+                const uint64_t v = (uint64_t)w * 32 + i;
+                const unsigned long long x = d.pr_res[v], deg = d.off[v + 1] - d.off[v];
+                d.pr_r[v] += x;
+                d.pr_c[v] = deg ? (17ull * x) / (20ull * deg) : 0ull;
+                d.pr_res[v] = 0ull;
+            }
+        }
+    }
+}
+
+// PRD output: rank = (r + res) * 2^-56, u64 -> fp64 -> fp32, both round-to-nearest
+__global__ void k_prd_output(DevState d) {
+    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < d.n; v += (uint64_t)gridDim.x * blockDim.x)
+        d.rank[v] = __double2float_rn(__ull2double_rn(d.pr_r[v] + d.pr_res[v]) * 0x1p-56);
 }
 
 __global__ void k_finalize_bfs(DevState d) {
@@ -800,6 +883,7 @@ void static_launch(const DevState& d, const Queues& q, const void* sbase, uint32
 void launch_static(int algo, const DevState& d, const Queues& q, const void* sbase, uint32_t ns, uint32_t nm,
                    uint32_t nh, uint32_t npieces, uint32_t piece, int max_ctas, cudaStream_t s) {
     switch (algo) {
+        case PRD: static_launch<PRD>(d, q, sbase, ns, nm, nh, npieces, piece, max_ctas, s); break;
         case BFS: static_launch<BFS>(d, q, sbase, ns, nm, nh, npieces, piece, max_ctas, s); break;
         case SSSP: static_launch<SSSP>(d, q, sbase, ns, nm, nh, npieces, piece, max_ctas, s); break;
         case CC: static_launch<CC>(d, q, sbase, ns, nm, nh, npieces, piece, max_ctas, s); break;
@@ -855,6 +939,7 @@ void launch_ondemand(int algo, const DevState& d, const Queues& q, const void* c
     switch (algo) {
         case SSSP: k_ondemand<SSSP><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
         case CC: k_ondemand<CC><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
+        case PRD: k_ondemand<PRD><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
         default: k_ondemand<PR><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
     }
     ++g_launches;
@@ -896,6 +981,12 @@ void launch_init(int algo, const DevState& d, uint32_t source, cudaStream_t s) {
             k_range_bits<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d.A, d.nwords, 0, d.n);
             ++g_launches;
             break;
+        case PRD: {
+            const unsigned long long res0 = (3ull << 56) / (20ull * d.n);   // floor((1-d) Q / n)
+            k_prd_init<<<gb, 256, 0, s>>>(d, res0);
+            ++g_launches;
+            break;
+        }
         default:
             cudaMemsetAsync(d.dang, 0, 2 * sizeof(double), s);
             k_pr_init<<<gb, 256, 0, s>>>(d);
@@ -909,6 +1000,7 @@ void launch_init(int algo, const DevState& d, uint32_t source, cudaStream_t s) {
 void launch_finalize(int algo, const DevState& d, bool dense, cudaStream_t s) {
     switch (algo) {
         case BFS: k_finalize_bfs<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d); break;
+        case PRD: k_finalize_prd<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d); break;
         case SSSP:
         case CC:
             if (dense) k_finalize_minlabel_dense<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d);
@@ -921,6 +1013,11 @@ void launch_finalize(int algo, const DevState& d, bool dense, cudaStream_t s) {
             break;
         }
     }
+    ++g_launches;
+}
+
+void launch_prd_output(const DevState& d, cudaStream_t s) {
+    k_prd_output<<<blocks_for(d.n, 256), 256, 0, s>>>(d);
     ++g_launches;
 }
 

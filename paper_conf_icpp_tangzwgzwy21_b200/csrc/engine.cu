@@ -32,7 +32,7 @@ namespace ascetic {
             throw Error(ASCETIC_ECUDA, std::string(#call) + ": " + cudaGetErrorString(e__));       \
     } while (0)
 
-enum { ALG_BFS = 0, ALG_SSSP = 1, ALG_CC = 2, ALG_PR = 3 };
+enum { ALG_BFS = 0, ALG_SSSP = 1, ALG_CC = 2, ALG_PR = 3, ALG_PRD = 4 };
 
 // ------------------------------------------------------------------ placer / partition
 Placement place(const uint64_t* off, uint64_t n, uint32_t b_e, uint64_t budget, double frac) {
@@ -122,6 +122,7 @@ Part::~Part() {
     free_regions();
     dfree(d_off_); dfree(d_A_); dfree(d_S_); dfree(d_next_); dfree(d_visited_);
     dfree(d_val_); dfree(d_snap_); dfree(d_rank_); dfree(d_contrib_); dfree(d_sum_); dfree(d_dang_);
+    dfree(d_pr_r_); dfree(d_pr_res_); dfree(d_pr_c_);
     dfree(d_hq_small_); dfree(d_hq_med_); dfree(d_hq_hub_); dfree(d_hub_pre_);
     dfree(d_mq_); dfree(d_mq_pre_); dfree(d_mq_src_); dfree(d_tile_first_);
     dfree(d_run_b_); dfree(d_run_e_); dfree(d_run_dst_);
@@ -200,7 +201,14 @@ void Part::alloc_vertex_state() {
 }
 
 void Part::alloc_algo_state(int algo) {
-    if (algo == ALG_PR) {
+    if (algo == ALG_PRD) {
+        if (!d_pr_r_) {
+            dalloc(&d_pr_r_, g_.n, &vertex_bytes_);
+            dalloc(&d_pr_res_, g_.n, &vertex_bytes_);
+            dalloc(&d_pr_c_, g_.n, &vertex_bytes_);
+        }
+        if (!d_rank_) dalloc(&d_rank_, g_.n, &vertex_bytes_);
+    } else if (algo == ALG_PR) {
         if (!d_rank_) {
             dalloc(&d_rank_, g_.n, &vertex_bytes_);
             dalloc(&d_contrib_, g_.n, &vertex_bytes_);
@@ -383,6 +391,8 @@ DevState Part::dev_state(uint32_t iter) const {
     d.vlo = vlo_; d.vhi = vhi_;
     d.static_arc0 = g_.off.empty() ? 0 : g_.off[stat_lo_];
     d.slot_of = hot_ ? d_slot_of_ : nullptr;
+    d.pr_r = d_pr_r_; d.pr_res = d_pr_res_; d.pr_c = d_pr_c_;
+    d.tau = prd_tau_;
     return d;
 }
 
@@ -438,6 +448,10 @@ void Part::transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsig
 
 void Part::begin(int algo, uint32_t source, uint32_t max_iters, bool timing) {
     algo_ = algo;
+    if (algo == ALG_PRD) {   // tau = floor(res0 * ppm / 1e6), res0 = floor(3 * 2^56 / (20 n))  (DESIGN R29)
+        const unsigned __int128 res0 = (3ull << 56) / (20ull * g_.n);
+        prd_tau_ = (uint64_t)(res0 * o_.prd_tol_ppm / 1000000u);
+    }
     max_iters_ = max_iters;
     gchunk_ = 0;
     prefetched_ = 0;
@@ -1075,6 +1089,10 @@ void Engine::set_option(int opt, int64_t value) {
             o_.placement_seed = (uint64_t)value;
             if (state_ == 2) state_ = 1;
             break;
+        case ASCETIC_OPT_PRD_TOL_PPM:
+            if (value < 0 || value > 1000000000ll) throw Error(ASCETIC_EINVAL, "PRD tolerance must be in [0, 1e9] ppm");
+            o_.prd_tol_ppm = (uint64_t)value;
+            break;
         case ASCETIC_OPT_REPLACE_POLICY:
             if (value < 0 || value > 2) throw Error(ASCETIC_EINVAL, "replace policy: 0 = by algorithm, 1 = cumulative, 2 = last");
             o_.replace_policy = (int)value;
@@ -1120,7 +1138,7 @@ void Engine::fork() {
 
 void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
     if (state_ != 2) throw Error(ASCETIC_ESTATE, state_ == 0 ? "run before load_csr" : "run before set_budget");
-    if (algo < 0 || algo > 3) throw Error(ASCETIC_EINVAL, "unknown algorithm");
+    if (algo < 0 || algo > 4) throw Error(ASCETIC_EINVAL, "unknown algorithm");
     if (algo == ALG_SSSP && g_.b_e != 8) throw Error(ASCETIC_EINVAL, "SSSP needs weights (ASCETIC_PAIRS or wgt)");
     if (algo != ALG_SSSP && g_.b_e != 4) throw Error(ASCETIC_EINVAL, "BFS/CC/PR take an unweighted CSR (b_e = 4)");
     if ((algo == ALG_BFS || algo == ALG_SSSP) && source >= g_.n) throw Error(ASCETIC_EINVAL, "source >= n");
@@ -1129,6 +1147,7 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         throw Error(ASCETIC_EINVAL, "CC and PR need ASCETIC_SYMMETRIC");
     if (g_.n == 0) throw Error(ASCETIC_EINVAL, "empty graph");
     if (o_.replace_k && o_.repartition) throw Error(ASCETIC_EINVAL, "replacement (§3.4) and Eq. 3 re-partition are exclusive");
+    if (algo == ALG_PRD && comm_.active()) throw Error(ASCETIC_EUNSUPPORTED, "PageRank-delta runs on one rank");
     if (o_.repartition && o_.placement != 0) throw Error(ASCETIC_EINVAL, "Eq. 3 re-partition shrinks a front prefix");
     CK(cudaSetDevice(device_));
     have_result_ = false;
@@ -1194,6 +1213,8 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         comm_.share_slices(rk, bounds_, 4, p0.cs());
         fork();
     }
+    if (algo == ALG_PRD)
+        for (auto& p : parts_) launch_prd_output(p->dev_state(t), p->cs());   // rank = fp32((r + res) 2^-56)
     if (parts_.size() > 1) join();
     for (auto& p : parts_) p->end();
     // ---- aggregate the local parts (one with NCCL; all emulated ranks otherwise)
@@ -1249,7 +1270,7 @@ void Engine::get_result(void* dst, uint64_t bytes) {
     if (!dst || bytes < 4 * g_.n) throw Error(ASCETIC_EINVAL, "result buffer must hold 4n bytes");
     CK(cudaSetDevice(device_));
     Part& p0 = *parts_[0];
-    const void* src = (last_algo_ == ALG_PR) ? (const void*)p0.rank_arr() : (const void*)p0.val();
+    const void* src = (last_algo_ == ALG_PR || last_algo_ == ALG_PRD) ? (const void*)p0.rank_arr() : (const void*)p0.val();
     CK(cudaMemcpy(dst, src, 4 * g_.n, cudaMemcpyDeviceToHost));
 }
 

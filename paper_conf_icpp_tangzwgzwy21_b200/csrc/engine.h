@@ -62,6 +62,7 @@ struct Options {
     int repartition = 0;          // Eq. 3 adaptive re-partition (off, as in the paper's evaluation)
     int placement = 0;            // initial static content: 0 = front prefix, 1 = rear suffix, 2 = random chunks
     uint64_t placement_seed = 1;  // seed of the random initial chunk set
+    uint64_t prd_tol_ppm = 10000; // PageRank-delta threshold, ppm of the initial residual (1-d)/n
     uint32_t replace_k = 0;       // §3.4 data replacement: chunk swaps examined per iteration (0 = off)
     int replace_policy = 0;       // hotness counter: 0 = by algorithm, 1 = cumulative, 2 = last iteration
 };
@@ -140,6 +141,8 @@ class Part {
     uint32_t *d_A_ = nullptr, *d_S_ = nullptr, *d_next_ = nullptr, *d_visited_ = nullptr;
     uint32_t *d_val_ = nullptr, *d_snap_ = nullptr;
     float *d_rank_ = nullptr, *d_contrib_ = nullptr;
+    unsigned long long *d_pr_r_ = nullptr, *d_pr_res_ = nullptr, *d_pr_c_ = nullptr;   // PageRank-delta
+    uint64_t prd_tau_ = 0;
     double *d_sum_ = nullptr, *d_dang_ = nullptr;
     uint32_t *d_hq_small_ = nullptr, *d_hq_med_ = nullptr, *d_hq_hub_ = nullptr, *d_hub_pre_ = nullptr;
     uint32_t *d_mq_ = nullptr, *d_run_b_ = nullptr, *d_run_e_ = nullptr, *d_tile_first_ = nullptr;
