@@ -213,8 +213,8 @@ int ascetic_set_option(int option, int64_t value);
  * ASCETIC_PRD (PageRank-delta, frontier-driven) is computed in 2^-56 fixed
  * point with integer atomics, d = 17/20: res_0 = floor(3*2^56/(20n)), A_t = {v : res[v] > tau};
  * each active u moves res[u] into r[u] and pushes floor(17 res[u] / (20 deg u)) along its
- * out-arcs; the result is fp32((r + res) 2^-56). Bit-exact against the oracle; one rank only
- * (EUNSUPPORTED under comm_init / emulate_ranks > 1); no ASCETIC_SYMMETRIC needed.
+ * out-arcs; the result is fp32((r + res) 2^-56). Bit-exact against the oracle (P > 1: the
+ * integer increments are SUM-exchanged); no ASCETIC_SYMMETRIC needed.
  * The static fill (one H2D of the front prefix) is part of the run unless KEEP_STATIC
  * kept it from a previous run. Results stay on the device until ascetic_get_result.
  */
@@ -233,7 +233,8 @@ int ascetic_get_result(void* host_dst, uint64_t bytes);
  * the out-lists of its range, has its own placer / Static Region / On-demand Region / transfer
  * engine under its own budget B, and keeps the vertex state replicated. One exchange per
  * iteration: OR of next-frontier bitmaps (BFS), MIN of values (SSSP, CC), SUM of the fp64
- * dangling mass + every rank's contrib slice (PR). Results equal the single-GPU run.
+ * dangling mass + every rank's contrib slice (PR), SUM of the u64 residual increments (PRD).
+ * Results equal the single-GPU run.
  *   ascetic_get_unique_id  rank 0: 128-byte NCCL unique id (EUNSUPPORTED if libnccl.so.2
  *                          cannot be loaded); share it out of band (torch.distributed)
  *   ascetic_comm_init      every rank, BEFORE load_csr; device = this rank's GPU

@@ -98,6 +98,7 @@ struct DevState {
     const uint32_t* slot_of;
     // PageRank-delta (fixed point 2^-56): rank, residual, push value; tau = activation threshold
     unsigned long long *pr_r, *pr_res, *pr_c;
+    unsigned long long* pr_inc;        // P > 1: this rank's increments (summed across ranks), else nullptr
     unsigned long long tau;
 };
 
@@ -154,6 +155,7 @@ void launch_or_reduce(uint32_t* dst, const uint32_t* gathered, uint32_t parts, u
 void launch_or_into(uint32_t* dst, const uint32_t* src, uint64_t nw, cudaStream_t s);
 void launch_min_into(uint32_t* dst, const uint32_t* src, uint64_t n, cudaStream_t s);
 void launch_add_f64(double* dst, const double* src, cudaStream_t s);
+void launch_add_u64(unsigned long long* dst, const unsigned long long* src, uint64_t n, cudaStream_t s);
 // bits := the vertex range [a, b)
 void launch_set_range_bits(uint32_t* bits, uint32_t nwords, uint64_t a, uint64_t b, cudaStream_t s);
 

@@ -131,6 +131,17 @@ void Comm::sum_f64(const std::vector<double*>& local, cudaStream_t s) {
     NC(nccl().AllReduce(local[0], local[0], 1, ncclFloat64, ncclSum, (ncclComm_t)nccl_comm_, s), "ncclAllReduce(sum)");
 }
 
+void Comm::sum_u64(const std::vector<unsigned long long*>& local, uint64_t n, cudaStream_t s) {
+    if (!active() || n == 0) return;
+    if (emulated_) {
+        for (size_t p = 1; p < local.size(); ++p) launch_add_u64(local[0], local[p], n, s);
+        for (size_t p = 1; p < local.size(); ++p)
+            CKc(cudaMemcpyAsync(local[p], local[0], n * 8, cudaMemcpyDeviceToDevice, s), "sum copy-back");
+        return;
+    }
+    NC(nccl().AllReduce(local[0], local[0], n, ncclUint64, ncclSum, (ncclComm_t)nccl_comm_, s), "ncclAllReduce(sum u64)");
+}
+
 void Comm::share_slices(const std::vector<void*>& local, const std::vector<uint64_t>& bounds, uint32_t elem_bytes,
                         cudaStream_t s) {
     if (!active()) return;

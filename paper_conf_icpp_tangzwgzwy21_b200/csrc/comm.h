@@ -3,6 +3,7 @@
 //   BFS       : OR of the next-frontier bitmaps        (NCCL has no bitwise OR: all-gather + OR kernel)
 //   SSSP / CC : MIN of the value arrays               (ncclAllReduce min)
 //   PR        : SUM of the fp64 dangling partials + every rank's contrib slice to all ranks
+//   PRD       : SUM of the u64 residual increments   (ncclAllReduce sum, exact: integers)
 // Two back ends behind one interface:
 //   NCCL     — across processes (libnccl.so.2 is dlopen'ed on first use, so single-GPU
 //              runs never load it and torch's own NCCL is reused when already loaded);
@@ -39,6 +40,8 @@ class Comm {
     void or_words(const std::vector<uint32_t*>& local, uint64_t nw, cudaStream_t s);
     void min_u32(const std::vector<uint32_t*>& local, uint64_t n, cudaStream_t s);
     void sum_f64(const std::vector<double*>& local, cudaStream_t s);
+    // element-wise SUM of n uint64 per rank (PageRank-delta residual increments), in place
+    void sum_u64(const std::vector<unsigned long long*>& local, uint64_t n, cudaStream_t s);
     // rank r owns elements [bounds[r], bounds[r+1]) of an elem_bytes array; afterwards every
     // rank holds every slice
     void share_slices(const std::vector<void*>& local, const std::vector<uint64_t>& bounds, uint32_t elem_bytes,

@@ -113,6 +113,7 @@ __device__ __forceinline__ uint32_t sat_add(uint32_t a, uint32_t w) {
 // order-independent); the one thread whose add crosses tau marks v for the next active set.
 __device__ __forceinline__ void prd_push(const DevState& d, uint32_t v, unsigned long long c) {
     if (c == 0) return;
+    if (d.pr_inc) { atomicAdd(d.pr_inc + v, c); return; }   // P > 1: summed across ranks, then finalize
     const unsigned long long old = atomicAdd(d.pr_res + v, c);
     if (old <= d.tau && old + c > d.tau) set_next(d, v);
 }
@@ -621,6 +622,39 @@ __global__ void k_finalize_prd(DevState d) {
     }
 }
 
+// PRD finalize after the cross-rank SUM of the increments (P > 1): res += inc over all vertices,
+// A_{t+1} = {v : res > tau}, the active absorb; identical on every rank (replicated state)
+__global__ void k_finalize_prd_dense(DevState d) {
+    for (uint32_t w = blockIdx.x * blockDim.x + threadIdx.x; w < d.nwords; w += gridDim.x * blockDim.x) {
+        uint32_t bits = 0;
+        const uint64_t v0 = (uint64_t)w * 32;
+        const uint32_t cnt = (uint32_t)min((uint64_t)32, d.n - v0);
+        for (uint32_t i = 0; i < cnt; ++i) {
+            const uint64_t v = v0 + i;
+            const unsigned long long inc = d.pr_inc[v];
+            if (!inc) continue;                      // res <= tau already (not active, unchanged)
+            d.pr_inc[v] = 0ull;
+            const unsigned long long x = d.pr_res[v] + inc;
+            if (x > d.tau) {
+                const unsigned long long deg = d.off[v + 1] - d.off[v];
+                bits |= 1u << i;
+                d.pr_r[v] += x;
+                d.pr_c[v] = deg ? (17ull * x) / (20ull * deg) : 0ull;
+                d.pr_res[v] = 0ull;
+            } else {
+                d.pr_res[v] = x;
+            }
+        }
+        d.A[w] = bits;
+        d.next[w] = 0;
+    }
+}
+
+__global__ void k_add_u64(unsigned long long* __restrict__ dst, const unsigned long long* __restrict__ src, uint64_t n) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+        dst[i] += src[i];
+}
+
 // PRD output: rank = (r + res) * 2^-56, u64 -> fp64 -> fp32, both round-to-nearest
 __global__ void k_prd_output(DevState d) {
     for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < d.n; v += (uint64_t)gridDim.x * blockDim.x)
@@ -1000,7 +1034,10 @@ void launch_init(int algo, const DevState& d, uint32_t source, cudaStream_t s) {
 void launch_finalize(int algo, const DevState& d, bool dense, cudaStream_t s) {
     switch (algo) {
         case BFS: k_finalize_bfs<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d); break;
-        case PRD: k_finalize_prd<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d); break;
+        case PRD:
+            if (dense) k_finalize_prd_dense<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d);
+            else k_finalize_prd<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d);
+            break;
         case SSSP:
         case CC:
             if (dense) k_finalize_minlabel_dense<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d);
@@ -1033,6 +1070,11 @@ void launch_or_into(uint32_t* dst, const uint32_t* src, uint64_t nw, cudaStream_
 
 void launch_min_into(uint32_t* dst, const uint32_t* src, uint64_t n, cudaStream_t s) {
     k_min_into<<<blocks_for(n, 256), 256, 0, s>>>(dst, src, n);
+    ++g_launches;
+}
+
+void launch_add_u64(unsigned long long* dst, const unsigned long long* src, uint64_t n, cudaStream_t s) {
+    k_add_u64<<<blocks_for(n, 256), 256, 0, s>>>(dst, src, n);
     ++g_launches;
 }
 

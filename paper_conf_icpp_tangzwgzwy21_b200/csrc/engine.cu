@@ -122,7 +122,7 @@ Part::~Part() {
     free_regions();
     dfree(d_off_); dfree(d_A_); dfree(d_S_); dfree(d_next_); dfree(d_visited_);
     dfree(d_val_); dfree(d_snap_); dfree(d_rank_); dfree(d_contrib_); dfree(d_sum_); dfree(d_dang_);
-    dfree(d_pr_r_); dfree(d_pr_res_); dfree(d_pr_c_);
+    dfree(d_pr_r_); dfree(d_pr_res_); dfree(d_pr_c_); dfree(d_pr_inc_);
     dfree(d_hq_small_); dfree(d_hq_med_); dfree(d_hq_hub_); dfree(d_hub_pre_);
     dfree(d_mq_); dfree(d_mq_pre_); dfree(d_mq_src_); dfree(d_tile_first_);
     dfree(d_run_b_); dfree(d_run_e_); dfree(d_run_dst_);
@@ -200,12 +200,17 @@ void Part::alloc_vertex_state() {
     if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_EHOSTMEM, "cudaHostAlloc run list"); }
 }
 
-void Part::alloc_algo_state(int algo) {
+void Part::alloc_algo_state(int algo, bool multi) {
+    multi_ = multi;
     if (algo == ALG_PRD) {
         if (!d_pr_r_) {
             dalloc(&d_pr_r_, g_.n, &vertex_bytes_);
             dalloc(&d_pr_res_, g_.n, &vertex_bytes_);
             dalloc(&d_pr_c_, g_.n, &vertex_bytes_);
+        }
+        if (multi && !d_pr_inc_) {
+            dalloc(&d_pr_inc_, g_.n, &vertex_bytes_);
+            CK(cudaMemset(d_pr_inc_, 0, g_.n * 8));
         }
         if (!d_rank_) dalloc(&d_rank_, g_.n, &vertex_bytes_);
     } else if (algo == ALG_PR) {
@@ -392,6 +397,7 @@ DevState Part::dev_state(uint32_t iter) const {
     d.static_arc0 = g_.off.empty() ? 0 : g_.off[stat_lo_];
     d.slot_of = hot_ ? d_slot_of_ : nullptr;
     d.pr_r = d_pr_r_; d.pr_res = d_pr_res_; d.pr_c = d_pr_c_;
+    d.pr_inc = multi_ ? d_pr_inc_ : nullptr;
     d.tau = prd_tau_;
     return d;
 }
@@ -1147,13 +1153,12 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         throw Error(ASCETIC_EINVAL, "CC and PR need ASCETIC_SYMMETRIC");
     if (g_.n == 0) throw Error(ASCETIC_EINVAL, "empty graph");
     if (o_.replace_k && o_.repartition) throw Error(ASCETIC_EINVAL, "replacement (§3.4) and Eq. 3 re-partition are exclusive");
-    if (algo == ALG_PRD && comm_.active()) throw Error(ASCETIC_EUNSUPPORTED, "PageRank-delta runs on one rank");
     if (o_.repartition && o_.placement != 0) throw Error(ASCETIC_EINVAL, "Eq. 3 re-partition shrinks a front prefix");
     CK(cudaSetDevice(device_));
     have_result_ = false;
     const bool multi = comm_.active();
     const bool timing = o_.timing != 0;
-    for (auto& p : parts_) p->alloc_algo_state(algo);
+    for (auto& p : parts_) p->alloc_algo_state(algo, multi);
     for (auto& p : parts_) p->begin(algo, source, max_iters, timing);
     Part& p0 = *parts_[0];
     std::vector<IterTotals> T(parts_.size());
@@ -1182,6 +1187,10 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
                 std::vector<uint32_t*> b;
                 for (auto& p : parts_) b.push_back(p->next());
                 comm_.or_words(b, nw, p0.cs());
+            } else if (algo == ALG_PRD) {
+                std::vector<unsigned long long*> b;
+                for (auto& p : parts_) b.push_back(p->prd_inc());
+                comm_.sum_u64(b, g_.n, p0.cs());
             } else {
                 std::vector<uint32_t*> b;
                 for (auto& p : parts_) b.push_back(p->val());

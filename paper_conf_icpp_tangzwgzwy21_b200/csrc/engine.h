@@ -85,7 +85,7 @@ class Part {
     Part(const HostGraph& g, const Options& o, int rank, uint64_t vlo, uint64_t vhi, int sm_count);
     ~Part();
     void alloc_vertex_state();
-    void alloc_algo_state(int algo);
+    void alloc_algo_state(int algo, bool multi);
     void upload_off();
     void set_budget(uint64_t bytes, double frac);
     void on_reload() { static_valid_ = false; }
@@ -115,6 +115,7 @@ class Part {
     uint32_t* val() const { return d_val_; }
     float* rank_arr() const { return d_rank_; }
     float* contrib() const { return d_contrib_; }
+    unsigned long long* prd_inc() const { return d_pr_inc_; }
     double* dang() const { return d_dang_; }
     uint64_t vertex_bytes() const { return vertex_bytes_; }
 
@@ -142,6 +143,8 @@ class Part {
     uint32_t *d_val_ = nullptr, *d_snap_ = nullptr;
     float *d_rank_ = nullptr, *d_contrib_ = nullptr;
     unsigned long long *d_pr_r_ = nullptr, *d_pr_res_ = nullptr, *d_pr_c_ = nullptr;   // PageRank-delta
+    unsigned long long* d_pr_inc_ = nullptr;   // P > 1: residual increments of this rank's pushes
+    bool multi_ = false;
     uint64_t prd_tau_ = 0;
     double *d_sum_ = nullptr, *d_dang_ = nullptr;
     uint32_t *d_hq_small_ = nullptr, *d_hq_med_ = nullptr, *d_hq_hub_ = nullptr, *d_hub_pre_ = nullptr;

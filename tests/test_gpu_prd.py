@@ -87,11 +87,27 @@ def test_prd_with_replacement(asc):
     _check(asc, g, 200000, its, st, asc.get_result().copy(), kswap=32, Ms=p.Ms)
 
 
-def test_prd_single_rank_only(asc):
-    g = gg.rmat(10, seed=54)
-    asc.emulate_ranks(2)
+@pytest.mark.parametrize("P", [2, 3, 4])
+def test_prd_emulated_ranks(asc, P):
+    """P ranks on one GPU: pushes into per-rank increment arrays, SUM exchange, dense finalize;
+    per-rank records and the fp32 ranks bit-exact against the oracle's multi-rank simulation."""
+    g = gg.rmat(13, seed=54)
+    budget = g.csr_bytes // (3 * P)
+    asc.emulate_ranks(P)
     asc.load_csr(g.off, g.nbr)
-    asc.set_budget(g.csr_bytes // 3)
-    with pytest.raises(asc.AsceticError) as e:
-        asc.run("prd", 0)
-    assert e.value.code == asc.EUNSUPPORTED
+    asc.set_option("prd_tol_ppm", 50000)
+    asc.set_budget(budget, 0.5)
+    asc.run("prd", 0)
+    st, its = asc.stats()
+    b = oracle.partition(g.off, P)
+    stat = np.zeros(g.n, dtype=np.uint8)
+    for k in range(P):
+        lo, hi = int(b[k]), int(b[k + 1])
+        stat[lo:lo + oracle.placer(g.off[lo:hi + 1] - g.off[lo], 4, budget, 0.5).s] = 1
+    oracle.set_prd_tol(50000)
+    ref = oracle.run("prd", g.off, g.nbr, is_static=stat, bounds=b)
+    np.testing.assert_array_equal(asc.get_result(), ref.values.astype(np.float32))
+    assert [i["rank"] for i in its] == [r["rank"] for r in ref.records]
+    for a, r in zip(its, ref.records):
+        for f in REC:
+            assert a[f] == r[f], (r["t"], r["rank"], f)

@@ -5,7 +5,8 @@ range from the library's own host partitioner (ascetic_partition) and place thei
 Region with the library's host placer (ascetic_place) under their own budget. They then
 run the per-iteration protocol of SURVEY §8(e) — classify the OWNED active vertices, push
 along owned out-lists, exchange (BFS: OR of next bitmaps by all-gather; CC: MIN all-reduce
-of labels; PR: SUM of dangling partials + all-gather of contrib slices), finalize on the
+of labels; PR: SUM of dangling partials + all-gather of contrib slices; PRD: SUM of the
+integer residual increments), finalize on the
 replicated state — with numpy standing in for the kernels and gloo for NCCL. Per-rank
 records and results must equal the oracle's multi-rank simulation and the P = 1 result.
 """
@@ -112,6 +113,30 @@ def _worker(rank, world, port, algo, q):
                 A = lab < snap                               # A_{t+1} from the exchanged values
                 t += 1
             vals = lab.astype(np.uint32)
+        elif algo == "prd":
+            # PageRank-delta (DESIGN R28-R30): integer residual increments, SUM all-reduce
+            s = 0
+            Q = 1 << 56
+            res0 = (3 * Q) // (20 * n)
+            tau = res0 * 10000 // 1000000
+            r = np.zeros(n, dtype=np.uint64)
+            res = np.full(n, res0, dtype=np.uint64)
+            A = res > tau
+            while A.any():
+                recs.append(_record(t, rank, A, stat_all, lo, hi, deg, 4, oracle.digest(A)))
+                r[A] += res[A]
+                c = np.where(A & (deg > 0), (17 * res) // (20 * np.maximum(deg, 1).astype(np.uint64)), 0).astype(np.uint64)
+                res[A] = 0
+                own = np.zeros(n, dtype=bool); own[lo:hi] = A[lo:hi]
+                sel = own[src_all]
+                inc = np.zeros(n, dtype=np.uint64)
+                np.add.at(inc, nbr[sel].astype(np.int64), c[src_all[sel]])
+                ti = torch.from_numpy(inc.view(np.int64).copy())
+                dist.all_reduce(ti)                          # exchange: SUM of the increments
+                res += ti.numpy().view(np.uint64)
+                A = res > tau
+                t += 1
+            vals = np.ldexp((r + res).astype(np.float64), -56)
         else:  # pr, pull
             s = 0
             iters = 6
@@ -146,7 +171,7 @@ def _worker(rank, world, port, algo, q):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("algo", ["bfs", "cc", "pr"])
+@pytest.mark.parametrize("algo", ["bfs", "cc", "pr", "prd"])
 def test_world2_gloo_protocol(algo):
     import graphgen as gg
     import oracle
@@ -170,7 +195,9 @@ def test_world2_gloo_protocol(algo):
                      bounds=np.array(bounds, dtype=np.uint64))
     got = [rec for t in range(len(per_rank[0])) for rk in range(2) for rec in [per_rank[rk][t]]]
     assert got == ref.records
-    if algo == "pr":
+    if algo == "prd":
+        np.testing.assert_array_equal(vals, ref.values)             # integer protocol: exact
+    elif algo == "pr":
         np.testing.assert_allclose(vals, ref.values, rtol=1e-12)
     else:
         np.testing.assert_array_equal(vals, ref.values)

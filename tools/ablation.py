@@ -28,19 +28,22 @@ def main():
         src = gg.sources(g, 1, seed=c["seed"])[0]
         asc.load_csr(g.off, g.nbr, pairs=g.pairs)
 
-        def one(label, nbytes, frac, overlap=1, rear=0, eq3=0, replace=0):
+        def one(label, nbytes, frac, overlap=1, rear=0, eq3=0, replace=0, run_algo=None, tol=10000):
             asc.set_option("overlap", overlap)
             asc.set_option("static_placement", rear)
             asc.set_option("repartition", eq3)
             asc.set_option("replace_chunks", replace)
+            asc.set_option("prd_tol_ppm", tol)
             asc.set_budget(nbytes, frac)
+            ra = run_algo or algo
             best = None
             for _ in range(2):
-                asc.run(algo, src, iters)
+                asc.run(ra, src, iters if ra == algo else 0)
                 st, _ = asc.stats(per_iter=False)
                 if best is None or st["time_run_s"] < best["time_run_s"]:
                     best = st
-            r = dict(config=key, study=label, repartitions=best["repartitions"],
+            r = dict(config=key, study=label if ra == algo else f"{label} ({ra}, tol {tol} ppm, "
+                     f"{best['iterations']} it)", repartitions=best["repartitions"],
                      budget_frac_of_csr=round(nbytes / g.csr_bytes, 3),
                      R=round(best["static_fraction_used"], 4), overlap=overlap, run_ms=round(best["time_run_s"] * 1e3, 2),
                      gteps=round(best["active_arcs_total"] / best["time_run_s"] / 1e9, 3),
@@ -57,15 +60,22 @@ def main():
         one("eq2", budget, -1.0)
         if only == "replace":
             # §3.4 data replacement: K chunk swaps per iteration, counter by algorithm
-            for K in [16, 256, 4096, 65536]:
+            for K in [16, 256, 4096]:
                 one("replace", budget, -1.0, replace=K)
+            for seed in [1, 2]:   # §5 random initial chunks
+                asc.set_option("placement_seed", seed)
+                one(f"random-fill seed {seed}", budget, -1.0, rear=2)
+        elif only == "prd":
+            # PageRank-delta (Subway's PR) on the config graph and budget
+            for tol in [10000, 300000]:
+                one("prd", budget, -1.0, run_algo="prd", tol=tol)
         elif os.environ.get("ABLATION_QUICK") != "1":
             for R in [0.0, 0.2, 0.4, 0.6, 0.8, 0.9, 0.95, 1.0]:
                 one("R-sweep", budget, R)
             one("overlap-off", budget, -1.0, overlap=0)
             for f in [0.25, 0.5, 0.75, 1.0]:
                 one("budget-sweep", int(f * g.csr_bytes), -1.0)
-        if only != "replace":
+        if only not in ("replace", "prd"):
             one("rear-fill", budget, -1.0, rear=1)
             one("eq3-repartition", budget, -1.0, eq3=1)
         asc.set_option("overlap", 1)
