@@ -1,6 +1,7 @@
 """Small end-to-end runs of every algorithm for compute-sanitizer (memcheck / racecheck /
 synccheck): tiny chunks (many chunk windows, lists split across chunks), hub splitting,
-gather and DMA transfer modes, and 2 emulated ranks. Checks results against the oracle."""
+gather and DMA transfer modes, and 2 emulated ranks; §3.4 replacement, random initial content
+and PageRank-delta. Checks results against the oracle."""
 import os
 import sys
 
@@ -41,6 +42,34 @@ def main():
                 ok = (np.max(np.abs(res - ref.values) / ref.values) < 1e-5) if algo == "pr" else np.array_equal(res, ref.values)
                 bad += 0 if ok else 1
                 print(f"world={world} {algo} xfer={xfer} cap={cap} hub={hub}: {'ok' if ok else 'MISMATCH'}", flush=True)
+    # §3.4 replacement, random initial content and PageRank-delta (one and two ranks)
+    for world in (1, 2):
+        asc.unload()
+        asc.emulate_ranks(world)
+        for algo, placement, K in [("bfs", 0, 8), ("sssp", 2, 8), ("cc", 2, 0), ("prd", 0, 4), ("prd", 2, 0)]:
+            g = gg.rmat(12, seed=6, weights=(algo == "sssp"))
+            src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+            asc.unload()
+            asc.load_csr(g.off, g.nbr, pairs=g.pairs)
+            asc.set_option("static_placement", placement)
+            asc.set_option("replace_chunks", K)
+            asc.set_option("chunk_cap", 4096)
+            asc.set_option("hub_degree", 64)
+            budget = g.csr_bytes // (3 * world)
+            asc.set_budget(budget)
+            asc.run(algo, src, 0)
+            res = asc.get_result()
+            bounds = oracle.partition(g.off, world)
+            ms = [oracle.placer(g.off[int(bounds[k]):int(bounds[k + 1]) + 1] - g.off[int(bounds[k])], g.b_e, budget).Ms
+                  for k in range(world)]
+            ref = oracle.run_hot(algo, g.off, g.nbr, static_bytes=ms, src=src, kswap=K, bounds=bounds,
+                                 random_seed=1 if placement == 2 else None)
+            exp = ref.values.astype(np.float32) if algo == "prd" else ref.values
+            ok = np.array_equal(res, exp)
+            bad += 0 if ok else 1
+            print(f"world={world} {algo} placement={placement} K={K}: {'ok' if ok else 'MISMATCH'}", flush=True)
+    for k, v in [("static_placement", 0), ("replace_chunks", 0), ("chunk_cap", 0), ("hub_degree", 2048)]:
+        asc.set_option(k, v)
     asc.unload()
     asc.emulate_ranks(1)
     print("mismatches:", bad)
