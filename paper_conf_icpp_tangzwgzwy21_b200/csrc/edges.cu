@@ -127,6 +127,53 @@ __device__ __forceinline__ void push_arc(const DevState& d, SrcVal<ALGO> sval, u
     else relax(d, id, sval);
 }
 
+// N arcs of one lane at once, in phases so the lane keeps N state loads (then N atomics) in
+// flight instead of one dependent load->atomic chain per arc: the static-hit kernels are
+// latency-bound on these random 4-byte accesses (vmask bit j = arc j valid).
+template <int ALGO, int N>
+__device__ __forceinline__ void push_batch(const DevState& d, const SrcVal<ALGO> (&sv)[N], const uint32_t (&id)[N],
+                                           const uint32_t (&w)[N], uint32_t vmask) {
+    if constexpr (ALGO == PRD) {
+        unsigned long long old[N];
+#pragma unroll
+        for (int j = 0; j < N; ++j) {
+            old[j] = ~0ull;
+            if (((vmask >> j) & 1u) && sv[j]) {
+                if (d.pr_inc) atomicAdd(d.pr_inc + id[j], sv[j]);
+                else old[j] = atomicAdd(d.pr_res + id[j], sv[j]);
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < N; ++j)
+            if (old[j] <= d.tau && old[j] + sv[j] > d.tau) set_next(d, id[j]);
+    } else if constexpr (ALGO == BFS) {
+        uint32_t vis[N], nx[N];
+#pragma unroll
+        for (int j = 0; j < N; ++j) vis[j] = ((vmask >> j) & 1u) ? ld_state_ro(d.visited + (id[j] >> 5)) : FULL;
+#pragma unroll
+        for (int j = 0; j < N; ++j) nx[j] = ((vmask >> j) & 1u) ? ld_state(d.next + (id[j] >> 5)) : FULL;
+#pragma unroll
+        for (int j = 0; j < N; ++j) {
+            const uint32_t bit = 1u << (id[j] & 31);
+            if (!((vis[j] | nx[j]) & bit)) atomicOr(d.next + (id[j] >> 5), bit);
+        }
+    } else {   // SSSP, CC: relax with the snapshot value
+        uint32_t cand[N], cur[N];
+#pragma unroll
+        for (int j = 0; j < N; ++j) {
+            cand[j] = (ALGO == SSSP) ? sat_add(sv[j], w[j]) : (uint32_t)sv[j];
+            cur[j] = ((vmask >> j) & 1u) ? ld_state(d.val + id[j]) : 0u;
+        }
+#pragma unroll
+        for (int j = 0; j < N; ++j) {
+            if (cand[j] < cur[j]) {
+                const uint32_t old = atomicMin(d.val + id[j], cand[j]);
+                if (cand[j] < old) set_next(d, id[j]);
+            }
+        }
+    }
+}
+
 __device__ __forceinline__ double pr_in(const DevState& d, uint32_t id) {
     return (double)__uint_as_float(ld_state_ro(reinterpret_cast<const uint32_t*>(d.contrib) + id));
 }
@@ -166,10 +213,24 @@ __device__ __forceinline__ double expand_list(const DevState& d, const void* bas
         }
         const unsigned long long qb = h >> 1, qe = a1 >> 1;
         const uint4* q = reinterpret_cast<const uint4*>(base);
-        for (unsigned long long k = qb + tid; k < qe; k += nthr) {
-            const uint4 x = ld_stream(q + sidx<REMAP, 16>(d, k));
-            push_arc<ALGO>(d, sval, x.x, x.y);
-            push_arc<ALGO>(d, sval, x.z, x.w);
+        // 4 x 16 B per lane per round (8 arcs): loads, then 8 state loads, then the atomics
+        for (unsigned long long k = qb + tid; k < qe; k += 4ull * nthr) {
+            uint4 x[4];
+            uint32_t vm = 0;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const unsigned long long kk = k + (unsigned long long)j * nthr;
+                x[j] = make_uint4(0u, 0u, 0u, 0u);
+                if (kk < qe) { x[j] = ld_stream(q + sidx<REMAP, 16>(d, kk)); vm |= 3u << (2 * j); }
+            }
+            SrcVal<ALGO> sv[8];
+            uint32_t id[8], w[8];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                sv[2 * j] = sv[2 * j + 1] = sval;
+                id[2 * j] = x[j].x; w[2 * j] = x[j].y; id[2 * j + 1] = x[j].z; w[2 * j + 1] = x[j].w;
+            }
+            push_batch<ALGO, 8>(d, sv, id, w, vm);
         }
         for (unsigned long long e = max(h, qe << 1) + tid; e < a1; e += nthr) {
             const uint2 x = ld_stream(arcs + sidx<REMAP, 8>(d, e));
@@ -184,13 +245,35 @@ __device__ __forceinline__ double expand_list(const DevState& d, const void* bas
         }
         const unsigned long long qb = h >> 2, qe = a1 >> 2;
         const uint4* q = reinterpret_cast<const uint4*>(base);
-        for (unsigned long long k = qb + tid; k < qe; k += nthr) {
-            const uint4 x = ld_stream(q + sidx<REMAP, 16>(d, k));
-            if (ALGO == PR) {
-                acc += pr_in(d, x.x) + pr_in(d, x.y) + pr_in(d, x.z) + pr_in(d, x.w);
+        // 2 x 16 B per lane per round (8 arcs) so 8 state loads / gathers are in flight
+        for (unsigned long long k = qb + tid; k < qe; k += 2ull * nthr) {
+            uint4 x[2];
+            uint32_t vm = 0;
+#pragma unroll
+            for (int j = 0; j < 2; ++j) {
+                const unsigned long long kk = k + (unsigned long long)j * nthr;
+                x[j] = make_uint4(0u, 0u, 0u, 0u);
+                if (kk < qe) { x[j] = ld_stream(q + sidx<REMAP, 16>(d, kk)); vm |= 15u << (4 * j); }
+            }
+            if constexpr (ALGO == PR) {
+                double v[8];
+#pragma unroll
+                for (int j = 0; j < 2; ++j) {
+                    const bool ok = (vm >> (4 * j)) & 1u;
+                    v[4 * j] = ok ? pr_in(d, x[j].x) : 0.0; v[4 * j + 1] = ok ? pr_in(d, x[j].y) : 0.0;
+                    v[4 * j + 2] = ok ? pr_in(d, x[j].z) : 0.0; v[4 * j + 3] = ok ? pr_in(d, x[j].w) : 0.0;
+                }
+                acc += ((v[0] + v[1]) + (v[2] + v[3])) + ((v[4] + v[5]) + (v[6] + v[7]));
             } else {
-                push_arc<ALGO>(d, sval, x.x, 0); push_arc<ALGO>(d, sval, x.y, 0);
-                push_arc<ALGO>(d, sval, x.z, 0); push_arc<ALGO>(d, sval, x.w, 0);
+                SrcVal<ALGO> sv[8];
+                uint32_t id[8], w[8];
+#pragma unroll
+                for (int j = 0; j < 2; ++j) {
+                    id[4 * j] = x[j].x; id[4 * j + 1] = x[j].y; id[4 * j + 2] = x[j].z; id[4 * j + 3] = x[j].w;
+                }
+#pragma unroll
+                for (int j = 0; j < 8; ++j) { sv[j] = sval; w[j] = 0u; }
+                push_batch<ALGO, 8>(d, sv, id, w, vm);
             }
         }
         for (unsigned long long e = max(h, qe << 2) + tid; e < a1; e += nthr) {
@@ -238,6 +321,39 @@ __global__ void __launch_bounds__(256) k_static_small(DevState d, const uint32_t
         }
         const uint32_t excl = incl - deg;
         const uint32_t total = __shfl_sync(FULL, incl, 31);
+        if constexpr (ALGO != PR) {
+            // 4 rounds of 32 arcs per warp at once: each lane maps, loads and pushes 4 arcs
+            for (uint32_t k0 = 0; k0 < total; k0 += 128) {
+                SrcVal<ALGO> sv[4];
+                uint32_t id[4], w[4], vm = 0;
+#pragma unroll
+                for (int b = 0; b < 4; ++b) {
+                    const uint32_t k = k0 + 32u * b + lane;
+                    int i = 0;
+#pragma unroll
+                    for (int step = 16; step >= 1; step >>= 1) {
+                        const uint32_t x = __shfl_sync(FULL, incl, i + step - 1);
+                        if (x <= k) i += step;
+                    }
+                    const unsigned long long ust = __shfl_sync(FULL, start, i);
+                    const uint32_t uex = __shfl_sync(FULL, excl, i);
+                    sv[b] = __shfl_sync(FULL, sval, i);
+                    id[b] = 0u; w[b] = 0u;
+                    if (k < total) {
+                        const unsigned long long e = ust + (k - uex) - d.static_arc0;
+                        if (ALGO == SSSP) {
+                            const uint2 x = ld_stream(reinterpret_cast<const uint2*>(sbase) + sidx<REMAP, 8>(d, e));
+                            id[b] = x.x; w[b] = x.y;
+                        } else {
+                            id[b] = ld_stream(reinterpret_cast<const uint32_t*>(sbase) + sidx<REMAP, 4>(d, e));
+                        }
+                        vm |= 1u << b;
+                    }
+                }
+                push_batch<ALGO, 4>(d, sv, id, w, vm);
+            }
+            continue;
+        }
         if (ALGO == PR) s_acc[wib][lane] = 0.0;
         __syncwarp();
         for (uint32_t k0 = 0; k0 < total; k0 += 32) {

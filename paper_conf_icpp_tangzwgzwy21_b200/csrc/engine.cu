@@ -598,8 +598,10 @@ void Part::expand(uint32_t t, const IterTotals& T) {
         CK(cudaEventRecord(static_go_, cs_));
         CK(cudaStreamWaitEvent(ss_, static_go_, 0));
         cudaEvent_t e0 = mark(ss_);
-        launch_static(algo_, d, q, d_static_, T.n_small, T.n_med, T.n_hub, T.n_pieces, kPieceArcs,
-                      (o_.static_ctas_per_sm > 0 ? o_.static_ctas_per_sm : 4) * sm_count_, ss_);
+        // persistent grid: 4 CTAs/SM leave room for the on-demand kernels; an iteration without
+        // misses (resident lists only) takes every slot
+        const int cps = o_.static_ctas_per_sm > 0 ? o_.static_ctas_per_sm : (T.miss_arcs ? 4 : 8);
+        launch_static(algo_, d, q, d_static_, T.n_small, T.n_med, T.n_hub, T.n_pieces, kPieceArcs, cps * sm_count_, ss_);
         CK(cudaGetLastError());
         span(e0, ss_, t, PH_STATIC);
         CK(cudaEventRecord(static_done_, ss_));
