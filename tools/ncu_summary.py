@@ -3,6 +3,8 @@
 usage: python tools/ncu_summary.py gpurun_out r01 [config]
 Writes profiles/<round>/ncu_summary.md, profiles/<round>/launch_shares.csv and
 profiles/ncu_traffic.json (per-launch DRAM traffic of each kernel class, read by bench.py).
+       python tools/ncu_summary.py gpurun_out r01 --captures-only NAME.md [title]
+summarises only the .ncu-rep captures into profiles/<round>/NAME.md.
 """
 import collections
 import csv
@@ -46,11 +48,37 @@ def to_bytes(v, unit):
     return float(v) * f if f else None
 
 
+def captures(src):
+    lines = []
+    for rep in sorted(x for x in os.listdir(src) if x.endswith(".ncu-rep")):
+        raw = subprocess.run(["ncu", "-i", os.path.join(src, rep), "--page", "raw", "--csv"],
+                             capture_output=True, text=True).stdout
+        rr = list(csv.reader(io.StringIO(raw)))
+        if len(rr) < 3:
+            continue
+        h, u = rr[0], rr[1]
+        for r in rr[2:]:
+            name = r[h.index("Kernel Name")].split("(ascetic::")[0].replace("void ", "").replace("ascetic::<unnamed>::", "")
+            lines += [f"## `{name}` (`{rep}`, `ncu --set full`)", "", "| metric | value | unit |", "|---|---|---|"]
+            for m, label in METRICS:
+                if m in h:
+                    i = h.index(m)
+                    lines.append(f"| {label} (`{m}`) | {r[i]} | {u[i]} |")
+            lines.append("")
+    return lines
+
+
 def main():
     src, rnd = sys.argv[1], sys.argv[2]
-    cfg = sys.argv[3] if len(sys.argv) > 3 else "c2"
     out_dir = os.path.join(ROOT, "profiles", rnd)
     os.makedirs(out_dir, exist_ok=True)
+    if len(sys.argv) > 4 and sys.argv[3] == "--captures-only":
+        title = sys.argv[5] if len(sys.argv) > 5 else "ncu captures"
+        lines = [f"# {title}", ""] + captures(src)
+        open(os.path.join(out_dir, sys.argv[4]), "w").write("\n".join(lines) + "\n")
+        print("\n".join(lines))
+        return
+    cfg = sys.argv[3] if len(sys.argv) > 3 else "c2"
     lines = [f"# ncu summary — round {rnd[1:]}, workload {cfg} (bench.py --steps 1 --warmup 3)", ""]
     # ---- launch list
     rows = list(csv.reader(open(os.path.join(src, "launches.csv"))))
