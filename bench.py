@@ -188,13 +188,14 @@ def main():
     h2d_peak = _h2d_peak(torch, dev)
     hbm_peak, hbm_src = _peaks()
 
-    # graph arcs generated straight into pinned host memory (the method's host Edgelist)
+    # graph offsets and arcs generated straight into pinned host memory (the method's host Edgelist)
     pinned = []
 
     def alloc(count, dtype):
-        t = torch.empty(max(1, count), dtype=torch.int32, pin_memory=True)
+        words = max(1, count) * np.dtype(dtype).itemsize // 4
+        t = torch.empty(words, dtype=torch.int32, pin_memory=True)
         pinned.append(t)
-        return t.numpy().view(np.uint32)
+        return t.numpy().view(dtype)
 
     t0 = time.time()
     g = gg.config_graph(args.config, alloc=alloc)

@@ -78,12 +78,12 @@ class Graph:
 
 
 def _export(h, pairs: bool, wseed: int, name: str, alloc=None) -> Graph:
-    """alloc(count, dtype) -> numpy array lets callers place the arcs (e.g. in pinned memory)."""
+    """alloc(count, dtype) -> numpy array lets callers place the offsets and arcs (e.g. in pinned memory)."""
     lib = _load()
     n = ctypes.c_uint32()
     m = ctypes.c_uint64()
     lib.gg_size(h, ctypes.byref(n), ctypes.byref(m))
-    off = np.empty(n.value + 1, dtype=np.uint64)
+    off = (alloc(n.value + 1, np.uint64) if alloc is not None else np.empty(n.value + 1, dtype=np.uint64))[:n.value + 1]
     cnt = (2 if pairs else 1) * m.value
     nbr = (alloc(cnt, np.uint32) if alloc is not None else np.empty(max(1, cnt), dtype=np.uint32))[:cnt]
     lib.gg_export(h, off.ctypes.data, nbr.ctypes.data if nbr.size else None, None, 1 if pairs else 0, wseed)

@@ -168,14 +168,16 @@ typedef struct {
  * Load a CSR graph ("The graph is presented in the CSR format").
  *   n       vertices (< 2^32 - 1)
  *   m       stored arcs (both directions for symmetric graphs)
- *   off     host uint64[n+1], off[0] = 0, non-decreasing, off[n] = m; copied to the device
+ *   off     host uint64[n+1], off[0] = 0, non-decreasing (checked on the device), off[n] = m
  *   nbr     host uint32[m] neighbour ids, or uint32[2m] (id, weight) pairs with ASCETIC_PAIRS
  *   wgt     host uint32[m] weights or NULL; if given (without PAIRS) the library builds
  *           its own interleaved pinned copy
  *   flags   ASCETIC_* load flags
  * Ownership: without ASCETIC_COPY the nbr array is pinned IN PLACE (cudaHostRegister,
- * read-only) and must stay alive and unmodified until ascetic_unload() or the next
- * load_csr. Memory already page-locked (cudaHostAlloc / torch pin_memory) is used as is.
+ * read-only) and the off array is used in place by the host planner; both must stay alive and
+ * unmodified until ascetic_unload() or the next load_csr. Memory already page-locked
+ * (cudaHostAlloc / torch pin_memory) is used as is (pinned off uploads at the link's rate).
+ * With ASCETIC_COPY the library keeps private copies of both.
  * Errors: EINVAL (off[0] != 0, non-monotone off, off[n] != m, ids >= n with VALIDATE,
  * wgt with PAIRS), EHOSTMEM (pinning), ENOMEM/ECUDA (device offsets).
  */

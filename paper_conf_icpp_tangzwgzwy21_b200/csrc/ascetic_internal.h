@@ -156,6 +156,8 @@ void launch_or_into(uint32_t* dst, const uint32_t* src, uint64_t nw, cudaStream_
 void launch_min_into(uint32_t* dst, const uint32_t* src, uint64_t n, cudaStream_t s);
 void launch_add_f64(double* dst, const double* src, cudaStream_t s);
 void launch_add_u64(unsigned long long* dst, const unsigned long long* src, uint64_t n, cudaStream_t s);
+// *bad := min{v : off[v+1] < off[v]} (left untouched when off[0..n] is non-decreasing)
+void launch_check_monotone(const unsigned long long* off, uint64_t n, unsigned long long* bad, cudaStream_t s);
 // bits := the vertex range [a, b)
 void launch_set_range_bits(uint32_t* bits, uint32_t nwords, uint64_t a, uint64_t b, cudaStream_t s);
 

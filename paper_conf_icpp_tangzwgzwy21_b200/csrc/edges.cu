@@ -866,6 +866,11 @@ __global__ void k_min_into(uint32_t* __restrict__ dst, const uint32_t* __restric
 
 __global__ void k_add_f64(double* dst, const double* src) { dst[0] += src[0]; }
 
+__global__ void k_check_monotone(const unsigned long long* __restrict__ off, uint64_t n, unsigned long long* bad) {
+    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
+        if (off[v + 1] < off[v]) atomicMin(bad, (unsigned long long)v);
+}
+
 // ------------------------------------------------------------------ §3.4 data replacement
 // Accesses of this iteration per 16 KiB chunk: every active list with deg > 0 is
 // in exactly one of the hit queues or the miss queue; its arcs [a, e) (rank-local) add their
@@ -1196,6 +1201,12 @@ void launch_add_u64(unsigned long long* dst, const unsigned long long* src, uint
 
 void launch_add_f64(double* dst, const double* src, cudaStream_t s) {
     k_add_f64<<<1, 1, 0, s>>>(dst, src);
+    ++g_launches;
+}
+
+void launch_check_monotone(const unsigned long long* off, uint64_t n, unsigned long long* bad, cudaStream_t s) {
+    if (!n) return;
+    k_check_monotone<<<blocks_for(n, 256), 256, 0, s>>>(off, n, bad);
     ++g_launches;
 }
 

@@ -237,7 +237,7 @@ void Part::alloc_algo_state(int algo, bool multi) {
 }
 
 void Part::upload_off() {
-    CK(cudaMemcpyAsync(d_off_, g_.off.data(), (g_.n + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice, cs_));
+    CK(cudaMemcpyAsync(d_off_, g_.off, (g_.n + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice, cs_));
     static_valid_ = false;
 }
 
@@ -264,13 +264,13 @@ void Part::layout_regions(uint64_t Ms) {
 }
 
 void Part::set_budget(uint64_t bytes, double frac) {
-    Placement p = place(g_.off.data() + vlo_, vhi_ - vlo_, g_.b_e, bytes, frac);
+    Placement p = place(g_.off + vlo_, vhi_ - vlo_, g_.b_e, bytes, frac);
     const uint64_t own = vhi_ - vlo_;
     stat_lo_ = vlo_;
     if (o_.placement == 1) {
         // rear initial content (§5): the suffix of whole lists that fits in Ms,
         // s_lo = min{v : b_e (off[vhi] - off[v]) <= Ms}
-        const uint64_t* off = g_.off.data();
+        const uint64_t* off = g_.off;
         const uint64_t lim = off[vhi_] - std::min<uint64_t>(p.Ms / g_.b_e, off[vhi_]);
         stat_lo_ = (uint64_t)(std::lower_bound(off + vlo_, off + vhi_ + 1, lim) - off);
         p.s = vhi_ - stat_lo_;
@@ -373,7 +373,7 @@ bool Part::maybe_repartition(const IterTotals& T) {
     const uint64_t delta = (uint64_t)std::floor(Ms * V / D);
     const uint64_t ms_new = (ms_cur_ - std::min(delta, ms_cur_)) / 16384ull * 16384ull;
     if (ms_new >= ms_cur_) return false;
-    const uint64_t* off = g_.off.data() + vlo_;
+    const uint64_t* off = g_.off + vlo_;
     const uint64_t lim = off[0] + ms_new / g_.b_e;
     const uint64_t s_new = (uint64_t)(std::upper_bound(off, off + (vhi_ - vlo_) + 1, lim) - off) - 1;
     CK(cudaStreamSynchronize(xs_));   // no transfer may still target the old chunk layout
@@ -394,7 +394,7 @@ DevState Part::dev_state(uint32_t iter) const {
     d.rank = d_rank_; d.contrib = d_contrib_; d.sum = d_sum_; d.dang = d_dang_;
     d.iter = iter;
     d.vlo = vlo_; d.vhi = vhi_;
-    d.static_arc0 = g_.off.empty() ? 0 : g_.off[stat_lo_];
+    d.static_arc0 = g_.off ? g_.off[stat_lo_] : 0;
     d.slot_of = hot_ ? d_slot_of_ : nullptr;
     d.pr_r = d_pr_r_; d.pr_res = d_pr_res_; d.pr_c = d_pr_c_;
     d.pr_inc = multi_ ? d_pr_inc_ : nullptr;
@@ -945,19 +945,6 @@ void Engine::load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_
     if ((flags & ASCETIC_PAIRS) && wgt) throw Error(ASCETIC_EINVAL, "wgt given together with ASCETIC_PAIRS");
     if (off[0] != 0) throw Error(ASCETIC_EINVAL, "off[0] != 0");
     if (off[n] != m) throw Error(ASCETIC_EINVAL, "off[n] != m");
-    {   // monotone offsets, checked in parallel
-        const unsigned nt = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
-        std::atomic<uint64_t> bad{~0ull};
-        std::vector<std::thread> th;
-        for (unsigned t = 0; t < nt; ++t)
-            th.emplace_back([&, t] {
-                const uint64_t a = n * t / nt, b = n * (t + 1) / nt;
-                for (uint64_t v = a; v < b; ++v)
-                    if (off[v + 1] < off[v]) { bad = v; return; }
-            });
-        for (auto& x : th) x.join();
-        if (bad != ~0ull) throw Error(ASCETIC_EINVAL, "off is not non-decreasing at v=" + std::to_string((uint64_t)bad));
-    }
     const bool pairs = (flags & ASCETIC_PAIRS) || wgt;
     const uint32_t b_e = pairs ? 8u : 4u;
     if (flags & ASCETIC_VALIDATE) {
@@ -975,16 +962,14 @@ void Engine::load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_
     if (same_shape) g_.release();
     have_result_ = false;
     g_.n = n; g_.m = m; g_.b_e = b_e; g_.flags = flags;
-    {   // host planning copy of the offsets (parallel memcpy)
-        g_.off.resize(n + 1);
-        const unsigned nt = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
-        std::vector<std::thread> th;
-        for (unsigned t = 0; t < nt; ++t)
-            th.emplace_back([&, t] {
-                const uint64_t a = (n + 1) * t / nt, b = (n + 1) * (t + 1) / nt;
-                std::memcpy(g_.off.data() + a, off + a, (b - a) * sizeof(uint64_t));
-            });
-        for (auto& x : th) x.join();
+    // offsets: used in place by the host planner (placer, partition, DMA planning) and DMA'd to
+    // the device (full speed when the caller's array is pinned); ASCETIC_COPY keeps a private copy
+    if (flags & ASCETIC_COPY) {
+        g_.off_own.assign(off, off + n + 1);
+        g_.off = g_.off_own.data();
+    } else {
+        g_.off_own.clear();
+        g_.off = off;
     }
     // ---- pin the edge array (the On-demand Engine's Edgelist)
     const size_t bytes = (size_t)b_e * m;
@@ -1030,7 +1015,7 @@ void Engine::load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_
     }
     // ---- rank parts: this process's ranks and their owned vertex ranges
     const int world = comm_.world();
-    bounds_ = partition(g_.off.data(), n, (uint32_t)world);
+    bounds_ = partition(g_.off, n, (uint32_t)world);
     if (!same_shape) {
         parts_.clear();
         if (comm_.emulated()) {
@@ -1044,6 +1029,20 @@ void Engine::load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_
     }
     for (auto& p : parts_) p->upload_off();   // offsets H2D on every load (also resets the static region)
     for (auto& p : parts_) CK(cudaStreamSynchronize(p->cs()));
+    {   // monotone offsets, checked on the device copy (one pass over 8(n+1) bytes of HBM)
+        unsigned long long* d_bad = nullptr;
+        CK(cudaMalloc(&d_bad, sizeof(unsigned long long)));
+        CK(cudaMemset(d_bad, 0xFF, sizeof(unsigned long long)));
+        launch_check_monotone(parts_[0]->dev_off(), n, d_bad, parts_[0]->cs());
+        unsigned long long bad = 0;
+        cudaError_t e = cudaMemcpy(&bad, d_bad, sizeof bad, cudaMemcpyDeviceToHost);
+        cudaFree(d_bad);
+        CK(e);
+        if (bad != ~0ull) {
+            unload();
+            throw Error(ASCETIC_EINVAL, "off is not non-decreasing at v=" + std::to_string(bad));
+        }
+    }
     state_ = 1;
 }
 
@@ -1289,8 +1288,9 @@ void Engine::unload() {
     if (device_ >= 0) cudaSetDevice(device_);
     parts_.clear();
     g_.release();
-    g_.off.clear();
-    g_.off.shrink_to_fit();
+    g_.off = nullptr;
+    g_.off_own.clear();
+    g_.off_own.shrink_to_fit();
     g_.n = g_.m = 0;
     state_ = 0;
     have_result_ = false;

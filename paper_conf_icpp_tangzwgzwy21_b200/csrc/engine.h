@@ -70,7 +70,8 @@ struct Options {
 struct HostGraph {
     uint64_t n = 0, m = 0;
     uint32_t b_e = 4, flags = 0;
-    std::vector<uint64_t> off;        // host copy: placer, partition, DMA planning
+    const uint64_t* off = nullptr;    // host offsets (caller's, or off_own): placer, partition, DMA planning
+    std::vector<uint64_t> off_own;    // private copy with ASCETIC_COPY
     const void* nbr = nullptr;        // b_e bytes per arc, pinned
     const void* nbr_dev = nullptr;    // device-visible alias (zero-copy)
     void* owned = nullptr;            // library-owned pinned copy
@@ -105,6 +106,7 @@ class Part {
     cudaEvent_t mark(cudaStream_t s);                               // open a timed span
 
     cudaStream_t cs() const { return cs_; }
+    const unsigned long long* dev_off() const { return d_off_; }
     cudaEvent_t sync_event() const { return sync_ev_; }
     DevState dev_state(uint32_t iter) const;
     const Placement& placement() const { return pl_; }
