@@ -14,7 +14,8 @@ SOURCES = ["frontier.cu", "edges.cu", "engine.cu", "comm.cu", "api.cpp"]
 HEADERS = ["ascetic_internal.h", "engine.h", "comm.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3", "-I", INCLUDE, "-I", CSRC]
+FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3", "-I", INCLUDE, "-I", CSRC] + \
+    os.environ.get("ASCETIC_NVCC_EXTRA", "").split()   # dev-only tuning builds (e.g. -DASC_U8=2)
 
 
 def _stale(target: str, deps: list[str]) -> bool:

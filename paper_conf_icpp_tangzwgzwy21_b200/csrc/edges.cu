@@ -20,6 +20,32 @@
 
 #include "ascetic_internal.h"
 
+// Batching factors of the static-hit kernels, per algorithm: 16-byte loads per lane per round
+// (8-byte arcs: SSSP; 4-byte arcs: the others) and 32-arc rounds per warp for short lists.
+// Measured on B200, resident RMAT-24 at 8 CTAs/SM (tools/gpu_ab2.sh, profiles/r01/static_batching_ab.md):
+// BFS gains nothing from batching (most arcs stop at the visited word), SSSP is best at 2/2
+// (-14 %), CC/PRD at 2/4 (-10 %). ASC_* override them for tuning builds.
+namespace ascetic { namespace {
+template <int ALGO> constexpr int kU8 = 2;
+template <int ALGO> constexpr int kU4 = (ALGO == 0) ? 1 : 2;
+template <int ALGO> constexpr int kSmallRounds = (ALGO == 0) ? 1 : (ALGO == 1 ? 2 : 4);
+} }
+#ifdef ASC_U8
+#define ASC_U8_OF(A) ASC_U8
+#else
+#define ASC_U8_OF(A) kU8<A>
+#endif
+#ifdef ASC_U4
+#define ASC_U4_OF(A) ASC_U4
+#else
+#define ASC_U4_OF(A) kU4<A>
+#endif
+#ifdef ASC_SMALL_ROUNDS
+#define ASC_SMALL_OF(A) ASC_SMALL_ROUNDS
+#else
+#define ASC_SMALL_OF(A) kSmallRounds<A>
+#endif
+
 namespace ascetic {
 
 unsigned long long g_launches = 0;
@@ -147,11 +173,15 @@ __device__ __forceinline__ void push_batch(const DevState& d, const SrcVal<ALGO>
         for (int j = 0; j < N; ++j)
             if (old[j] <= d.tau && old[j] + sv[j] > d.tau) set_next(d, id[j]);
     } else if constexpr (ALGO == BFS) {
+        // visited words first (most arcs stop there), then the next words of the survivors only
         uint32_t vis[N], nx[N];
 #pragma unroll
         for (int j = 0; j < N; ++j) vis[j] = ((vmask >> j) & 1u) ? ld_state_ro(d.visited + (id[j] >> 5)) : FULL;
 #pragma unroll
-        for (int j = 0; j < N; ++j) nx[j] = ((vmask >> j) & 1u) ? ld_state(d.next + (id[j] >> 5)) : FULL;
+        for (int j = 0; j < N; ++j) {
+            const uint32_t bit = 1u << (id[j] & 31);
+            nx[j] = (vis[j] & bit) ? FULL : ld_state(d.next + (id[j] >> 5));
+        }
 #pragma unroll
         for (int j = 0; j < N; ++j) {
             const uint32_t bit = 1u << (id[j] & 31);
@@ -213,24 +243,25 @@ __device__ __forceinline__ double expand_list(const DevState& d, const void* bas
         }
         const unsigned long long qb = h >> 1, qe = a1 >> 1;
         const uint4* q = reinterpret_cast<const uint4*>(base);
-        // 4 x 16 B per lane per round (8 arcs): loads, then 8 state loads, then the atomics
-        for (unsigned long long k = qb + tid; k < qe; k += 4ull * nthr) {
-            uint4 x[4];
+        // U x 16 B per lane per round (2U arcs): loads, then the state loads, then the atomics
+        constexpr int U = ASC_U8_OF(ALGO);
+        for (unsigned long long k = qb + tid; k < qe; k += (unsigned long long)U * nthr) {
+            uint4 x[U];
             uint32_t vm = 0;
 #pragma unroll
-            for (int j = 0; j < 4; ++j) {
+            for (int j = 0; j < U; ++j) {
                 const unsigned long long kk = k + (unsigned long long)j * nthr;
                 x[j] = make_uint4(0u, 0u, 0u, 0u);
                 if (kk < qe) { x[j] = ld_stream(q + sidx<REMAP, 16>(d, kk)); vm |= 3u << (2 * j); }
             }
-            SrcVal<ALGO> sv[8];
-            uint32_t id[8], w[8];
+            SrcVal<ALGO> sv[2 * U];
+            uint32_t id[2 * U], w[2 * U];
 #pragma unroll
-            for (int j = 0; j < 4; ++j) {
+            for (int j = 0; j < U; ++j) {
                 sv[2 * j] = sv[2 * j + 1] = sval;
                 id[2 * j] = x[j].x; w[2 * j] = x[j].y; id[2 * j + 1] = x[j].z; w[2 * j + 1] = x[j].w;
             }
-            push_batch<ALGO, 8>(d, sv, id, w, vm);
+            push_batch<ALGO, 2 * U>(d, sv, id, w, vm);
         }
         for (unsigned long long e = max(h, qe << 1) + tid; e < a1; e += nthr) {
             const uint2 x = ld_stream(arcs + sidx<REMAP, 8>(d, e));
@@ -245,35 +276,31 @@ __device__ __forceinline__ double expand_list(const DevState& d, const void* bas
         }
         const unsigned long long qb = h >> 2, qe = a1 >> 2;
         const uint4* q = reinterpret_cast<const uint4*>(base);
-        // 2 x 16 B per lane per round (8 arcs) so 8 state loads / gathers are in flight
-        for (unsigned long long k = qb + tid; k < qe; k += 2ull * nthr) {
-            uint4 x[2];
-            uint32_t vm = 0;
-#pragma unroll
-            for (int j = 0; j < 2; ++j) {
-                const unsigned long long kk = k + (unsigned long long)j * nthr;
-                x[j] = make_uint4(0u, 0u, 0u, 0u);
-                if (kk < qe) { x[j] = ld_stream(q + sidx<REMAP, 16>(d, kk)); vm |= 15u << (4 * j); }
-            }
+        // push algorithms: 2 x 16 B per lane per round (8 arcs) so 8 state loads are in flight;
+        // PR keeps 1 x 16 B per round (its 4 contrib gathers are independent loads already)
+        constexpr int U = (ALGO == PR) ? 1 : ASC_U4_OF(ALGO);
+        for (unsigned long long k = qb + tid; k < qe; k += (unsigned long long)U * nthr) {
             if constexpr (ALGO == PR) {
-                double v[8];
-#pragma unroll
-                for (int j = 0; j < 2; ++j) {
-                    const bool ok = (vm >> (4 * j)) & 1u;
-                    v[4 * j] = ok ? pr_in(d, x[j].x) : 0.0; v[4 * j + 1] = ok ? pr_in(d, x[j].y) : 0.0;
-                    v[4 * j + 2] = ok ? pr_in(d, x[j].z) : 0.0; v[4 * j + 3] = ok ? pr_in(d, x[j].w) : 0.0;
-                }
-                acc += ((v[0] + v[1]) + (v[2] + v[3])) + ((v[4] + v[5]) + (v[6] + v[7]));
+                const uint4 x = ld_stream(q + sidx<REMAP, 16>(d, k));
+                acc += pr_in(d, x.x) + pr_in(d, x.y) + pr_in(d, x.z) + pr_in(d, x.w);
             } else {
-                SrcVal<ALGO> sv[8];
-                uint32_t id[8], w[8];
+                uint4 x[U];
+                uint32_t vm = 0;
 #pragma unroll
-                for (int j = 0; j < 2; ++j) {
+                for (int j = 0; j < U; ++j) {
+                    const unsigned long long kk = k + (unsigned long long)j * nthr;
+                    x[j] = make_uint4(0u, 0u, 0u, 0u);
+                    if (kk < qe) { x[j] = ld_stream(q + sidx<REMAP, 16>(d, kk)); vm |= 15u << (4 * j); }
+                }
+                SrcVal<ALGO> sv[4 * U];
+                uint32_t id[4 * U], w[4 * U];
+#pragma unroll
+                for (int j = 0; j < U; ++j) {
                     id[4 * j] = x[j].x; id[4 * j + 1] = x[j].y; id[4 * j + 2] = x[j].z; id[4 * j + 3] = x[j].w;
                 }
 #pragma unroll
-                for (int j = 0; j < 8; ++j) { sv[j] = sval; w[j] = 0u; }
-                push_batch<ALGO, 8>(d, sv, id, w, vm);
+                for (int j = 0; j < 4 * U; ++j) { sv[j] = sval; w[j] = 0u; }
+                push_batch<ALGO, 4 * U>(d, sv, id, w, vm);
             }
         }
         for (unsigned long long e = max(h, qe << 2) + tid; e < a1; e += nthr) {
@@ -322,12 +349,14 @@ __global__ void __launch_bounds__(256) k_static_small(DevState d, const uint32_t
         const uint32_t excl = incl - deg;
         const uint32_t total = __shfl_sync(FULL, incl, 31);
         if constexpr (ALGO != PR) {
-            // 4 rounds of 32 arcs per warp at once: each lane maps, loads and pushes 4 arcs
-            for (uint32_t k0 = 0; k0 < total; k0 += 128) {
-                SrcVal<ALGO> sv[4];
-                uint32_t id[4], w[4], vm = 0;
+            // ASC_SMALL_ROUNDS rounds of 32 arcs per warp at once: each lane maps, loads and pushes
+            // one arc per round
+            constexpr int B = ASC_SMALL_OF(ALGO);
+            for (uint32_t k0 = 0; k0 < total; k0 += 32u * B) {
+                SrcVal<ALGO> sv[B];
+                uint32_t id[B], w[B], vm = 0;
 #pragma unroll
-                for (int b = 0; b < 4; ++b) {
+                for (int b = 0; b < B; ++b) {
                     const uint32_t k = k0 + 32u * b + lane;
                     int i = 0;
 #pragma unroll
@@ -350,7 +379,7 @@ __global__ void __launch_bounds__(256) k_static_small(DevState d, const uint32_t
                         vm |= 1u << b;
                     }
                 }
-                push_batch<ALGO, 4>(d, sv, id, w, vm);
+                push_batch<ALGO, B>(d, sv, id, w, vm);
             }
             continue;
         }
