@@ -74,3 +74,40 @@ def test_c3_full_pr(asc):
         assert i["miss_bytes"] == 4 * (g.m - int(g.off[p.s]))
         assert i["active_arcs"] == g.m
     assert st["h2d_payload_bytes"] == 43 * 4 * (g.m - int(g.off[p.s]))
+
+
+_C2 = {}
+
+
+def _c2():
+    if "g" not in _C2:
+        _C2["g"] = gg.config_graph("c2")
+    return _C2["g"]
+
+
+@pytest.mark.parametrize("placement,K", [(0, 256), (2, 0)])
+def test_c2_full_replacement_and_random_fill(asc, placement, K):
+    """§3.4 replacement (K = 256 swaps per iteration) and the random initial chunks at the bench
+    size: values, every record (incl. swaps, swap bytes, |S|) and all bytes bit-exact."""
+    g = _c2()
+    budget = gg.config_budget("c2", g)
+    asc.load_csr(g.off, g.nbr, pairs=True)
+    asc.set_option("static_placement", placement)
+    asc.set_option("replace_chunks", K)
+    try:
+        asc.set_budget(budget)
+        src = gg.sources(g, 8, seed=2)[0]
+        asc.run("sssp", src)
+        st, its = asc.stats()
+        res = asc.get_result()
+    finally:
+        asc.set_option("static_placement", 0)
+        asc.set_option("replace_chunks", 0)
+    p = oracle.placer(g.off, 8, budget)
+    ref = oracle.run_hot("sssp", g.off, g.nbr, static_bytes=p.Ms, src=src, kswap=K,
+                         random_seed=1 if placement == 2 else None)
+    np.testing.assert_array_equal(res, ref.values)
+    f = REC + ["swaps", "replace_bytes"]
+    assert [{k: i[k] for k in f} for i in its] == [{k: r[k] for k in f} for r in ref.records]
+    assert [i["s_static"] for i in its] == [r["s"] for r in ref.records]
+    assert st["h2d_payload_bytes"] == ref.h2d_payload and st["h2d_replace_bytes"] == ref.replace_bytes

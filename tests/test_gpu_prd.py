@@ -111,3 +111,14 @@ def test_prd_emulated_ranks(asc, P):
     for a, r in zip(its, ref.records):
         for f in REC:
             assert a[f] == r[f], (r["t"], r["rank"], f)
+
+
+def test_prd_rmat20_parity(asc):
+    """A larger PageRank-delta run (RMAT-20, 33 M arcs, many chunk windows and hub pieces)."""
+    g = gg.rmat(20, seed=55)
+    budget = g.csr_bytes // 2
+    asc.load_csr(g.off, g.nbr)
+    asc.set_budget(budget)
+    asc.run("prd", 0)
+    st, its = asc.stats()
+    _check(asc, g, 10000, its, st, asc.get_result().copy())

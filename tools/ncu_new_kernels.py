@@ -25,6 +25,17 @@ def main():
         print("replace", st["swaps_total"], st["h2d_replace_bytes"], st["time_run_s"])
         asc.set_option("replace_chunks", 0)
         asc.unload()
+    if which == "resident":   # static-hit kernels alone (budget above the CSR), SSSP and CC
+        for algo in ("sssp", "cc"):
+            g = gg.rmat(23, seed=2, weights=(algo == "sssp"))
+            src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+            asc.load_csr(g.off, g.nbr, pairs=g.pairs)
+            asc.set_budget(int(g.csr_bytes * 1.2))
+            for _ in range(2):
+                asc.run(algo, src)
+            st, _ = asc.stats(per_iter=False)
+            print("resident", algo, st["time_static_s"], st["static_arcs"])
+            asc.unload()
     if which in ("all", "prd"):
         g = gg.rmat(22, seed=3)
         asc.load_csr(g.off, g.nbr)
