@@ -340,7 +340,7 @@ def main():
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         e2e_ms = float(tt.item())
         e2e_arcs, h2d_b, d2h_b = _sum_ranks(e2e_arcs), _sum_ranks(h2d_b), _sum_ranks(d2h_b)
-    e2e = {"value": e2e_arcs / (e2e_ms / 1e3) / 1e9, "unit": "GTEPS",
+    e2e = {"value": e2e_arcs / (e2e_ms / 1e3) / 1e9 if e2e_ms > 0 else None, "unit": "GTEPS",
            "h2d_bytes_per_step": h2d_b // max(1, args.e2e_steps), "d2h_bytes_per_step": d2h_b // max(1, args.e2e_steps),
            "steps": args.e2e_steps, "ms_per_step": e2e_ms / max(1, args.e2e_steps),
            "host_ms_per_call": {k: round(v, 3) for k, v in e2e_parts.items()}}
