@@ -96,8 +96,13 @@ typedef enum {
     ASCETIC_OPT_REPLACE_POLICY = 15, /* hotness counter: 0 = by algorithm (default: cumulative for
                                       BFS/SSSP/CC, last iteration for PR), 1 = cumulative, 2 = last iteration */
     ASCETIC_OPT_PLACEMENT_SEED = 16, /* seed of the random initial content (default 1). Set before set_budget. */
-    ASCETIC_OPT_PRD_TOL_PPM = 17     /* PageRank-delta activation threshold tau in ppm of the initial residual
+    ASCETIC_OPT_PRD_TOL_PPM = 17,    /* PageRank-delta activation threshold tau in ppm of the initial residual
                                       (1-d)/n (default 10000 = 1 %) */
+    ASCETIC_OPT_FUSED_EXCHANGE = 18  /* P > 1, BFS/SSSP/CC/PRD: 1 = fuse the per-iteration exchange into the
+                                      finalize kernel, which reads every rank's next bitmap / values /
+                                      increments straight from peer memory (CUDA IPC over NVLink with the NCCL
+                                      back end; the other parts' buffers when emulated), between stream-ordered
+                                      barriers; 0 (default) = NCCL collectives. Results are identical. */
 } ascetic_option;
 
 typedef struct {

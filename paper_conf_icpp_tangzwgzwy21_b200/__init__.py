@@ -36,7 +36,8 @@ SYMMETRIC, COPY, VALIDATE, PAIRS = 1, 2, 4, 8
 OPTIONS = {"chunk_cap": 1, "xfer_mode": 2, "dma_min_run": 3, "overlap": 4, "keep_static": 5,
            "hub_degree": 6, "timing": 7, "gather_ctas": 8, "chunk_buffers": 9, "static_ctas_per_sm": 10,
            "prefetch": 11, "repartition": 12, "static_placement": 13, "replace_chunks": 14,
-           "replace_policy": 15, "placement_seed": 16, "prd_tol_ppm": 17}
+           "replace_policy": 15, "placement_seed": 16, "prd_tol_ppm": 17,
+           "fused_exchange": 18}
 INF = 0xFFFFFFFF
 
 

@@ -148,6 +148,9 @@ void launch_copy_chunks(const void* host_dev, uint64_t x0, uint64_t D, const uin
 void launch_static_bits(const DevState& d, const uint32_t* slot_of, uint32_t b_e, cudaStream_t s);
 // dense = values were exchanged (P > 1): SSSP/CC rebuild A from val < snap over all vertices
 void launch_finalize(int algo, const DevState& d, bool dense, cudaStream_t s);
+// fused exchange + finalize (P > 1): peers = device array of P pointers to every rank's buffer
+// (BFS: next bitmaps, SSSP/CC: values, PRD: residual increments)
+void launch_finalize_peers(int algo, const DevState& d, const void* const* peers, int P, cudaStream_t s);
 // PRD: rank[v] = fp32((r + res) 2^-56)
 void launch_prd_output(const DevState& d, cudaStream_t s);
 // collectives' device side (comm.cu drives them)

@@ -86,6 +86,11 @@ void Comm::init_emulated(int world) {
 }
 
 void Comm::destroy() {
+    for (auto& e : peers_)
+        for (int p = 0; p < (int)e.second.size(); ++p)
+            if (p != rank_ && e.second[p]) cudaIpcCloseMemHandle(e.second[p]);
+    peers_.clear();
+    if (barrier_buf_) { cudaFree(barrier_buf_); barrier_buf_ = nullptr; }
     if (nccl_comm_) { nccl().CommDestroy((ncclComm_t)nccl_comm_); nccl_comm_ = nullptr; }
     if (scratch_) { cudaFree(scratch_); scratch_ = nullptr; scratch_words_ = 0; }
     world_ = 1; rank_ = 0; emulated_ = false;
@@ -140,6 +145,39 @@ void Comm::sum_u64(const std::vector<unsigned long long*>& local, uint64_t n, cu
         return;
     }
     NC(nccl().AllReduce(local[0], local[0], n, ncclUint64, ncclSum, (ncclComm_t)nccl_comm_, s), "ncclAllReduce(sum u64)");
+}
+
+std::vector<void*> Comm::open_peers(void* local) {
+    if (emulated_ || !active()) throw Error(ASCETIC_EINVAL, "open_peers needs the NCCL back end");
+    for (auto& e : peers_)
+        if (e.first == local) return e.second;
+    cudaIpcMemHandle_t h;
+    CKc(cudaIpcGetMemHandle(&h, local), "cudaIpcGetMemHandle");
+    char* dbuf = nullptr;
+    CKc(cudaMalloc(&dbuf, sizeof h * (size_t)(world_ + 1)), "ipc handle buffer");
+    CKc(cudaMemcpy(dbuf + sizeof h * (size_t)world_, &h, sizeof h, cudaMemcpyHostToDevice), "ipc handle H2D");
+    NC(nccl().AllGather(dbuf + sizeof h * (size_t)world_, dbuf, sizeof h, ncclInt8, (ncclComm_t)nccl_comm_, 0),
+       "ncclAllGather(ipc handles)");
+    std::vector<cudaIpcMemHandle_t> all(world_);
+    cudaError_t e = cudaMemcpy(all.data(), dbuf, sizeof h * (size_t)world_, cudaMemcpyDeviceToHost);
+    cudaFree(dbuf);
+    CKc(e, "ipc handles D2H");
+    std::vector<void*> ptrs(world_, nullptr);
+    for (int p = 0; p < world_; ++p) {
+        if (p == rank_) { ptrs[p] = local; continue; }
+        CKc(cudaIpcOpenMemHandle(&ptrs[p], all[p], cudaIpcMemLazyEnablePeerAccess), "cudaIpcOpenMemHandle");
+    }
+    peers_.emplace_back(local, ptrs);
+    return ptrs;
+}
+
+void Comm::barrier(cudaStream_t s) {
+    if (emulated_ || !active()) return;
+    if (!barrier_buf_) {
+        CKc(cudaMalloc(&barrier_buf_, sizeof(int)), "barrier buffer");
+        CKc(cudaMemset(barrier_buf_, 0, sizeof(int)), "barrier buffer");
+    }
+    NC(nccl().AllReduce(barrier_buf_, barrier_buf_, 1, ncclInt32, ncclMax, (ncclComm_t)nccl_comm_, s), "barrier");
 }
 
 void Comm::share_slices(const std::vector<void*>& local, const std::vector<uint64_t>& bounds, uint32_t elem_bytes,

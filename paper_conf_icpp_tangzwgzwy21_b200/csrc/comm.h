@@ -42,6 +42,12 @@ class Comm {
     void sum_f64(const std::vector<double*>& local, cudaStream_t s);
     // element-wise SUM of n uint64 per rank (PageRank-delta residual increments), in place
     void sum_u64(const std::vector<unsigned long long*>& local, uint64_t n, cudaStream_t s);
+    // Fused exchange support (NCCL back end): map every rank's `local` device allocation into this
+    // process with CUDA IPC (handles all-gathered over NCCL; cached per pointer); returns the
+    // world pointers, this rank's own at index rank(). Collective: every rank calls it.
+    std::vector<void*> open_peers(void* local);
+    // stream-ordered barrier over all ranks (a 4-byte ncclAllReduce); no-op when emulated
+    void barrier(cudaStream_t s);
     // rank r owns elements [bounds[r], bounds[r+1]) of an elem_bytes array; afterwards every
     // rank holds every slice
     void share_slices(const std::vector<void*>& local, const std::vector<uint64_t>& bounds, uint32_t elem_bytes,
@@ -53,6 +59,8 @@ class Comm {
     void* nccl_comm_ = nullptr;
     uint32_t* scratch_ = nullptr;
     uint64_t scratch_words_ = 0;
+    int* barrier_buf_ = nullptr;
+    std::vector<std::pair<void*, std::vector<void*>>> peers_;   // local pointer -> world pointers (IPC)
 };
 
 }  // namespace ascetic

@@ -795,6 +795,79 @@ __global__ void k_finalize_prd_dense(DevState d) {
     }
 }
 
+// ---- fused exchange + finalize (P > 1): each rank reads every rank's buffer straight from peer
+// memory (NVLink peers mapped with CUDA IPC; the other parts' buffers when ranks are emulated on
+// one GPU) and builds A_{t+1} in the same pass — no gathered copy, no separate reduce kernel.
+// Loads bypass L1 (ld.global.cg): the peers wrote these buffers before the stream barrier.
+template <typename T>
+__device__ __forceinline__ T ld_peer(const T* p) { return __ldcg(p); }
+
+// BFS: A = (OR_p next_p) & ~visited; every rank applies the same update to its replicated state
+__global__ void k_finalize_bfs_peers(DevState d, const uint32_t* const* __restrict__ peers, int P) {
+    for (uint32_t w = blockIdx.x * blockDim.x + threadIdx.x; w < d.nwords; w += gridDim.x * blockDim.x) {
+        uint32_t nx = 0;
+        for (int p = 0; p < P; ++p) nx |= ld_peer(peers[p] + w);
+        const uint32_t vis = d.visited[w];
+        const uint32_t nw = nx & ~vis;
+        d.A[w] = nw;
+        if (nw) {
+            d.visited[w] = vis | nw;
+            uint32_t b = nw;
+            while (b) {
+                const int i = __ffs(b) - 1;
+                b &= b - 1;
+                d.val[(uint64_t)w * 32 + i] = d.iter + 1;
+            }
+        }
+    }
+}
+
+// SSSP / CC: val = MIN_p val_p, A = {v : val < snap}, snap = val (a peer may be writing its own
+// val with the same minimum concurrently: every value read is >= the minimum, so MIN is exact)
+__global__ void k_finalize_min_peers(DevState d, const uint32_t* const* __restrict__ peers, int P) {
+    for (uint32_t w = blockIdx.x * blockDim.x + threadIdx.x; w < d.nwords; w += gridDim.x * blockDim.x) {
+        uint32_t bits = 0;
+        const uint64_t v0 = (uint64_t)w * 32;
+        const uint32_t cnt = (uint32_t)min((uint64_t)32, d.n - v0);
+        for (uint32_t i = 0; i < cnt; ++i) {
+            uint32_t x = kInf;
+            for (int p = 0; p < P; ++p) x = min(x, ld_peer(peers[p] + v0 + i));
+            const uint32_t y = d.snap[v0 + i];
+            if (x < y) { bits |= 1u << i; d.snap[v0 + i] = x; }
+            if (x != d.val[v0 + i]) d.val[v0 + i] = x;
+        }
+        d.A[w] = bits;
+        d.next[w] = 0;
+    }
+}
+
+// PRD: res += SUM_p inc_p (integers: exact in any order), A = {res > tau}, absorb
+__global__ void k_finalize_prd_peers(DevState d, const unsigned long long* const* __restrict__ peers, int P) {
+    for (uint32_t w = blockIdx.x * blockDim.x + threadIdx.x; w < d.nwords; w += gridDim.x * blockDim.x) {
+        uint32_t bits = 0;
+        const uint64_t v0 = (uint64_t)w * 32;
+        const uint32_t cnt = (uint32_t)min((uint64_t)32, d.n - v0);
+        for (uint32_t i = 0; i < cnt; ++i) {
+            const uint64_t v = v0 + i;
+            unsigned long long inc = 0;
+            for (int p = 0; p < P; ++p) inc += ld_peer(peers[p] + v);
+            if (!inc) continue;
+            const unsigned long long x = d.pr_res[v] + inc;
+            if (x > d.tau) {
+                const unsigned long long deg = d.off[v + 1] - d.off[v];
+                bits |= 1u << i;
+                d.pr_r[v] += x;
+                d.pr_c[v] = deg ? (17ull * x) / (20ull * deg) : 0ull;
+                d.pr_res[v] = 0ull;
+            } else {
+                d.pr_res[v] = x;
+            }
+        }
+        d.A[w] = bits;
+        d.next[w] = 0;
+    }
+}
+
 __global__ void k_add_u64(unsigned long long* __restrict__ dst, const unsigned long long* __restrict__ src, uint64_t n) {
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
         dst[i] += src[i];
@@ -1220,6 +1293,20 @@ void launch_or_into(uint32_t* dst, const uint32_t* src, uint64_t nw, cudaStream_
 
 void launch_min_into(uint32_t* dst, const uint32_t* src, uint64_t n, cudaStream_t s) {
     k_min_into<<<blocks_for(n, 256), 256, 0, s>>>(dst, src, n);
+    ++g_launches;
+}
+
+void launch_finalize_peers(int algo, const DevState& d, const void* const* peers, int P, cudaStream_t s) {
+    const unsigned g = blocks_for(d.nwords, 256);
+    switch (algo) {
+        case BFS: k_finalize_bfs_peers<<<g, 256, 0, s>>>(d, reinterpret_cast<const uint32_t* const*>(peers), P); break;
+        case SSSP:
+        case CC: k_finalize_min_peers<<<g, 256, 0, s>>>(d, reinterpret_cast<const uint32_t* const*>(peers), P); break;
+        case PRD:
+            k_finalize_prd_peers<<<g, 256, 0, s>>>(d, reinterpret_cast<const unsigned long long* const*>(peers), P);
+            break;
+        default: return;
+    }
     ++g_launches;
 }
 

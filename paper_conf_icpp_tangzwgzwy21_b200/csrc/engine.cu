@@ -120,7 +120,8 @@ Part::~Part() {
     if (cs_) cudaStreamSynchronize(cs_);
     if (xs_) cudaStreamSynchronize(xs_);
     free_regions();
-    dfree(d_off_); dfree(d_A_); dfree(d_S_); dfree(d_next_); dfree(d_visited_);
+    dfree(d_off_); dfree(d_A_); dfree(d_S_); dfree(d_next_); dfree(d_visited_); dfree(d_next2_);
+    if (d_peers_) { cudaFree((void*)d_peers_); d_peers_ = nullptr; }
     dfree(d_val_); dfree(d_snap_); dfree(d_rank_); dfree(d_contrib_); dfree(d_sum_); dfree(d_dang_);
     dfree(d_pr_r_); dfree(d_pr_res_); dfree(d_pr_c_); dfree(d_pr_inc_);
     dfree(d_hq_small_); dfree(d_hq_med_); dfree(d_hq_hub_); dfree(d_hub_pre_);
@@ -389,7 +390,7 @@ bool Part::maybe_repartition(const IterTotals& T) {
 DevState Part::dev_state(uint32_t iter) const {
     DevState d;
     d.off = d_off_; d.n = g_.n; d.nwords = nwords_;
-    d.A = d_A_; d.S = d_S_; d.next = d_next_; d.visited = d_visited_;
+    d.A = d_A_; d.S = d_S_; d.next = (fused_ && (iter & 1u)) ? d_next2_ : d_next_; d.visited = d_visited_;
     d.val = d_val_; d.snap = d_snap_;
     d.rank = d_rank_; d.contrib = d_contrib_; d.sum = d_sum_; d.dang = d_dang_;
     d.iter = iter;
@@ -809,6 +810,43 @@ void Part::replace(uint32_t t) {
     host_s_ += std::chrono::duration<double>(std::chrono::steady_clock::now() - th0).count();
 }
 
+// ---- fused exchange: the finalize reads every rank's buffer from peer memory
+void Part::set_fused(bool on) {
+    fused_ = on;
+    if (on && !d_next2_) {
+        dalloc(&d_next2_, nwords_, &vertex_bytes_);
+        CK(cudaMemset(d_next2_, 0, (size_t)std::max<uint32_t>(nwords_, 1) * 4));
+    }
+}
+
+void Part::set_peers(int kind, const std::vector<void*>& ptrs) {
+    const int P = (int)ptrs.size();
+    if (!d_peers_ || peer_world_ != P) {
+        if (d_peers_) cudaFree((void*)d_peers_);
+        CK(cudaMalloc((void**)&d_peers_, 3 * (size_t)P * sizeof(void*)));
+        peer_world_ = P;
+    }
+    CK(cudaMemcpyAsync(d_peers_ + (size_t)kind * P, ptrs.data(), (size_t)P * sizeof(void*), cudaMemcpyHostToDevice, cs_));
+    CK(cudaStreamSynchronize(cs_));
+}
+
+void Part::finalize_fused(uint32_t t) {
+    join_static();
+    cudaEvent_t e0 = mark(cs_);
+    const int kind = algo_ == ALG_BFS ? (int)(t & 1u) : 2;
+    launch_finalize_peers(algo_, dev_state(t), d_peers_ + (size_t)kind * peer_world_, peer_world_, cs_);
+    CK(cudaGetLastError());
+    span(e0, cs_, t, PH_FIN);
+}
+
+void Part::clear_next(uint32_t b) {
+    CK(cudaMemsetAsync(next_buf((int)b), 0, (size_t)nwords_ * 4, cs_));
+}
+
+void Part::clear_prd_inc() {
+    if (d_pr_inc_) CK(cudaMemsetAsync(d_pr_inc_, 0, g_.n * 8, cs_));
+}
+
 void Part::finalize(uint32_t t, bool dense) {
     // ---- next active set, after the static-hit kernels
     join_static();
@@ -1100,6 +1138,7 @@ void Engine::set_option(int opt, int64_t value) {
             if (value < 0 || value > 1000000000ll) throw Error(ASCETIC_EINVAL, "PRD tolerance must be in [0, 1e9] ppm");
             o_.prd_tol_ppm = (uint64_t)value;
             break;
+        case ASCETIC_OPT_FUSED_EXCHANGE: o_.fused_exchange = value ? 1 : 0; break;
         case ASCETIC_OPT_REPLACE_POLICY:
             if (value < 0 || value > 2) throw Error(ASCETIC_EINVAL, "replace policy: 0 = by algorithm, 1 = cumulative, 2 = last");
             o_.replace_policy = (int)value;
@@ -1160,6 +1199,23 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
     const bool multi = comm_.active();
     const bool timing = o_.timing != 0;
     for (auto& p : parts_) p->alloc_algo_state(algo, multi);
+    for (auto& p : parts_) p->set_fused(false);
+    // fused exchange (P > 1, BFS/SSSP/CC/PRD): every part gets the world's buffer pointers
+    const bool fused = multi && o_.fused_exchange && algo != ALG_PR;
+    if (fused) {
+        for (auto& p : parts_) p->set_fused(true);
+        for (int kind = 0; kind < 3; ++kind) {
+            if (kind < 2 && algo != ALG_BFS) continue;
+            auto local = [&](Part& p) -> void* {
+                if (kind < 2) return p.next_buf(kind);
+                return algo == ALG_PRD ? (void*)p.prd_inc() : (void*)p.val();
+            };
+            std::vector<void*> world;
+            if (comm_.emulated()) for (auto& p : parts_) world.push_back(local(*p));
+            else world = comm_.open_peers(local(*parts_[0]));
+            for (auto& p : parts_) p->set_peers(kind, world);
+        }
+    }
     for (auto& p : parts_) p->begin(algo, source, max_iters, timing);
     Part& p0 = *parts_[0];
     std::vector<IterTotals> T(parts_.size());
@@ -1178,6 +1234,25 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
             }
         }
         for (size_t i = 0; i < parts_.size(); ++i) parts_[i]->expand(t, T[i]);
+        if (fused) {
+            // barrier 1: every rank's edge kernels are done before anyone reads its buffer
+            for (auto& p : parts_) p->join_static();
+            cudaEvent_t e0 = p0.mark(p0.cs());
+            if (comm_.emulated()) { join(); fork(); } else comm_.barrier(p0.cs());
+            p0.span(e0, p0.cs(), t, PH_XCH);
+            // BFS: the other next buffer was last read before this barrier: clear it for t+1
+            if (algo == ALG_BFS) for (auto& p : parts_) p->clear_next((t + 1) & 1u);
+            for (auto& p : parts_) p->finalize_fused(t);
+            if (algo != ALG_BFS) {
+                // barrier 2: nobody overwrites its values / increments while a peer still reads them
+                cudaEvent_t e1 = p0.mark(p0.cs());
+                if (comm_.emulated()) { join(); fork(); } else comm_.barrier(p0.cs());
+                p0.span(e1, p0.cs(), t, PH_XCH);
+                if (algo == ALG_PRD) for (auto& p : parts_) p->clear_prd_inc();
+            }
+            for (auto& p : parts_) p->replace(t);
+            continue;
+        }
         if (multi && algo != ALG_PR) {
             // ---- exchange: OR of next bitmaps (BFS), MIN of values (SSSP, CC)
             for (auto& p : parts_) p->join_static();

@@ -63,6 +63,7 @@ struct Options {
     int placement = 0;            // initial static content: 0 = front prefix, 1 = rear suffix, 2 = random chunks
     uint64_t placement_seed = 1;  // seed of the random initial chunk set
     uint64_t prd_tol_ppm = 10000; // PageRank-delta threshold, ppm of the initial residual (1-d)/n
+    int fused_exchange = 0;       // P > 1: exchange fused into finalize over peer memory (NVLink / IPC)
     uint32_t replace_k = 0;       // §3.4 data replacement: chunk swaps examined per iteration (0 = off)
     int replace_policy = 0;       // hotness counter: 0 = by algorithm, 1 = cumulative, 2 = last iteration
 };
@@ -101,6 +102,13 @@ class Part {
     void replace(uint32_t t);                      // §3.4: hotness update + chunk swaps (effective at t+1)
     void join_static();   // cs waits for this iteration's static-hit kernels
     void finalize(uint32_t t, bool dense);
+    // fused exchange (P > 1): the peer tables and the finalize that reads every rank's buffer
+    void set_fused(bool on);   // this run uses the fused exchange (allocates the second next buffer)
+    void set_peers(int kind, const std::vector<void*>& ptrs);   // kind 0/1: next[0/1], 2: val or inc
+    void finalize_fused(uint32_t t);
+    void clear_next(uint32_t b);
+    void clear_prd_inc();
+    uint32_t* next_buf(int b) const { return b ? d_next2_ : d_next_; }
     void end();
     void span(cudaEvent_t a, cudaStream_t s, uint32_t t, int ph);   // close a timed span
     cudaEvent_t mark(cudaStream_t s);                               // open a timed span
@@ -147,6 +155,10 @@ class Part {
     unsigned long long *d_pr_r_ = nullptr, *d_pr_res_ = nullptr, *d_pr_c_ = nullptr;   // PageRank-delta
     unsigned long long* d_pr_inc_ = nullptr;   // P > 1: residual increments of this rank's pushes
     bool multi_ = false;
+    bool fused_ = false;
+    uint32_t* d_next2_ = nullptr;              // fused exchange: next bitmaps double-buffered by iteration parity
+    const void** d_peers_ = nullptr;           // [3][world] device pointers (next0, next1, val/inc)
+    int peer_world_ = 0;
     uint64_t prd_tau_ = 0;
     double *d_sum_ = nullptr, *d_dang_ = nullptr;
     uint32_t *d_hq_small_ = nullptr, *d_hq_med_ = nullptr, *d_hq_hub_ = nullptr, *d_hub_pre_ = nullptr;
