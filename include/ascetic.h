@@ -245,6 +245,9 @@ int ascetic_get_result(void* host_dst, uint64_t bytes);
  *   ascetic_get_unique_id  rank 0: 128-byte NCCL unique id (EUNSUPPORTED if libnccl.so.2
  *                          cannot be loaded); share it out of band (torch.distributed)
  *   ascetic_comm_init      every rank, BEFORE load_csr; device = this rank's GPU
+ *                          world = 1 with a unique id builds a one-rank NCCL communicator
+ *                          (the exchange path runs through NCCL; used to test it on one GPU);
+ *                          world = 1 with uid128 = NULL drops any communicator
  *   ascetic_emulate_ranks  drive `world` ranks from THIS process on its one GPU (each rank a
  *                          full engine with its own device state; collectives by device copies).
  *                          Same per-rank code path and per-rank statistics; for testing the

@@ -71,7 +71,10 @@ void Comm::init_nccl(int rank, int world, const void* uid128) {
     destroy();
     if (world < 1 || rank < 0 || rank >= world) throw Error(ASCETIC_EINVAL, "bad rank/world");
     world_ = world; rank_ = rank; emulated_ = false;
-    if (world == 1) return;
+    // world 1 without an id: no communicator (single GPU). world 1 WITH an id: a one-rank NCCL
+    // communicator, so the whole exchange path (collectives, barriers, IPC handle exchange)
+    // runs through NCCL on one GPU — how that path is exercised without a multi-GPU box.
+    if (world == 1 && !uid128) return;
     ncclUniqueId id;
     std::memcpy(&id, uid128, sizeof id);
     ncclComm_t c = nullptr;
@@ -86,10 +89,8 @@ void Comm::init_emulated(int world) {
 }
 
 void Comm::destroy() {
-    for (auto& e : peers_)
-        for (int p = 0; p < (int)e.second.size(); ++p)
-            if (p != rank_ && e.second[p]) cudaIpcCloseMemHandle(e.second[p]);
-    peers_.clear();
+    for (auto& m : peer_maps_) cudaIpcCloseMemHandle(m.ptr);
+    peer_maps_.clear();
     if (barrier_buf_) { cudaFree(barrier_buf_); barrier_buf_ = nullptr; }
     if (nccl_comm_) { nccl().CommDestroy((ncclComm_t)nccl_comm_); nccl_comm_ = nullptr; }
     if (scratch_) { cudaFree(scratch_); scratch_ = nullptr; scratch_words_ = 0; }
@@ -149,8 +150,9 @@ void Comm::sum_u64(const std::vector<unsigned long long*>& local, uint64_t n, cu
 
 std::vector<void*> Comm::open_peers(void* local) {
     if (emulated_ || !active()) throw Error(ASCETIC_EINVAL, "open_peers needs the NCCL back end");
-    for (auto& e : peers_)
-        if (e.first == local) return e.second;
+    // Always collective: every rank all-gathers its current handle, whatever its cache holds
+    // (a rank that re-allocated while another did not must not leave that one waiting in a
+    // skipped all-gather). A peer mapping is reused only while the peer's handle is unchanged.
     cudaIpcMemHandle_t h;
     CKc(cudaIpcGetMemHandle(&h, local), "cudaIpcGetMemHandle");
     char* dbuf = nullptr;
@@ -165,9 +167,15 @@ std::vector<void*> Comm::open_peers(void* local) {
     std::vector<void*> ptrs(world_, nullptr);
     for (int p = 0; p < world_; ++p) {
         if (p == rank_) { ptrs[p] = local; continue; }
+        for (auto& m : peer_maps_)
+            if (m.rank == p && std::memcmp(m.handle, &all[p], sizeof h) == 0) { ptrs[p] = m.ptr; break; }
+        if (ptrs[p]) continue;
         CKc(cudaIpcOpenMemHandle(&ptrs[p], all[p], cudaIpcMemLazyEnablePeerAccess), "cudaIpcOpenMemHandle");
+        PeerMap m;
+        m.rank = p; m.ptr = ptrs[p];
+        std::memcpy(m.handle, &all[p], sizeof h);
+        peer_maps_.push_back(m);
     }
-    peers_.emplace_back(local, ptrs);
     return ptrs;
 }
 

@@ -30,7 +30,7 @@ class Comm {
     void destroy();
     ~Comm() { destroy(); }
 
-    bool active() const { return world_ > 1; }
+    bool active() const { return world_ > 1 || nccl_comm_ != nullptr; }
     bool emulated() const { return emulated_; }
     int world() const { return world_; }
     int rank() const { return rank_; }
@@ -43,7 +43,7 @@ class Comm {
     // element-wise SUM of n uint64 per rank (PageRank-delta residual increments), in place
     void sum_u64(const std::vector<unsigned long long*>& local, uint64_t n, cudaStream_t s);
     // Fused exchange support (NCCL back end): map every rank's `local` device allocation into this
-    // process with CUDA IPC (handles all-gathered over NCCL; cached per pointer); returns the
+    // process with CUDA IPC (handles all-gathered over NCCL on every call; a peer's mapping is reused while its handle is unchanged); returns the
     // world pointers, this rank's own at index rank(). Collective: every rank calls it.
     std::vector<void*> open_peers(void* local);
     // stream-ordered barrier over all ranks (a 4-byte ncclAllReduce); no-op when emulated
@@ -60,7 +60,12 @@ class Comm {
     uint32_t* scratch_ = nullptr;
     uint64_t scratch_words_ = 0;
     int* barrier_buf_ = nullptr;
-    std::vector<std::pair<void*, std::vector<void*>>> peers_;   // local pointer -> world pointers (IPC)
+    struct PeerMap {   // an opened CUDA IPC mapping of a peer's allocation
+        int rank;
+        unsigned char handle[64];   // CUDA_IPC_HANDLE_SIZE
+        void* ptr;
+    };
+    std::vector<PeerMap> peer_maps_;
 };
 
 }  // namespace ascetic
