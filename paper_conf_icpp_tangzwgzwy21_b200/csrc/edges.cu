@@ -16,6 +16,7 @@
 //    queue's 64-bit prefix (one global binary search per CTA).
 //  * the gather is a zero-copy SM copy: host arcs are read through the mapped pinned
 //    CSR with the same arc->source map, so the host never needs the request list.
+#include <cstdlib>
 #include <type_traits>
 
 #include "ascetic_internal.h"
@@ -521,12 +522,9 @@ __device__ __forceinline__ uint32_t warp_map(const unsigned long long* s_pre, ui
 
 // ------------------------------------------------------------------ on-demand compute
 template <int ALGO>
-__global__ void __launch_bounds__(256) k_ondemand(DevState d, Queues q, const void* __restrict__ chunk,
-                                                  unsigned long long lo, unsigned long long hi) {
-    __shared__ unsigned long long s_pre[kEdgeTile + 1];
-    __shared__ uint32_t s_u[kEdgeTile + 1];
-    __shared__ SrcVal<ALGO> s_v[kEdgeTile + 1];
-    const unsigned long long t = (lo >> kEdgeTileShift) + blockIdx.x;
+__device__ __forceinline__ void ondemand_tile(const DevState& d, const Queues& q, const void* __restrict__ chunk,
+                                              unsigned long long lo, unsigned long long hi, unsigned long long t,
+                                              unsigned long long* s_pre, uint32_t* s_u, SrcVal<ALGO>* s_v) {
     const Tile x = tile_of(q, t, lo, hi);
     for (uint32_t k = threadIdx.x; k < x.cnt; k += blockDim.x) {
         s_pre[k] = __ldg(q.mq_pre + x.i0 + k);
@@ -620,6 +618,20 @@ __global__ void __launch_bounds__(256) k_ondemand(DevState d, Queues q, const vo
     }
 }
 
+// one CTA per 2048-arc tile of the chunk window, or a capped grid striding over the tiles
+template <int ALGO>
+__global__ void __launch_bounds__(256) k_ondemand(DevState d, Queues q, const void* __restrict__ chunk,
+                                                  unsigned long long lo, unsigned long long hi) {
+    __shared__ unsigned long long s_pre[kEdgeTile + 1];
+    __shared__ uint32_t s_u[kEdgeTile + 1];
+    __shared__ SrcVal<ALGO> s_v[kEdgeTile + 1];
+    const unsigned long long t0 = lo >> kEdgeTileShift, t1 = (hi - 1) >> kEdgeTileShift;
+    for (unsigned long long t = t0 + blockIdx.x; t <= t1; t += gridDim.x) {
+        if (t != t0 + blockIdx.x) __syncthreads();   // the previous tile's warps are done with smem
+        ondemand_tile<ALGO>(d, q, chunk, lo, hi, t, s_pre, s_u, s_v);
+    }
+}
+
 // BFS needs no source: 128-bit loads straight over the chunk.
 __global__ void __launch_bounds__(256) k_ondemand_bfs(DevState d, const uint32_t* __restrict__ chunk,
                                                       unsigned long long len) {
@@ -677,6 +689,113 @@ __global__ void __launch_bounds__(256) k_gather(Queues q, const void* __restrict
         for (int g = 0; g < 8; ++g) {
             const unsigned long long a = pw + 32ull * g + lane;
             if (a < pe) dst[a - lo] = v[g];
+        }
+    }
+}
+
+// 16-byte cover gather (default). Measured on the box (tools/zc_align.cu, profiles/r01/zc_align.log):
+// zero-copy reads of random host runs reach ~44 GB/s with 4-byte loads, ~48 with 8-byte and
+// ~50 with 16-byte loads, even when the runs start 4-byte aligned and the 16-byte cover is read
+// (the extra bytes sit in sectors that are fetched anyway). So lanes here load 16-byte-aligned
+// units of host memory: per warp segment of 256 stream arcs, the missed vertices are grouped
+// into pieces (maximal runs whose lists are adjacent on the host: one stream->host offset per
+// piece), each piece's cover units are enumerated across the warp (a unit shared by two
+// vertices of one piece is loaded once), and every lane stores the piece words its unit holds
+// at their stream position. `hoff` = the host array's byte offset from its 16-byte-aligned base.
+template <int BE>
+__global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restrict__ host, uint32_t hoff,
+                                                  uint32_t* __restrict__ chunk, unsigned long long lo,
+                                                  unsigned long long hi) {
+    __shared__ unsigned long long s_pre[kEdgeTile + 1];
+    __shared__ unsigned long long s_src[kEdgeTile + 1];
+    constexpr unsigned long long AW = BE / 4;                 // words per arc
+    const unsigned long long w_off = hoff / 4;                // host word index of arc 0
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const unsigned long long t0 = lo >> kEdgeTileShift, t1 = (hi - 1) >> kEdgeTileShift;
+    for (unsigned long long t = t0 + blockIdx.x; t <= t1; t += gridDim.x) {
+        const Tile x = tile_of(q, t, lo, hi);
+        __syncthreads();
+        for (uint32_t k = threadIdx.x; k < x.cnt; k += blockDim.x) {
+            s_pre[k] = __ldg(q.mq_pre + x.i0 + k);
+            s_src[k] = __ldg(q.mq_src + x.i0 + k);
+        }
+        __syncthreads();
+        const unsigned long long pw = x.t_lo + (unsigned long long)warp * 256ull;
+        if (pw >= x.t_hi) continue;
+        const unsigned long long pe = min(x.t_hi, pw + 256ull);
+        const uint32_t kfirst = find_local(s_pre, 0, x.cnt, pw);
+        const uint32_t klast = find_local(s_pre, kfirst, x.cnt, pe - 1);
+        for (uint32_t kb = kfirst; kb <= klast; kb += 32) {
+            // lane <-> vertex j of the segment: stream arcs [a0, a1), host arcs [h0, h1)
+            const uint32_t j = kb + (uint32_t)lane;
+            const bool v = j <= klast;
+            unsigned long long a0 = 0, a1 = 0, h0 = 0;
+            if (v) {
+                const unsigned long long pj = s_pre[j];
+                const unsigned long long ej = (j + 1 < x.cnt) ? s_pre[j + 1] : ~0ull;
+                a0 = max(pw, pj);
+                a1 = max(a0, min(pe, ej));
+                h0 = s_src[j] + (a0 - pj);
+            }
+            const unsigned long long h1 = h0 + (a1 - a0);
+            const unsigned long long ph1 = __shfl_up_sync(FULL, h1, 1);
+            const bool start = v && (lane == 0 || h0 != ph1);
+            const uint32_t smask = __ballot_sync(FULL, start);
+            const uint32_t vmask = __ballot_sync(FULL, v);
+            const int ps = 31 - __clz(smask & ((2u << lane) - 1u));          // this lane's piece start
+            const uint32_t after = lane == 31 ? 0u : (smask & ~((2u << lane) - 1u));
+            const int pl = after ? (__ffs(after) - 2) : (31 - __clz(vmask)); // and its last lane
+            const unsigned long long W0 = w_off + __shfl_sync(FULL, h0, ps) * AW;   // piece host words [W0, W1)
+            const unsigned long long W1 = w_off + __shfl_sync(FULL, h1, pl) * AW;
+            const unsigned long long D0 = (__shfl_sync(FULL, a0, ps) - lo) * AW;    // chunk word of W0
+            const unsigned long long hw0 = w_off + h0 * AW, hw1 = w_off + h1 * AW;
+            // cover units of this lane's words not already covered by the previous lane of the piece
+            const unsigned long long u0 = start ? (hw0 >> 2) : ((hw0 + 3) >> 2);
+            const unsigned long long u1 = (hw1 + 3) >> 2;
+            const uint32_t cnt = (v && hw1 > hw0 && u1 > u0) ? (uint32_t)(u1 - u0) : 0u;
+            uint32_t incl = cnt;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(FULL, incl, o);
+                if (lane >= o) incl += y;
+            }
+            const uint32_t excl = incl - cnt;
+            const uint32_t total = __shfl_sync(FULL, incl, 31);
+            for (uint32_t b = 0; b < total; b += 128) {
+                // 4 groups of 32 units: all loads first (4 x 16 B in flight per lane), then the stores
+                uint4 val[4];
+                unsigned long long uw[4], pw0[4], pw1[4], pd0[4];
+#pragma unroll
+                for (int g = 0; g < 4; ++g) {
+                    const uint32_t tt = b + 32u * g + (uint32_t)lane;
+                    int i = 0;
+#pragma unroll
+                    for (int step = 16; step >= 1; step >>= 1) {
+                        const uint32_t y = __shfl_sync(FULL, incl, i + step - 1);
+                        if (y <= tt) i += step;
+                    }
+                    const unsigned long long uo = __shfl_sync(FULL, u0, i);
+                    const uint32_t eo = __shfl_sync(FULL, excl, i);
+                    pw0[g] = __shfl_sync(FULL, W0, i);
+                    pw1[g] = __shfl_sync(FULL, W1, i);
+                    pd0[g] = __shfl_sync(FULL, D0, i);
+                    uw[g] = ~0ull;
+                    if (tt < total) {
+                        uw[g] = uo + (tt - eo);
+                        val[g] = host[uw[g]];
+                    }
+                }
+#pragma unroll
+                for (int g = 0; g < 4; ++g) {
+                    if (uw[g] == ~0ull) continue;
+                    const uint32_t wv[4] = {val[g].x, val[g].y, val[g].z, val[g].w};
+#pragma unroll
+                    for (int c = 0; c < 4; ++c) {
+                        const unsigned long long w = uw[g] * 4 + c;
+                        if (w >= pw0[g] && w < pw1[g]) chunk[pd0[g] + (w - pw0[g])] = wv[c];
+                    }
+                }
+            }
         }
     }
 }
@@ -1192,7 +1311,9 @@ void launch_ondemand(int algo, const DevState& d, const Queues& q, const void* c
         ++g_launches;
         return;
     }
-    const unsigned tiles = (unsigned)(((hi - 1) >> kEdgeTileShift) - (lo >> kEdgeTileShift) + 1);
+    unsigned tiles = (unsigned)(((hi - 1) >> kEdgeTileShift) - (lo >> kEdgeTileShift) + 1);
+    static const int cap = [] { const char* e = std::getenv("ASC_OND_CTAS"); return e ? std::atoi(e) : 0; }();
+    if (cap > 0 && tiles > (unsigned)cap) tiles = (unsigned)cap;
     switch (algo) {
         case SSSP: k_ondemand<SSSP><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
         case CC: k_ondemand<CC><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
@@ -1207,8 +1328,27 @@ void launch_gather(const Queues& q, const void* host_nbr, uint32_t b_e, void* ch
     if (hi <= lo) return;
     const unsigned long long tiles = ((hi - 1) >> kEdgeTileShift) - (lo >> kEdgeTileShift) + 1;
     const unsigned grid = (unsigned)(tiles < (unsigned long long)max_ctas ? tiles : (unsigned long long)max_ctas);
-    if (b_e == 8) k_gather<8><<<grid, 256, 0, s>>>(q, host_nbr, chunk, lo, hi);
-    else k_gather<4><<<grid, 256, 0, s>>>(q, host_nbr, chunk, lo, hi);
+    // dev knob: extra dynamic shared memory per gather CTA caps how many gather CTAs share an SM
+    static const int dsm = [] {
+        const char* e = std::getenv("ASC_GATHER_DSMEM");
+        const int v = e ? std::atoi(e) : 0;
+        if (v > 0) {
+            cudaFuncSetAttribute(k_gather<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, v);
+            cudaFuncSetAttribute(k_gather<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, v);
+        }
+        return v;
+    }();
+    static const bool old = [] { const char* e = std::getenv("ASC_GATHER_OLD"); return e && std::atoi(e); }();
+    if (old) {
+        if (b_e == 8) k_gather<8><<<grid, 256, dsm, s>>>(q, host_nbr, chunk, lo, hi);
+        else k_gather<4><<<grid, 256, dsm, s>>>(q, host_nbr, chunk, lo, hi);
+    } else {
+        const uintptr_t hp = reinterpret_cast<uintptr_t>(host_nbr);
+        const uint4* base = reinterpret_cast<const uint4*>(hp & ~(uintptr_t)15);
+        const uint32_t hoff = (uint32_t)(hp & 15);
+        if (b_e == 8) k_gather16<8><<<grid, 256, 0, s>>>(q, base, hoff, reinterpret_cast<uint32_t*>(chunk), lo, hi);
+        else k_gather16<4><<<grid, 256, 0, s>>>(q, base, hoff, reinterpret_cast<uint32_t*>(chunk), lo, hi);
+    }
     ++g_launches;
 }
 
