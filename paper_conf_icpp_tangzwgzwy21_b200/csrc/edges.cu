@@ -521,18 +521,38 @@ __device__ __forceinline__ uint32_t warp_map(const unsigned long long* s_pre, ui
 }
 
 // ------------------------------------------------------------------ on-demand compute
-template <int ALGO>
+// Tile metadata either staged in shared memory (SMEM) or read straight from the queues (L1-cached):
+// the zero-shared-memory variant can co-reside with any kernel whatever the SM's L1/shared split.
+template <int ALGO, bool SMEM>
+struct TileView {
+    const unsigned long long* pre;
+    const uint32_t* u;
+    const SrcVal<ALGO>* v;
+    const DevState* d;
+    __device__ __forceinline__ uint32_t vtx(uint32_t k) const { return SMEM ? u[k] : __ldg(u + k); }
+    __device__ __forceinline__ SrcVal<ALGO> val(uint32_t k) const { return SMEM ? v[k] : src_val<ALGO>(*d, __ldg(u + k)); }
+};
+
+template <int ALGO, bool SMEM>
 __device__ __forceinline__ void ondemand_tile(const DevState& d, const Queues& q, const void* __restrict__ chunk,
                                               unsigned long long lo, unsigned long long hi, unsigned long long t,
-                                              unsigned long long* s_pre, uint32_t* s_u, SrcVal<ALGO>* s_v) {
+                                              unsigned long long* s_pre_, uint32_t* s_u_, SrcVal<ALGO>* s_v_) {
     const Tile x = tile_of(q, t, lo, hi);
-    for (uint32_t k = threadIdx.x; k < x.cnt; k += blockDim.x) {
-        s_pre[k] = __ldg(q.mq_pre + x.i0 + k);
-        const uint32_t u = __ldg(q.mq + x.i0 + k);
-        s_u[k] = u;
-        if (ALGO != PR) s_v[k] = src_val<ALGO>(d, u);
+    if (SMEM) {
+        for (uint32_t k = threadIdx.x; k < x.cnt; k += blockDim.x) {
+            s_pre_[k] = __ldg(q.mq_pre + x.i0 + k);
+            const uint32_t u = __ldg(q.mq + x.i0 + k);
+            s_u_[k] = u;
+            if (ALGO != PR) s_v_[k] = src_val<ALGO>(d, u);
+        }
+        __syncthreads();
     }
-    __syncthreads();
+    TileView<ALGO, SMEM> tv;
+    tv.pre = SMEM ? s_pre_ : q.mq_pre + x.i0;
+    tv.u = SMEM ? s_u_ : q.mq + x.i0;
+    tv.v = s_v_;
+    tv.d = &d;
+    const unsigned long long* s_pre = tv.pre;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const unsigned long long pw = x.t_lo + (unsigned long long)warp * 256ull;
     if (pw >= x.t_hi) return;
@@ -549,7 +569,7 @@ __device__ __forceinline__ void ondemand_tile(const DevState& d, const Queues& q
             k = __shfl_sync(FULL, mk, 31);
             const unsigned long long a = p + lane;
             id[g] = kInf;
-            c[g] = s_v[mk];
+            c[g] = tv.val(mk);
             if (a < pe) id[g] = ld_stream(reinterpret_cast<const uint32_t*>(chunk) + (a - lo));
         }
 #pragma unroll
@@ -569,10 +589,10 @@ __device__ __forceinline__ void ondemand_tile(const DevState& d, const Queues& q
                 if (ALGO == SSSP) {
                     const uint2 e = ld_stream(reinterpret_cast<const uint2*>(chunk) + (a - lo));
                     id[g] = e.x;
-                    cand[g] = sat_add(s_v[mk], e.y);
+                    cand[g] = sat_add(tv.val(mk), e.y);
                 } else {
                     id[g] = ld_stream(reinterpret_cast<const uint32_t*>(chunk) + (a - lo));
-                    cand[g] = s_v[mk];
+                    cand[g] = tv.val(mk);
                 }
             }
         }
@@ -613,7 +633,7 @@ __device__ __forceinline__ void ondemand_tile(const DevState& d, const Queues& q
                 if (lane >= o && ok2 == key) v += y;
             }
             const int nk = __shfl_down_sync(FULL, key, 1);
-            if (ok && (lane == 31 || nk != key)) atomicAdd(d.sum + s_u[mk8[g]], v);
+            if (ok && (lane == 31 || nk != key)) atomicAdd(d.sum + tv.vtx(mk8[g]), v);
         }
     }
 }
@@ -628,8 +648,16 @@ __global__ void __launch_bounds__(256) k_ondemand(DevState d, Queues q, const vo
     const unsigned long long t0 = lo >> kEdgeTileShift, t1 = (hi - 1) >> kEdgeTileShift;
     for (unsigned long long t = t0 + blockIdx.x; t <= t1; t += gridDim.x) {
         if (t != t0 + blockIdx.x) __syncthreads();   // the previous tile's warps are done with smem
-        ondemand_tile<ALGO>(d, q, chunk, lo, hi, t, s_pre, s_u, s_v);
+        ondemand_tile<ALGO, true>(d, q, chunk, lo, hi, t, s_pre, s_u, s_v);
     }
+}
+
+template <int ALGO>
+__global__ void __launch_bounds__(256) k_ondemand_g(DevState d, Queues q, const void* __restrict__ chunk,
+                                                    unsigned long long lo, unsigned long long hi) {
+    const unsigned long long t0 = lo >> kEdgeTileShift, t1 = (hi - 1) >> kEdgeTileShift;
+    for (unsigned long long t = t0 + blockIdx.x; t <= t1; t += gridDim.x)
+        ondemand_tile<ALGO, false>(d, q, chunk, lo, hi, t, nullptr, nullptr, nullptr);
 }
 
 // BFS needs no source: 128-bit loads straight over the chunk.
@@ -702,24 +730,28 @@ __global__ void __launch_bounds__(256) k_gather(Queues q, const void* __restrict
 // piece), each piece's cover units are enumerated across the warp (a unit shared by two
 // vertices of one piece is loaded once), and every lane stores the piece words its unit holds
 // at their stream position. `hoff` = the host array's byte offset from its 16-byte-aligned base.
-template <int BE>
+template <int BE, bool SMEM>
 __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restrict__ host, uint32_t hoff,
                                                   uint32_t* __restrict__ chunk, unsigned long long lo,
                                                   unsigned long long hi) {
-    __shared__ unsigned long long s_pre[kEdgeTile + 1];
-    __shared__ unsigned long long s_src[kEdgeTile + 1];
+    __shared__ unsigned long long sm_pre[SMEM ? kEdgeTile + 1 : 1];
+    __shared__ unsigned long long sm_src[SMEM ? kEdgeTile + 1 : 1];
     constexpr unsigned long long AW = BE / 4;                 // words per arc
     const unsigned long long w_off = hoff / 4;                // host word index of arc 0
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const unsigned long long t0 = lo >> kEdgeTileShift, t1 = (hi - 1) >> kEdgeTileShift;
     for (unsigned long long t = t0 + blockIdx.x; t <= t1; t += gridDim.x) {
         const Tile x = tile_of(q, t, lo, hi);
-        __syncthreads();
-        for (uint32_t k = threadIdx.x; k < x.cnt; k += blockDim.x) {
-            s_pre[k] = __ldg(q.mq_pre + x.i0 + k);
-            s_src[k] = __ldg(q.mq_src + x.i0 + k);
+        const unsigned long long* s_pre = SMEM ? sm_pre : q.mq_pre + x.i0;
+        const unsigned long long* s_src = SMEM ? sm_src : q.mq_src + x.i0;
+        if (SMEM) {
+            __syncthreads();
+            for (uint32_t k = threadIdx.x; k < x.cnt; k += blockDim.x) {
+                sm_pre[k] = __ldg(q.mq_pre + x.i0 + k);
+                sm_src[k] = __ldg(q.mq_src + x.i0 + k);
+            }
+            __syncthreads();
         }
-        __syncthreads();
         const unsigned long long pw = x.t_lo + (unsigned long long)warp * 256ull;
         if (pw >= x.t_hi) continue;
         const unsigned long long pe = min(x.t_hi, pw + 256ull);
@@ -1235,9 +1267,27 @@ inline unsigned blocks_for(unsigned long long n, int per_block, unsigned cap = 1
     return (unsigned)(b > cap ? cap : b);
 }
 
+// Every kernel that can run concurrently with another (static-hit, on-demand, gather, chunk copy)
+// asks for the same L1/shared carveout (maximum shared). With the default per-kernel choice an SM
+// running only k_static_med (no shared memory) is configured for maximum L1, and the on-demand
+// kernel launched next (33 KB of shared memory per CTA) finds no SM it can use until the 9 ms
+// static kernel drains: measured on C3 as one 8-11 ms on-demand kernel per iteration (ASCETIC_TRACE=2)
+// that stalled chunk-buffer reuse and idled the host link ~5 ms per iteration.
+template <typename K>
+void carve(K* k, const char* env = "ASC_CARVE") {
+    const char* e = std::getenv(env);
+    const int pct = e ? std::atoi(e) : -1;   // dev A/B: percent of the maximum shared memory
+    if (pct < 0) return;
+    cudaFuncSetAttribute(reinterpret_cast<const void*>(k), cudaFuncAttributePreferredSharedMemoryCarveout, pct);
+}
+
 template <int ALGO, bool REMAP>
 void static_launch_t(const DevState& d, const Queues& q, const void* sbase, uint32_t ns, uint32_t nm, uint32_t nh,
                      uint32_t npieces, uint32_t piece, int max_ctas, cudaStream_t s) {
+    static const bool carved = (carve(k_static_small<ALGO, REMAP>, "ASC_CARVE_STATIC"),
+                                carve(k_static_med<ALGO, REMAP>, "ASC_CARVE_STATIC"),
+                                carve(k_static_hub<ALGO, REMAP>, "ASC_CARVE_STATIC"), true);
+    (void)carved;
     auto cap = [&](unsigned long long b) { return (unsigned)(b < (unsigned long long)max_ctas ? b : max_ctas); };
     if (ns) { k_static_small<ALGO, REMAP><<<cap((ns + 255) / 256), 256, 0, s>>>(d, q.hq_small, ns, sbase); ++g_launches; }
     if (nm) { k_static_med<ALGO, REMAP><<<cap((nm + 7) / 8), 256, 0, s>>>(d, q.hq_med, nm, sbase); ++g_launches; }
@@ -1271,6 +1321,8 @@ void launch_chunk_access(const DevState& d, const Queues& q, uint32_t n_small, u
                          uint32_t b_e, uint32_t* acc, cudaStream_t s) {
     const unsigned long long total = (unsigned long long)n_small + n_med + n_hub + q.n_missq;
     if (!total) return;
+    static const bool carved = (carve(k_chunk_access), true);
+    (void)carved;
     const uint32_t epc_shift = kChunkShift - (b_e == 8 ? 3 : 2);
     k_chunk_access<<<blocks_for(total, 256), 256, 0, s>>>(d, q, n_small, n_med, n_hub, epc_shift, acc);
     ++g_launches;
@@ -1288,6 +1340,8 @@ void launch_apply_swaps(const DevState& d, uint32_t* slot_of, const uint32_t* sw
 void launch_copy_chunks(const void* host_dev, uint64_t x0, uint64_t D, const uint32_t* ids, const uint32_t* slots,
                         uint32_t count, void* dst, cudaStream_t s) {
     if (!count) return;
+    static const bool carved = (carve(k_copy_chunks), true);
+    (void)carved;
     // 64 CTAs x 16 KiB = 1 MiB of host reads in flight (the transfer engine's sizing)
     k_copy_chunks<<<count < 64u ? count : 64u, 256, 0, s>>>(reinterpret_cast<const char*>(host_dev), x0, D, ids, slots,
                                                           count, reinterpret_cast<char*>(dst));
@@ -1311,9 +1365,27 @@ void launch_ondemand(int algo, const DevState& d, const Queues& q, const void* c
         ++g_launches;
         return;
     }
+    static const bool carved = (carve(k_ondemand<SSSP>), carve(k_ondemand<CC>), carve(k_ondemand<PRD>),
+                                carve(k_ondemand<PR>), carve(k_ondemand_bfs), true);
+    (void)carved;
     unsigned tiles = (unsigned)(((hi - 1) >> kEdgeTileShift) - (lo >> kEdgeTileShift) + 1);
     static const int cap = [] { const char* e = std::getenv("ASC_OND_CTAS"); return e ? std::atoi(e) : 0; }();
     if (cap > 0 && tiles > (unsigned)cap) tiles = (unsigned)cap;
+    // Zero-shared-memory variant by default: the staged one (33 KB per CTA, ASC_OND_SMEM=1) cannot
+    // start on SMs whose L1/shared split was chosen for a shared-memory-free static kernel, and
+    // waited out each 9 ms k_static_med on C3 (one 8-11 ms on-demand kernel per iteration that
+    // stalled chunk-buffer reuse: 35-38 ms of link gaps per 6 iterations -> 0.7 ms; ASCETIC_TRACE=2).
+    static const bool gv = [] { const char* e = std::getenv("ASC_OND_SMEM"); return !(e && std::atoi(e)); }();
+    if (gv) {
+        switch (algo) {
+            case SSSP: k_ondemand_g<SSSP><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
+            case CC: k_ondemand_g<CC><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
+            case PRD: k_ondemand_g<PRD><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
+            default: k_ondemand_g<PR><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
+        }
+        ++g_launches;
+        return;
+    }
     switch (algo) {
         case SSSP: k_ondemand<SSSP><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
         case CC: k_ondemand<CC><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
@@ -1338,6 +1410,8 @@ void launch_gather(const Queues& q, const void* host_nbr, uint32_t b_e, void* ch
         }
         return v;
     }();
+    static const bool carved = (carve(k_gather<4>), carve(k_gather<8>), carve(k_gather16<4, true>), carve(k_gather16<8, true>), true);
+    (void)carved;
     static const bool old = [] { const char* e = std::getenv("ASC_GATHER_OLD"); return e && std::atoi(e); }();
     if (old) {
         if (b_e == 8) k_gather<8><<<grid, 256, dsm, s>>>(q, host_nbr, chunk, lo, hi);
@@ -1346,8 +1420,17 @@ void launch_gather(const Queues& q, const void* host_nbr, uint32_t b_e, void* ch
         const uintptr_t hp = reinterpret_cast<uintptr_t>(host_nbr);
         const uint4* base = reinterpret_cast<const uint4*>(hp & ~(uintptr_t)15);
         const uint32_t hoff = (uint32_t)(hp & 15);
-        if (b_e == 8) k_gather16<8><<<grid, 256, 0, s>>>(q, base, hoff, reinterpret_cast<uint32_t*>(chunk), lo, hi);
-        else k_gather16<4><<<grid, 256, 0, s>>>(q, base, hoff, reinterpret_cast<uint32_t*>(chunk), lo, hi);
+        // tile metadata staged in shared memory (A/B: the zero-shared-memory variant, ASC_GATHER_SMEM=0,
+        // gathers at the same rate but its L1 metadata reads slow the concurrent static kernels)
+        static const bool sm = [] { const char* e = std::getenv("ASC_GATHER_SMEM"); return !(e && !std::atoi(e)); }();
+        uint32_t* c = reinterpret_cast<uint32_t*>(chunk);
+        if (sm) {
+            if (b_e == 8) k_gather16<8, true><<<grid, 256, 0, s>>>(q, base, hoff, c, lo, hi);
+            else k_gather16<4, true><<<grid, 256, 0, s>>>(q, base, hoff, c, lo, hi);
+        } else {
+            if (b_e == 8) k_gather16<8, false><<<grid, 256, 0, s>>>(q, base, hoff, c, lo, hi);
+            else k_gather16<4, false><<<grid, 256, 0, s>>>(q, base, hoff, c, lo, hi);
+        }
     }
     ++g_launches;
 }

@@ -420,11 +420,11 @@ cudaEvent_t Part::mark(cudaStream_t s) {
     return e;
 }
 
-void Part::span(cudaEvent_t a, cudaStream_t s, uint32_t t, int ph) {
+void Part::span(cudaEvent_t a, cudaStream_t s, uint32_t t, int ph, int sub) {
     if (!timing_) return;
     cudaEvent_t e = pool_.get();
     CK(cudaEventRecord(e, s));
-    spans_.push_back({a, e, t, ph});
+    spans_.push_back({a, e, t, ph, sub});
 }
 
 // ---- transfer engine: chunk = miss-stream arcs [lo, hi). mode 1: zero-copy SM gather over
@@ -600,13 +600,24 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     if (T.n_small + T.n_med + T.n_hub) {
         CK(cudaEventRecord(static_go_, cs_));
         CK(cudaStreamWaitEvent(ss_, static_go_, 0));
-        cudaEvent_t e0 = mark(ss_);
         // persistent grid: 4 CTAs/SM leave room for the on-demand kernels; an iteration without
         // misses (resident lists only) takes every slot
         const int cps = o_.static_ctas_per_sm > 0 ? o_.static_ctas_per_sm : (T.miss_arcs ? 4 : 8);
-        launch_static(algo_, d, q, d_static_, T.n_small, T.n_med, T.n_hub, T.n_pieces, kPieceArcs, cps * sm_count_, ss_);
-        CK(cudaGetLastError());
-        span(e0, ss_, t, PH_STATIC);
+        static const bool split = [] { const char* e = std::getenv("ASCETIC_TRACE"); return e && e[0] == '2'; }();
+        if (split && timing_) {   // timeline of the three degree buckets (dev: ASCETIC_TRACE=2)
+            for (int b = 0; b < 3; ++b) {
+                cudaEvent_t e0 = mark(ss_);
+                launch_static(algo_, d, q, d_static_, b == 0 ? T.n_small : 0, b == 1 ? T.n_med : 0,
+                              b == 2 ? T.n_hub : 0, T.n_pieces, kPieceArcs, cps * sm_count_, ss_);
+                CK(cudaGetLastError());
+                span(e0, ss_, t, PH_STATIC, 1 + b);
+            }
+        } else {
+            cudaEvent_t e0 = mark(ss_);
+            launch_static(algo_, d, q, d_static_, T.n_small, T.n_med, T.n_hub, T.n_pieces, kPieceArcs, cps * sm_count_, ss_);
+            CK(cudaGetLastError());
+            span(e0, ss_, t, PH_STATIC);
+        }
         CK(cudaEventRecord(static_done_, ss_));
         static_pending_ = true;
         static_launched_ = true;
@@ -875,10 +886,11 @@ void Part::end() {
     for (const Span& sp : spans_) {
         float a = 0.f;
         CK(cudaEventElapsedTime(&a, sp.a, sp.b));
-        if (trace && trace[0] == '1') {   // timeline: rank iter kernel-class start end (ms from run start)
+        if (trace && (trace[0] == '1' || trace[0] == '2')) {   // timeline: rank iter kernel-class start end (ms from run start)
             float s0 = 0.f;
             CK(cudaEventElapsedTime(&s0, ev_start_, sp.a));
-            std::fprintf(stderr, "TRACE %d %u %s %.4f %.4f\n", rank_, sp.iter, kPhName[sp.ph], s0, s0 + a);
+            static const char* kSub[4] = {"", "_small", "_med", "_hub"};
+            std::fprintf(stderr, "TRACE %d %u %s%s %.4f %.4f\n", rank_, sp.iter, kPhName[sp.ph], kSub[sp.sub & 3], s0, s0 + a);
         }
         ph[sp.ph] += a;
         if (sp.iter < iters.size()) {

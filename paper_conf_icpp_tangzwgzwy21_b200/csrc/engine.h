@@ -110,7 +110,7 @@ class Part {
     void clear_prd_inc();
     uint32_t* next_buf(int b) const { return b ? d_next2_ : d_next_; }
     void end();
-    void span(cudaEvent_t a, cudaStream_t s, uint32_t t, int ph);   // close a timed span
+    void span(cudaEvent_t a, cudaStream_t s, uint32_t t, int ph, int sub = 0);   // close a timed span
     cudaEvent_t mark(cudaStream_t s);                               // open a timed span
 
     cudaStream_t cs() const { return cs_; }
@@ -196,7 +196,7 @@ class Part {
     uint32_t max_iters_ = 0;
     cudaEvent_t ev_classified_ = nullptr;
     EventPool pool_;
-    struct Span { cudaEvent_t a, b; uint32_t iter; int ph; };
+    struct Span { cudaEvent_t a, b; uint32_t iter; int ph; int sub; };
     std::vector<Span> spans_;
     cudaEvent_t ev_start_ = nullptr, ev_fill0_ = nullptr, ev_fill1_ = nullptr;
     double host_s_ = 0.0;
