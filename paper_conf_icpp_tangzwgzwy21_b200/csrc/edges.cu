@@ -1267,12 +1267,11 @@ inline unsigned blocks_for(unsigned long long n, int per_block, unsigned cap = 1
     return (unsigned)(b > cap ? cap : b);
 }
 
-// Every kernel that can run concurrently with another (static-hit, on-demand, gather, chunk copy)
-// asks for the same L1/shared carveout (maximum shared). With the default per-kernel choice an SM
-// running only k_static_med (no shared memory) is configured for maximum L1, and the on-demand
-// kernel launched next (33 KB of shared memory per CTA) finds no SM it can use until the 9 ms
-// static kernel drains: measured on C3 as one 8-11 ms on-demand kernel per iteration (ASCETIC_TRACE=2)
-// that stalled chunk-buffer reuse and idled the host link ~5 ms per iteration.
+// Dev A/B knob (ASC_CARVE / ASC_CARVE_STATIC = percent of the maximum shared memory): pin the
+// L1/shared carveout of the kernels that run concurrently. Measured on C3/C2 and left off: a
+// uniform maximum-shared split made the static-hit kernels 2.5-3x slower (they live on L1 hits of
+// the vertex state), and 25-60 % splits for the static kernels let the on-demand kernels co-run but
+// slowed both; the on-demand kernels instead use no shared memory at all (launch_ondemand).
 template <typename K>
 void carve(K* k, const char* env = "ASC_CARVE") {
     const char* e = std::getenv(env);
