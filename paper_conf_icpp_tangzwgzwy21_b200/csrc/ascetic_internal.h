@@ -132,7 +132,7 @@ void launch_static(int algo, const DevState& d, const Queues& q, const void* sta
                    uint32_t piece_arcs, int max_ctas, cudaStream_t s);
 void launch_ondemand(int algo, const DevState& d, const Queues& q,
                      const void* chunk, unsigned long long lo, unsigned long long hi, cudaStream_t s);
-void launch_gather(const Queues& q, const void* host_nbr, uint32_t b_e, void* chunk,
+void launch_gather(const Queues& q, const void* host_nbr, uint64_t m, uint32_t b_e, void* chunk,
                    unsigned long long lo, unsigned long long hi, int max_ctas, cudaStream_t s);
 // §3.4: per-chunk accesses (active arcs) of this iteration's hit + miss queues into acc
 void launch_chunk_access(const DevState& d, const Queues& q, uint32_t n_small, uint32_t n_med, uint32_t n_hub,

@@ -721,6 +721,16 @@ __global__ void __launch_bounds__(256) k_gather(Queues q, const void* __restrict
     }
 }
 
+// host (mapped pinned) 16-byte load, not allocated in L1: read once, and keeping it out of L1
+// leaves the concurrent static-hit kernels their L1 hits on vertex state (C2 static 14.9 -> 12.1 ms,
+// C4-shaped 13.8 -> 11.0 ms; the gather rate is unchanged)
+__device__ __forceinline__ uint4 ld_host16(const uint4* p) {
+    uint4 x;
+    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(x.x), "=r"(x.y), "=r"(x.z), "=r"(x.w) : "l"(p));
+    return x;
+}
+
 // 16-byte cover gather (default). Measured on the box (tools/zc_align.cu, profiles/r01/zc_align.log):
 // zero-copy reads of random host runs reach ~44 GB/s with 4-byte loads, ~48 with 8-byte and
 // ~50 with 16-byte loads, even when the runs start 4-byte aligned and the 16-byte cover is read
@@ -732,8 +742,8 @@ __global__ void __launch_bounds__(256) k_gather(Queues q, const void* __restrict
 // at their stream position. `hoff` = the host array's byte offset from its 16-byte-aligned base.
 template <int BE, bool SMEM>
 __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restrict__ host, uint32_t hoff,
-                                                  uint32_t* __restrict__ chunk, unsigned long long lo,
-                                                  unsigned long long hi) {
+                                                  unsigned long long w_end, uint32_t* __restrict__ chunk,
+                                                  unsigned long long lo, unsigned long long hi) {
     __shared__ unsigned long long sm_pre[SMEM ? kEdgeTile + 1 : 1];
     __shared__ unsigned long long sm_src[SMEM ? kEdgeTile + 1 : 1];
     constexpr unsigned long long AW = BE / 4;                 // words per arc
@@ -814,12 +824,24 @@ __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restr
                     uw[g] = ~0ull;
                     if (tt < total) {
                         uw[g] = uo + (tt - eo);
-                        val[g] = host[uw[g]];
+                        // the array's first / last unit may stick out of [w_off, w_end): read those
+                        // word by word in the store phase, never outside the caller's array
+                        if (uw[g] * 4 >= w_off && uw[g] * 4 + 4 <= w_end) val[g] = ld_host16(host + uw[g]);
                     }
                 }
 #pragma unroll
                 for (int g = 0; g < 4; ++g) {
                     if (uw[g] == ~0ull) continue;
+                    if (!(uw[g] * 4 >= w_off && uw[g] * 4 + 4 <= w_end)) {
+                        const uint32_t* hw = reinterpret_cast<const uint32_t*>(host) + uw[g] * 4;
+                        uint32_t x4[4];
+#pragma unroll
+                        for (int c = 0; c < 4; ++c) {
+                            const unsigned long long w = uw[g] * 4 + c;
+                            x4[c] = (w >= w_off && w < w_end) ? hw[c] : 0u;
+                        }
+                        val[g] = make_uint4(x4[0], x4[1], x4[2], x4[3]);
+                    }
                     const uint32_t wv[4] = {val[g].x, val[g].y, val[g].z, val[g].w};
 #pragma unroll
                     for (int c = 0; c < 4; ++c) {
@@ -1394,7 +1416,7 @@ void launch_ondemand(int algo, const DevState& d, const Queues& q, const void* c
     ++g_launches;
 }
 
-void launch_gather(const Queues& q, const void* host_nbr, uint32_t b_e, void* chunk,
+void launch_gather(const Queues& q, const void* host_nbr, uint64_t m, uint32_t b_e, void* chunk,
                    unsigned long long lo, unsigned long long hi, int max_ctas, cudaStream_t s) {
     if (hi <= lo) return;
     const unsigned long long tiles = ((hi - 1) >> kEdgeTileShift) - (lo >> kEdgeTileShift) + 1;
@@ -1423,12 +1445,13 @@ void launch_gather(const Queues& q, const void* host_nbr, uint32_t b_e, void* ch
         // gathers at the same rate but its L1 metadata reads slow the concurrent static kernels)
         static const bool sm = [] { const char* e = std::getenv("ASC_GATHER_SMEM"); return !(e && !std::atoi(e)); }();
         uint32_t* c = reinterpret_cast<uint32_t*>(chunk);
+        const unsigned long long w_end = hoff / 4 + m * (b_e / 4);   // host words from the aligned base
         if (sm) {
-            if (b_e == 8) k_gather16<8, true><<<grid, 256, 0, s>>>(q, base, hoff, c, lo, hi);
-            else k_gather16<4, true><<<grid, 256, 0, s>>>(q, base, hoff, c, lo, hi);
+            if (b_e == 8) k_gather16<8, true><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
+            else k_gather16<4, true><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
         } else {
-            if (b_e == 8) k_gather16<8, false><<<grid, 256, 0, s>>>(q, base, hoff, c, lo, hi);
-            else k_gather16<4, false><<<grid, 256, 0, s>>>(q, base, hoff, c, lo, hi);
+            if (b_e == 8) k_gather16<8, false><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
+            else k_gather16<4, false><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
         }
     }
     ++g_launches;

@@ -436,7 +436,7 @@ void Part::transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsig
         // and congests the memory system for the concurrently running edge kernels
         // (measured: 64 CTAs at b_e = 8 -> same 47 GB/s, 3x faster on-demand kernels than 296)
         const int ctas = o_.gather_ctas ? o_.gather_ctas : (int)(64u * 8u / g_.b_e);
-        launch_gather(q, g_.nbr_dev, g_.b_e, d_chunk_[buf], lo, hi, ctas, xs_);
+        launch_gather(q, g_.nbr_dev, g_.m, g_.b_e, d_chunk_[buf], lo, hi, ctas, xs_);
         return;
     }
     size_t r = std::upper_bound(rdst_.begin(), rdst_.end(), lo) - rdst_.begin();
