@@ -144,7 +144,7 @@ def run_reference(args, ws, rank):
               + f" on the {args.config} graph (n={g.n}, m={g.m})")
     out = {"metric": METRIC, "value": v, "unit": "GTEPS", "impl": "reference", "n_gpus": ws,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": secs / args.steps * 1e3,
-           "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32" if algo != "pr" else "f64",
+           "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32" if algo != "pr" else "f64",
            "data": "synthetic", "config": {"workload": f"{args.config}: {c['desc']}", "budget_bytes": budget,
                                            "n": g.n, "m": g.m, "h2d_gb_per_run": h2d / args.steps / 1e9},
            "cpu_baseline": {"value": v, "unit": "GTEPS", "cores": oracle.threads(), "kind": "oracle",
