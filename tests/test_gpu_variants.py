@@ -1,0 +1,56 @@
+"""The A/B kernel variants kept behind dev environment switches (DESIGN.md §5/§6) stay correct:
+each runs in a fresh process (the switches are read once per process) through the C ABI and is
+checked against the oracle: the shared-memory-staged on-demand kernel (ASC_OND_SMEM=1), the
+arc-per-lane 4/8-byte gather (ASC_GATHER_OLD=1) and the zero-shared-memory 16-byte gather
+(ASC_GATHER_SMEM=0)."""
+import os
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+SCRIPT = r"""
+import sys
+sys.path.insert(0, %(root)r)
+import numpy as np
+import graphgen as gg, oracle
+import paper_conf_icpp_tangzwgzwy21_b200 as asc
+for algo in ["bfs", "sssp", "cc", "pr", "prd"]:
+    g = gg.rmat(12, seed=21, weights=(algo == "sssp"))
+    src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+    it = 6 if algo == "pr" else 0
+    asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True)
+    asc.set_option("chunk_cap", 3000)
+    asc.set_option("xfer_mode", 1)
+    asc.set_budget(g.csr_bytes // 4, 0.3)
+    asc.run(algo, src, it)
+    st, its = asc.stats()
+    res = asc.get_result().copy()
+    p = oracle.placer(g.off, g.b_e, g.csr_bytes // 4, 0.3)
+    ref = oracle.run(algo, g.off, g.nbr, src=src, max_iters=it, is_static=oracle.static_prefix(g.n, p.s))
+    if algo == "pr":
+        assert (np.abs(res - ref.values) / ref.values).max() <= 1e-5
+    else:
+        exp = ref.values.astype(np.float32) if algo == "prd" else ref.values
+        assert np.array_equal(res, exp), algo
+    assert [i["digest"] for i in its] == [r["digest"] for r in ref.records], algo
+    assert st["h2d_payload_bytes"] == ref.h2d_payload, algo
+print("variant ok")
+"""
+
+
+@pytest.mark.parametrize("env", ["ASC_OND_SMEM=1", "ASC_GATHER_OLD=1", "ASC_GATHER_SMEM=0"])
+def test_dev_variants_match_oracle(env):
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    k, v = env.split("=")
+    e = dict(os.environ)
+    e[k] = v
+    r = subprocess.run([sys.executable, "-c", SCRIPT % {"root": ROOT}], env=e, capture_output=True, text=True,
+                       timeout=600)
+    assert r.returncode == 0 and "variant ok" in r.stdout, r.stdout[-2000:] + r.stderr[-2000:]
