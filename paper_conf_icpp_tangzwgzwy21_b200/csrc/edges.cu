@@ -1289,26 +1289,9 @@ inline unsigned blocks_for(unsigned long long n, int per_block, unsigned cap = 1
     return (unsigned)(b > cap ? cap : b);
 }
 
-// Dev A/B knob (ASC_CARVE / ASC_CARVE_STATIC = percent of the maximum shared memory): pin the
-// L1/shared carveout of the kernels that run concurrently. Measured on C3/C2 and left off: a
-// uniform maximum-shared split made the static-hit kernels 2.5-3x slower (they live on L1 hits of
-// the vertex state), and 25-60 % splits for the static kernels let the on-demand kernels co-run but
-// slowed both; the on-demand kernels instead use no shared memory at all (launch_ondemand).
-template <typename K>
-void carve(K* k, const char* env = "ASC_CARVE") {
-    const char* e = std::getenv(env);
-    const int pct = e ? std::atoi(e) : -1;   // dev A/B: percent of the maximum shared memory
-    if (pct < 0) return;
-    cudaFuncSetAttribute(reinterpret_cast<const void*>(k), cudaFuncAttributePreferredSharedMemoryCarveout, pct);
-}
-
 template <int ALGO, bool REMAP>
 void static_launch_t(const DevState& d, const Queues& q, const void* sbase, uint32_t ns, uint32_t nm, uint32_t nh,
                      uint32_t npieces, uint32_t piece, int max_ctas, cudaStream_t s) {
-    static const bool carved = (carve(k_static_small<ALGO, REMAP>, "ASC_CARVE_STATIC"),
-                                carve(k_static_med<ALGO, REMAP>, "ASC_CARVE_STATIC"),
-                                carve(k_static_hub<ALGO, REMAP>, "ASC_CARVE_STATIC"), true);
-    (void)carved;
     auto cap = [&](unsigned long long b) { return (unsigned)(b < (unsigned long long)max_ctas ? b : max_ctas); };
     if (ns) { k_static_small<ALGO, REMAP><<<cap((ns + 255) / 256), 256, 0, s>>>(d, q.hq_small, ns, sbase); ++g_launches; }
     if (nm) { k_static_med<ALGO, REMAP><<<cap((nm + 7) / 8), 256, 0, s>>>(d, q.hq_med, nm, sbase); ++g_launches; }
@@ -1342,8 +1325,6 @@ void launch_chunk_access(const DevState& d, const Queues& q, uint32_t n_small, u
                          uint32_t b_e, uint32_t* acc, cudaStream_t s) {
     const unsigned long long total = (unsigned long long)n_small + n_med + n_hub + q.n_missq;
     if (!total) return;
-    static const bool carved = (carve(k_chunk_access), true);
-    (void)carved;
     const uint32_t epc_shift = kChunkShift - (b_e == 8 ? 3 : 2);
     k_chunk_access<<<blocks_for(total, 256), 256, 0, s>>>(d, q, n_small, n_med, n_hub, epc_shift, acc);
     ++g_launches;
@@ -1361,8 +1342,6 @@ void launch_apply_swaps(const DevState& d, uint32_t* slot_of, const uint32_t* sw
 void launch_copy_chunks(const void* host_dev, uint64_t x0, uint64_t D, const uint32_t* ids, const uint32_t* slots,
                         uint32_t count, void* dst, cudaStream_t s) {
     if (!count) return;
-    static const bool carved = (carve(k_copy_chunks), true);
-    (void)carved;
     // 64 CTAs x 16 KiB = 1 MiB of host reads in flight (the transfer engine's sizing)
     k_copy_chunks<<<count < 64u ? count : 64u, 256, 0, s>>>(reinterpret_cast<const char*>(host_dev), x0, D, ids, slots,
                                                           count, reinterpret_cast<char*>(dst));
@@ -1386,12 +1365,7 @@ void launch_ondemand(int algo, const DevState& d, const Queues& q, const void* c
         ++g_launches;
         return;
     }
-    static const bool carved = (carve(k_ondemand<SSSP>), carve(k_ondemand<CC>), carve(k_ondemand<PRD>),
-                                carve(k_ondemand<PR>), carve(k_ondemand_bfs), true);
-    (void)carved;
     unsigned tiles = (unsigned)(((hi - 1) >> kEdgeTileShift) - (lo >> kEdgeTileShift) + 1);
-    static const int cap = [] { const char* e = std::getenv("ASC_OND_CTAS"); return e ? std::atoi(e) : 0; }();
-    if (cap > 0 && tiles > (unsigned)cap) tiles = (unsigned)cap;
     // Zero-shared-memory variant by default: the staged one (33 KB per CTA, ASC_OND_SMEM=1) cannot
     // start on SMs whose L1/shared split was chosen for a shared-memory-free static kernel, and
     // waited out each 9 ms k_static_med on C3 (one 8-11 ms on-demand kernel per iteration that
@@ -1421,22 +1395,10 @@ void launch_gather(const Queues& q, const void* host_nbr, uint64_t m, uint32_t b
     if (hi <= lo) return;
     const unsigned long long tiles = ((hi - 1) >> kEdgeTileShift) - (lo >> kEdgeTileShift) + 1;
     const unsigned grid = (unsigned)(tiles < (unsigned long long)max_ctas ? tiles : (unsigned long long)max_ctas);
-    // dev knob: extra dynamic shared memory per gather CTA caps how many gather CTAs share an SM
-    static const int dsm = [] {
-        const char* e = std::getenv("ASC_GATHER_DSMEM");
-        const int v = e ? std::atoi(e) : 0;
-        if (v > 0) {
-            cudaFuncSetAttribute(k_gather<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, v);
-            cudaFuncSetAttribute(k_gather<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, v);
-        }
-        return v;
-    }();
-    static const bool carved = (carve(k_gather<4>), carve(k_gather<8>), carve(k_gather16<4, true>), carve(k_gather16<8, true>), true);
-    (void)carved;
     static const bool old = [] { const char* e = std::getenv("ASC_GATHER_OLD"); return e && std::atoi(e); }();
     if (old) {
-        if (b_e == 8) k_gather<8><<<grid, 256, dsm, s>>>(q, host_nbr, chunk, lo, hi);
-        else k_gather<4><<<grid, 256, dsm, s>>>(q, host_nbr, chunk, lo, hi);
+        if (b_e == 8) k_gather<8><<<grid, 256, 0, s>>>(q, host_nbr, chunk, lo, hi);
+        else k_gather<4><<<grid, 256, 0, s>>>(q, host_nbr, chunk, lo, hi);
     } else {
         const uintptr_t hp = reinterpret_cast<uintptr_t>(host_nbr);
         const uint4* base = reinterpret_cast<const uint4*>(hp & ~(uintptr_t)15);

@@ -154,9 +154,7 @@ void Part::alloc_vertex_state() {
     // iterations, whose static pull is HBM-bound, by 20 %).
     int lo_pri = 0, hi_pri = 0;
     CK(cudaDeviceGetStreamPriorityRange(&lo_pri, &hi_pri));
-    int cs_pri = lo_pri;
-    if (const char* e = std::getenv("ASC_CS_PRI_UP")) cs_pri = std::max(hi_pri, lo_pri - std::atoi(e));   // dev knob
-    CK(cudaStreamCreateWithPriority(&cs_, cudaStreamNonBlocking, cs_pri));
+    CK(cudaStreamCreateWithPriority(&cs_, cudaStreamNonBlocking, lo_pri));
     CK(cudaStreamCreateWithPriority(&xs_, cudaStreamNonBlocking, hi_pri));
     CK(cudaStreamCreateWithPriority(&ss_, cudaStreamNonBlocking, lo_pri));
     for (int i = 0; i < kMaxBuffers; ++i) {
