@@ -740,7 +740,7 @@ __device__ __forceinline__ uint4 ld_host16(const uint4* p) {
 // piece), each piece's cover units are enumerated across the warp (a unit shared by two
 // vertices of one piece is loaded once), and every lane stores the piece words its unit holds
 // at their stream position. `hoff` = the host array's byte offset from its 16-byte-aligned base.
-template <int BE, bool SMEM>
+template <int BE, bool SMEM, int NG = 4>
 __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restrict__ host, uint32_t hoff,
                                                   unsigned long long w_end, uint32_t* __restrict__ chunk,
                                                   unsigned long long lo, unsigned long long hi) {
@@ -803,12 +803,12 @@ __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restr
             }
             const uint32_t excl = incl - cnt;
             const uint32_t total = __shfl_sync(FULL, incl, 31);
-            for (uint32_t b = 0; b < total; b += 128) {
-                // 4 groups of 32 units: all loads first (4 x 16 B in flight per lane), then the stores
-                uint4 val[4];
-                unsigned long long uw[4], pw0[4], pw1[4], pd0[4];
+            for (uint32_t b = 0; b < total; b += 32u * NG) {
+                // NG groups of 32 units: all loads first (NG x 16 B in flight per lane), then the stores
+                uint4 val[NG];
+                unsigned long long uw[NG], pw0[NG], pw1[NG], pd0[NG];
 #pragma unroll
-                for (int g = 0; g < 4; ++g) {
+                for (int g = 0; g < NG; ++g) {
                     const uint32_t tt = b + 32u * g + (uint32_t)lane;
                     int i = 0;
 #pragma unroll
@@ -830,7 +830,7 @@ __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restr
                     }
                 }
 #pragma unroll
-                for (int g = 0; g < 4; ++g) {
+                for (int g = 0; g < NG; ++g) {
                     if (uw[g] == ~0ull) continue;
                     if (!(uw[g] * 4 >= w_off && uw[g] * 4 + 4 <= w_end)) {
                         const uint32_t* hw = reinterpret_cast<const uint32_t*>(host) + uw[g] * 4;
@@ -1408,9 +1408,22 @@ void launch_gather(const Queues& q, const void* host_nbr, uint64_t m, uint32_t b
         static const bool sm = [] { const char* e = std::getenv("ASC_GATHER_SMEM"); return !(e && !std::atoi(e)); }();
         uint32_t* c = reinterpret_cast<uint32_t*>(chunk);
         const unsigned long long w_end = hoff / 4 + m * (b_e / 4);   // host words from the aligned base
+        // units loaded per lane per round (A/B knob ASC_GATHER_NG): a 256-arc warp segment of 8-byte
+        // arcs is 128 units plus up to one per piece boundary, so 4 per lane (128) usually needs a
+        // second, nearly empty round. C2 A/B on B200 (profiles/r01/gather_ng_ab.log): NG 4 -> 6 =
+        // 44.6-44.7 -> 45.0 GB/s, +0.6 % GTEPS; 5 and 8 within noise of 6. 4-byte arcs: 64 units, 4 fits.
+        static const int ng = [] { const char* e = std::getenv("ASC_GATHER_NG"); return e ? std::atoi(e) : 0; }();
         if (sm) {
-            if (b_e == 8) k_gather16<8, true><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
-            else k_gather16<4, true><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
+            if (b_e == 8) {
+                if (ng == 5) k_gather16<8, true, 5><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
+                else if (ng == 4) k_gather16<8, true, 4><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
+                else if (ng == 8) k_gather16<8, true, 8><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
+                else k_gather16<8, true, 6><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
+            } else {
+                if (ng == 2) k_gather16<4, true, 2><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
+                else if (ng == 3) k_gather16<4, true, 3><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
+                else k_gather16<4, true><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
+            }
         } else {
             if (b_e == 8) k_gather16<8, false><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
             else k_gather16<4, false><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);

@@ -1,8 +1,9 @@
 """The A/B kernel variants kept behind dev environment switches (DESIGN.md §5/§6) stay correct:
 each runs in a fresh process (the switches are read once per process) through the C ABI and is
 checked against the oracle: the shared-memory-staged on-demand kernel (ASC_OND_SMEM=1), the
-arc-per-lane 4/8-byte gather (ASC_GATHER_OLD=1) and the zero-shared-memory 16-byte gather
-(ASC_GATHER_SMEM=0)."""
+arc-per-lane 4/8-byte gather (ASC_GATHER_OLD=1), the zero-shared-memory 16-byte gather
+(ASC_GATHER_SMEM=0) and the 16-byte gather's other loads-per-lane-per-round settings
+(ASC_GATHER_NG; default 6 for 8-byte arcs, 4 for 4-byte arcs)."""
 import os
 import subprocess
 import sys
@@ -43,7 +44,8 @@ print("variant ok")
 """
 
 
-@pytest.mark.parametrize("env", ["ASC_OND_SMEM=1", "ASC_GATHER_OLD=1", "ASC_GATHER_SMEM=0"])
+@pytest.mark.parametrize("env", ["ASC_OND_SMEM=1", "ASC_GATHER_OLD=1", "ASC_GATHER_SMEM=0", "ASC_GATHER_NG=4",
+                                 "ASC_GATHER_NG=5", "ASC_GATHER_NG=8", "ASC_GATHER_NG=2", "ASC_GATHER_NG=3"])
 def test_dev_variants_match_oracle(env):
     import torch
     if not torch.cuda.is_available():
