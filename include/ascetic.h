@@ -98,11 +98,18 @@ typedef enum {
     ASCETIC_OPT_PLACEMENT_SEED = 16, /* seed of the random initial content (default 1). Set before set_budget. */
     ASCETIC_OPT_PRD_TOL_PPM = 17,    /* PageRank-delta activation threshold tau in ppm of the initial residual
                                       (1-d)/n (default 10000 = 1 %) */
-    ASCETIC_OPT_FUSED_EXCHANGE = 18  /* P > 1, BFS/SSSP/CC/PRD: 1 = fuse the per-iteration exchange into the
+    ASCETIC_OPT_FUSED_EXCHANGE = 18, /* P > 1, BFS/SSSP/CC/PRD: 1 = fuse the per-iteration exchange into the
                                       finalize kernel, which reads every rank's next bitmap / values /
                                       increments straight from peer memory (CUDA IPC over NVLink with the NCCL
                                       back end; the other parts' buffers when emulated), between stream-ordered
                                       barriers; 0 (default) = NCCL collectives. Results are identical. */
+    ASCETIC_OPT_SPARSE_EXCHANGE = 19 /* P > 1, SSSP/CC, collectives path: d >= 1 = sparse MIN exchange (SURVEY
+                                      §8(e)): each rank packs the (id, value) pairs it lowered this iteration, the
+                                      pairs are all-gathered and applied with atomicMin, whenever every rank has at
+                                      most max(1, n / (d * P)) of them (else the dense ncclAllReduce(min) of n
+                                      values); one 4P-byte host read per iteration decides. 0 (default) = dense
+                                      always. 8 keeps the all-gather under the all-reduce's bytes. Results are
+                                      identical. */
 } ascetic_option;
 
 typedef struct {
@@ -148,6 +155,8 @@ typedef struct {
     uint64_t h2d_replace_bytes;   /* §3.4 swapped-in chunk bytes (ASCETIC_OPT_REPLACE_CHUNKS) */
     uint64_t swaps_total;         /* §3.4 chunk swaps performed */
     double time_replace_s;        /* copy-stream time of the swap DMAs */
+    uint64_t sparse_exchanges;    /* iterations whose exchange went sparse (ASCETIC_OPT_SPARSE_EXCHANGE) */
+    uint64_t sparse_exchange_bytes; /* (id, value) pair bytes all ranks contributed to those exchanges */
 } ascetic_stats_t;
 
 typedef struct {

@@ -157,6 +157,12 @@ void launch_prd_output(const DevState& d, cudaStream_t s);
 void launch_or_reduce(uint32_t* dst, const uint32_t* gathered, uint32_t parts, uint64_t nw, cudaStream_t s);
 void launch_or_into(uint32_t* dst, const uint32_t* src, uint64_t nw, cudaStream_t s);
 void launch_min_into(uint32_t* dst, const uint32_t* src, uint64_t n, cudaStream_t s);
+// sparse MIN exchange (SSSP / CC): pack this rank's improved (id, value) pairs (count zeroed first;
+// at most cap written, *count = the full number), and apply P ranks' pairs (rank `skip` left out)
+void launch_sparse_pack(const uint32_t* next, const uint32_t* val, uint32_t nwords, void* pairs, uint32_t cap,
+                        uint32_t* count, cudaStream_t s);
+void launch_sparse_apply(uint32_t* val, uint32_t* next, const void* pairs, uint64_t stride, const uint32_t* counts,
+                         int P, int skip, uint32_t cap, cudaStream_t s);
 void launch_add_f64(double* dst, const double* src, cudaStream_t s);
 void launch_add_u64(unsigned long long* dst, const unsigned long long* src, uint64_t n, cudaStream_t s);
 // *bad := min{v : off[v+1] < off[v]} (left untouched when off[0..n] is non-decreasing)

@@ -94,6 +94,9 @@ void Comm::destroy() {
     if (barrier_buf_) { cudaFree(barrier_buf_); barrier_buf_ = nullptr; }
     if (nccl_comm_) { nccl().CommDestroy((ncclComm_t)nccl_comm_); nccl_comm_ = nullptr; }
     if (scratch_) { cudaFree(scratch_); scratch_ = nullptr; scratch_words_ = 0; }
+    if (sp_counts_) { cudaFree(sp_counts_); sp_counts_ = nullptr; }
+    if (sp_counts_host_) { cudaFreeHost(sp_counts_host_); sp_counts_host_ = nullptr; }
+    if (sp_gather_) { cudaFree(sp_gather_); sp_gather_ = nullptr; sp_gather_bytes_ = 0; }
     world_ = 1; rank_ = 0; emulated_ = false;
 }
 
@@ -124,6 +127,47 @@ void Comm::min_u32(const std::vector<uint32_t*>& local, uint64_t n, cudaStream_t
         return;
     }
     NC(nccl().AllReduce(local[0], local[0], n, ncclUint32, ncclMin, (ncclComm_t)nccl_comm_, s), "ncclAllReduce(min)");
+}
+
+bool Comm::sparse_min(const std::vector<uint32_t*>& val, const std::vector<uint32_t*>& next,
+                      const std::vector<void*>& pairs, const std::vector<uint32_t*>& count, uint32_t cap,
+                      cudaStream_t s, uint64_t* bytes_out) {
+    if (!active()) return true;
+    const int L = (int)val.size();   // local ranks: world when emulated, 1 with NCCL
+    if (!sp_counts_host_) CKc(cudaMallocHost(&sp_counts_host_, sizeof(uint32_t) * (size_t)std::max(world_, L)), "sparse counts");
+    if (emulated_) {
+        for (int i = 0; i < L; ++i)
+            CKc(cudaMemcpyAsync(sp_counts_host_ + i, count[i], 4, cudaMemcpyDeviceToHost, s), "sparse counts d2h");
+    } else {
+        if (!sp_counts_) CKc(cudaMalloc(&sp_counts_, sizeof(uint32_t) * (size_t)world_), "sparse counts");
+        NC(nccl().AllGather(count[0], sp_counts_, 1, ncclUint32, (ncclComm_t)nccl_comm_, s), "ncclAllGather(sparse counts)");
+        CKc(cudaMemcpyAsync(sp_counts_host_, sp_counts_, 4 * (size_t)world_, cudaMemcpyDeviceToHost, s), "sparse counts d2h");
+    }
+    CKc(cudaStreamSynchronize(s), "sparse counts sync");
+    uint32_t maxc = 0;
+    uint64_t total = 0;
+    for (int r = 0; r < world_; ++r) { maxc = std::max(maxc, sp_counts_host_[r]); total += sp_counts_host_[r]; }
+    if (maxc > cap) return false;
+    if (bytes_out) *bytes_out = total * 8ull;
+    if (maxc == 0) return true;
+    if (emulated_) {
+        // every part applies every other part's pairs; all packs were enqueued before, on s
+        for (int q = 0; q < L; ++q)
+            for (int p = 0; p < L; ++p)
+                if (p != q) launch_sparse_apply(val[q], next[q], pairs[p], 0, count[p], 1, -1, maxc, s);
+        return true;
+    }
+    const uint64_t need = (uint64_t)world_ * maxc * 8ull;
+    if (sp_gather_bytes_ < need) {
+        if (sp_gather_) cudaFree(sp_gather_);
+        const uint64_t want = (uint64_t)world_ * cap * 8ull;   // sized once for the largest exchange
+        CKc(cudaMalloc(&sp_gather_, want), "sparse gather");
+        sp_gather_bytes_ = want;
+    }
+    NC(nccl().AllGather(pairs[0], sp_gather_, 2ull * maxc, ncclUint32, (ncclComm_t)nccl_comm_, s),
+       "ncclAllGather(sparse pairs)");
+    launch_sparse_apply(val[0], next[0], sp_gather_, maxc, sp_counts_, world_, rank_, maxc, s);
+    return true;
 }
 
 void Comm::sum_f64(const std::vector<double*>& local, cudaStream_t s) {

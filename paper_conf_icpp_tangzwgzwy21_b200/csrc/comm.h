@@ -39,6 +39,14 @@ class Comm {
     // (1 with NCCL, world with emulation). Everything is enqueued on `s`.
     void or_words(const std::vector<uint32_t*>& local, uint64_t nw, cudaStream_t s);
     void min_u32(const std::vector<uint32_t*>& local, uint64_t n, cudaStream_t s);
+    // sparse MIN (SSSP / CC, small frontiers): every rank's (id, value) improvement pairs
+    // (pairs[i]: count[i] of them, device u32, packed by launch_sparse_pack with capacity cap) go to
+    // every rank and are applied by atomicMin + next bit. Reads the counts on the host (one sync);
+    // returns false, having changed nothing, when some rank has more than cap pairs (the caller then
+    // runs min_u32). All ranks take the same decision: they see the same counts.
+    bool sparse_min(const std::vector<uint32_t*>& val, const std::vector<uint32_t*>& next,
+                    const std::vector<void*>& pairs, const std::vector<uint32_t*>& count, uint32_t cap,
+                    cudaStream_t s, uint64_t* bytes_out = nullptr);
     void sum_f64(const std::vector<double*>& local, cudaStream_t s);
     // element-wise SUM of n uint64 per rank (PageRank-delta residual increments), in place
     void sum_u64(const std::vector<unsigned long long*>& local, uint64_t n, cudaStream_t s);
@@ -60,6 +68,10 @@ class Comm {
     uint32_t* scratch_ = nullptr;
     uint64_t scratch_words_ = 0;
     int* barrier_buf_ = nullptr;
+    uint32_t* sp_counts_ = nullptr;      // device: all ranks' pair counts (NCCL)
+    uint32_t* sp_counts_host_ = nullptr; // pinned: the same on the host
+    void* sp_gather_ = nullptr;          // device: all ranks' pairs (NCCL), world x cap
+    uint64_t sp_gather_bytes_ = 0;
     struct PeerMap {   // an opened CUDA IPC mapping of a peer's allocation
         int rank;
         unsigned char handle[64];   // CUDA_IPC_HANDLE_SIZE

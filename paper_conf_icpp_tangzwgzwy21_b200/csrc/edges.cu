@@ -1139,6 +1139,59 @@ __global__ void k_min_into(uint32_t* __restrict__ dst, const uint32_t* __restric
         dst[i] = min(dst[i], src[i]);
 }
 
+// sparse MIN exchange (SSSP / CC): this rank's improvements of the iteration as
+// (id, value) pairs. A vertex's next bit is set iff this rank lowered its value below the
+// iteration-start snapshot, which every rank shares, so the pairs of all ranks reproduce the MIN.
+// Order of the pairs is irrelevant (MIN commutes); `count` may exceed `cap` (then the caller
+// falls back to the dense exchange and nothing past cap is written).
+__global__ void __launch_bounds__(256) k_sparse_pack(const uint32_t* __restrict__ next, const uint32_t* __restrict__ val,
+                                                     uint32_t nwords, uint2* __restrict__ out, uint32_t cap,
+                                                     uint32_t* __restrict__ count) {
+    const int lane = threadIdx.x & 31;
+    for (uint32_t w0 = blockIdx.x * blockDim.x; w0 < nwords; w0 += gridDim.x * blockDim.x) {   // warp-uniform trip count
+        const uint32_t w = w0 + threadIdx.x;
+        const uint32_t bits = w < nwords ? next[w] : 0u;
+        const uint32_t c = __popc(bits);
+        uint32_t incl = c;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(FULL, incl, o);
+            if (lane >= o) incl += y;
+        }
+        const uint32_t tot = __shfl_sync(FULL, incl, 31);
+        uint32_t base = 0;
+        if (lane == 31 && tot) base = atomicAdd(count, tot);
+        base = __shfl_sync(FULL, base, 31);
+        uint32_t i = base + incl - c;
+        uint32_t b = bits;
+        while (b) {
+            const int k = __ffs(b) - 1;
+            b &= b - 1;
+            const uint32_t v = w * 32u + (uint32_t)k;
+            if (i < cap) out[i] = make_uint2(v, val[v]);
+            ++i;
+        }
+    }
+}
+
+// apply the other ranks' pairs: val = min(val, x), next bit set (every pair is below the shared
+// snapshot, so the vertex is active at t+1 whichever rank lowered it). pairs of rank p at
+// pairs + p * stride, counts[p] of them; rank `skip` (this one) is left out.
+__global__ void __launch_bounds__(256) k_sparse_apply(uint32_t* __restrict__ val, uint32_t* __restrict__ next,
+                                                      const uint2* __restrict__ pairs, uint64_t stride,
+                                                      const uint32_t* __restrict__ counts, int P, int skip, uint32_t cap) {
+    for (int p = 0; p < P; ++p) {
+        if (p == skip) continue;
+        const uint32_t c = min(counts[p], cap);
+        const uint2* src = pairs + (uint64_t)p * stride;
+        for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < c; i += gridDim.x * blockDim.x) {
+            const uint2 x = src[i];
+            atomicMin(val + x.x, x.y);
+            atomicOr(next + (x.x >> 5), 1u << (x.x & 31u));
+        }
+    }
+}
+
 __global__ void k_add_f64(double* dst, const double* src) { dst[0] += src[0]; }
 
 __global__ void k_check_monotone(const unsigned long long* __restrict__ off, uint64_t n, unsigned long long* bad) {
@@ -1508,6 +1561,20 @@ void launch_or_reduce(uint32_t* dst, const uint32_t* gathered, uint32_t parts, u
 
 void launch_or_into(uint32_t* dst, const uint32_t* src, uint64_t nw, cudaStream_t s) {
     k_or_into<<<blocks_for(nw, 256), 256, 0, s>>>(dst, src, nw);
+    ++g_launches;
+}
+
+void launch_sparse_pack(const uint32_t* next, const uint32_t* val, uint32_t nwords, void* pairs, uint32_t cap,
+                        uint32_t* count, cudaStream_t s) {
+    cudaMemsetAsync(count, 0, 4, s);
+    k_sparse_pack<<<blocks_for(nwords, 256), 256, 0, s>>>(next, val, nwords, reinterpret_cast<uint2*>(pairs), cap, count);
+    ++g_launches;
+}
+
+void launch_sparse_apply(uint32_t* val, uint32_t* next, const void* pairs, uint64_t stride, const uint32_t* counts,
+                         int P, int skip, uint32_t cap, cudaStream_t s) {
+    k_sparse_apply<<<blocks_for(cap, 256, 148u * 4u), 256, 0, s>>>(val, next, reinterpret_cast<const uint2*>(pairs),
+                                                                    stride, counts, P, skip, cap);
     ++g_launches;
 }
 

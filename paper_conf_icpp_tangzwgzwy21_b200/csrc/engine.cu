@@ -1151,6 +1151,10 @@ void Engine::set_option(int opt, int64_t value) {
             o_.prd_tol_ppm = (uint64_t)value;
             break;
         case ASCETIC_OPT_FUSED_EXCHANGE: o_.fused_exchange = value ? 1 : 0; break;
+        case ASCETIC_OPT_SPARSE_EXCHANGE:
+            if (value < 0 || value > 0xFFFFFFFFll) throw Error(ASCETIC_EINVAL, "sparse exchange divisor must be in [0, 2^32)");
+            o_.sparse_exchange = (uint32_t)value;
+            break;
         case ASCETIC_OPT_REPLACE_POLICY:
             if (value < 0 || value > 2) throw Error(ASCETIC_EINVAL, "replace policy: 0 = by algorithm, 1 = cumulative, 2 = last");
             o_.replace_policy = (int)value;
@@ -1232,8 +1236,10 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
     Part& p0 = *parts_[0];
     std::vector<IterTotals> T(parts_.size());
     uint32_t t = 0;
+    uint64_t sparse_iters = 0, sparse_bytes = 0;
     for (t = 0;; ++t) {
         if (max_iters && t == max_iters) break;
+        bool dense_fin = true;   // false after a sparse exchange: A_{t+1} = the merged next bitmap
         for (auto& p : parts_) p->classify(t);
         for (size_t i = 0; i < parts_.size(); ++i) T[i] = parts_[i]->wait_classify();
         if (T[0].nA == 0) break;   // |A_t| is counted over the replicated bitmap: identical on every rank
@@ -1280,14 +1286,38 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
                 for (auto& p : parts_) b.push_back(p->prd_inc());
                 comm_.sum_u64(b, g_.n, p0.cs());
             } else {
-                std::vector<uint32_t*> b;
-                for (auto& p : parts_) b.push_back(p->val());
-                comm_.min_u32(b, g_.n, p0.cs());
+                std::vector<uint32_t*> b, nx;
+                for (auto& p : parts_) { b.push_back(p->val()); nx.push_back(p->next()); }
+                bool sparse = false;
+                if (o_.sparse_exchange) {
+                    // the (id, value) pairs each rank lowered, when few; else dense MIN
+                    const uint64_t c = std::max<uint64_t>(1, g_.n / ((uint64_t)o_.sparse_exchange * comm_.world()));
+                    const uint32_t cap = (uint32_t)std::min<uint64_t>(c, g_.n);
+                    if (sp_cap_ != cap || sp_pairs_.size() != parts_.size()) {
+                        free_sparse();
+                        for (size_t i = 0; i < parts_.size(); ++i) {
+                            void* pp = nullptr;
+                            uint32_t* cc = nullptr;
+                            CK(cudaMalloc(&pp, (size_t)cap * 8));
+                            CK(cudaMalloc(&cc, 4));
+                            sp_pairs_.push_back(pp);
+                            sp_cnt_.push_back(cc);
+                        }
+                        sp_cap_ = cap;
+                    }
+                    for (size_t i = 0; i < parts_.size(); ++i)
+                        launch_sparse_pack(nx[i], b[i], (uint32_t)nw, sp_pairs_[i], cap, sp_cnt_[i], p0.cs());
+                    uint64_t bytes = 0;
+                    sparse = comm_.sparse_min(b, nx, sp_pairs_, sp_cnt_, cap, p0.cs(), &bytes);
+                    if (sparse) { ++sparse_iters; sparse_bytes += bytes; }
+                }
+                if (!sparse) comm_.min_u32(b, g_.n, p0.cs());
+                dense_fin = !sparse;
             }
             p0.span(e0, p0.cs(), t, PH_XCH);
             fork();
         }
-        for (auto& p : parts_) p->finalize(t, multi);
+        for (auto& p : parts_) p->finalize(t, multi && dense_fin);
         if (multi && algo == ALG_PR) {
             // ---- exchange: SUM of the fp64 dangling partials, every rank's contrib slice to all
             join();
@@ -1343,6 +1373,8 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         st_.kernel_launches = std::max(st_.kernel_launches, s.kernel_launches);
     }
     st_.iterations = t;
+    st_.sparse_exchanges = sparse_iters;
+    st_.sparse_exchange_bytes = sparse_bytes;
     st_.world = (uint32_t)comm_.world();
     st_.rank = (uint32_t)comm_.rank();
     st_.gteps = st_.time_run_s > 0 ? (double)st_.active_arcs_total / st_.time_run_s / 1e9 : 0.0;
@@ -1371,8 +1403,17 @@ void Engine::get_result(void* dst, uint64_t bytes) {
     CK(cudaMemcpy(dst, src, 4 * g_.n, cudaMemcpyDeviceToHost));
 }
 
+void Engine::free_sparse() {
+    for (void* p : sp_pairs_) if (p) cudaFree(p);
+    for (uint32_t* c : sp_cnt_) if (c) cudaFree(c);
+    sp_pairs_.clear();
+    sp_cnt_.clear();
+    sp_cap_ = 0;
+}
+
 void Engine::unload() {
     if (device_ >= 0) cudaSetDevice(device_);
+    free_sparse();
     parts_.clear();
     g_.release();
     g_.off = nullptr;

@@ -64,6 +64,7 @@ struct Options {
     uint64_t placement_seed = 1;  // seed of the random initial chunk set
     uint64_t prd_tol_ppm = 10000; // PageRank-delta threshold, ppm of the initial residual (1-d)/n
     int fused_exchange = 0;       // P > 1: exchange fused into finalize over peer memory (NVLink / IPC)
+    uint32_t sparse_exchange = 0; // P > 1, SSSP/CC: sparse MIN when every rank has <= n/(d P) pairs (0 = off)
     uint32_t replace_k = 0;       // §3.4 data replacement: chunk swaps examined per iteration (0 = off)
     int replace_policy = 0;       // hotness counter: 0 = by algorithm, 1 = cumulative, 2 = last iteration
 };
@@ -254,6 +255,11 @@ class Engine {
     bool have_result_ = false;
     ascetic_stats_t st_{};
     std::vector<ascetic_iter_stats_t> iters_;
+    // sparse MIN exchange buffers, one per local part: (id, value) pairs and their count
+    std::vector<void*> sp_pairs_;
+    std::vector<uint32_t*> sp_cnt_;
+    uint32_t sp_cap_ = 0;
+    void free_sparse();
 };
 
 }  // namespace ascetic

@@ -117,3 +117,42 @@ def test_fused_exchange_matches_oracle(asc, P, algo):
     finally:
         asc.set_option("fused_exchange", 0)
         asc.set_option("chunk_cap", 0)
+
+
+@pytest.mark.parametrize("P", [2, 3, 5])
+@pytest.mark.parametrize("algo", ["sssp", "cc"])
+@pytest.mark.parametrize("d", [8, 2000])
+def test_sparse_exchange_matches_oracle(asc, P, algo, d):
+    """ASCETIC_OPT_SPARSE_EXCHANGE: each rank's lowered (id, value) pairs are
+    exchanged and applied with atomicMin when every rank has at most n/(d P) of them, else the
+    dense MIN runs. d = 8: mostly sparse; d = 2000: a cap of 1 pair, so nearly every iteration
+    falls back to dense. Values and every per-rank record equal the oracle either way."""
+    g = gg.rmat(12, seed=35, weights=(algo == "sssp"))
+    src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+    budget = g.csr_bytes // (4 * P)
+    asc.emulate_ranks(P)
+    asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True)
+    asc.set_option("sparse_exchange", d)
+    asc.set_option("chunk_cap", 4096)
+    try:
+        asc.set_budget(budget, 0.4)
+        for rep in range(2):                        # second run reuses the pair buffers
+            asc.run(algo, src)
+            st, its = asc.stats()
+            res = asc.get_result().copy()
+            bounds = oracle.partition(g.off, P)
+            ref = oracle.run(algo, g.off, g.nbr, src=src, is_static=_rank_static(g, bounds, budget, 0.4),
+                             bounds=bounds)
+            np.testing.assert_array_equal(res, ref.values)
+            assert [{f: i[f] for f in REC} for i in its] == [{f: r[f] for f in REC} for r in ref.records]
+            if d == 8:
+                assert st["sparse_exchanges"] >= 1 and st["sparse_exchange_bytes"] > 0
+            else:
+                assert st["sparse_exchanges"] < st["iterations"]
+        asc.set_option("sparse_exchange", 0)         # back to dense on the same parts
+        asc.run(algo, src)
+        np.testing.assert_array_equal(asc.get_result(), ref.values)
+        assert asc.stats()[0]["sparse_exchanges"] == 0
+    finally:
+        asc.set_option("sparse_exchange", 0)
+        asc.set_option("chunk_cap", 0)

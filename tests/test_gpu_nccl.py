@@ -76,3 +76,27 @@ def test_nccl_one_rank_reload_reopens_peers(asc):
             np.testing.assert_array_equal(asc.get_result(), ref.values)
     finally:
         asc.set_option("fused_exchange", 0)
+
+
+@pytest.mark.parametrize("algo", ["sssp", "cc"])
+def test_nccl_one_rank_sparse_exchange(asc, algo):
+    """ASCETIC_OPT_SPARSE_EXCHANGE through libnccl: the count and pair all-gathers run on the
+    one-rank communicator (nothing foreign to apply), the finalize takes the merged next bitmap."""
+    g = gg.rmat(12, seed=39, weights=(algo == "sssp"))
+    src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+    budget = g.csr_bytes // 4
+    asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True)
+    asc.set_option("sparse_exchange", 8)
+    asc.set_option("chunk_cap", 4096)
+    try:
+        asc.set_budget(budget, 0.4)
+        p = oracle.placer(g.off, g.b_e, budget, 0.4)
+        ref = oracle.run(algo, g.off, g.nbr, src=src, is_static=oracle.static_prefix(g.n, p.s))
+        asc.run(algo, src)
+        st, its = asc.stats()
+        assert st["world"] == 1 and st["sparse_exchanges"] >= 1
+        np.testing.assert_array_equal(asc.get_result(), ref.values)
+        assert [{f: i[f] for f in REC} for i in its] == [{f: r[f] for f in REC} for r in ref.records]
+    finally:
+        asc.set_option("sparse_exchange", 0)
+        asc.set_option("chunk_cap", 0)

@@ -97,6 +97,51 @@ def _worker(rank, world, port, algo, q):
                 A = nxt
                 t += 1
             vals = level.astype(np.uint32)
+        elif algo == "cc_sparse":
+            # CC with the sparse MIN exchange (ASCETIC_OPT_SPARSE_EXCHANGE, d = 8): each rank's
+            # lowered (id, label) pairs, all-gathered padded to the largest count and applied with
+            # MIN, when every rank has at most n / (8 P) of them; else the dense MIN all-reduce
+            s = 0
+            cap = max(1, n // (8 * world))
+            lab = np.arange(n, dtype=np.int64)
+            A = np.ones(n, dtype=bool)
+            n_sparse = n_dense = 0
+            while A.any():
+                recs.append(_record(t, rank, A, stat_all, lo, hi, deg, 4, oracle.digest(A)))
+                snap = lab.copy()
+                own = np.zeros(n, dtype=bool); own[lo:hi] = A[lo:hi]
+                sel = own[src_all]
+                np.minimum.at(lab, nbr[sel].astype(np.int64), snap[src_all[sel]])
+                ids = np.flatnonzero(lab < snap)                 # this rank's next bits
+                cnt = torch.tensor([ids.size], dtype=torch.int64)
+                cnts = [torch.zeros_like(cnt) for _ in range(world)]
+                dist.all_gather(cnts, cnt)
+                maxc = max(int(c.item()) for c in cnts)
+                if maxc <= cap:
+                    buf = torch.zeros((maxc, 2), dtype=torch.int64)
+                    buf[: ids.size, 0] = torch.from_numpy(ids)
+                    buf[: ids.size, 1] = torch.from_numpy(lab[ids])
+                    bufs = [torch.zeros_like(buf) for _ in range(world)]
+                    dist.all_gather(bufs, buf)
+                    nxt = np.zeros(n, dtype=bool)
+                    nxt[ids] = True
+                    for r_, (b_, c_) in enumerate(zip(bufs, cnts)):
+                        if r_ == rank:
+                            continue
+                        pr = b_[: int(c_.item())].numpy()
+                        np.minimum.at(lab, pr[:, 0], pr[:, 1])
+                        nxt[pr[:, 0]] = True
+                    A = nxt                                      # A_{t+1} = the merged next bits
+                    n_sparse += 1
+                else:
+                    tl = torch.from_numpy(lab)
+                    dist.all_reduce(tl, op=dist.ReduceOp.MIN)
+                    lab = tl.numpy().copy()
+                    A = lab < snap
+                    n_dense += 1
+                t += 1
+            assert n_sparse >= 1 and n_dense >= 1, (n_sparse, n_dense)
+            vals = lab.astype(np.uint32)
         elif algo == "cc":
             s = 0
             lab = np.arange(n, dtype=np.int64)
@@ -171,7 +216,7 @@ def _worker(rank, world, port, algo, q):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("algo", ["bfs", "cc", "pr", "prd"])
+@pytest.mark.parametrize("algo", ["bfs", "cc", "cc_sparse", "pr", "prd"])
 def test_world2_gloo_protocol(algo):
     import graphgen as gg
     import oracle
@@ -191,7 +236,7 @@ def test_world2_gloo_protocol(algo):
     o_pl = oracle.placer(g.off[bounds[0]:bounds[1] + 1] - g.off[bounds[0]], 4, g.csr_bytes // 6, 0.5)
     assert pl["s"] == o_pl.s and pl["static_bytes"] == o_pl.static_bytes and pl["cap"] == o_pl.cap
     iters = 6 if algo == "pr" else 0
-    ref = oracle.run(algo, g.off, g.nbr, src=s, max_iters=iters, is_static=stat.astype(np.uint8),
+    ref = oracle.run(algo.replace("_sparse", ""), g.off, g.nbr, src=s, max_iters=iters, is_static=stat.astype(np.uint8),
                      bounds=np.array(bounds, dtype=np.uint64))
     got = [rec for t in range(len(per_rank[0])) for rk in range(2) for rec in [per_rank[rk][t]]]
     assert got == ref.records
