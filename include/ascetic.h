@@ -103,13 +103,14 @@ typedef enum {
                                       increments straight from peer memory (CUDA IPC over NVLink with the NCCL
                                       back end; the other parts' buffers when emulated), between stream-ordered
                                       barriers; 0 (default) = NCCL collectives. Results are identical. */
-    ASCETIC_OPT_SPARSE_EXCHANGE = 19 /* P > 1, SSSP/CC, collectives path: d >= 1 = sparse MIN exchange (SURVEY
-                                      §8(e)): each rank packs the (id, value) pairs it lowered this iteration, the
-                                      pairs are all-gathered and applied with atomicMin, whenever every rank has at
-                                      most max(1, n / (d * P)) of them (else the dense ncclAllReduce(min) of n
-                                      values); one 4P-byte host read per iteration decides. 0 (default) = dense
-                                      always. 8 keeps the all-gather under the all-reduce's bytes. Results are
-                                      identical. */
+    ASCETIC_OPT_SPARSE_EXCHANGE = 19 /* P > 1, BFS/SSSP/CC, collectives path: d >= 1 = sparse exchange (SURVEY
+                                      §8(e)): each rank packs the (id, value) pairs it set in its next bitmap this
+                                      iteration (lowered values; BFS: newly reached ids), the pairs are
+                                      all-gathered and applied with atomicMin + next bit, whenever every rank has
+                                      at most max(1, n / (d * P)) of them (BFS: n / (64 d P), a pair replaces a
+                                      bitmap bit), else the dense ncclAllReduce(min) / bitmap OR; one 4P-byte host
+                                      read per iteration decides. 0 (default) = dense always. 8 keeps the
+                                      all-gather under the all-reduce's bytes. Results are identical. */
 } ascetic_option;
 
 typedef struct {

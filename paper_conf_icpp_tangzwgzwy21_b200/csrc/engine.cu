@@ -1277,41 +1277,52 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
             join();
             cudaEvent_t e0 = p0.mark(p0.cs());
             const uint64_t nw = (g_.n + 31) / 32;
+            // SURVEY §8(e) sparse form (BFS / SSSP / CC): the ids (and values) each rank set in its
+            // next bitmap this iteration, when every rank has at most `cap` of them; else dense
+            auto try_sparse = [&](uint64_t cap64) -> bool {
+                if (!o_.sparse_exchange) return false;
+                const uint32_t cap = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(cap64, g_.n));
+                if (sp_cap_ != cap || sp_pairs_.size() != parts_.size()) {
+                    free_sparse();
+                    for (size_t i = 0; i < parts_.size(); ++i) {
+                        void* pp = nullptr;
+                        uint32_t* cc = nullptr;
+                        CK(cudaMalloc(&pp, (size_t)cap * 8));
+                        CK(cudaMalloc(&cc, 4));
+                        sp_pairs_.push_back(pp);
+                        sp_cnt_.push_back(cc);
+                    }
+                    sp_cap_ = cap;
+                }
+                std::vector<uint32_t*> b, nx;
+                for (auto& p : parts_) { b.push_back(p->val()); nx.push_back(p->next()); }
+                for (size_t i = 0; i < parts_.size(); ++i)
+                    launch_sparse_pack(nx[i], b[i], (uint32_t)nw, sp_pairs_[i], cap, sp_cnt_[i], p0.cs());
+                uint64_t bytes = 0;
+                const bool ok = comm_.sparse_min(b, nx, sp_pairs_, sp_cnt_, cap, p0.cs(), &bytes);
+                if (ok) { ++sparse_iters; sparse_bytes += bytes; }
+                return ok;
+            };
+            const uint64_t dP = (uint64_t)std::max<uint32_t>(1, o_.sparse_exchange) * (uint64_t)comm_.world();
             if (algo == ALG_BFS) {
-                std::vector<uint32_t*> b;
-                for (auto& p : parts_) b.push_back(p->next());
-                comm_.or_words(b, nw, p0.cs());
+                // BFS levels: a discovering rank holds t+1, the others INF, so MIN is right too;
+                // a pair (8 B) replaces a bitmap bit: cap n / (64 d P)
+                if (!try_sparse(g_.n / (64 * dP))) {
+                    std::vector<uint32_t*> b;
+                    for (auto& p : parts_) b.push_back(p->next());
+                    comm_.or_words(b, nw, p0.cs());
+                }
             } else if (algo == ALG_PRD) {
                 std::vector<unsigned long long*> b;
                 for (auto& p : parts_) b.push_back(p->prd_inc());
                 comm_.sum_u64(b, g_.n, p0.cs());
             } else {
-                std::vector<uint32_t*> b, nx;
-                for (auto& p : parts_) { b.push_back(p->val()); nx.push_back(p->next()); }
-                bool sparse = false;
-                if (o_.sparse_exchange) {
-                    // the (id, value) pairs each rank lowered, when few; else dense MIN
-                    const uint64_t c = std::max<uint64_t>(1, g_.n / ((uint64_t)o_.sparse_exchange * comm_.world()));
-                    const uint32_t cap = (uint32_t)std::min<uint64_t>(c, g_.n);
-                    if (sp_cap_ != cap || sp_pairs_.size() != parts_.size()) {
-                        free_sparse();
-                        for (size_t i = 0; i < parts_.size(); ++i) {
-                            void* pp = nullptr;
-                            uint32_t* cc = nullptr;
-                            CK(cudaMalloc(&pp, (size_t)cap * 8));
-                            CK(cudaMalloc(&cc, 4));
-                            sp_pairs_.push_back(pp);
-                            sp_cnt_.push_back(cc);
-                        }
-                        sp_cap_ = cap;
-                    }
-                    for (size_t i = 0; i < parts_.size(); ++i)
-                        launch_sparse_pack(nx[i], b[i], (uint32_t)nw, sp_pairs_[i], cap, sp_cnt_[i], p0.cs());
-                    uint64_t bytes = 0;
-                    sparse = comm_.sparse_min(b, nx, sp_pairs_, sp_cnt_, cap, p0.cs(), &bytes);
-                    if (sparse) { ++sparse_iters; sparse_bytes += bytes; }
+                const bool sparse = try_sparse(g_.n / dP);
+                if (!sparse) {
+                    std::vector<uint32_t*> b;
+                    for (auto& p : parts_) b.push_back(p->val());
+                    comm_.min_u32(b, g_.n, p0.cs());
                 }
-                if (!sparse) comm_.min_u32(b, g_.n, p0.cs());
                 dense_fin = !sparse;
             }
             p0.span(e0, p0.cs(), t, PH_XCH);

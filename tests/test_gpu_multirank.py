@@ -120,13 +120,14 @@ def test_fused_exchange_matches_oracle(asc, P, algo):
 
 
 @pytest.mark.parametrize("P", [2, 3, 5])
-@pytest.mark.parametrize("algo", ["sssp", "cc"])
-@pytest.mark.parametrize("d", [8, 2000])
+@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc"])
+@pytest.mark.parametrize("d", [1, 8, 2000])
 def test_sparse_exchange_matches_oracle(asc, P, algo, d):
-    """ASCETIC_OPT_SPARSE_EXCHANGE: each rank's lowered (id, value) pairs are
-    exchanged and applied with atomicMin when every rank has at most n/(d P) of them, else the
-    dense MIN runs. d = 8: mostly sparse; d = 2000: a cap of 1 pair, so nearly every iteration
-    falls back to dense. Values and every per-rank record equal the oracle either way."""
+    """ASCETIC_OPT_SPARSE_EXCHANGE: each rank's lowered (id, value) pairs (BFS:
+    newly reached ids) are exchanged and applied with atomicMin + next bit when every rank has at
+    most n/(d P) of them (BFS n/(64 d P)), else the dense MIN / OR runs. d = 1, 8: mostly sparse;
+    d = 2000: a cap of 1 pair, so nearly every iteration falls back to dense. Values and every
+    per-rank record equal the oracle either way."""
     g = gg.rmat(12, seed=35, weights=(algo == "sssp"))
     src = int(np.argmax(np.diff(g.off.astype(np.int64))))
     budget = g.csr_bytes // (4 * P)
@@ -145,7 +146,7 @@ def test_sparse_exchange_matches_oracle(asc, P, algo, d):
                              bounds=bounds)
             np.testing.assert_array_equal(res, ref.values)
             assert [{f: i[f] for f in REC} for i in its] == [{f: r[f] for f in REC} for r in ref.records]
-            if d == 8:
+            if d == 1 or (d == 8 and algo != "bfs"):
                 assert st["sparse_exchanges"] >= 1 and st["sparse_exchange_bytes"] > 0
             else:
                 assert st["sparse_exchanges"] < st["iterations"]

@@ -78,7 +78,7 @@ def test_nccl_one_rank_reload_reopens_peers(asc):
         asc.set_option("fused_exchange", 0)
 
 
-@pytest.mark.parametrize("algo", ["sssp", "cc"])
+@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc"])
 def test_nccl_one_rank_sparse_exchange(asc, algo):
     """ASCETIC_OPT_SPARSE_EXCHANGE through libnccl: the count and pair all-gathers run on the
     one-rank communicator (nothing foreign to apply), the finalize takes the merged next bitmap."""
@@ -86,7 +86,7 @@ def test_nccl_one_rank_sparse_exchange(asc, algo):
     src = int(np.argmax(np.diff(g.off.astype(np.int64))))
     budget = g.csr_bytes // 4
     asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True)
-    asc.set_option("sparse_exchange", 8)
+    asc.set_option("sparse_exchange", 1)
     asc.set_option("chunk_cap", 4096)
     try:
         asc.set_budget(budget, 0.4)
