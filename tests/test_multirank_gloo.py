@@ -97,6 +97,45 @@ def _worker(rank, world, port, algo, q):
                 A = nxt
                 t += 1
             vals = level.astype(np.uint32)
+        elif algo == "bfs_sparse":
+            # BFS with the sparse exchange (d = 1): newly reached ids, all-gathered padded to the
+            # largest count, when every rank has at most n / (64 P); else the bitmap OR
+            s = int(np.argmax(deg))
+            cap = max(1, n // (64 * world))
+            level = np.full(n, INF, dtype=np.uint64)
+            level[s] = 0
+            A = np.zeros(n, dtype=bool); A[s] = True
+            visited = A.copy()
+            n_sparse = n_dense = 0
+            while A.any():
+                recs.append(_record(t, rank, A, stat_all, lo, hi, deg, 4, oracle.digest(A)))
+                own = np.zeros(n, dtype=bool); own[lo:hi] = A[lo:hi]
+                sel = own[src_all]
+                nxt = np.zeros(n, dtype=bool)
+                nxt[nbr[sel]] = True
+                nxt &= ~visited
+                ids = np.flatnonzero(nxt)
+                cnt = torch.tensor([ids.size], dtype=torch.int64)
+                cnts = [torch.zeros_like(cnt) for _ in range(world)]
+                dist.all_gather(cnts, cnt)
+                maxc = max(int(c.item()) for c in cnts)
+                if maxc <= cap:
+                    buf = torch.zeros(maxc, dtype=torch.int64)
+                    buf[: ids.size] = torch.from_numpy(ids)
+                    bufs = [torch.zeros_like(buf) for _ in range(world)]
+                    dist.all_gather(bufs, buf)
+                    for b_, c_ in zip(bufs, cnts):
+                        nxt[b_[: int(c_.item())].numpy()] = True
+                    n_sparse += 1
+                else:
+                    nxt = _or_allgather(nxt)
+                    n_dense += 1
+                visited |= nxt
+                level[nxt] = t + 1
+                A = nxt
+                t += 1
+            assert n_sparse >= 1 and n_dense >= 1, (n_sparse, n_dense)
+            vals = level.astype(np.uint32)
         elif algo == "cc_sparse":
             # CC with the sparse MIN exchange (ASCETIC_OPT_SPARSE_EXCHANGE, d = 8): each rank's
             # lowered (id, label) pairs, all-gathered padded to the largest count and applied with
@@ -216,7 +255,7 @@ def _worker(rank, world, port, algo, q):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("algo", ["bfs", "cc", "cc_sparse", "pr", "prd"])
+@pytest.mark.parametrize("algo", ["bfs", "bfs_sparse", "cc", "cc_sparse", "pr", "prd"])
 def test_world2_gloo_protocol(algo):
     import graphgen as gg
     import oracle
