@@ -129,6 +129,20 @@ void Comm::min_u32(const std::vector<uint32_t*>& local, uint64_t n, cudaStream_t
     NC(nccl().AllReduce(local[0], local[0], n, ncclUint32, ncclMin, (ncclComm_t)nccl_comm_, s), "ncclAllReduce(min)");
 }
 
+void Comm::reserve_sparse(uint32_t cap, int local_parts) {
+    if (!active()) return;
+    if (!sp_counts_host_)
+        CKc(cudaMallocHost(&sp_counts_host_, sizeof(uint32_t) * (size_t)std::max(world_, local_parts)), "sparse counts");
+    if (emulated_) return;
+    if (!sp_counts_) CKc(cudaMalloc(&sp_counts_, sizeof(uint32_t) * (size_t)world_), "sparse counts");
+    const uint64_t want = (uint64_t)world_ * cap * 8ull;
+    if (sp_gather_bytes_ < want) {
+        if (sp_gather_) cudaFree(sp_gather_);
+        CKc(cudaMalloc(&sp_gather_, want), "sparse gather");
+        sp_gather_bytes_ = want;
+    }
+}
+
 bool Comm::sparse_min(const std::vector<uint32_t*>& val, const std::vector<uint32_t*>& next,
                       const std::vector<void*>& pairs, const std::vector<uint32_t*>& count, uint32_t cap,
                       cudaStream_t s, uint64_t* bytes_out) {

@@ -44,6 +44,8 @@ class Comm {
     // every rank and are applied by atomicMin + next bit. Reads the counts on the host (one sync);
     // returns false, having changed nothing, when some rank has more than cap pairs (the caller then
     // runs min_u32). All ranks take the same decision: they see the same counts.
+    // allocate sparse_min's host count buffer and (NCCL) its gather buffer for `cap` pairs per rank
+    void reserve_sparse(uint32_t cap, int local_parts);
     bool sparse_min(const std::vector<uint32_t*>& val, const std::vector<uint32_t*>& next,
                     const std::vector<void*>& pairs, const std::vector<uint32_t*>& count, uint32_t cap,
                     cudaStream_t s, uint64_t* bytes_out = nullptr);

@@ -1232,6 +1232,28 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
             for (auto& p : parts_) p->set_peers(kind, world);
         }
     }
+    // sparse exchange (collectives path, BFS / SSSP / CC): pair buffers sized before the timed run.
+    // cap = n / (d P) pairs per rank; BFS n / (64 d P), a pair (8 B) replacing one bitmap bit
+    const bool sparse_on = multi && !fused && o_.sparse_exchange &&
+                           (algo == ALG_BFS || algo == ALG_SSSP || algo == ALG_CC);
+    if (sparse_on) {
+        const uint64_t dP = (uint64_t)o_.sparse_exchange * (uint64_t)comm_.world();
+        const uint64_t c64 = algo == ALG_BFS ? g_.n / (64 * dP) : g_.n / dP;
+        const uint32_t cap = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(c64, g_.n));
+        if (sp_cap_ != cap || sp_pairs_.size() != parts_.size()) {
+            free_sparse();
+            for (size_t i = 0; i < parts_.size(); ++i) {
+                void* pp = nullptr;
+                uint32_t* cc = nullptr;
+                CK(cudaMalloc(&pp, (size_t)cap * 8));
+                CK(cudaMalloc(&cc, 4));
+                sp_pairs_.push_back(pp);
+                sp_cnt_.push_back(cc);
+            }
+            sp_cap_ = cap;
+        }
+        comm_.reserve_sparse(cap, (int)parts_.size());
+    }
     for (auto& p : parts_) p->begin(algo, source, max_iters, timing);
     Part& p0 = *parts_[0];
     std::vector<IterTotals> T(parts_.size());
@@ -1279,21 +1301,9 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
             const uint64_t nw = (g_.n + 31) / 32;
             // SURVEY §8(e) sparse form (BFS / SSSP / CC): the ids (and values) each rank set in its
             // next bitmap this iteration, when every rank has at most `cap` of them; else dense
-            auto try_sparse = [&](uint64_t cap64) -> bool {
-                if (!o_.sparse_exchange) return false;
-                const uint32_t cap = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(cap64, g_.n));
-                if (sp_cap_ != cap || sp_pairs_.size() != parts_.size()) {
-                    free_sparse();
-                    for (size_t i = 0; i < parts_.size(); ++i) {
-                        void* pp = nullptr;
-                        uint32_t* cc = nullptr;
-                        CK(cudaMalloc(&pp, (size_t)cap * 8));
-                        CK(cudaMalloc(&cc, 4));
-                        sp_pairs_.push_back(pp);
-                        sp_cnt_.push_back(cc);
-                    }
-                    sp_cap_ = cap;
-                }
+            auto try_sparse = [&]() -> bool {
+                if (!sparse_on) return false;
+                const uint32_t cap = sp_cap_;
                 std::vector<uint32_t*> b, nx;
                 for (auto& p : parts_) { b.push_back(p->val()); nx.push_back(p->next()); }
                 for (size_t i = 0; i < parts_.size(); ++i)
@@ -1303,11 +1313,9 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
                 if (ok) { ++sparse_iters; sparse_bytes += bytes; }
                 return ok;
             };
-            const uint64_t dP = (uint64_t)std::max<uint32_t>(1, o_.sparse_exchange) * (uint64_t)comm_.world();
             if (algo == ALG_BFS) {
-                // BFS levels: a discovering rank holds t+1, the others INF, so MIN is right too;
-                // a pair (8 B) replaces a bitmap bit: cap n / (64 d P)
-                if (!try_sparse(g_.n / (64 * dP))) {
+                // BFS levels: a discovering rank holds t+1, the others INF, so MIN is right too
+                if (!try_sparse()) {
                     std::vector<uint32_t*> b;
                     for (auto& p : parts_) b.push_back(p->next());
                     comm_.or_words(b, nw, p0.cs());
@@ -1317,7 +1325,7 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
                 for (auto& p : parts_) b.push_back(p->prd_inc());
                 comm_.sum_u64(b, g_.n, p0.cs());
             } else {
-                const bool sparse = try_sparse(g_.n / dP);
+                const bool sparse = try_sparse();
                 if (!sparse) {
                     std::vector<uint32_t*> b;
                     for (auto& p : parts_) b.push_back(p->val());
