@@ -369,6 +369,18 @@ def main():
         cpu = {"value": a_ / s_t / 1e9, "unit": "GTEPS", "cores": oracle.threads(), "kind": "oracle",
                "sample": f"{runs} full oracle {algo.upper()} runs" + (f" of {it_} iterations" if algo == "pr" else "")
                          + f" from the bench sources on the same {args.config} graph ({s_t:.1f} s)"}
+        if args.config in ("c1", "c2"):
+            # a single-thread oracle figure too, for C1/C2: one run from the first source
+            k0 = oracle.threads()
+            oracle.set_threads(1)
+            try:
+                t0 = time.perf_counter()
+                r = oracle.run(algo, g.off, g.nbr, src=srcs[0], max_iters=it_, is_static=stc)
+                t1 = time.perf_counter() - t0
+            finally:
+                oracle.set_threads(k0)
+            cpu["single_thread"] = {"value": r.active_arcs_total / t1 / 1e9, "unit": "GTEPS", "cores": 1,
+                                    "sample": f"1 full oracle {algo.upper()} run from source {srcs[0]} ({t1:.1f} s)"}
 
     out = {"metric": METRIC, "value": value, "unit": "GTEPS", "n_gpus": ws, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,

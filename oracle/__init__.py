@@ -77,6 +77,7 @@ def _load():
         lib.or_random_chunks.argtypes = [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_void_p]
         lib.or_set_prd_tol.argtypes = [ctypes.c_uint64]
         lib.or_threads.restype = ctypes.c_int
+        lib.or_set_threads.argtypes = [ctypes.c_int]
         lib.or_classify.argtypes = [ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p,
                                     ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
                                     ctypes.c_void_p, ctypes.c_void_p]
@@ -86,6 +87,12 @@ def _load():
 
 def threads() -> int:
     return int(_load().or_threads())
+
+
+def set_threads(k: int) -> None:
+    """OpenMP threads of the following runs (timing only; results do not depend on it except the
+    fp64 summation order of PR's dangling mass)."""
+    _load().or_set_threads(int(k))
 
 
 @dataclass
