@@ -226,6 +226,8 @@ def main():
         step(i)
     torch.cuda.synchronize()
 
+    g500_edges = 0
+    deg64 = np.diff(g.off.astype(np.int64)) if algo == "bfs" else None
     clocks = Clocks(local)
     clocks.start()
     per = []
@@ -243,6 +245,11 @@ def main():
         torch.cuda.synchronize()
         total_ms += e0.elapsed_time(e1)
         per.append(st)
+        if algo == "bfs":
+            # Graph500 TEPS: undirected edges in the reached component, read after the
+            # timed region; the graphs are symmetric, so that is half the reached vertices' arcs
+            lv = asc.get_result()
+            g500_edges += int(deg64[lv != 0xFFFFFFFF].sum()) // 2
     clk = clocks.stop()
     if ws > 1:
         tt = torch.tensor([total_ms], device=dev, dtype=torch.float64)
@@ -399,6 +406,7 @@ def main():
                                      ": 1D edge-balanced vertex ranges, per-rank static region and budget, "
                                      "NCCL exchange per iteration (OR / MIN / SUM + slice broadcast)")},
            "gteps_excl_fill": value_excl_fill,
+           "graph500_gteps": (g500_edges / (total_ms / 1e3) / 1e9) if algo == "bfs" else None,
            "roofline": roofline, "link": link, "cpu_baseline": cpu, "e2e": e2e,
            "gpu_launches": int(sum(s["kernel_launches"] for s in per)),
            "library_ms_per_step": lib_ms / args.steps,
