@@ -166,6 +166,8 @@ def main():
     ap.add_argument("--ref-pr-iters", type=int, default=2, help="PR iterations per reference step (bounded)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--xfer", type=int, default=0)
+    ap.add_argument("--sparse-exchange", type=int, default=0,
+                    help="N > 1, BFS/SSSP/CC: ASCETIC_OPT_SPARSE_EXCHANGE divisor d (0 = dense exchange)")
     args = ap.parse_args()
     ws, rank, local = _dist()
     if args.warmup < 3:
@@ -216,6 +218,7 @@ def main():
     asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True)
     asc.set_budget(budget)
     asc.set_option("xfer_mode", args.xfer)
+    asc.set_option("sparse_exchange", args.sparse_exchange)
     l2_flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
 
     def step(i):
@@ -335,6 +338,7 @@ def main():
         h1 = time.perf_counter()
         asc.set_budget(budget)
         asc.set_option("xfer_mode", args.xfer)
+        asc.set_option("sparse_exchange", args.sparse_exchange)
         h2 = time.perf_counter()
         asc.run(algo, srcs[k % len(srcs)], iters)
         h3 = time.perf_counter()
@@ -404,7 +408,10 @@ def main():
                       "graph_gen_s": round(gen_s, 2),
                       "parallelism": f"{ws} process(es), one GPU each" + ("" if ws == 1 else
                                      ": 1D edge-balanced vertex ranges, per-rank static region and budget, "
-                                     "NCCL exchange per iteration (OR / MIN / SUM + slice broadcast)")},
+                                     "NCCL exchange per iteration (OR / MIN / SUM + slice broadcast)"
+                                     + (f"; sparse exchange d={args.sparse_exchange}, "
+                                        f"{sum(s_['sparse_exchanges'] for s_ in per)} sparse iterations"
+                                        if args.sparse_exchange else ""))},
            "gteps_excl_fill": value_excl_fill,
            "graph500_gteps": (g500_edges / (total_ms / 1e3) / 1e9) if algo == "bfs" else None,
            "roofline": roofline, "link": link, "cpu_baseline": cpu, "e2e": e2e,
