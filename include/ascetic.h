@@ -70,7 +70,8 @@ typedef enum {
     ASCETIC_OPT_HUB_DEGREE = 6,    /* hit-queue degree at/above which a list is split across CTAs (default 2048) */
     ASCETIC_OPT_TIMING = 7,        /* 1 (default) = per-iteration phase timing with CUDA events */
     ASCETIC_OPT_GATHER_CTAS = 8,   /* persistent CTAs of the zero-copy gather; 0 (default) = 512 / b_e (~1 MiB in flight) */
-    ASCETIC_OPT_CHUNK_BUFFERS = 9, /* On-demand Region C split into N buffers of C/N (2..8, default 3); set before set_budget */
+    ASCETIC_OPT_CHUNK_BUFFERS = 9, /* On-demand Region C split into N buffers of C/N (2..8; 0 = auto (default): 3, or 2
+                                    when C/3 < 4 MiB); set before set_budget */
     ASCETIC_OPT_STATIC_CTAS_PER_SM = 10, /* persistent grid of the static-hit kernels, CTAs per SM (0 = default 4) */
     ASCETIC_OPT_PREFETCH = 11,     /* 1 (default): PR issues the next iteration's first chunk DMAs at the end of the
                                       current one (A_t = V, so the miss stream repeats); 0 = off */

@@ -281,7 +281,11 @@ void Part::set_budget(uint64_t bytes, double frac) {
         throw Error(ASCETIC_ENOMEM, "budget leaves an On-demand chunk below 16 bytes (cap=" + std::to_string(p.cap) + ")");
     // On-demand Region C split into nb chunk buffers of floor(C/nb/16)*16 bytes (the placer's
     // `cap` is the 2-buffer figure; more buffers give the pipeline slack, same C)
-    const int nb = std::max(2, std::min(kMaxBuffers, o_.chunk_buffers));
+    // auto (0): 3 buffers, or 2 when a third of C is under 4 MiB: per-chunk latency (~25 us of
+    // gather + on-demand launch) then dominates and fewer, larger chunks win (C1 A/B on B200:
+    // 2 / 3 / 4 buffers = 0.99 / 1.14 / 1.29 ms per run, profiles/r01/c1_chunk_buffers.log)
+    const int nb = o_.chunk_buffers ? std::max(2, std::min(kMaxBuffers, o_.chunk_buffers))
+                                    : (p.C / 3 < (4ull << 20) ? 2 : 3);
     // chunk buffers never need more than the rank's whole payload D
     const uint64_t per_buf = std::min<uint64_t>(p.C / (uint64_t)nb, std::max<uint64_t>(p.D, 16)) / 16 * 16;
     if (p.s < own && per_buf < 16)
@@ -1164,7 +1168,7 @@ void Engine::set_option(int opt, int64_t value) {
             o_.static_ctas_per_sm = (int)value;
             break;
         case ASCETIC_OPT_CHUNK_BUFFERS:
-            if (value < 2 || value > 8) throw Error(ASCETIC_EINVAL, "chunk buffers must be in [2, 8]");
+            if (value != 0 && (value < 2 || value > 8)) throw Error(ASCETIC_EINVAL, "chunk buffers must be 0 (auto) or in [2, 8]");
             o_.chunk_buffers = (int)value;
             if (state_ == 2) state_ = 1;   // takes effect at the next set_budget
             break;

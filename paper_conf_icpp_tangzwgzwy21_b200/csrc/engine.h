@@ -55,8 +55,9 @@ struct Options {
     uint32_t hub_deg = 2048;
     int timing = 1;
     int gather_ctas = 0;
-    int chunk_buffers = 3;   // On-demand Region split into this many chunk buffers of C/N bytes
-                             // (3 absorbs one slow on-demand kernel without stalling the link)
+    int chunk_buffers = 0;   // On-demand Region split into this many chunk buffers of C/N bytes;
+                             // 0 = auto: 3 (absorbs one slow on-demand kernel without stalling the
+                             // link), 2 when C/3 < 4 MiB (chunks that small are latency-bound)
     int static_ctas_per_sm = 0;   // persistent grid of the static-hit kernels (0 = 4 per SM)
     int prefetch = 1;             // PR: issue the next iteration's first chunk transfers early
     int repartition = 0;          // Eq. 3 adaptive re-partition (off, as in the paper's evaluation)

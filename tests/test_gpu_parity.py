@@ -240,7 +240,7 @@ def test_options_do_not_change_results(asc, opt, val):
             assert st["h2d_static_fill_bytes"] == 0
         else:
             assert st["h2d_static_fill_bytes"] == p.static_bytes
-    defaults = {"overlap": 1, "keep_static": 0, "chunk_buffers": 3, "gather_ctas": 0, "static_ctas_per_sm": 0,
+    defaults = {"overlap": 1, "keep_static": 0, "chunk_buffers": 0, "gather_ctas": 0, "static_ctas_per_sm": 0,
                 "timing": 1}
     asc.set_option(opt, defaults[opt])
 
@@ -261,7 +261,7 @@ def test_pr_cross_iteration_prefetch(asc, prefetch, nbuf):
     st, its = asc.stats()
     res = asc.get_result().copy()
     asc.set_option("prefetch", 1)
-    asc.set_option("chunk_buffers", 3)
+    asc.set_option("chunk_buffers", 0)
     asc.set_option("xfer_mode", 0)
     asc.set_option("chunk_cap", 0)
     p = oracle.placer(g.off, 4, g.csr_bytes // 3, 0.5)
