@@ -125,7 +125,8 @@ typedef struct {
     uint64_t static_reserved;     /* Ms = R*B floored to 16 KiB */
     uint64_t static_bytes;        /* b_e * off[s] actually resident */
     uint64_t ondemand_bytes;      /* C = B - Ms */
-    uint64_t chunk_cap;           /* bytes per on-demand chunk buffer (2 buffers) */
+    uint64_t chunk_cap;           /* bytes per on-demand chunk buffer: floor(C / chunk_buffers / 16) * 16 (or the
+                                     CHUNK_CAP option, if smaller) */
     double static_fraction_used;  /* R */
     uint64_t h2d_payload_bytes;   /* Σ_t miss bytes (the parity target) */
     uint64_t h2d_static_fill_bytes;
@@ -159,6 +160,8 @@ typedef struct {
     double time_replace_s;        /* copy-stream time of the swap DMAs */
     uint64_t sparse_exchanges;    /* iterations whose exchange went sparse (ASCETIC_OPT_SPARSE_EXCHANGE) */
     uint64_t sparse_exchange_bytes; /* (id, value) pair bytes all ranks contributed to those exchanges */
+    uint32_t chunk_buffers;       /* On-demand Region buffers in use (auto: 3, or 2 when C/3 < 4 MiB) */
+    uint32_t reserved0;
 } ascetic_stats_t;
 
 typedef struct {
@@ -205,9 +208,11 @@ int ascetic_load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_t
  *   bytes            B = Static Region + On-demand Region (vertex state is accounted outside)
  *   static_fraction  R in [0,1] fixes the split; < 0 selects Eq. 2 with K = 0.10,
  *                    clamped to [0,1]. NaN or > 1 => EINVAL.
- * Ms = floor(R*B / 16 KiB) * 16 KiB (<= D), s = max{v : b_e*off[v] <= Ms}, C = B - Ms,
- * chunk cap = floor(C/2/16)*16. Allocates the static buffer (b_e*off[s] bytes) and two
- * chunk buffers once. ENOMEM if s < n and the chunk cap is below 16 bytes, or allocation fails.
+ * Ms = floor(R*B / 16 KiB) * 16 KiB (<= D), s = max{v : b_e*off[v] <= Ms}, C = B - Ms.
+ * C is split into N chunk buffers (ASCETIC_OPT_CHUNK_BUFFERS; auto: 3, or 2 when C/3 < 4 MiB) of
+ * floor(C/N/16)*16 bytes each (ascetic_placement_t.cap is the 2-buffer figure). Allocates one
+ * arena of Ms + N buffers (<= B) once. ENOMEM if s < n and a buffer is below 16 bytes, or
+ * allocation fails.
  */
 int ascetic_set_budget(uint64_t bytes, double static_fraction);
 

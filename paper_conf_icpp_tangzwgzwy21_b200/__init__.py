@@ -63,7 +63,8 @@ class Stats(ctypes.Structure):
                 ("time_finalize_s", ctypes.c_double), ("time_host_s", ctypes.c_double),
                 ("repartitions", ctypes.c_uint64), ("h2d_replace_bytes", ctypes.c_uint64),
                 ("swaps_total", ctypes.c_uint64), ("time_replace_s", ctypes.c_double),
-                ("sparse_exchanges", ctypes.c_uint64), ("sparse_exchange_bytes", ctypes.c_uint64)]
+                ("sparse_exchanges", ctypes.c_uint64), ("sparse_exchange_bytes", ctypes.c_uint64),
+                ("chunk_buffers", ctypes.c_uint32), ("reserved0", ctypes.c_uint32)]
 
 
 class IterStats(ctypes.Structure):

@@ -20,6 +20,7 @@
 namespace ascetic {
 
 constexpr uint32_t kInf = 0xFFFFFFFFu;
+constexpr double kFxOne = 4611686018427387904.0;         // 2^62: PR sums are < 2 (Σ_v sum = Σ r <= 1)
 constexpr int kClassifyWarps = 8;                       // words per tile = 8 * 32
 constexpr int kTileWords = kClassifyWarps * 32;         // 256 words = 8192 vertices
 constexpr uint32_t kSmallDeg = 32;                      // hit lists shorter than this: warp-cooperative
@@ -88,8 +89,11 @@ struct DevState {
     uint32_t* snap;
     float* rank;
     float* contrib;
-    double* sum;
-    double* dang;          // [0] = current dangling mass, [1] = next
+    // PR pull sums and dangling mass in 2^-62 fixed point (u64): every fp64 partial (a row, a hub
+    // piece, a chunk segment of a row) is rounded once to the grid and added as an integer, so the
+    // totals do not depend on the order the atomics land in (bitwise-reproducible ranks, DESIGN R31)
+    unsigned long long* sum;
+    unsigned long long* dang;   // [0] = current dangling mass, [1] = next
     uint32_t iter;         // t
     uint64_t vlo, vhi;     // owned vertex range (PR finalize)
     unsigned long long static_arc0;   // first arc held by the Static Region (off[vlo])
@@ -163,7 +167,6 @@ void launch_sparse_pack(const uint32_t* next, const uint32_t* val, uint32_t nwor
                         uint32_t* count, cudaStream_t s);
 void launch_sparse_apply(uint32_t* val, uint32_t* next, const void* pairs, uint64_t stride, const uint32_t* counts,
                          int P, int skip, uint32_t cap, cudaStream_t s);
-void launch_add_f64(double* dst, const double* src, cudaStream_t s);
 void launch_add_u64(unsigned long long* dst, const unsigned long long* src, uint64_t n, cudaStream_t s);
 // *bad := min{v : off[v+1] < off[v]} (left untouched when off[0..n] is non-decreasing)
 void launch_check_monotone(const unsigned long long* off, uint64_t n, unsigned long long* bad, cudaStream_t s);

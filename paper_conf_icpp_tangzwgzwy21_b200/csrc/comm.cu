@@ -184,17 +184,6 @@ bool Comm::sparse_min(const std::vector<uint32_t*>& val, const std::vector<uint3
     return true;
 }
 
-void Comm::sum_f64(const std::vector<double*>& local, cudaStream_t s) {
-    if (!active()) return;
-    if (emulated_) {
-        for (size_t p = 1; p < local.size(); ++p) launch_add_f64(local[0], local[p], s);
-        for (size_t p = 1; p < local.size(); ++p)
-            CKc(cudaMemcpyAsync(local[p], local[0], 8, cudaMemcpyDeviceToDevice, s), "sum copy-back");
-        return;
-    }
-    NC(nccl().AllReduce(local[0], local[0], 1, ncclFloat64, ncclSum, (ncclComm_t)nccl_comm_, s), "ncclAllReduce(sum)");
-}
-
 void Comm::sum_u64(const std::vector<unsigned long long*>& local, uint64_t n, cudaStream_t s) {
     if (!active() || n == 0) return;
     if (emulated_) {

@@ -2,7 +2,7 @@
 // is single-GPU). One process per GPU, 1D vertex ranges, replicated vertex state:
 //   BFS       : OR of the next-frontier bitmaps        (NCCL has no bitwise OR: all-gather + OR kernel)
 //   SSSP / CC : MIN of the value arrays               (ncclAllReduce min)
-//   PR        : SUM of the fp64 dangling partials + every rank's contrib slice to all ranks
+//   PR        : SUM of the 2^-62 fixed-point dangling partials (exact) + every rank's contrib slice to all ranks
 //   PRD       : SUM of the u64 residual increments   (ncclAllReduce sum, exact: integers)
 // Two back ends behind one interface:
 //   NCCL     — across processes (libnccl.so.2 is dlopen'ed on first use, so single-GPU
@@ -49,7 +49,6 @@ class Comm {
     bool sparse_min(const std::vector<uint32_t*>& val, const std::vector<uint32_t*>& next,
                     const std::vector<void*>& pairs, const std::vector<uint32_t*>& count, uint32_t cap,
                     cudaStream_t s, uint64_t* bytes_out = nullptr);
-    void sum_f64(const std::vector<double*>& local, cudaStream_t s);
     // element-wise SUM of n uint64 per rank (PageRank-delta residual increments), in place
     void sum_u64(const std::vector<unsigned long long*>& local, uint64_t n, cudaStream_t s);
     // Fused exchange support (NCCL back end): map every rank's `local` device allocation into this

@@ -68,6 +68,10 @@ __device__ __forceinline__ SrcVal<ALGO> src_val(const DevState& d, uint32_t u) {
 }
 constexpr double kDamp = 0.85;
 
+// PR fixed point (DESIGN R31): one round-to-nearest per fp64 partial, integer sums thereafter
+__device__ __forceinline__ unsigned long long to_fx(double x) { return __double2ull_rn(x * kFxOne); }
+__device__ __forceinline__ double from_fx(unsigned long long x) { return __ull2double_rn(x) * (1.0 / kFxOne); }
+
 // ------------------------------------------------------------------ L2 policy loads
 // Adjacency lists and chunks are read once: stream them with L2 evict_first so they do not
 // push the randomly accessed vertex state (dist / labels / bitmaps / contrib, the part of
@@ -421,7 +425,7 @@ __global__ void __launch_bounds__(256) k_static_small(DevState d, const uint32_t
                 }
             }
         }
-        if (ALGO == PR && valid) d.sum[u] = s_acc[wib][lane];
+        if (ALGO == PR && valid) d.sum[u] = to_fx(s_acc[wib][lane]);
         __syncwarp();
     }
 }
@@ -439,7 +443,7 @@ __global__ void __launch_bounds__(256) k_static_med(DevState d, const uint32_t* 
         double acc = expand_list<ALGO, REMAP>(d, sbase, a0 - d.static_arc0, a1 - d.static_arc0, sval, lane, 32);
         if (ALGO == PR) {
             acc = warp_sum_d(acc);
-            if (lane == 0) d.sum[u] = acc;
+            if (lane == 0) d.sum[u] = to_fx(acc);
         }
     }
 }
@@ -467,7 +471,7 @@ __global__ void __launch_bounds__(256) k_static_hub(DevState d, const uint32_t* 
             if (threadIdx.x == 0) {
                 double t = 0.0;
                 for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += s_red[w];
-                atomicAdd(d.sum + u, t);
+                atomicAdd(d.sum + u, to_fx(t));
             }
             __syncthreads();
         }
@@ -521,36 +525,25 @@ __device__ __forceinline__ uint32_t warp_map(const unsigned long long* s_pre, ui
 }
 
 // ------------------------------------------------------------------ on-demand compute
-// Tile metadata either staged in shared memory (SMEM) or read straight from the queues (L1-cached):
-// the zero-shared-memory variant can co-reside with any kernel whatever the SM's L1/shared split.
-template <int ALGO, bool SMEM>
+// Tile metadata is read straight from the queues (L1-cached), no shared memory: the kernel can
+// co-reside with any kernel whatever the SM's L1/shared split (a 33 KB/CTA staged variant could
+// not start on SMs configured for the shared-memory-free static kernels).
+template <int ALGO>
 struct TileView {
     const unsigned long long* pre;
     const uint32_t* u;
-    const SrcVal<ALGO>* v;
     const DevState* d;
-    __device__ __forceinline__ uint32_t vtx(uint32_t k) const { return SMEM ? u[k] : __ldg(u + k); }
-    __device__ __forceinline__ SrcVal<ALGO> val(uint32_t k) const { return SMEM ? v[k] : src_val<ALGO>(*d, __ldg(u + k)); }
+    __device__ __forceinline__ uint32_t vtx(uint32_t k) const { return __ldg(u + k); }
+    __device__ __forceinline__ SrcVal<ALGO> val(uint32_t k) const { return src_val<ALGO>(*d, __ldg(u + k)); }
 };
 
-template <int ALGO, bool SMEM>
+template <int ALGO>
 __device__ __forceinline__ void ondemand_tile(const DevState& d, const Queues& q, const void* __restrict__ chunk,
-                                              unsigned long long lo, unsigned long long hi, unsigned long long t,
-                                              unsigned long long* s_pre_, uint32_t* s_u_, SrcVal<ALGO>* s_v_) {
+                                              unsigned long long lo, unsigned long long hi, unsigned long long t) {
     const Tile x = tile_of(q, t, lo, hi);
-    if (SMEM) {
-        for (uint32_t k = threadIdx.x; k < x.cnt; k += blockDim.x) {
-            s_pre_[k] = __ldg(q.mq_pre + x.i0 + k);
-            const uint32_t u = __ldg(q.mq + x.i0 + k);
-            s_u_[k] = u;
-            if (ALGO != PR) s_v_[k] = src_val<ALGO>(d, u);
-        }
-        __syncthreads();
-    }
-    TileView<ALGO, SMEM> tv;
-    tv.pre = SMEM ? s_pre_ : q.mq_pre + x.i0;
-    tv.u = SMEM ? s_u_ : q.mq + x.i0;
-    tv.v = s_v_;
+    TileView<ALGO> tv;
+    tv.pre = q.mq_pre + x.i0;
+    tv.u = q.mq + x.i0;
     tv.d = &d;
     const unsigned long long* s_pre = tv.pre;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -633,31 +626,17 @@ __device__ __forceinline__ void ondemand_tile(const DevState& d, const Queues& q
                 if (lane >= o && ok2 == key) v += y;
             }
             const int nk = __shfl_down_sync(FULL, key, 1);
-            if (ok && (lane == 31 || nk != key)) atomicAdd(d.sum + tv.vtx(mk8[g]), v);
+            if (ok && (lane == 31 || nk != key)) atomicAdd(d.sum + tv.vtx(mk8[g]), to_fx(v));
         }
     }
 }
 
-// one CTA per 2048-arc tile of the chunk window, or a capped grid striding over the tiles
-template <int ALGO>
-__global__ void __launch_bounds__(256) k_ondemand(DevState d, Queues q, const void* __restrict__ chunk,
-                                                  unsigned long long lo, unsigned long long hi) {
-    __shared__ unsigned long long s_pre[kEdgeTile + 1];
-    __shared__ uint32_t s_u[kEdgeTile + 1];
-    __shared__ SrcVal<ALGO> s_v[kEdgeTile + 1];
-    const unsigned long long t0 = lo >> kEdgeTileShift, t1 = (hi - 1) >> kEdgeTileShift;
-    for (unsigned long long t = t0 + blockIdx.x; t <= t1; t += gridDim.x) {
-        if (t != t0 + blockIdx.x) __syncthreads();   // the previous tile's warps are done with smem
-        ondemand_tile<ALGO, true>(d, q, chunk, lo, hi, t, s_pre, s_u, s_v);
-    }
-}
-
+// one CTA per 2048-arc tile of the chunk window
 template <int ALGO>
 __global__ void __launch_bounds__(256) k_ondemand_g(DevState d, Queues q, const void* __restrict__ chunk,
                                                     unsigned long long lo, unsigned long long hi) {
     const unsigned long long t0 = lo >> kEdgeTileShift, t1 = (hi - 1) >> kEdgeTileShift;
-    for (unsigned long long t = t0 + blockIdx.x; t <= t1; t += gridDim.x)
-        ondemand_tile<ALGO, false>(d, q, chunk, lo, hi, t, nullptr, nullptr, nullptr);
+    for (unsigned long long t = t0 + blockIdx.x; t <= t1; t += gridDim.x) ondemand_tile<ALGO>(d, q, chunk, lo, hi, t);
 }
 
 // BFS needs no source: 128-bit loads straight over the chunk.
@@ -675,52 +654,6 @@ __global__ void __launch_bounds__(256) k_ondemand_bfs(DevState d, const uint32_t
 }
 
 // ------------------------------------------------------------------ zero-copy gather (transfer engine)
-// Persistent CTAs stride over the chunk's tiles. Each warp copies its 256 arcs as 8 groups
-// of 32 consecutive arcs: all 8 host loads are issued before the first store, so every
-// lane keeps 8 PCIe reads in flight; consecutive arcs of a run are consecutive host
-// addresses, so each group is one contiguous 128/256-byte read.
-template <int BE>
-__global__ void __launch_bounds__(256) k_gather(Queues q, const void* __restrict__ host, void* __restrict__ chunk,
-                                                unsigned long long lo, unsigned long long hi) {
-    using T = typename std::conditional<BE == 8, unsigned long long, uint32_t>::type;
-    __shared__ unsigned long long s_pre[kEdgeTile + 1];
-    __shared__ unsigned long long s_src[kEdgeTile + 1];
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const T* __restrict__ src = reinterpret_cast<const T*>(host);
-    T* __restrict__ dst = reinterpret_cast<T*>(chunk);
-    const unsigned long long t0 = lo >> kEdgeTileShift, t1 = (hi - 1) >> kEdgeTileShift;
-    for (unsigned long long t = t0 + blockIdx.x; t <= t1; t += gridDim.x) {
-        const Tile x = tile_of(q, t, lo, hi);
-        __syncthreads();
-        for (uint32_t k = threadIdx.x; k < x.cnt; k += blockDim.x) {
-            s_pre[k] = __ldg(q.mq_pre + x.i0 + k);
-            s_src[k] = __ldg(q.mq_src + x.i0 + k);
-        }
-        __syncthreads();
-        const unsigned long long pw = x.t_lo + (unsigned long long)warp * 256ull;
-        if (pw >= x.t_hi) continue;
-        const unsigned long long pe = min(x.t_hi, pw + 256ull);
-        uint32_t k = find_local(s_pre, 0, x.cnt, pw);
-        unsigned long long from[8];
-#pragma unroll
-        for (int g = 0; g < 8; ++g) {
-            const unsigned long long p = pw + 32ull * g;
-            const uint32_t mk = warp_map(s_pre, x.cnt, k, p, lane);
-            k = __shfl_sync(FULL, mk, 31);
-            from[g] = s_src[mk] + (p + lane - s_pre[mk]);
-        }
-        T v[8];
-#pragma unroll
-        for (int g = 0; g < 8; ++g)
-            if (pw + 32ull * g + lane < pe) v[g] = src[from[g]];
-#pragma unroll
-        for (int g = 0; g < 8; ++g) {
-            const unsigned long long a = pw + 32ull * g + lane;
-            if (a < pe) dst[a - lo] = v[g];
-        }
-    }
-}
-
 // host (mapped pinned) 16-byte load, not allocated in L1: read once, and keeping it out of L1
 // leaves the concurrent static-hit kernels their L1 hits on vertex state (C2 static 14.9 -> 12.1 ms,
 // C4-shaped 13.8 -> 11.0 ms; the gather rate is unchanged)
@@ -740,28 +673,26 @@ __device__ __forceinline__ uint4 ld_host16(const uint4* p) {
 // piece), each piece's cover units are enumerated across the warp (a unit shared by two
 // vertices of one piece is loaded once), and every lane stores the piece words its unit holds
 // at their stream position. `hoff` = the host array's byte offset from its 16-byte-aligned base.
-template <int BE, bool SMEM, int NG = 4>
+template <int BE, int NG>
 __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restrict__ host, uint32_t hoff,
                                                   unsigned long long w_end, uint32_t* __restrict__ chunk,
                                                   unsigned long long lo, unsigned long long hi) {
-    __shared__ unsigned long long sm_pre[SMEM ? kEdgeTile + 1 : 1];
-    __shared__ unsigned long long sm_src[SMEM ? kEdgeTile + 1 : 1];
+    // tile metadata staged in shared memory (reading it through L1 instead gathers at the same rate,
+    // but its L1 traffic slows the concurrent static-hit kernels)
+    __shared__ unsigned long long s_pre[kEdgeTile + 1];
+    __shared__ unsigned long long s_src[kEdgeTile + 1];
     constexpr unsigned long long AW = BE / 4;                 // words per arc
     const unsigned long long w_off = hoff / 4;                // host word index of arc 0
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const unsigned long long t0 = lo >> kEdgeTileShift, t1 = (hi - 1) >> kEdgeTileShift;
     for (unsigned long long t = t0 + blockIdx.x; t <= t1; t += gridDim.x) {
         const Tile x = tile_of(q, t, lo, hi);
-        const unsigned long long* s_pre = SMEM ? sm_pre : q.mq_pre + x.i0;
-        const unsigned long long* s_src = SMEM ? sm_src : q.mq_src + x.i0;
-        if (SMEM) {
-            __syncthreads();
-            for (uint32_t k = threadIdx.x; k < x.cnt; k += blockDim.x) {
-                sm_pre[k] = __ldg(q.mq_pre + x.i0 + k);
-                sm_src[k] = __ldg(q.mq_src + x.i0 + k);
-            }
-            __syncthreads();
+        __syncthreads();
+        for (uint32_t k = threadIdx.x; k < x.cnt; k += blockDim.x) {
+            s_pre[k] = __ldg(q.mq_pre + x.i0 + k);
+            s_src[k] = __ldg(q.mq_src + x.i0 + k);
         }
+        __syncthreads();
         const unsigned long long pw = x.t_lo + (unsigned long long)warp * 256ull;
         if (pw >= x.t_hi) continue;
         const unsigned long long pe = min(x.t_hi, pw + 256ull);
@@ -898,7 +829,7 @@ __global__ void k_pr_init(DevState d) {
         if (!deg) dang += r0;
     }
     dang = warp_sum_d(dang);
-    if ((threadIdx.x & 31) == 0 && dang != 0.0) atomicAdd(d.dang, dang);
+    if ((threadIdx.x & 31) == 0 && dang != 0.0) atomicAdd(d.dang, to_fx(dang));
 }
 
 // PRD (DESIGN R28-R30): r = 0, res = res0; A_0 = {v : res0 > tau} absorbs at once
@@ -1089,21 +1020,21 @@ __global__ void k_finalize_minlabel(DevState d) {
 }
 
 // r' = (1-d)/n + d (sum + dang/n) in fp64, stored fp32; contrib = fp32(r'/deg);
-// next dangling mass accumulated from the fp64 r'.
+// next dangling mass accumulated from the fp64 r', per warp, into the fixed-point total.
 __global__ void k_finalize_pr(DevState d, int cur) {
     const double inv_n = 1.0 / (double)d.n;
-    const double dc = d.dang[cur];
+    const double dc = from_fx(d.dang[cur]);
     double dn = 0.0;
     for (uint64_t v = d.vlo + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < d.vhi;
          v += (uint64_t)gridDim.x * blockDim.x) {
-        const double r = (1.0 - kDamp) * inv_n + kDamp * (d.sum[v] + dc * inv_n);
+        const double r = (1.0 - kDamp) * inv_n + kDamp * (from_fx(d.sum[v]) + dc * inv_n);
         const unsigned long long deg = __ldg(d.off + v + 1) - __ldg(d.off + v);
         d.rank[v] = (float)r;
         d.contrib[v] = deg ? (float)(r / (double)deg) : 0.0f;
         if (!deg) dn += r;
     }
     dn = warp_sum_d(dn);
-    if ((threadIdx.x & 31) == 0 && dn != 0.0) atomicAdd(d.dang + (cur ^ 1), dn);
+    if ((threadIdx.x & 31) == 0 && dn != 0.0) atomicAdd(d.dang + (cur ^ 1), to_fx(dn));
 }
 
 // P > 1: values were MIN-exchanged, so A_{t+1} = {v : val[v] < snap[v]} over every vertex
@@ -1191,8 +1122,6 @@ __global__ void __launch_bounds__(256) k_sparse_apply(uint32_t* __restrict__ val
         }
     }
 }
-
-__global__ void k_add_f64(double* dst, const double* src) { dst[0] += src[0]; }
 
 __global__ void k_check_monotone(const unsigned long long* __restrict__ off, uint64_t n, unsigned long long* bad) {
     for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
@@ -1418,27 +1347,12 @@ void launch_ondemand(int algo, const DevState& d, const Queues& q, const void* c
         ++g_launches;
         return;
     }
-    unsigned tiles = (unsigned)(((hi - 1) >> kEdgeTileShift) - (lo >> kEdgeTileShift) + 1);
-    // Zero-shared-memory variant by default: the staged one (33 KB per CTA, ASC_OND_SMEM=1) cannot
-    // start on SMs whose L1/shared split was chosen for a shared-memory-free static kernel, and
-    // waited out each 9 ms k_static_med on C3 (one 8-11 ms on-demand kernel per iteration that
-    // stalled chunk-buffer reuse: 35-38 ms of link gaps per 6 iterations -> 0.7 ms; ASCETIC_TRACE=2).
-    static const bool gv = [] { const char* e = std::getenv("ASC_OND_SMEM"); return !(e && std::atoi(e)); }();
-    if (gv) {
-        switch (algo) {
-            case SSSP: k_ondemand_g<SSSP><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
-            case CC: k_ondemand_g<CC><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
-            case PRD: k_ondemand_g<PRD><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
-            default: k_ondemand_g<PR><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
-        }
-        ++g_launches;
-        return;
-    }
+    const unsigned tiles = (unsigned)(((hi - 1) >> kEdgeTileShift) - (lo >> kEdgeTileShift) + 1);
     switch (algo) {
-        case SSSP: k_ondemand<SSSP><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
-        case CC: k_ondemand<CC><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
-        case PRD: k_ondemand<PRD><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
-        default: k_ondemand<PR><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
+        case SSSP: k_ondemand_g<SSSP><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
+        case CC: k_ondemand_g<CC><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
+        case PRD: k_ondemand_g<PRD><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
+        default: k_ondemand_g<PR><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
     }
     ++g_launches;
 }
@@ -1448,40 +1362,17 @@ void launch_gather(const Queues& q, const void* host_nbr, uint64_t m, uint32_t b
     if (hi <= lo) return;
     const unsigned long long tiles = ((hi - 1) >> kEdgeTileShift) - (lo >> kEdgeTileShift) + 1;
     const unsigned grid = (unsigned)(tiles < (unsigned long long)max_ctas ? tiles : (unsigned long long)max_ctas);
-    static const bool old = [] { const char* e = std::getenv("ASC_GATHER_OLD"); return e && std::atoi(e); }();
-    if (old) {
-        if (b_e == 8) k_gather<8><<<grid, 256, 0, s>>>(q, host_nbr, chunk, lo, hi);
-        else k_gather<4><<<grid, 256, 0, s>>>(q, host_nbr, chunk, lo, hi);
-    } else {
-        const uintptr_t hp = reinterpret_cast<uintptr_t>(host_nbr);
-        const uint4* base = reinterpret_cast<const uint4*>(hp & ~(uintptr_t)15);
-        const uint32_t hoff = (uint32_t)(hp & 15);
-        // tile metadata staged in shared memory (A/B: the zero-shared-memory variant, ASC_GATHER_SMEM=0,
-        // gathers at the same rate but its L1 metadata reads slow the concurrent static kernels)
-        static const bool sm = [] { const char* e = std::getenv("ASC_GATHER_SMEM"); return !(e && !std::atoi(e)); }();
-        uint32_t* c = reinterpret_cast<uint32_t*>(chunk);
-        const unsigned long long w_end = hoff / 4 + m * (b_e / 4);   // host words from the aligned base
-        // units loaded per lane per round (A/B knob ASC_GATHER_NG): a 256-arc warp segment of 8-byte
-        // arcs is 128 units plus up to one per piece boundary, so 4 per lane (128) usually needs a
-        // second, nearly empty round. C2 A/B on B200 (profiles/r01/gather_ng_ab.log): NG 4 -> 6 =
-        // 44.6-44.7 -> 45.0 GB/s, +0.6 % GTEPS; 5 and 8 within noise of 6. 4-byte arcs: 64 units, 4 fits.
-        static const int ng = [] { const char* e = std::getenv("ASC_GATHER_NG"); return e ? std::atoi(e) : 0; }();
-        if (sm) {
-            if (b_e == 8) {
-                if (ng == 5) k_gather16<8, true, 5><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
-                else if (ng == 4) k_gather16<8, true, 4><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
-                else if (ng == 8) k_gather16<8, true, 8><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
-                else k_gather16<8, true, 6><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
-            } else {
-                if (ng == 2) k_gather16<4, true, 2><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
-                else if (ng == 3) k_gather16<4, true, 3><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
-                else k_gather16<4, true><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
-            }
-        } else {
-            if (b_e == 8) k_gather16<8, false><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
-            else k_gather16<4, false><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
-        }
-    }
+    const uintptr_t hp = reinterpret_cast<uintptr_t>(host_nbr);
+    const uint4* base = reinterpret_cast<const uint4*>(hp & ~(uintptr_t)15);
+    const uint32_t hoff = (uint32_t)(hp & 15);
+    uint32_t* c = reinterpret_cast<uint32_t*>(chunk);
+    const unsigned long long w_end = hoff / 4 + m * (b_e / 4);   // host words from the aligned base
+    // units loaded per lane per round: a 256-arc warp segment of 8-byte arcs is 128 units plus up to
+    // one per piece boundary, so 4 per lane (128) usually needs a second, nearly empty round; 6 took
+    // C2's gather from 44.6-44.7 to 45.0 GB/s (profiles/r01/gather_ng_ab.log; 5 and 8 within noise of
+    // 6). 4-byte arcs: 64 units per segment, 4 per lane fits.
+    if (b_e == 8) k_gather16<8, 6><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
+    else k_gather16<4, 4><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
     ++g_launches;
 }
 
@@ -1518,7 +1409,7 @@ void launch_init(int algo, const DevState& d, uint32_t source, cudaStream_t s) {
             break;
         }
         default:
-            cudaMemsetAsync(d.dang, 0, 2 * sizeof(double), s);
+            cudaMemsetAsync(d.dang, 0, 2 * sizeof(unsigned long long), s);
             k_pr_init<<<gb, 256, 0, s>>>(d);
             ++g_launches;
             k_range_bits<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d.A, d.nwords, 0, d.n);
@@ -1541,7 +1432,7 @@ void launch_finalize(int algo, const DevState& d, bool dense, cudaStream_t s) {
             break;
         default: {
             const int cur = (int)(d.iter & 1u);
-            cudaMemsetAsync(d.dang + (cur ^ 1), 0, sizeof(double), s);
+            cudaMemsetAsync(d.dang + (cur ^ 1), 0, sizeof(unsigned long long), s);
             k_finalize_pr<<<blocks_for(d.vhi > d.vlo ? d.vhi - d.vlo : 1, 256), 256, 0, s>>>(d, cur);
             break;
         }
@@ -1599,11 +1490,6 @@ void launch_finalize_peers(int algo, const DevState& d, const void* const* peers
 
 void launch_add_u64(unsigned long long* dst, const unsigned long long* src, uint64_t n, cudaStream_t s) {
     k_add_u64<<<blocks_for(n, 256), 256, 0, s>>>(dst, src, n);
-    ++g_launches;
-}
-
-void launch_add_f64(double* dst, const double* src, cudaStream_t s) {
-    k_add_f64<<<1, 1, 0, s>>>(dst, src);
     ++g_launches;
 }
 

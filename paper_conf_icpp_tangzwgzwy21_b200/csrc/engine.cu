@@ -15,6 +15,7 @@
 #include "engine.h"
 
 #include <algorithm>
+#include <array>
 #include <atomic>
 #include <chrono>
 #include <cmath>
@@ -352,6 +353,12 @@ void Part::set_budget(uint64_t bytes, double frac) {
         CK(cudaMemcpyAsync(d_init_, init_chunks_.data(), hNS_ * 4, cudaMemcpyHostToDevice, cs_));
         hot_dirty_ = true;   // begin() installs the initial slots
     }
+    // what the Static Region holds: a kept region (ASCETIC_OPT_KEEP_STATIC) is only reused when the
+    // placement, its first vertex, its size and the slot layout are all unchanged
+    const std::array<uint64_t, 6> key = {(uint64_t)o_.placement, o_.placement == 2 ? o_.placement_seed : 0ull,
+                                         stat_lo_, p.s, hot_ ? p.Ms : 0ull, (uint64_t)hot_};
+    if (key != static_key_) static_valid_ = false;
+    static_key_ = key;
     CK(cudaStreamSynchronize(cs_));
 }
 
@@ -580,7 +587,7 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     is.s_static = T.nS;
     const DevState d = dev_state(t);
     const Queues q = queues(T);
-    if (algo_ == ALG_PR) CK(cudaMemsetAsync(d_sum_ + vlo_, 0, (vhi_ - vlo_) * sizeof(double), cs_));
+    if (algo_ == ALG_PR) CK(cudaMemsetAsync(d_sum_ + vlo_, 0, (vhi_ - vlo_) * sizeof(unsigned long long), cs_));
     // ---- Static Computing, overlapping the transfer, on its own stream so
     // the on-demand kernels (and through them the chunk buffers' reuse) never queue behind it;
     // finalize joins it. The static buffer holds host arcs [off[vlo], off[vlo+s]); kernels
@@ -944,6 +951,7 @@ void Part::end() {
     st.static_bytes = pl_.static_bytes;
     st.ondemand_bytes = pl_.C;
     st.chunk_cap = cap_;
+    st.chunk_buffers = (uint32_t)nbuf_;
     st.static_fraction_used = pl_.R;
     st.h2d_other_bytes = 0;
     st.time_run_s = ms / 1e3;
@@ -1010,8 +1018,11 @@ void Engine::load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_
     CK(cudaSetDevice(device_));
     CK(cudaDeviceGetAttribute(&sm_count_, cudaDevAttrMultiProcessorCount, device_));
     // same shape: keep every device allocation and stream (a reload is then offsets H2D and
-    // host bookkeeping only); otherwise start from scratch
-    const bool same_shape = state_ != 0 && n == g_.n && m == g_.m && b_e == g_.b_e;
+    // host bookkeeping only); otherwise start from scratch. The rank ranges are part of the shape:
+    // a part's owned range [vlo, vhi) and its range-sized queues are fixed at construction, so a
+    // graph with the same n and m but other edge-balanced bounds rebuilds the parts.
+    bool same_shape = state_ != 0 && n == g_.n && m == g_.m && b_e == g_.b_e;
+    if (same_shape && comm_.world() > 1) same_shape = partition(off, n, (uint32_t)comm_.world()) == bounds_;
     if (state_ != 0 && !same_shape) unload();
     if (same_shape) g_.release();
     have_result_ = false;
@@ -1342,14 +1353,15 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         }
         for (auto& p : parts_) p->finalize(t, multi && dense_fin);
         if (multi && algo == ALG_PR) {
-            // ---- exchange: SUM of the fp64 dangling partials, every rank's contrib slice to all
+            // ---- exchange: SUM of the fixed-point dangling partials (exact, so the total is the same
+            // for every P), every rank's contrib slice to all
             join();
             cudaEvent_t e0 = p0.mark(p0.cs());
-            std::vector<double*> dg;
+            std::vector<unsigned long long*> dg;
             std::vector<void*> cb;
             const int nxt = (int)((t + 1) & 1u);
             for (auto& p : parts_) { dg.push_back(p->dang() + nxt); cb.push_back(p->contrib()); }
-            comm_.sum_f64(dg, p0.cs());
+            comm_.sum_u64(dg, 1, p0.cs());
             comm_.share_slices(cb, bounds_, 4, p0.cs());
             p0.span(e0, p0.cs(), t, PH_XCH);
             fork();

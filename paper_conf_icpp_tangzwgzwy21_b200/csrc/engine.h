@@ -7,6 +7,7 @@
 //               (classify -> static + transfer + on-demand -> exchange -> finalize) and owns
 //               the Comm (NCCL across processes, or P ranks emulated on one GPU)
 #pragma once
+#include <array>
 #include <cstdint>
 #include <memory>
 #include <stdexcept>
@@ -128,7 +129,7 @@ class Part {
     float* rank_arr() const { return d_rank_; }
     float* contrib() const { return d_contrib_; }
     unsigned long long* prd_inc() const { return d_pr_inc_; }
-    double* dang() const { return d_dang_; }
+    unsigned long long* dang() const { return d_dang_; }
     uint64_t vertex_bytes() const { return vertex_bytes_; }
 
     // results of the last run
@@ -162,7 +163,7 @@ class Part {
     const void** d_peers_ = nullptr;           // [3][world] device pointers (next0, next1, val/inc)
     int peer_world_ = 0;
     uint64_t prd_tau_ = 0;
-    double *d_sum_ = nullptr, *d_dang_ = nullptr;
+    unsigned long long *d_sum_ = nullptr, *d_dang_ = nullptr;   // PR, 2^-62 fixed point
     uint32_t *d_hq_small_ = nullptr, *d_hq_med_ = nullptr, *d_hq_hub_ = nullptr, *d_hub_pre_ = nullptr;
     uint32_t *d_mq_ = nullptr, *d_run_b_ = nullptr, *d_run_e_ = nullptr, *d_tile_first_ = nullptr;
     unsigned long long *d_mq_pre_ = nullptr, *d_mq_src_ = nullptr, *d_run_dst_ = nullptr;
@@ -186,6 +187,7 @@ class Part {
     int nbuf_ = 2, nbuf_alloc_ = 0;   // chunk buffers in use / allocated
     uint64_t cap_ = 0, static_alloc_ = 0, chunk_alloc_ = 0;
     bool static_valid_ = false;
+    std::array<uint64_t, 6> static_key_{};   // placement, seed, first static vertex, s, slot bytes, slots on
     // streams / events
     cudaStream_t cs_ = nullptr, xs_ = nullptr, ss_ = nullptr;   // compute, copy, static-hit streams
     cudaEvent_t ready_[kMaxBuffers] = {}, consumed_[kMaxBuffers] = {};

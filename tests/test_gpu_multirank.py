@@ -119,6 +119,25 @@ def test_fused_exchange_matches_oracle(asc, P, algo):
         asc.set_option("chunk_cap", 0)
 
 
+def _bfs_sparse_prediction(g, levels, bounds, iters, d, P):
+    """(sparse iterations, pair bytes) of the BFS sparse exchange, from the oracle's levels."""
+    n = g.n
+    deg = np.diff(g.off.astype(np.int64))
+    src_of = np.repeat(np.arange(n, dtype=np.int64), deg)
+    dst = g.nbr.astype(np.int64)
+    lv = levels.astype(np.int64)
+    cap = max(1, n // (64 * d * P))
+    sparse, byt = 0, 0
+    for t in range(iters):
+        hit = (lv[src_of] == t) & (lv[dst] == t + 1)
+        counts = [np.unique(dst[hit & (src_of >= int(bounds[r])) & (src_of < int(bounds[r + 1]))]).size
+                  for r in range(P)]
+        if max(counts) <= cap:
+            sparse += 1
+            byt += 8 * sum(counts)
+    return sparse, byt
+
+
 @pytest.mark.parametrize("P", [2, 3, 5])
 @pytest.mark.parametrize("algo", ["bfs", "sssp", "cc"])
 @pytest.mark.parametrize("d", [1, 8, 2000])
@@ -146,9 +165,16 @@ def test_sparse_exchange_matches_oracle(asc, P, algo, d):
                              bounds=bounds)
             np.testing.assert_array_equal(res, ref.values)
             assert [{f: i[f] for f in REC} for i in its] == [{f: r[f] for f in REC} for r in ref.records]
-            if d == 1 or (d == 8 and algo != "bfs"):
-                assert st["sparse_exchanges"] >= 1                # (the last BFS level may be 0 pairs)
-                assert algo == "bfs" or st["sparse_exchange_bytes"] > 0
+            if algo == "bfs":
+                # exact: rank r's pairs at level t are the ids it newly reached, i.e. the level-(t+1)
+                # vertices adjacent to its owned level-t vertices; the level goes sparse iff every
+                # rank has at most max(1, n / (64 d P)) of them, and moves 8 bytes per pair
+                cnt, byt = _bfs_sparse_prediction(g, ref.values, bounds, st["iterations"], d, P)
+                assert st["sparse_exchanges"] == cnt and st["sparse_exchange_bytes"] == byt
+                if d == 1:
+                    assert byt > 0
+            elif d == 1 or d == 8:
+                assert st["sparse_exchanges"] >= 1 and st["sparse_exchange_bytes"] > 0
             else:
                 assert st["sparse_exchanges"] < st["iterations"]
         asc.set_option("sparse_exchange", 0)         # back to dense on the same parts

@@ -219,7 +219,7 @@ def test_load_variants_copy_wgt_validate(asc):
 
 
 @pytest.mark.parametrize("opt,val", [("overlap", 0), ("keep_static", 1), ("chunk_buffers", 2),
-                                     ("chunk_buffers", 8), ("gather_ctas", 1), ("static_ctas_per_sm", 1),
+                                     ("chunk_buffers", 3), ("chunk_buffers", 8), ("gather_ctas", 1), ("static_ctas_per_sm", 1),
                                      ("timing", 0)])
 def test_options_do_not_change_results(asc, opt, val):
     """Tuning knobs change scheduling only: results, records and bytes stay bit-exact."""
@@ -364,3 +364,45 @@ def test_gather_unaligned_host_arrays(asc, algo, shift):
             _pr_ok(res, ref.values)
         else:
             np.testing.assert_array_equal(res, ref.values)
+
+
+@pytest.mark.parametrize("mib,nb", [(11, 2), (13, 3)])
+def test_auto_chunk_buffers(asc, mib, nb):
+    """Auto chunk buffers (option 0): 3 buffers of C/3, or 2 when C/3 < 4 MiB; results unchanged."""
+    g = gg.config_graph("c1")
+    budget = mib << 20
+    asc.load_csr(g.off, g.nbr)
+    asc.set_option("chunk_buffers", 0)
+    asc.set_budget(budget, 0.0)                            # R = 0: C = B
+    src = gg.sources(g, 1, seed=1)[0]
+    asc.run("bfs", src)
+    st, its = asc.stats()
+    assert st["chunk_buffers"] == nb
+    assert st["chunk_cap"] == min(budget // nb, 4 * g.m) // 16 * 16
+    ref = _oracle("bfs", g, src, 0)
+    np.testing.assert_array_equal(asc.get_result(), ref.values)
+    _check_records(its, ref)
+
+
+def test_pr_bitwise_reproducible(asc):
+    """PR sums are combined in 2^-62 fixed point (integer atomics), so two runs with the same
+    options give bitwise-identical fp32 ranks, whatever order the hub-piece and chunk-segment
+    partials land in (DESIGN R31); still within the tolerance of the fp64 oracle."""
+    g = gg.rmat(14, seed=31)
+    asc.load_csr(g.off, g.nbr)
+    asc.set_option("hub_degree", 64)                       # many multi-CTA hub rows
+    asc.set_option("chunk_cap", 3000)                      # rows split across chunks and segments
+    asc.set_option("xfer_mode", 1)
+    asc.set_budget(g.csr_bytes // 3, 0.4)
+    runs = []
+    for _ in range(3):
+        asc.run("pr", 0, 12)
+        runs.append(asc.get_result().copy())
+    asc.set_option("hub_degree", 2048)
+    asc.set_option("chunk_cap", 0)
+    asc.set_option("xfer_mode", 0)
+    assert all(np.array_equal(r.view(np.uint32), runs[0].view(np.uint32)) for r in runs[1:])
+    p = oracle.placer(g.off, 4, g.csr_bytes // 3, 0.4)
+    ref = _oracle("pr", g, 0, p.s, max_iters=12)
+    _pr_ok(runs[0], ref.values)
+    assert abs(runs[0].astype(np.float64).sum() - 1.0) <= 1e-5
