@@ -127,6 +127,58 @@ def _config(args, c, g) -> dict:
             if c["algo"] in ("bfs", "sssp") else None}
 
 
+def shared_graph(config: str, barrier, local_rank: int, tag: str, alloc_local=None):
+    """N > 1 on one node: local rank 0 generates the CSR ONCE into shared files (/dev/shm when it has
+    room, else ASCETIC_SHM_DIR or /tmp), every rank maps them MAP_SHARED, so host RAM holds one copy
+    whatever N is; each rank's library then pins only the arcs of its own rows.
+    Returns (graph, cleanup, generation seconds)."""
+    import graphgen as gg
+    c = gg.CONFIGS[config]
+    est = 8 * ((1 << c["scale"]) + 1) + (8 if c["algo"] == "sssp" else 4) * 2 * c["tuples"]
+    d = "/dev/shm"
+    try:
+        st = os.statvfs(d)
+        if st.f_bavail * st.f_frsize < est * 1.05:
+            d = os.environ.get("ASCETIC_SHM_DIR", "/tmp")
+    except OSError:
+        d = os.environ.get("ASCETIC_SHM_DIR", "/tmp")
+    base = os.path.join(d, f"ascetic_{config}_{tag}")
+    gen_s = 0.0
+    if local_rank == 0:
+        files = []
+
+        def alloc(count, dtype):
+            path = f"{base}.{len(files)}"
+            files.append(path)
+            return np.memmap(path, dtype=dtype, mode="w+", shape=(max(1, count),))
+
+        t0 = time.time()
+        g = gg.config_graph(config, alloc=alloc)
+        gen_s = time.time() - t0
+        for a in (g.off, g.nbr):
+            if isinstance(a.base, np.memmap):
+                a.base.flush()
+        json.dump({"n": g.n, "m": g.m, "pairs": g.pairs, "files": files}, open(base + ".json.tmp", "w"))
+        os.replace(base + ".json.tmp", base + ".json")
+    barrier()
+    meta = json.load(open(base + ".json"))
+    n, m, pairs = meta["n"], meta["m"], meta["pairs"]
+    off = np.memmap(meta["files"][0], dtype=np.uint64, mode="r")[: n + 1]
+    cnt = (2 if pairs else 1) * m
+    nbr = np.memmap(meta["files"][1], dtype=np.uint32, mode="r")[:cnt]
+    g = gg.Graph(n=n, m=m, off=off, nbr=nbr, pairs=pairs, name=config)
+
+    def cleanup():
+        barrier()
+        if local_rank == 0:
+            for f in meta["files"] + [base + ".json"]:
+                try:
+                    os.unlink(f)
+                except OSError:
+                    pass
+    return g, cleanup, gen_s
+
+
 def run_reference(args, ws, rank):
     """--impl reference: the oracle as it stands, on the host cores, same config/metric/unit."""
     if rank != 0:
@@ -213,9 +265,13 @@ def main():
         pinned.append(t)
         return t.numpy().view(dtype)
 
-    t0 = time.time()
-    g = gg.config_graph(args.config, alloc=alloc)
-    gen_s = time.time() - t0
+    cleanup = None
+    if ws > 1:
+        g, cleanup, gen_s = shared_graph(args.config, dist.barrier, local, os.environ.get("MASTER_PORT", "0"))
+    else:
+        t0 = time.time()
+        g = gg.config_graph(args.config, alloc=alloc)
+        gen_s = time.time() - t0
     srcs = gg.sources(g, 8, seed=c["seed"])
     if ws > 1:
         # 1D edge-balanced ranges, one per GPU; NCCL exchange inside the library.
@@ -465,6 +521,8 @@ def main():
     if rank == 0:
         print(json.dumps(out), flush=True)
     asc.unload()
+    if cleanup is not None:
+        cleanup()
     if ws > 1:
         dist.destroy_process_group()
     return 0

@@ -104,7 +104,7 @@ typedef enum {
                                       increments straight from peer memory (CUDA IPC over NVLink with the NCCL
                                       back end; the other parts' buffers when emulated), between stream-ordered
                                       barriers; 0 (default) = NCCL collectives. Results are identical. */
-    ASCETIC_OPT_SPARSE_EXCHANGE = 19 /* P > 1, BFS/SSSP/CC, collectives path: d >= 1 = sparse exchange (SURVEY
+    ASCETIC_OPT_SPARSE_EXCHANGE = 19,/* P > 1, BFS/SSSP/CC, collectives path: d >= 1 = sparse exchange (SURVEY
                                       §8(e)): each rank packs the (id, value) pairs it set in its next bitmap this
                                       iteration (lowered values; BFS: newly reached ids), the pairs are
                                       all-gathered and applied with atomicMin + next bit, whenever every rank has
@@ -112,6 +112,11 @@ typedef enum {
                                       bitmap bit), else the dense ncclAllReduce(min) / bitmap OR; one 4P-byte host
                                       read per iteration decides. 0 (default) = dense always. 8 keeps the
                                       all-gather under the all-reduce's bytes. Results are identical. */
+    ASCETIC_OPT_RELAX_MODE = 20      /* SSSP/CC min updates: 1 = atomicMin, and the thread whose atomic lowered the
+                                      value sets the vertex's next-frontier bit; 2 = fire-and-forget RED.MIN, and
+                                      the finalize derives A_{t+1} = {v : val < snap} in one dense pass (Jacobi:
+                                      the same set); 0 = auto (default). The sparse exchange forces 1. Results are
+                                      identical. */
 } ascetic_option;
 
 typedef struct {

@@ -37,7 +37,7 @@ OPTIONS = {"chunk_cap": 1, "xfer_mode": 2, "dma_min_run": 3, "overlap": 4, "keep
            "hub_degree": 6, "timing": 7, "gather_ctas": 8, "chunk_buffers": 9, "static_ctas_per_sm": 10,
            "prefetch": 11, "repartition": 12, "static_placement": 13, "replace_chunks": 14,
            "replace_policy": 15, "placement_seed": 16, "prd_tol_ppm": 17,
-           "fused_exchange": 18, "sparse_exchange": 19}
+           "fused_exchange": 18, "sparse_exchange": 19, "relax_mode": 20}
 INF = 0xFFFFFFFF
 
 

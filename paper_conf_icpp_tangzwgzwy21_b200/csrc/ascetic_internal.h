@@ -104,6 +104,7 @@ struct DevState {
     unsigned long long *pr_r, *pr_res, *pr_c;
     unsigned long long* pr_inc;        // P > 1: this rank's increments (summed across ranks), else nullptr
     unsigned long long tau;
+    uint32_t red_min;                  // SSSP/CC: fire-and-forget RED.MIN + dense finalize (no next bits)
 };
 
 constexpr uint32_t kNoSlot = 0xFFFFFFFFu;

@@ -4,6 +4,7 @@
 #include <dlfcn.h>
 #include <nccl.h>   // types and enums only; every function is resolved with dlsym
 
+#include <algorithm>
 #include <cstring>
 
 #include "ascetic_internal.h"
@@ -21,6 +22,8 @@ struct NcclApi {
     ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t, cudaStream_t) = nullptr;
     ncclResult_t (*AllGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
     ncclResult_t (*Broadcast)(const void*, void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*Send)(const void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*Recv)(void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
     ncclResult_t (*GroupStart)() = nullptr;
     ncclResult_t (*GroupEnd)() = nullptr;
     const char* (*GetErrorString)(ncclResult_t) = nullptr;
@@ -44,6 +47,8 @@ NcclApi& nccl() {
     api.AllReduce = (decltype(api.AllReduce))sym("ncclAllReduce");
     api.AllGather = (decltype(api.AllGather))sym("ncclAllGather");
     api.Broadcast = (decltype(api.Broadcast))sym("ncclBroadcast");
+    api.Send = (decltype(api.Send))sym("ncclSend");
+    api.Recv = (decltype(api.Recv))sym("ncclRecv");
     api.GroupStart = (decltype(api.GroupStart))sym("ncclGroupStart");
     api.GroupEnd = (decltype(api.GroupEnd))sym("ncclGroupEnd");
     api.GetErrorString = (decltype(api.GetErrorString))sym("ncclGetErrorString");
@@ -108,14 +113,33 @@ void Comm::or_words(const std::vector<uint32_t*>& local, uint64_t nw, cudaStream
             CKc(cudaMemcpyAsync(local[p], local[0], nw * 4, cudaMemcpyDeviceToDevice, s), "or copy-back");
         return;
     }
-    const uint64_t need = nw * (uint64_t)world_;
+    // NCCL has no bitwise OR: reduce-scatter-OR by point-to-point slices, then all-gather the ORed
+    // slices. Rank r owns words [r*S, min((r+1)*S, nw)), S = ceil(nw/P); every rank sends each peer
+    // that peer's slice and ORs the P copies of its own: 2 (P-1)/P * nw words on the wire per rank
+    // (an all-gather of whole bitmaps + local OR would move (P-1) * nw).
+    const uint64_t P = (uint64_t)world_, me = (uint64_t)rank_;
+    const uint64_t S = (nw + P - 1) / P;
+    auto len = [&](uint64_t r) -> uint64_t { return r * S >= nw ? 0 : std::min(S, nw - r * S); };
+    const uint64_t need = 2 * P * S;
     if (scratch_words_ < need) {
         if (scratch_) cudaFree(scratch_);
         CKc(cudaMalloc(&scratch_, need * 4), "exchange scratch");
         scratch_words_ = need;
     }
-    NC(nccl().AllGather(local[0], scratch_, nw, ncclUint32, (ncclComm_t)nccl_comm_, s), "ncclAllGather(bitmap)");
-    launch_or_reduce(local[0], scratch_, (uint32_t)world_, nw, s);
+    uint32_t* recv = scratch_;           // [P][len(me)]: every rank's copy of my slice
+    uint32_t* gath = scratch_ + P * S;   // [P][S]: the ORed slices, gathered in place
+    const uint64_t lm = len(me);
+    if (lm) CKc(cudaMemcpyAsync(recv + me * lm, local[0] + me * S, lm * 4, cudaMemcpyDeviceToDevice, s), "own slice");
+    NC(nccl().GroupStart(), "ncclGroupStart");
+    for (uint64_t r = 0; r < P; ++r) {
+        if (r == me) continue;
+        if (len(r)) NC(nccl().Send(local[0] + r * S, len(r), ncclUint32, (int)r, (ncclComm_t)nccl_comm_, s), "ncclSend(slice)");
+        if (lm) NC(nccl().Recv(recv + r * lm, lm, ncclUint32, (int)r, (ncclComm_t)nccl_comm_, s), "ncclRecv(slice)");
+    }
+    NC(nccl().GroupEnd(), "ncclGroupEnd");
+    if (lm) launch_or_reduce(gath + me * S, recv, (uint32_t)P, lm, s);
+    NC(nccl().AllGather(gath + me * S, gath, S, ncclUint32, (ncclComm_t)nccl_comm_, s), "ncclAllGather(ORed slices)");
+    CKc(cudaMemcpyAsync(local[0], gath, nw * 4, cudaMemcpyDeviceToDevice, s), "bitmap copy-back");
 }
 
 void Comm::min_u32(const std::vector<uint32_t*>& local, uint64_t n, cudaStream_t s) {

@@ -1,6 +1,7 @@
 // comm.h — the per-iteration exchange of the multi-GPU path (the paper itself
 // is single-GPU). One process per GPU, 1D vertex ranges, replicated vertex state:
-//   BFS       : OR of the next-frontier bitmaps        (NCCL has no bitwise OR: all-gather + OR kernel)
+//   BFS       : OR of the next-frontier bitmaps        (NCCL has no bitwise OR: reduce-scatter-OR over
+//               point-to-point slices + OR kernel, then all-gather of the ORed slices)
 //   SSSP / CC : MIN of the value arrays               (ncclAllReduce min)
 //   PR        : SUM of the 2^-62 fixed-point dangling partials (exact) + every rank's contrib slice to all ranks
 //   PRD       : SUM of the u64 residual increments   (ncclAllReduce sum, exact: integers)

@@ -129,10 +129,22 @@ __device__ __forceinline__ void bfs_visit(const DevState& d, uint32_t v) {
     atomicOr(d.next + wi, bit);
 }
 
+// SSSP / CC relax. Two forms with the same A_{t+1} (Jacobi: the set of vertices whose value ends
+// the iteration below its snapshot): d.red_min = 0 waits for atomicMin's old value and sets the
+// next bit when it lowered it; d.red_min = 1 issues a fire-and-forget RED.MIN and the dense
+// finalize derives A_{t+1} = {v : val < snap} (no dependent atomic chain per improving arc).
+__device__ __forceinline__ void min_update(const DevState& d, uint32_t v, uint32_t cand) {
+    if (d.red_min) {
+        atomicMin(d.val + v, cand);                      // result unused: compiles to RED.E.MIN
+    } else {
+        const uint32_t old = atomicMin(d.val + v, cand);
+        if (cand < old) set_next(d, v);
+    }
+}
+
 __device__ __forceinline__ void relax(const DevState& d, uint32_t v, uint32_t cand) {
     if (cand >= ld_state(d.val + v)) return;            // values only decrease within an iteration
-    const uint32_t old = atomicMin(d.val + v, cand);
-    if (cand < old) set_next(d, v);
+    min_update(d, v, cand);
 }
 
 __device__ __forceinline__ uint32_t sat_add(uint32_t a, uint32_t w) {
@@ -201,10 +213,7 @@ __device__ __forceinline__ void push_batch(const DevState& d, const SrcVal<ALGO>
         }
 #pragma unroll
         for (int j = 0; j < N; ++j) {
-            if (cand[j] < cur[j]) {
-                const uint32_t old = atomicMin(d.val + id[j], cand[j]);
-                if (cand[j] < old) set_next(d, id[j]);
-            }
+            if (cand[j] < cur[j]) min_update(d, id[j], cand[j]);
         }
     }
 }
@@ -593,10 +602,7 @@ __device__ __forceinline__ void ondemand_tile(const DevState& d, const Queues& q
         for (int g = 0; g < 8; ++g) cur[g] = id[g] != kInf ? ld_state(d.val + id[g]) : 0u;
 #pragma unroll
         for (int g = 0; g < 8; ++g) {
-            if (id[g] != kInf && cand[g] < cur[g]) {
-                const uint32_t old = atomicMin(d.val + id[g], cand[g]);
-                if (cand[g] < old) set_next(d, id[g]);
-            }
+            if (id[g] != kInf && cand[g] < cur[g]) min_update(d, id[g], cand[g]);
         }
     } else {
         // PR pull: partial row sums of the chunk's arcs. Same 3 phases: map + chunk loads,
@@ -871,31 +877,38 @@ __global__ void k_finalize_prd(DevState d) {
     }
 }
 
+// Dense finalize kernels (after an exchange, or reading peers): one thread per vertex, one warp per
+// 32-vertex bitmap word built with a ballot, so every warp load instruction reads 128 contiguous bytes
+// of each value array (one line, also when the array is a peer's over NVLink) and lane 0 writes the word.
+#define FOR_EACH_WORD_WARP(d, w, v, lane)                                                                     \
+    const int lane = threadIdx.x & 31;                                                                        \
+    for (uint64_t w = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < (d).nwords;                \
+         w += ((uint64_t)gridDim.x * blockDim.x) >> 5)                                                       \
+        if (const uint64_t v = w * 32 + (uint64_t)lane; true)
+
 // PRD finalize after the cross-rank SUM of the increments (P > 1): res += inc over all vertices,
 // A_{t+1} = {v : res > tau}, the active absorb; identical on every rank (replicated state)
-__global__ void k_finalize_prd_dense(DevState d) {
-    for (uint32_t w = blockIdx.x * blockDim.x + threadIdx.x; w < d.nwords; w += gridDim.x * blockDim.x) {
-        uint32_t bits = 0;
-        const uint64_t v0 = (uint64_t)w * 32;
-        const uint32_t cnt = (uint32_t)min((uint64_t)32, d.n - v0);
-        for (uint32_t i = 0; i < cnt; ++i) {
-            const uint64_t v = v0 + i;
+__global__ void __launch_bounds__(256) k_finalize_prd_dense(DevState d) {
+    FOR_EACH_WORD_WARP(d, w, v, lane) {
+        bool act = false;
+        if (v < d.n) {
             const unsigned long long inc = d.pr_inc[v];
-            if (!inc) continue;                      // res <= tau already (not active, unchanged)
-            d.pr_inc[v] = 0ull;
-            const unsigned long long x = d.pr_res[v] + inc;
-            if (x > d.tau) {
-                const unsigned long long deg = d.off[v + 1] - d.off[v];
-                bits |= 1u << i;
-                d.pr_r[v] += x;
-                d.pr_c[v] = deg ? (17ull * x) / (20ull * deg) : 0ull;
-                d.pr_res[v] = 0ull;
-            } else {
-                d.pr_res[v] = x;
+            if (inc) {                                   // inc = 0: res <= tau already (not active, unchanged)
+                d.pr_inc[v] = 0ull;
+                const unsigned long long x = d.pr_res[v] + inc;
+                if (x > d.tau) {
+                    const unsigned long long deg = d.off[v + 1] - d.off[v];
+                    act = true;
+                    d.pr_r[v] += x;
+                    d.pr_c[v] = deg ? (17ull * x) / (20ull * deg) : 0ull;
+                    d.pr_res[v] = 0ull;
+                } else {
+                    d.pr_res[v] = x;
+                }
             }
         }
-        d.A[w] = bits;
-        d.next[w] = 0;
+        const uint32_t bits = __ballot_sync(FULL, act);
+        if (lane == 0) { d.A[w] = bits; d.next[w] = 0; }
     }
 }
 
@@ -928,47 +941,44 @@ __global__ void k_finalize_bfs_peers(DevState d, const uint32_t* const* __restri
 
 // SSSP / CC: val = MIN_p val_p, A = {v : val < snap}, snap = val (a peer may be writing its own
 // val with the same minimum concurrently: every value read is >= the minimum, so MIN is exact)
-__global__ void k_finalize_min_peers(DevState d, const uint32_t* const* __restrict__ peers, int P) {
-    for (uint32_t w = blockIdx.x * blockDim.x + threadIdx.x; w < d.nwords; w += gridDim.x * blockDim.x) {
-        uint32_t bits = 0;
-        const uint64_t v0 = (uint64_t)w * 32;
-        const uint32_t cnt = (uint32_t)min((uint64_t)32, d.n - v0);
-        for (uint32_t i = 0; i < cnt; ++i) {
+__global__ void __launch_bounds__(256) k_finalize_min_peers(DevState d, const uint32_t* const* __restrict__ peers, int P) {
+    FOR_EACH_WORD_WARP(d, w, v, lane) {
+        bool act = false;
+        if (v < d.n) {
             uint32_t x = kInf;
-            for (int p = 0; p < P; ++p) x = min(x, ld_peer(peers[p] + v0 + i));
-            const uint32_t y = d.snap[v0 + i];
-            if (x < y) { bits |= 1u << i; d.snap[v0 + i] = x; }
-            if (x != d.val[v0 + i]) d.val[v0 + i] = x;
+            for (int p = 0; p < P; ++p) x = min(x, ld_peer(peers[p] + v));
+            const uint32_t y = d.snap[v];
+            if (x < y) { act = true; d.snap[v] = x; }
+            if (x != d.val[v]) d.val[v] = x;
         }
-        d.A[w] = bits;
-        d.next[w] = 0;
+        const uint32_t bits = __ballot_sync(FULL, act);
+        if (lane == 0) { d.A[w] = bits; d.next[w] = 0; }
     }
 }
 
 // PRD: res += SUM_p inc_p (integers: exact in any order), A = {res > tau}, absorb
-__global__ void k_finalize_prd_peers(DevState d, const unsigned long long* const* __restrict__ peers, int P) {
-    for (uint32_t w = blockIdx.x * blockDim.x + threadIdx.x; w < d.nwords; w += gridDim.x * blockDim.x) {
-        uint32_t bits = 0;
-        const uint64_t v0 = (uint64_t)w * 32;
-        const uint32_t cnt = (uint32_t)min((uint64_t)32, d.n - v0);
-        for (uint32_t i = 0; i < cnt; ++i) {
-            const uint64_t v = v0 + i;
+__global__ void __launch_bounds__(256) k_finalize_prd_peers(DevState d, const unsigned long long* const* __restrict__ peers,
+                                                            int P) {
+    FOR_EACH_WORD_WARP(d, w, v, lane) {
+        bool act = false;
+        if (v < d.n) {
             unsigned long long inc = 0;
             for (int p = 0; p < P; ++p) inc += ld_peer(peers[p] + v);
-            if (!inc) continue;
-            const unsigned long long x = d.pr_res[v] + inc;
-            if (x > d.tau) {
-                const unsigned long long deg = d.off[v + 1] - d.off[v];
-                bits |= 1u << i;
-                d.pr_r[v] += x;
-                d.pr_c[v] = deg ? (17ull * x) / (20ull * deg) : 0ull;
-                d.pr_res[v] = 0ull;
-            } else {
-                d.pr_res[v] = x;
+            if (inc) {
+                const unsigned long long x = d.pr_res[v] + inc;
+                if (x > d.tau) {
+                    const unsigned long long deg = d.off[v + 1] - d.off[v];
+                    act = true;
+                    d.pr_r[v] += x;
+                    d.pr_c[v] = deg ? (17ull * x) / (20ull * deg) : 0ull;
+                    d.pr_res[v] = 0ull;
+                } else {
+                    d.pr_res[v] = x;
+                }
             }
         }
-        d.A[w] = bits;
-        d.next[w] = 0;
+        const uint32_t bits = __ballot_sync(FULL, act);
+        if (lane == 0) { d.A[w] = bits; d.next[w] = 0; }
     }
 }
 
@@ -1038,17 +1048,15 @@ __global__ void k_finalize_pr(DevState d, int cur) {
 }
 
 // P > 1: values were MIN-exchanged, so A_{t+1} = {v : val[v] < snap[v]} over every vertex
-__global__ void k_finalize_minlabel_dense(DevState d) {
-    for (uint32_t w = blockIdx.x * blockDim.x + threadIdx.x; w < d.nwords; w += gridDim.x * blockDim.x) {
-        uint32_t bits = 0;
-        const uint64_t v0 = (uint64_t)w * 32;
-        const uint32_t cnt = (uint32_t)min((uint64_t)32, d.n - v0);
-        for (uint32_t i = 0; i < cnt; ++i) {
-            const uint32_t x = d.val[v0 + i], y = d.snap[v0 + i];
-            if (x < y) { bits |= 1u << i; d.snap[v0 + i] = x; }
+__global__ void __launch_bounds__(256) k_finalize_minlabel_dense(DevState d) {
+    FOR_EACH_WORD_WARP(d, w, v, lane) {
+        bool act = false;
+        if (v < d.n) {
+            const uint32_t x = d.val[v], y = d.snap[v];
+            if (x < y) { act = true; d.snap[v] = x; }
         }
-        d.A[w] = bits;
-        d.next[w] = 0;
+        const uint32_t bits = __ballot_sync(FULL, act);
+        if (lane == 0) { d.A[w] = bits; d.next[w] = 0; }
     }
 }
 
@@ -1422,12 +1430,12 @@ void launch_finalize(int algo, const DevState& d, bool dense, cudaStream_t s) {
     switch (algo) {
         case BFS: k_finalize_bfs<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d); break;
         case PRD:
-            if (dense) k_finalize_prd_dense<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d);
+            if (dense) k_finalize_prd_dense<<<blocks_for(d.nwords, 8), 256, 0, s>>>(d);
             else k_finalize_prd<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d);
             break;
         case SSSP:
         case CC:
-            if (dense) k_finalize_minlabel_dense<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d);
+            if (dense) k_finalize_minlabel_dense<<<blocks_for(d.nwords, 8), 256, 0, s>>>(d);
             else k_finalize_minlabel<<<blocks_for(d.nwords, 256), 256, 0, s>>>(d);
             break;
         default: {
@@ -1475,13 +1483,13 @@ void launch_min_into(uint32_t* dst, const uint32_t* src, uint64_t n, cudaStream_
 }
 
 void launch_finalize_peers(int algo, const DevState& d, const void* const* peers, int P, cudaStream_t s) {
-    const unsigned g = blocks_for(d.nwords, 256);
+    const unsigned g = blocks_for(d.nwords, 256), gw = blocks_for(d.nwords, 8);
     switch (algo) {
         case BFS: k_finalize_bfs_peers<<<g, 256, 0, s>>>(d, reinterpret_cast<const uint32_t* const*>(peers), P); break;
         case SSSP:
-        case CC: k_finalize_min_peers<<<g, 256, 0, s>>>(d, reinterpret_cast<const uint32_t* const*>(peers), P); break;
+        case CC: k_finalize_min_peers<<<gw, 256, 0, s>>>(d, reinterpret_cast<const uint32_t* const*>(peers), P); break;
         case PRD:
-            k_finalize_prd_peers<<<g, 256, 0, s>>>(d, reinterpret_cast<const unsigned long long* const*>(peers), P);
+            k_finalize_prd_peers<<<gw, 256, 0, s>>>(d, reinterpret_cast<const unsigned long long* const*>(peers), P);
             break;
         default: return;
     }

@@ -108,7 +108,7 @@ static void dfree(T*& p) {
 }
 
 void HostGraph::release() {
-    if (registered) { cudaHostUnregister(registered); registered = nullptr; }
+    if (registered) { cudaHostUnregister(registered); registered = nullptr; reg_bytes = 0; }
     if (owned) { cudaFreeHost(owned); owned = nullptr; }
     nbr = nbr_dev = nullptr;
 }
@@ -411,6 +411,7 @@ DevState Part::dev_state(uint32_t iter) const {
     d.pr_r = d_pr_r_; d.pr_res = d_pr_res_; d.pr_c = d_pr_c_;
     d.pr_inc = multi_ ? d_pr_inc_ : nullptr;
     d.tau = prd_tau_;
+    d.red_min = red_min_ ? 1u : 0u;
     return d;
 }
 
@@ -873,7 +874,7 @@ void Part::finalize(uint32_t t, bool dense) {
     // ---- next active set, after the static-hit kernels
     join_static();
     cudaEvent_t e0 = mark(cs_);
-    launch_finalize(algo_, dev_state(t), dense, cs_);
+    launch_finalize(algo_, dev_state(t), dense || red_min_, cs_);
     CK(cudaGetLastError());
     span(e0, cs_, t, PH_FIN);
 }
@@ -1024,7 +1025,7 @@ void Engine::load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_
     bool same_shape = state_ != 0 && n == g_.n && m == g_.m && b_e == g_.b_e;
     if (same_shape && comm_.world() > 1) same_shape = partition(off, n, (uint32_t)comm_.world()) == bounds_;
     if (state_ != 0 && !same_shape) unload();
-    if (same_shape) g_.release();
+    if (g_.owned) { cudaFreeHost(g_.owned); g_.owned = nullptr; }   // a registration may be kept (below)
     have_result_ = false;
     g_.n = n; g_.m = m; g_.b_e = b_e; g_.flags = flags;
     // offsets: used in place by the host planner (placer, partition, DMA planning) and DMA'd to
@@ -1036,51 +1037,83 @@ void Engine::load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_
         g_.off_own.clear();
         g_.off = off;
     }
-    // ---- pin the edge array (the On-demand Engine's Edgelist)
+    // ---- rank ranges first: with one process per GPU a rank only ever reads the arcs of its own rows
+    const int world = comm_.world();
+    std::vector<uint64_t> nb = partition(off, n, (uint32_t)world);
+    uint64_t a0 = 0, a1 = m;                         // arcs this process may read from the host
+    if (!comm_.emulated() && world > 1) {
+        a0 = std::min<uint64_t>(off[nb[comm_.rank()]], m);
+        a1 = std::max<uint64_t>(a0, std::min<uint64_t>(off[nb[comm_.rank() + 1]], m));
+    }
+    // ---- pin the edge array (the On-demand Engine's Edgelist): this process's arc range
+    // only (ranks share one host CSR, each pins its owned rows). Host arc x is always
+    // addressed as nbr + b_e x; for a private copy of a slice `nbr` is the copy's virtual base.
     const size_t bytes = (size_t)b_e * m;
     if (bytes > 0) {
         const bool need_copy = (flags & ASCETIC_COPY) || wgt;
         if (need_copy) {
-            cudaError_t e = cudaHostAlloc(&g_.owned, bytes, cudaHostAllocPortable | cudaHostAllocMapped);
+            if (g_.registered) { cudaHostUnregister(g_.registered); g_.registered = nullptr; g_.reg_bytes = 0; }
+            // bytes [f0, f1) of the b_e layout, 16-byte aligned so the gather's cover units stay inside
+            const uint64_t f0 = (uint64_t)b_e * a0 / 16 * 16;
+            const uint64_t f1 = std::min<uint64_t>(((uint64_t)b_e * a1 + 15) / 16 * 16, bytes);
+            cudaError_t e = cudaHostAlloc(&g_.owned, std::max<uint64_t>(f1 - f0, 16), cudaHostAllocPortable | cudaHostAllocMapped);
             if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_EHOSTMEM, "cudaHostAlloc failed"); }
             if (wgt) {
                 uint32_t* dst = (uint32_t*)g_.owned;
+                const uint64_t e0 = f0 / 8, e1 = f1 / 8;   // interleaved (id, w): 8 bytes per arc
                 const unsigned nt = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
                 std::vector<std::thread> th;
                 for (unsigned t = 0; t < nt; ++t)
                     th.emplace_back([=] {
-                        for (uint64_t e2 = t; e2 < m; e2 += nt) { dst[2 * e2] = nbr[e2]; dst[2 * e2 + 1] = wgt[e2]; }
+                        for (uint64_t e2 = e0 + t; e2 < e1; e2 += nt) {
+                            dst[2 * (e2 - e0)] = nbr[e2];
+                            dst[2 * (e2 - e0) + 1] = wgt[e2];
+                        }
                     });
                 for (auto& x : th) x.join();
             } else {
-                std::memcpy(g_.owned, nbr, bytes);
+                std::memcpy(g_.owned, (const char*)nbr + f0, f1 - f0);
             }
-            g_.nbr = g_.owned;
+            g_.nbr = (const char*)g_.owned - f0;
+            void* dp = nullptr;
+            CK(cudaHostGetDevicePointer(&dp, g_.owned, 0));
+            g_.nbr_dev = (const char*)dp - f0;
         } else {
+            // whole pages covering this process's arcs, clipped to the caller's array
+            const uintptr_t base = (uintptr_t)nbr, pg = 4096;
+            const uintptr_t lo = std::max<uintptr_t>(base, (base + (uintptr_t)b_e * a0) / pg * pg);
+            const uintptr_t hi = std::min<uintptr_t>(base + bytes, (base + (uintptr_t)b_e * a1 + pg - 1) / pg * pg);
+            const size_t rb = std::max<size_t>(hi > lo ? hi - lo : 0, 1);
+            const bool keep = g_.registered == (void*)lo && g_.reg_bytes == rb;   // same range as before
+            if (g_.registered && !keep) { cudaHostUnregister(g_.registered); g_.registered = nullptr; g_.reg_bytes = 0; }
             cudaPointerAttributes attr{};
-            cudaError_t e = cudaPointerGetAttributes(&attr, nbr);
+            cudaError_t e = keep ? cudaSuccess : cudaPointerGetAttributes(&attr, (const void*)lo);
             if (e != cudaSuccess) cudaGetLastError();
-            if (e == cudaSuccess && attr.type == cudaMemoryTypeHost) {
-                g_.nbr = nbr;                       // already page-locked (cudaHostAlloc / pin_memory)
-            } else {
-                e = cudaHostRegister((void*)nbr, bytes,
-                                     cudaHostRegisterPortable | cudaHostRegisterMapped | cudaHostRegisterReadOnly);
+            uintptr_t dbase = lo;                 // host address whose device alias is looked up
+            if (!keep && e == cudaSuccess && attr.type == cudaMemoryTypeHost) {
+                dbase = base;                     // already page-locked by the caller (cudaHostAlloc / pin_memory)
+            } else if (!keep) {
+                e = cudaHostRegister((void*)lo, rb, cudaHostRegisterPortable | cudaHostRegisterMapped | cudaHostRegisterReadOnly);
                 if (e != cudaSuccess) {
                     cudaGetLastError();
-                    e = cudaHostRegister((void*)nbr, bytes, cudaHostRegisterPortable | cudaHostRegisterMapped);
+                    e = cudaHostRegister((void*)lo, rb, cudaHostRegisterPortable | cudaHostRegisterMapped);
                 }
                 if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_EHOSTMEM, std::string("cudaHostRegister: ") + cudaGetErrorString(e)); }
-                g_.registered = (void*)nbr;
-                g_.nbr = nbr;
+                g_.registered = (void*)lo;
+                g_.reg_bytes = rb;
             }
+            g_.nbr = nbr;
+            void* dp = nullptr;
+            CK(cudaHostGetDevicePointer(&dp, (void*)dbase, 0));
+            g_.nbr_dev = (const char*)dp - (dbase - base);
         }
-        void* dp = nullptr;
-        CK(cudaHostGetDevicePointer(&dp, (void*)g_.nbr, 0));
-        g_.nbr_dev = dp;
+    } else {
+        g_.release();
     }
+    g_.arc_lo = a0;
+    g_.arc_hi = a1;
     // ---- rank parts: this process's ranks and their owned vertex ranges
-    const int world = comm_.world();
-    bounds_ = partition(g_.off, n, (uint32_t)world);
+    bounds_ = nb;
     if (!same_shape) {
         parts_.clear();
         if (comm_.emulated()) {
@@ -1178,6 +1211,10 @@ void Engine::set_option(int opt, int64_t value) {
             if (value < 0 || value > 64) throw Error(ASCETIC_EINVAL, "static CTAs per SM must be in [0, 64]");
             o_.static_ctas_per_sm = (int)value;
             break;
+        case ASCETIC_OPT_RELAX_MODE:
+            if (value < 0 || value > 2) throw Error(ASCETIC_EINVAL, "relax mode: 0 = auto, 1 = atomicMin + next bit, 2 = RED.MIN + dense finalize");
+            o_.relax_mode = (int)value;
+            break;
         case ASCETIC_OPT_CHUNK_BUFFERS:
             if (value != 0 && (value < 2 || value > 8)) throw Error(ASCETIC_EINVAL, "chunk buffers must be 0 (auto) or in [2, 8]");
             o_.chunk_buffers = (int)value;
@@ -1269,6 +1306,10 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         }
         comm_.reserve_sparse(cap, (int)parts_.size());
     }
+    // SSSP/CC min updates: RED.MIN + dense finalize, unless the sparse exchange needs this rank's next
+    // bits (it packs exactly the ids this rank lowered)
+    const bool red = (algo == ALG_SSSP || algo == ALG_CC) && !sparse_on && o_.relax_mode == 2;
+    for (auto& p : parts_) p->set_red_min(red);
     for (auto& p : parts_) p->begin(algo, source, max_iters, timing);
     Part& p0 = *parts_[0];
     std::vector<IterTotals> T(parts_.size());

@@ -69,6 +69,7 @@ struct Options {
     uint32_t sparse_exchange = 0; // P > 1, SSSP/CC: sparse MIN when every rank has <= n/(d P) pairs (0 = off)
     uint32_t replace_k = 0;       // §3.4 data replacement: chunk swaps examined per iteration (0 = off)
     int replace_policy = 0;       // hotness counter: 0 = by algorithm, 1 = cumulative, 2 = last iteration
+    int relax_mode = 0;           // SSSP/CC min update: 0 = auto, 1 = atomicMin + next bit, 2 = RED.MIN + dense finalize
 };
 
 struct HostGraph {
@@ -79,7 +80,9 @@ struct HostGraph {
     const void* nbr = nullptr;        // b_e bytes per arc, pinned
     const void* nbr_dev = nullptr;    // device-visible alias (zero-copy)
     void* owned = nullptr;            // library-owned pinned copy
-    void* registered = nullptr;       // pinned in place by us
+    void* registered = nullptr;       // pinned in place by us: [registered, registered + reg_bytes)
+    size_t reg_bytes = 0;
+    uint64_t arc_lo = 0, arc_hi = 0;  // host arcs this process reads (its ranks' rows; all with emulation)
     void release();
 };
 
@@ -107,6 +110,7 @@ class Part {
     void finalize(uint32_t t, bool dense);
     // fused exchange (P > 1): the peer tables and the finalize that reads every rank's buffer
     void set_fused(bool on);   // this run uses the fused exchange (allocates the second next buffer)
+    void set_red_min(bool on) { red_min_ = on; }   // SSSP/CC: RED.MIN updates, A_{t+1} from val < snap
     void set_peers(int kind, const std::vector<void*>& ptrs);   // kind 0/1: next[0/1], 2: val or inc
     void finalize_fused(uint32_t t);
     void clear_next(uint32_t b);
@@ -159,6 +163,7 @@ class Part {
     unsigned long long* d_pr_inc_ = nullptr;   // P > 1: residual increments of this rank's pushes
     bool multi_ = false;
     bool fused_ = false;
+    bool red_min_ = false;
     uint32_t* d_next2_ = nullptr;              // fused exchange: next bitmaps double-buffered by iteration parity
     const void** d_peers_ = nullptr;           // [3][world] device pointers (next0, next1, val/inc)
     int peer_world_ = 0;

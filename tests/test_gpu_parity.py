@@ -220,7 +220,7 @@ def test_load_variants_copy_wgt_validate(asc):
 
 @pytest.mark.parametrize("opt,val", [("overlap", 0), ("keep_static", 1), ("chunk_buffers", 2),
                                      ("chunk_buffers", 3), ("chunk_buffers", 8), ("gather_ctas", 1), ("static_ctas_per_sm", 1),
-                                     ("timing", 0)])
+                                     ("timing", 0), ("relax_mode", 1), ("relax_mode", 2)])
 def test_options_do_not_change_results(asc, opt, val):
     """Tuning knobs change scheduling only: results, records and bytes stay bit-exact."""
     g = gg.rmat(12, seed=14, weights=True)
@@ -241,7 +241,7 @@ def test_options_do_not_change_results(asc, opt, val):
         else:
             assert st["h2d_static_fill_bytes"] == p.static_bytes
     defaults = {"overlap": 1, "keep_static": 0, "chunk_buffers": 0, "gather_ctas": 0, "static_ctas_per_sm": 0,
-                "timing": 1}
+                "timing": 1, "relax_mode": 0}
     asc.set_option(opt, defaults[opt])
 
 
@@ -406,3 +406,23 @@ def test_pr_bitwise_reproducible(asc):
     ref = _oracle("pr", g, 0, p.s, max_iters=12)
     _pr_ok(runs[0], ref.values)
     assert abs(runs[0].astype(np.float64).sum() - 1.0) <= 1e-5
+
+
+@pytest.mark.parametrize("mode", [1, 2])
+@pytest.mark.parametrize("algo", ["sssp", "cc"])
+def test_relax_modes_resident_and_out_of_core(asc, mode, algo):
+    """Both SSSP/CC min-update forms (atomicMin + next bit, RED.MIN + dense finalize) give the same
+    values, active sets and bytes, resident (all lists static) and out of core."""
+    g = gg.rmat(13, seed=19, weights=(algo == "sssp"))
+    src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+    asc.set_option("relax_mode", mode)
+    try:
+        for budget in (10 * g.csr_bytes, g.csr_bytes // 4):
+            st, its, res = _run(asc, g, algo, src=src, budget=budget)
+            p = oracle.placer(g.off, g.b_e, budget)
+            ref = _oracle(algo, g, src, p.s)
+            np.testing.assert_array_equal(res, ref.values)
+            _check_records(its, ref)
+            assert st["h2d_payload_bytes"] == ref.h2d_payload
+    finally:
+        asc.set_option("relax_mode", 0)

@@ -56,16 +56,18 @@ def main():
             lv = asc.get_result().copy()
             act = lv == t
         else:
+            # A_0 = V (CC) or {src} (SSSP); A_t = {v : r_t < r_(t-1)}, r_t = values after t iterations
             if t == 0:
                 act = np.zeros(g.n, bool)
                 if algo == "cc":
                     act[:] = True
+                    prev = np.arange(g.n, dtype=np.uint32)
                 else:
                     act[src] = True
-                asc.run(algo, src, 1)
-                prev = asc.get_result().copy()
+                    prev = np.full(g.n, 0xFFFFFFFF, dtype=np.uint32)
+                    prev[src] = 0
             else:
-                asc.run(algo, src, t + 1)
+                asc.run(algo, src, t)
                 cur = asc.get_result().copy()
                 act = cur < prev
                 prev = cur
