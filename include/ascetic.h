@@ -112,11 +112,17 @@ typedef enum {
                                       bitmap bit), else the dense ncclAllReduce(min) / bitmap OR; one 4P-byte host
                                       read per iteration decides. 0 (default) = dense always. 8 keeps the
                                       all-gather under the all-reduce's bytes. Results are identical. */
-    ASCETIC_OPT_RELAX_MODE = 20      /* SSSP/CC min updates: 1 = atomicMin, and the thread whose atomic lowered the
+    ASCETIC_OPT_RELAX_MODE = 20,     /* SSSP/CC min updates: 1 = atomicMin, and the thread whose atomic lowered the
                                       value sets the vertex's next-frontier bit; 2 = fire-and-forget RED.MIN, and
                                       the finalize derives A_{t+1} = {v : val < snap} in one dense pass (Jacobi:
-                                      the same set); 0 = auto (default). The sparse exchange forces 1. Results are
-                                      identical. */
+                                      the same set); 0 = auto (default) = 2 (resident static-hit kernels 5-15 % faster). The sparse
+                                      exchange forces 1. Results are identical. */
+    ASCETIC_OPT_CE_MIN_RUN = 21,     /* bytes (default 1 MiB, 0 = off): in gather-mode iterations the miss runs of at
+                                      least this many bytes are copied by the copy engines (one cudaMemcpyAsync per
+                                      run piece, on a second copy stream) while the SM gather moves the rest */
+    ASCETIC_OPT_GAP_BRIDGE = 22      /* bytes (default 256, 0 = off): the SM gather also loads (and discards) host holes
+                                      of at most this size between consecutive pieces, so one contiguous read
+                                      replaces two (the link charges per contiguous region) */
 } ascetic_option;
 
 typedef struct {
@@ -135,7 +141,7 @@ typedef struct {
     double static_fraction_used;  /* R */
     uint64_t h2d_payload_bytes;   /* Σ_t miss bytes (the parity target) */
     uint64_t h2d_static_fill_bytes;
-    uint64_t h2d_other_bytes;     /* padding/metadata H2D (expected 0) */
+    uint64_t h2d_other_bytes;     /* metadata H2D: the long-run stream intervals of hybrid gather iterations */
     uint64_t d2h_bytes;           /* run lists + counters read back */
     uint64_t active_arcs_total;   /* Σ_t Σ_{v∈A_t} deg(v) */
     uint64_t chunks_total;
@@ -167,6 +173,9 @@ typedef struct {
     uint64_t sparse_exchange_bytes; /* (id, value) pair bytes all ranks contributed to those exchanges */
     uint32_t chunk_buffers;       /* On-demand Region buffers in use (auto: 3, or 2 when C/3 < 4 MiB) */
     uint32_t reserved0;
+    uint64_t gather_ce_bytes;     /* part of gather_bytes moved by the copy engines (long runs, CE_MIN_RUN) */
+    uint64_t gather_load_bytes;   /* host bytes the SM gather loaded: 16-byte cover units incl. bridged holes
+                                     (vs gather_bytes - gather_ce_bytes of payload: the over-fetch) */
 } ascetic_stats_t;
 
 typedef struct {

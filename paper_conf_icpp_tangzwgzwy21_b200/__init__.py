@@ -37,7 +37,8 @@ OPTIONS = {"chunk_cap": 1, "xfer_mode": 2, "dma_min_run": 3, "overlap": 4, "keep
            "hub_degree": 6, "timing": 7, "gather_ctas": 8, "chunk_buffers": 9, "static_ctas_per_sm": 10,
            "prefetch": 11, "repartition": 12, "static_placement": 13, "replace_chunks": 14,
            "replace_policy": 15, "placement_seed": 16, "prd_tol_ppm": 17,
-           "fused_exchange": 18, "sparse_exchange": 19, "relax_mode": 20}
+           "fused_exchange": 18, "sparse_exchange": 19, "relax_mode": 20,
+           "ce_min_run": 21, "gap_bridge": 22}
 INF = 0xFFFFFFFF
 
 
@@ -64,7 +65,8 @@ class Stats(ctypes.Structure):
                 ("repartitions", ctypes.c_uint64), ("h2d_replace_bytes", ctypes.c_uint64),
                 ("swaps_total", ctypes.c_uint64), ("time_replace_s", ctypes.c_double),
                 ("sparse_exchanges", ctypes.c_uint64), ("sparse_exchange_bytes", ctypes.c_uint64),
-                ("chunk_buffers", ctypes.c_uint32), ("reserved0", ctypes.c_uint32)]
+                ("chunk_buffers", ctypes.c_uint32), ("reserved0", ctypes.c_uint32),
+                ("gather_ce_bytes", ctypes.c_uint64), ("gather_load_bytes", ctypes.c_uint64)]
 
 
 class IterStats(ctypes.Structure):

@@ -137,8 +137,17 @@ void launch_static(int algo, const DevState& d, const Queues& q, const void* sta
                    uint32_t piece_arcs, int max_ctas, cudaStream_t s);
 void launch_ondemand(int algo, const DevState& d, const Queues& q,
                      const void* chunk, unsigned long long lo, unsigned long long hi, cudaStream_t s);
+// zero-copy gather of miss-stream arcs [lo, hi) into chunk; skips the vertices inside the sorted long
+// stream intervals lint[2i, 2i+1) (copied by the copy engines), bridges host holes <= gap_bytes;
+// adds the number of 16-byte host units it loads to *cover
 void launch_gather(const Queues& q, const void* host_nbr, uint64_t m, uint32_t b_e, void* chunk,
-                   unsigned long long lo, unsigned long long hi, int max_ctas, cudaStream_t s);
+                   unsigned long long lo, unsigned long long hi, int max_ctas, const unsigned long long* lint,
+                   uint32_t nlint, uint32_t gap_bytes, unsigned long long* cover, cudaStream_t s);
+// long miss runs (>= min_arcs arcs): append (b, e, dst) of each into out[3*i] (mapped host memory,
+// unordered, at most cap), count into *count; `flag` set to 1 by the last CTA (host spin target)
+void launch_long_runs(const uint32_t* run_b, const uint32_t* run_e, const unsigned long long* run_dst, uint32_t n_runs,
+                      const unsigned long long* off, unsigned long long min_arcs, unsigned long long* out, uint32_t cap,
+                      uint32_t* count, uint32_t* done, uint32_t* flag, cudaStream_t s);
 // §3.4: per-chunk accesses (active arcs) of this iteration's hit + miss queues into acc
 void launch_chunk_access(const DevState& d, const Queues& q, uint32_t n_small, uint32_t n_med, uint32_t n_hub,
                          uint32_t b_e, uint32_t* acc, cudaStream_t s);

@@ -679,10 +679,19 @@ __device__ __forceinline__ uint4 ld_host16(const uint4* p) {
 // piece), each piece's cover units are enumerated across the warp (a unit shared by two
 // vertices of one piece is loaded once), and every lane stores the piece words its unit holds
 // at their stream position. `hoff` = the host array's byte offset from its 16-byte-aligned base.
+// Gap bridging: SM reads of host memory are charged per contiguous region (tools/zc_gran.cu: ~90 M
+// random regions/s whatever their size up to 512 B), and consecutive miss runs are mostly separated by
+// a few bytes (profiles/r02/run_profile_c4.log: 89-96 % of the gaps < 16 B), so a piece whose next
+// piece starts at most `gap_words` later also loads the hole units between them (not stored): the
+// warp instruction then reads one contiguous block instead of two.
+// Long runs: stream intervals lint[2i, 2i+1) (sorted, disjoint; whole vertices) go through the copy
+// engines instead (Part::transfer_chunk); their vertices are skipped here.
 template <int BE, int NG>
 __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restrict__ host, uint32_t hoff,
                                                   unsigned long long w_end, uint32_t* __restrict__ chunk,
-                                                  unsigned long long lo, unsigned long long hi) {
+                                                  unsigned long long lo, unsigned long long hi,
+                                                  const unsigned long long* __restrict__ lint, uint32_t nlint,
+                                                  uint32_t gap_words, unsigned long long* __restrict__ cover) {
     // tile metadata staged in shared memory (reading it through L1 instead gathers at the same rate,
     // but its L1 traffic slows the concurrent static-hit kernels)
     __shared__ unsigned long long s_pre[kEdgeTile + 1];
@@ -704,10 +713,17 @@ __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restr
         const unsigned long long pe = min(x.t_hi, pw + 256ull);
         const uint32_t kfirst = find_local(s_pre, 0, x.cnt, pw);
         const uint32_t klast = find_local(s_pre, kfirst, x.cnt, pe - 1);
+        // long intervals that can touch this segment: the last one starting at or before pw, and the next
+        uint32_t li = 0;
+        if (nlint) {
+            uint32_t L = 0, R = nlint;                               // first interval starting after pw
+            while (L < R) { const uint32_t mid = (L + R) >> 1; if (__ldg(lint + 2 * mid) <= pw) L = mid + 1; else R = mid; }
+            li = L ? L - 1 : 0;
+        }
         for (uint32_t kb = kfirst; kb <= klast; kb += 32) {
             // lane <-> vertex j of the segment: stream arcs [a0, a1), host arcs [h0, h1)
             const uint32_t j = kb + (uint32_t)lane;
-            const bool v = j <= klast;
+            bool v = j <= klast;
             unsigned long long a0 = 0, a1 = 0, h0 = 0;
             if (v) {
                 const unsigned long long pj = s_pre[j];
@@ -715,22 +731,34 @@ __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restr
                 a0 = max(pw, pj);
                 a1 = max(a0, min(pe, ej));
                 h0 = s_src[j] + (a0 - pj);
+                // a vertex inside a long run (runs are whole vertices) is the copy engines' job
+                for (uint32_t k = li; k < li + 2 && k < nlint; ++k)
+                    if (a0 >= __ldg(lint + 2 * k) && a0 < __ldg(lint + 2 * k + 1)) v = false;
+                if (!v) a0 = a1 = h0 = 0;
             }
             const unsigned long long h1 = h0 + (a1 - a0);
             const unsigned long long ph1 = __shfl_up_sync(FULL, h1, 1);
-            const bool start = v && (lane == 0 || h0 != ph1);
+            const bool pv = __shfl_up_sync(FULL, v, 1);
+            const bool start = v && (lane == 0 || !pv || h0 != ph1);
             const uint32_t smask = __ballot_sync(FULL, start);
             const uint32_t vmask = __ballot_sync(FULL, v);
+            const uint32_t brk = __ballot_sync(FULL, start || !v);          // piece boundaries and holes
             const int ps = 31 - __clz(smask & ((2u << lane) - 1u));          // this lane's piece start
-            const uint32_t after = lane == 31 ? 0u : (smask & ~((2u << lane) - 1u));
+            const uint32_t after = lane == 31 ? 0u : (brk & ~((2u << lane) - 1u));
             const int pl = after ? (__ffs(after) - 2) : (31 - __clz(vmask)); // and its last lane
-            const unsigned long long W0 = w_off + __shfl_sync(FULL, h0, ps) * AW;   // piece host words [W0, W1)
-            const unsigned long long W1 = w_off + __shfl_sync(FULL, h1, pl) * AW;
-            const unsigned long long D0 = (__shfl_sync(FULL, a0, ps) - lo) * AW;    // chunk word of W0
+            const unsigned long long W0 = w_off + __shfl_sync(FULL, h0, ps & 31) * AW;   // piece host words [W0, W1)
+            const unsigned long long W1 = w_off + __shfl_sync(FULL, h1, pl & 31) * AW;
+            const unsigned long long D0 = (__shfl_sync(FULL, a0, ps & 31) - lo) * AW;    // chunk word of W0
             const unsigned long long hw0 = w_off + h0 * AW, hw1 = w_off + h1 * AW;
             // cover units of this lane's words not already covered by the previous lane of the piece
             const unsigned long long u0 = start ? (hw0 >> 2) : ((hw0 + 3) >> 2);
-            const unsigned long long u1 = (hw1 + 3) >> 2;
+            unsigned long long u1 = (hw1 + 3) >> 2;
+            // bridge to the next piece of this group when the hole is at most gap_words: its units are
+            // loaded by this (the piece's last) lane and fall outside [W0, W1), so nothing is stored
+            const unsigned long long nh0 = __shfl_down_sync(FULL, hw0, 1);
+            const bool nstart = __shfl_down_sync(FULL, start, 1);
+            if (v && lane == pl && lane < 31 && nstart && nh0 > hw1 && nh0 - hw1 <= gap_words)
+                u1 = max(u1, nh0 >> 2);
             const uint32_t cnt = (v && hw1 > hw0 && u1 > u0) ? (uint32_t)(u1 - u0) : 0u;
             uint32_t incl = cnt;
 #pragma unroll
@@ -740,6 +768,7 @@ __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restr
             }
             const uint32_t excl = incl - cnt;
             const uint32_t total = __shfl_sync(FULL, incl, 31);
+            if (lane == 0 && total) atomicAdd(cover, (unsigned long long)total);   // 16-byte units read
             for (uint32_t b = 0; b < total; b += 32u * NG) {
                 // NG groups of 32 units: all loads first (NG x 16 B in flight per lane), then the stores
                 uint4 val[NG];
@@ -787,6 +816,33 @@ __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restr
                     }
                 }
             }
+        }
+    }
+}
+
+// Long miss runs for the copy engines: runs are maximal id ranges of M_t, so a run's host bytes are
+// one contiguous range b_e [off[b], off[e]); those >= min_arcs arcs are appended (unordered) with
+// their stream offset into mapped host memory for the host to sort and issue as DMAs.
+__global__ void __launch_bounds__(256) k_long_runs(const uint32_t* __restrict__ run_b, const uint32_t* __restrict__ run_e,
+                                                   const unsigned long long* __restrict__ run_dst, uint32_t n_runs,
+                                                   const unsigned long long* __restrict__ off, unsigned long long min_arcs,
+                                                   unsigned long long* out, uint32_t cap, uint32_t* count,
+                                                   uint32_t* done, uint32_t* flag) {
+    for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < n_runs; r += gridDim.x * blockDim.x) {
+        const uint32_t b = run_b[r], e = run_e[r];
+        if (__ldg(off + e) - __ldg(off + b) >= min_arcs) {
+            const uint32_t i = atomicAdd(count, 1u);
+            if (i < cap) { out[3 * i] = b; out[3 * i + 1] = e; out[3 * i + 2] = run_dst[r]; }
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence_system();                                    // this CTA's host writes first
+        if (atomicAdd(done, 1u) == gridDim.x - 1) {
+            __threadfence();
+            flag[1] = *reinterpret_cast<volatile uint32_t*>(count);
+            __threadfence_system();
+            *reinterpret_cast<volatile uint32_t*>(flag) = 1u;
         }
     }
 }
@@ -1366,7 +1422,8 @@ void launch_ondemand(int algo, const DevState& d, const Queues& q, const void* c
 }
 
 void launch_gather(const Queues& q, const void* host_nbr, uint64_t m, uint32_t b_e, void* chunk,
-                   unsigned long long lo, unsigned long long hi, int max_ctas, cudaStream_t s) {
+                   unsigned long long lo, unsigned long long hi, int max_ctas, const unsigned long long* lint,
+                   uint32_t nlint, uint32_t gap_bytes, unsigned long long* cover, cudaStream_t s) {
     if (hi <= lo) return;
     const unsigned long long tiles = ((hi - 1) >> kEdgeTileShift) - (lo >> kEdgeTileShift) + 1;
     const unsigned grid = (unsigned)(tiles < (unsigned long long)max_ctas ? tiles : (unsigned long long)max_ctas);
@@ -1379,8 +1436,18 @@ void launch_gather(const Queues& q, const void* host_nbr, uint64_t m, uint32_t b
     // one per piece boundary, so 4 per lane (128) usually needs a second, nearly empty round; 6 took
     // C2's gather from 44.6-44.7 to 45.0 GB/s (profiles/r01/gather_ng_ab.log; 5 and 8 within noise of
     // 6). 4-byte arcs: 64 units per segment, 4 per lane fits.
-    if (b_e == 8) k_gather16<8, 6><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
-    else k_gather16<4, 4><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi);
+    if (b_e == 8) k_gather16<8, 6><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi, lint, nlint, gap_bytes / 4, cover);
+    else k_gather16<4, 4><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi, lint, nlint, gap_bytes / 4, cover);
+    ++g_launches;
+}
+
+void launch_long_runs(const uint32_t* run_b, const uint32_t* run_e, const unsigned long long* run_dst, uint32_t n_runs,
+                      const unsigned long long* off, unsigned long long min_arcs, unsigned long long* out, uint32_t cap,
+                      uint32_t* count, uint32_t* done, uint32_t* flag, cudaStream_t s) {
+    cudaMemsetAsync(count, 0, 4, s);
+    cudaMemsetAsync(done, 0, 4, s);
+    k_long_runs<<<blocks_for(n_runs ? n_runs : 1, 256, 148u * 4u), 256, 0, s>>>(run_b, run_e, run_dst, n_runs, off,
+                                                                                min_arcs, out, cap, count, done, flag);
     ++g_launches;
 }
 

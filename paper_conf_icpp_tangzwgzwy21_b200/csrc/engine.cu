@@ -131,11 +131,21 @@ Part::~Part() {
     dfree(d_tile_agg_); dfree(d_tile_incl_); dfree(d_tile_flag_); dfree(d_tot_);
     if (h_tot_) cudaFreeHost(h_tot_);
     if (h_runs_) cudaFreeHost(h_runs_);
+    if (h_long_) cudaFreeHost(h_long_);
+    if (h_long_flag_) cudaFreeHost(h_long_flag_);
+    for (int i = 0; i < 2; ++i) { if (h_lint_[i]) cudaFreeHost(h_lint_[i]); dfree(d_lint_[i]); }
+    dfree(d_long_cnt_); dfree(d_cover_);
+    for (int i = 0; i < kMaxBuffers; ++i) {
+        if (ce_done_[i]) cudaEventDestroy(ce_done_[i]);
+        if (xfer_go_[i]) cudaEventDestroy(xfer_go_[i]);
+    }
+    if (xs2_) { cudaStreamSynchronize(xs2_); cudaStreamDestroy(xs2_); }
     for (int i = 0; i < kMaxBuffers; ++i) {
         if (ready_[i]) cudaEventDestroy(ready_[i]);
         if (consumed_[i]) cudaEventDestroy(consumed_[i]);
     }
     if (ev_classified_) cudaEventDestroy(ev_classified_);
+    if (ev_long_) cudaEventDestroy(ev_long_);
     free_hot();
     if (ev_acc_) cudaEventDestroy(ev_acc_);
     if (ev_swapped_) cudaEventDestroy(ev_swapped_);
@@ -158,14 +168,18 @@ void Part::alloc_vertex_state() {
     CK(cudaStreamCreateWithPriority(&cs_, cudaStreamNonBlocking, lo_pri));
     CK(cudaStreamCreateWithPriority(&xs_, cudaStreamNonBlocking, hi_pri));
     CK(cudaStreamCreateWithPriority(&ss_, cudaStreamNonBlocking, lo_pri));
+    CK(cudaStreamCreateWithPriority(&xs2_, cudaStreamNonBlocking, hi_pri));
     for (int i = 0; i < kMaxBuffers; ++i) {
         CK(cudaEventCreateWithFlags(&ready_[i], cudaEventDisableTiming));
         CK(cudaEventCreateWithFlags(&consumed_[i], cudaEventDisableTiming));
+        CK(cudaEventCreateWithFlags(&ce_done_[i], cudaEventDisableTiming));
+        CK(cudaEventCreateWithFlags(&xfer_go_[i], cudaEventDisableTiming));
     }
     CK(cudaEventCreateWithFlags(&static_go_, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&static_done_, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&sync_ev_, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&ev_classified_, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&ev_long_, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&ev_acc_, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&ev_swapped_, cudaEventDisableTiming));
     const uint64_t n = g_.n, m = g_.m;
@@ -200,6 +214,13 @@ void Part::alloc_vertex_state() {
     if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_EHOSTMEM, "cudaHostAlloc totals"); }
     e = cudaHostAlloc((void**)&h_runs_, 2ull * kRunsHostMax * sizeof(uint32_t), cudaHostAllocMapped | cudaHostAllocPortable);
     if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_EHOSTMEM, "cudaHostAlloc run list"); }
+    e = cudaHostAlloc((void**)&h_long_, 3ull * kLongMax * 8, cudaHostAllocMapped | cudaHostAllocPortable);
+    if (e == cudaSuccess) e = cudaHostAlloc((void**)&h_long_flag_, 8, cudaHostAllocMapped | cudaHostAllocPortable);
+    for (int i = 0; i < 2 && e == cudaSuccess; ++i) e = cudaHostAlloc((void**)&h_lint_[i], 2ull * kLongMax * 8, cudaHostAllocPortable);
+    if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_EHOSTMEM, "cudaHostAlloc long-run lists"); }
+    dalloc(&d_long_cnt_, 2, &vertex_bytes_);
+    for (int i = 0; i < 2; ++i) dalloc(&d_lint_[i], 2ull * kLongMax, &vertex_bytes_);
+    dalloc(&d_cover_, 1, &vertex_bytes_);
 }
 
 void Part::alloc_algo_state(int algo, bool multi) {
@@ -441,12 +462,43 @@ void Part::span(cudaEvent_t a, cudaStream_t s, uint32_t t, int ph, int sub) {
 // the miss queue; mode 2: copy-engine DMA of the run pieces intersecting the window.
 void Part::transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsigned long long hi, int mode) {
     if (mode == 1) {
+        const uint32_t b_e = g_.b_e;
+        // the long runs of the window go to the copy engines on the second copy stream, concurrently
+        // with the SM gather of the rest; both start after this chunk's buffer is free (xfer_go) and
+        // the chunk is ready when both are done
+        bool ce = false;
+        if (nlint_) {
+            size_t r = std::upper_bound(ldst_.begin(), ldst_.end(), lo) - ldst_.begin();
+            r = r ? r - 1 : 0;
+            const char* host = (const char*)g_.nbr;
+            char* dst = (char*)d_chunk_[buf];
+            for (; r < lb_.size(); ++r) {
+                const unsigned long long a0 = g_.off[lb_[r]], a1 = g_.off[le_[r]];
+                const unsigned long long s0 = ldst_[r], s1 = s0 + (a1 - a0);
+                if (s0 >= hi) break;
+                const unsigned long long p0 = std::max(s0, lo), p1 = std::min(s1, hi);
+                if (p1 <= p0) continue;
+                if (!ce) {
+                    CK(cudaEventRecord(xfer_go_[buf], xs_));
+                    CK(cudaStreamWaitEvent(xs2_, xfer_go_[buf], 0));
+                    ce = true;
+                }
+                CK(cudaMemcpyAsync(dst + (p0 - lo) * b_e, host + (a0 + (p0 - s0)) * b_e, (p1 - p0) * b_e,
+                                   cudaMemcpyHostToDevice, xs2_));
+                st.gather_ce_bytes += (p1 - p0) * b_e;
+            }
+        }
         // default grid keeps ~1 MiB of PCIe reads in flight (CTAs x 256 lanes x 8 loads x b_e):
         // enough to saturate the link (~20 us of it), while a deeper queue only adds latency
         // and congests the memory system for the concurrently running edge kernels
         // (measured: 64 CTAs at b_e = 8 -> same 47 GB/s, 3x faster on-demand kernels than 296)
-        const int ctas = o_.gather_ctas ? o_.gather_ctas : (int)(64u * 8u / g_.b_e);
-        launch_gather(q, g_.nbr_dev, g_.m, g_.b_e, d_chunk_[buf], lo, hi, ctas, xs_);
+        const int ctas = o_.gather_ctas ? o_.gather_ctas : (int)(64u * 8u / b_e);
+        launch_gather(q, g_.nbr_dev, g_.m, b_e, d_chunk_[buf], lo, hi, ctas, nlint_ ? d_lint_[lint_buf_] : nullptr,
+                      nlint_, o_.gap_bridge, d_cover_, xs_);
+        if (ce) {
+            CK(cudaEventRecord(ce_done_[buf], xs2_));
+            CK(cudaStreamWaitEvent(xs_, ce_done_[buf], 0));
+        }
         return;
     }
     size_t r = std::upper_bound(rdst_.begin(), rdst_.end(), lo) - rdst_.begin();
@@ -463,6 +515,58 @@ void Part::transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsig
         CK(cudaMemcpyAsync(dst + (p0 - lo) * b_e, host + (a0 + (p0 - s0)) * b_e, (p1 - p0) * b_e,
                            cudaMemcpyHostToDevice, xs_));
     }
+}
+
+// Gather-mode iteration with runs of >= ce_min_run bytes: the copy engines move those (one
+// cudaMemcpyAsync each, ~55 GB/s when long) while the SM gather does the many short ones. A small
+// kernel lists the long runs into mapped memory; the host sorts them by stream position and hands
+// the gather their stream intervals (H2D on the copy stream, before this iteration's gathers).
+uint32_t Part::plan_long_runs(const IterTotals& T) {
+    nlint_ = 0;
+    lb_.clear(); le_.clear(); ldst_.clear();
+    const unsigned long long min_arcs = std::max<uint64_t>(1, o_.ce_min_run / g_.b_e);
+    *reinterpret_cast<volatile uint32_t*>(&h_long_flag_[0]) = 0;
+    launch_long_runs(d_run_b_, d_run_e_, d_run_dst_, T.n_runs, d_off_, min_arcs, h_long_, kLongMax, d_long_cnt_,
+                     d_long_cnt_ + 1, h_long_flag_, cs_);
+    CK(cudaGetLastError());
+    CK(cudaEventRecord(ev_long_, cs_));
+    const volatile uint32_t* flag = h_long_flag_;
+    uint32_t spins = 0;
+    while (!flag[0]) {
+        if ((++spins & 1023u) == 0) {
+            const cudaError_t e = cudaEventQuery(ev_long_);
+            if (e == cudaSuccess) break;
+            if (e != cudaErrorNotReady) CK(e);
+        }
+    }
+    if (!flag[0]) CK(cudaEventSynchronize(ev_long_));
+    std::atomic_thread_fence(std::memory_order_acquire);
+    const uint32_t c0 = flag[1];
+    const uint32_t cnt = std::min<uint32_t>(c0, kLongMax);
+    st.d2h_bytes += 8 + 24ull * cnt;
+    if (!cnt) return 0;
+    std::vector<uint32_t> idx(cnt);
+    const volatile unsigned long long* L = h_long_;
+    std::vector<unsigned long long> raw(3ull * cnt);
+    for (uint64_t i = 0; i < 3ull * cnt; ++i) raw[i] = L[i];
+    for (uint32_t i = 0; i < cnt; ++i) idx[i] = i;
+    std::sort(idx.begin(), idx.end(), [&](uint32_t a, uint32_t b) { return raw[3 * a + 2] < raw[3 * b + 2]; });
+    lint_buf_ ^= 1u;
+    unsigned long long* li = h_lint_[lint_buf_];
+    for (uint32_t k = 0; k < cnt; ++k) {
+        const uint32_t i = idx[k];
+        lb_.push_back((uint32_t)raw[3 * i]);
+        le_.push_back((uint32_t)raw[3 * i + 1]);
+        ldst_.push_back(raw[3 * i + 2]);
+        li[2 * k] = raw[3 * i + 2];
+        li[2 * k + 1] = raw[3 * i + 2] + (g_.off[raw[3 * i + 1]] - g_.off[raw[3 * i]]);
+    }
+    // staging buffer of parity p is rewritten two iterations later, after this copy ran (the host
+    // reaches iteration t+2 only once classify(t+2) finished, which follows every chunk of t+1)
+    CK(cudaMemcpyAsync(d_lint_[lint_buf_], li, 16ull * cnt, cudaMemcpyHostToDevice, xs_));
+    st.h2d_other_bytes += 16ull * cnt;
+    nlint_ = cnt;
+    return cnt;
 }
 
 void Part::begin(int algo, uint32_t source, uint32_t max_iters, bool timing) {
@@ -506,6 +610,7 @@ void Part::begin(int algo, uint32_t source, uint32_t max_iters, bool timing) {
     launches0_ = g_launches;
     ev_start_ = pool_.get(); ev_fill0_ = pool_.get(); ev_fill1_ = pool_.get();
     CK(cudaEventRecord(ev_start_, cs_));
+    CK(cudaMemsetAsync(d_cover_, 0, 8, cs_));
     // ---- static fill: ONE DMA of this rank's front prefix, counted in the run
     CK(cudaStreamWaitEvent(xs_, ev_start_, 0));
     CK(cudaEventRecord(ev_fill0_, xs_));
@@ -634,6 +739,7 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     }
     st.static_arcs += T.hit_arcs;
     st.ondemand_arcs += T.miss_arcs;
+    nlint_ = 0;
     // ---- On-demand request, fragmented into chunks
     const unsigned long long cap_arcs = cap_ / b_e;
     const unsigned long long miss = T.miss_arcs;
@@ -658,6 +764,7 @@ void Part::expand(uint32_t t, const IterTotals& T) {
             unsigned long long acc = 0;
             for (uint32_t r = 0; r < T.n_runs; ++r) { rdst_[r] = acc; acc += g_.off[re_[r]] - g_.off[rb_[r]]; }
         }
+        if (mode == 1 && o_.ce_min_run && T.n_runs && miss * b_e >= 2 * o_.ce_min_run) plan_long_runs(T);
         if (!o_.overlap && static_pending_) CK(cudaStreamWaitEvent(xs_, static_done_, 0));   // ablation
     }
     // chunks already transferred at the end of the previous iteration (PR prefetch) must be
@@ -954,7 +1061,11 @@ void Part::end() {
     st.chunk_cap = cap_;
     st.chunk_buffers = (uint32_t)nbuf_;
     st.static_fraction_used = pl_.R;
-    st.h2d_other_bytes = 0;
+    {
+        unsigned long long units = 0;
+        CK(cudaMemcpy(&units, d_cover_, 8, cudaMemcpyDeviceToHost));
+        st.gather_load_bytes = units * 16ull;
+    }
     st.time_run_s = ms / 1e3;
     st.time_fill_s = fill_ms / 1e3;
     st.time_classify_s = ph[PH_CLS] / 1e3;
@@ -1215,6 +1326,14 @@ void Engine::set_option(int opt, int64_t value) {
             if (value < 0 || value > 2) throw Error(ASCETIC_EINVAL, "relax mode: 0 = auto, 1 = atomicMin + next bit, 2 = RED.MIN + dense finalize");
             o_.relax_mode = (int)value;
             break;
+        case ASCETIC_OPT_CE_MIN_RUN:
+            if (value < 0) throw Error(ASCETIC_EINVAL, "copy-engine minimum run must be >= 0 bytes");
+            o_.ce_min_run = (uint64_t)value;
+            break;
+        case ASCETIC_OPT_GAP_BRIDGE:
+            if (value < 0 || value > 65536) throw Error(ASCETIC_EINVAL, "gap bridge must be in [0, 65536] bytes");
+            o_.gap_bridge = (uint32_t)value;
+            break;
         case ASCETIC_OPT_CHUNK_BUFFERS:
             if (value != 0 && (value < 2 || value > 8)) throw Error(ASCETIC_EINVAL, "chunk buffers must be 0 (auto) or in [2, 8]");
             o_.chunk_buffers = (int)value;
@@ -1306,9 +1425,10 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         }
         comm_.reserve_sparse(cap, (int)parts_.size());
     }
-    // SSSP/CC min updates: RED.MIN + dense finalize, unless the sparse exchange needs this rank's next
-    // bits (it packs exactly the ids this rank lowered)
-    const bool red = (algo == ALG_SSSP || algo == ALG_CC) && !sparse_on && o_.relax_mode == 2;
+    // SSSP/CC min updates: RED.MIN + dense finalize (default: resident RMAT-24 static-hit kernels -15 %
+    // SSSP / -11 % CC, friendster-shaped CC -5 %, profiles/r02/resident_ab.md), unless the sparse
+    // exchange needs this rank's next bits (it packs exactly the ids this rank lowered)
+    const bool red = (algo == ALG_SSSP || algo == ALG_CC) && !sparse_on && o_.relax_mode != 1;
     for (auto& p : parts_) p->set_red_min(red);
     for (auto& p : parts_) p->begin(algo, source, max_iters, timing);
     Part& p0 = *parts_[0];
@@ -1439,6 +1559,9 @@ void Engine::run(int algo, uint32_t source, uint32_t max_iters) {
         st_.static_arcs += s.static_arcs;
         st_.ondemand_arcs += s.ondemand_arcs;
         st_.gather_bytes += s.gather_bytes;
+        st_.gather_ce_bytes += s.gather_ce_bytes;
+        st_.gather_load_bytes += s.gather_load_bytes;
+        st_.h2d_other_bytes += s.h2d_other_bytes;
         st_.dma_bytes += s.dma_bytes;
         st_.static_bytes += s.static_bytes;
         st_.vertex_state_bytes += s.vertex_state_bytes;

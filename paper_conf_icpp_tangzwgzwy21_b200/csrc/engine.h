@@ -70,6 +70,8 @@ struct Options {
     uint32_t replace_k = 0;       // §3.4 data replacement: chunk swaps examined per iteration (0 = off)
     int replace_policy = 0;       // hotness counter: 0 = by algorithm, 1 = cumulative, 2 = last iteration
     int relax_mode = 0;           // SSSP/CC min update: 0 = auto, 1 = atomicMin + next bit, 2 = RED.MIN + dense finalize
+    uint64_t ce_min_run = 1ull << 20;   // gather-mode iterations: runs >= this many bytes go to the copy engines (0 = off)
+    uint32_t gap_bridge = 256;          // gather: also load host holes <= this many bytes between pieces (0 = off)
 };
 
 struct HostGraph {
@@ -142,6 +144,7 @@ class Part {
 
   private:
     void transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsigned long long hi, int mode);
+    uint32_t plan_long_runs(const IterTotals& T);   // gather mode: the long runs for the copy engines
     Queues queues(const IterTotals& T) const;
     void free_regions();
     void layout_regions(uint64_t Ms);
@@ -226,6 +229,19 @@ class Part {
     // DMA planning scratch
     std::vector<uint32_t> rb_, re_;
     std::vector<unsigned long long> rdst_;
+    // hybrid gather: long runs by the copy engines on a second copy stream, the rest by the SM gather
+    static constexpr uint32_t kLongMax = 1u << 16;
+    unsigned long long* h_long_ = nullptr;          // mapped: (b, e, dst) x kLongMax, unordered
+    uint32_t* h_long_flag_ = nullptr;               // mapped: [0] ready, [1] count
+    uint32_t* d_long_cnt_ = nullptr;                // device: count, done
+    unsigned long long* h_lint_[2] = {};            // pinned staging of the sorted stream intervals (by parity)
+    unsigned long long* d_lint_[2] = {};            // device copies read by the gather
+    uint32_t nlint_ = 0, lint_buf_ = 0;
+    std::vector<uint32_t> lb_, le_;                  // this iteration's long runs, by stream position
+    std::vector<unsigned long long> ldst_;
+    cudaStream_t xs2_ = nullptr;
+    cudaEvent_t ce_done_[kMaxBuffers] = {}, xfer_go_[kMaxBuffers] = {}, ev_long_ = nullptr;
+    unsigned long long* d_cover_ = nullptr;          // gather: 16-byte units loaded (link bytes / 16)
     static constexpr uint32_t kPieceArcs = 4096;
     static constexpr uint32_t kRunsHostMax = 8192;
 };

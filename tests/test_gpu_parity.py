@@ -220,7 +220,8 @@ def test_load_variants_copy_wgt_validate(asc):
 
 @pytest.mark.parametrize("opt,val", [("overlap", 0), ("keep_static", 1), ("chunk_buffers", 2),
                                      ("chunk_buffers", 3), ("chunk_buffers", 8), ("gather_ctas", 1), ("static_ctas_per_sm", 1),
-                                     ("timing", 0), ("relax_mode", 1), ("relax_mode", 2)])
+                                     ("timing", 0), ("relax_mode", 1), ("relax_mode", 2), ("ce_min_run", 0),
+                                     ("ce_min_run", 2048), ("gap_bridge", 0), ("gap_bridge", 4096)])
 def test_options_do_not_change_results(asc, opt, val):
     """Tuning knobs change scheduling only: results, records and bytes stay bit-exact."""
     g = gg.rmat(12, seed=14, weights=True)
@@ -241,7 +242,7 @@ def test_options_do_not_change_results(asc, opt, val):
         else:
             assert st["h2d_static_fill_bytes"] == p.static_bytes
     defaults = {"overlap": 1, "keep_static": 0, "chunk_buffers": 0, "gather_ctas": 0, "static_ctas_per_sm": 0,
-                "timing": 1, "relax_mode": 0}
+                "timing": 1, "relax_mode": 0, "ce_min_run": 1 << 20, "gap_bridge": 256}
     asc.set_option(opt, defaults[opt])
 
 
@@ -426,3 +427,45 @@ def test_relax_modes_resident_and_out_of_core(asc, mode, algo):
             assert st["h2d_payload_bytes"] == ref.h2d_payload
     finally:
         asc.set_option("relax_mode", 0)
+
+
+@pytest.mark.parametrize("shift", [0, 1])
+@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pr"])
+def test_hybrid_gather_copy_engine_long_runs(asc, algo, shift):
+    """Gather-mode iterations with long runs: runs >= CE_MIN_RUN bytes go to the copy engines on a
+    second copy stream while the SM gather (skipping their vertices, bridging small holes) moves the
+    rest of each chunk window. Small windows cut long runs across chunks; the host array may start
+    off a 16-byte boundary. Values, records and bytes equal the oracle's; the CE path must run."""
+    cfg = ALGO_GRAPHS[algo]
+    g = gg.rmat(cfg["scale"], seed=23, weights=cfg["weights"])
+    buf = np.zeros(g.nbr.size + 8, dtype=np.uint32)
+    base = (-(buf.ctypes.data // 4)) % 4
+    nbr = buf[base + shift: base + shift + g.nbr.size]
+    nbr[:] = g.nbr
+    src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+    iters = 6 if algo == "pr" else 0
+    ce_total = 0
+    for cap, ce in ((3000, 1024), (1 << 16, 256), (1 << 16, 4096)):
+        asc.load_csr(g.off, nbr, pairs=g.pairs, symmetric=True)
+        asc.set_option("chunk_cap", cap)
+        asc.set_option("xfer_mode", 1)
+        asc.set_option("ce_min_run", ce)
+        asc.set_option("gap_bridge", 64)
+        asc.set_budget(g.csr_bytes // 4, 0.3)
+        asc.run(algo, src, iters)
+        st, its = asc.stats()
+        res = asc.get_result().copy()
+        for k, v in (("chunk_cap", 0), ("xfer_mode", 0), ("ce_min_run", 1 << 20), ("gap_bridge", 256)):
+            asc.set_option(k, v)
+        p = oracle.placer(g.off, g.b_e, g.csr_bytes // 4, 0.3)
+        ref = _oracle(algo, g, src, p.s, max_iters=iters)
+        _check_records(its, ref)
+        assert st["h2d_payload_bytes"] == ref.h2d_payload == st["gather_bytes"]
+        if algo == "pr":
+            _pr_ok(res, ref.values)
+        else:
+            np.testing.assert_array_equal(res, ref.values)
+        ce_total += st["gather_ce_bytes"]
+        # the SM gather loads at least the payload it moves (cover units, bridged holes)
+        assert st["gather_load_bytes"] >= st["gather_bytes"] - st["gather_ce_bytes"]
+    assert ce_total > 0
