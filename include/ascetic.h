@@ -68,7 +68,9 @@ typedef enum {
     ASCETIC_OPT_OVERLAP = 4,       /* 1 (default) = static compute overlaps the transfer; 0 = serialize (ablation, Fig. 8) */
     ASCETIC_OPT_KEEP_STATIC = 5,   /* 1 = keep the Static Region filled across runs (fill counted once) ; default 0 */
     ASCETIC_OPT_HUB_DEGREE = 6,    /* hit-queue degree at/above which a list is split across CTAs (default 2048) */
-    ASCETIC_OPT_TIMING = 7,        /* 1 (default) = per-iteration phase timing with CUDA events */
+    ASCETIC_OPT_TIMING = 7,        /* CUDA-event phase timing: 1 (default) = per-phase spans in iterations with >= 2^20
+                                      active arcs or >= 4 MiB of misses, one span (the iteration) otherwise;
+                                      2 = every phase of every iteration; 0 = off */
     ASCETIC_OPT_GATHER_CTAS = 8,   /* persistent CTAs of the zero-copy gather; 0 (default) = 512 / b_e (~1 MiB in flight) */
     ASCETIC_OPT_CHUNK_BUFFERS = 9, /* On-demand Region C split into N buffers of C/N (2..8; 0 = auto (default): 3, or 2
                                     when C/3 < 4 MiB); set before set_budget */
@@ -120,9 +122,10 @@ typedef enum {
     ASCETIC_OPT_CE_MIN_RUN = 21,     /* bytes (default 1 MiB, 0 = off): in gather-mode iterations the miss runs of at
                                       least this many bytes are copied by the copy engines (one cudaMemcpyAsync per
                                       run piece, on a second copy stream) while the SM gather moves the rest */
-    ASCETIC_OPT_GAP_BRIDGE = 22      /* bytes (default 256, 0 = off): the SM gather also loads (and discards) host holes
-                                      of at most this size between consecutive pieces, so one contiguous read
-                                      replaces two (the link charges per contiguous region) */
+    ASCETIC_OPT_GAP_BRIDGE = 22      /* bytes (default 0 = off): the SM gather also loads (and discards) host holes of
+                                      at most this size between consecutive pieces of a warp's group, so the warp
+                                      reads one contiguous block instead of two. Measured: no gain at 64 B, -1 % at
+                                      256 B, -2..3 % at 1 KiB on C2/C4 (the link is not charged per block) */
 } ascetic_option;
 
 typedef struct {

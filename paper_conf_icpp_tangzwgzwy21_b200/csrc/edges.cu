@@ -679,11 +679,12 @@ __device__ __forceinline__ uint4 ld_host16(const uint4* p) {
 // piece), each piece's cover units are enumerated across the warp (a unit shared by two
 // vertices of one piece is loaded once), and every lane stores the piece words its unit holds
 // at their stream position. `hoff` = the host array's byte offset from its 16-byte-aligned base.
-// Gap bridging: SM reads of host memory are charged per contiguous region (tools/zc_gran.cu: ~90 M
-// random regions/s whatever their size up to 512 B), and consecutive miss runs are mostly separated by
-// a few bytes (profiles/r02/run_profile_c4.log: 89-96 % of the gaps < 16 B), so a piece whose next
-// piece starts at most `gap_words` later also loads the hole units between them (not stored): the
-// warp instruction then reads one contiguous block instead of two.
+// Gap bridging (option, off by default): a piece whose next piece starts at most `gap_words` later
+// also loads the hole units between them (not stored), so the warp instruction reads one contiguous
+// block instead of two. Random SM reads run at ~90 M regions/s up to 512 B each (tools/zc_gran.cu)
+// and 89-96 % of the gaps between C4's miss runs are < 16 B (profiles/r02/run_profile_c4.log), but
+// bridging did not raise the rate (profiles/r02/gather_ab_c4.log): regions adjacent inside one
+// instruction are not what the link charges for.
 // Long runs: stream intervals lint[2i, 2i+1) (sorted, disjoint; whole vertices) go through the copy
 // engines instead (Part::transfer_chunk); their vertices are skipped here.
 template <int BE, int NG>

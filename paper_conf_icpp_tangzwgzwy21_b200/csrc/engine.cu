@@ -35,6 +35,14 @@ namespace ascetic {
 
 enum { ALG_BFS = 0, ALG_SSSP = 1, ALG_CC = 2, ALG_PR = 3, ALG_PRD = 4 };
 
+// ASCETIC_TRACE (the one environment knob; tracing only, never a kernel choice): 1 = print every timed
+// span of a run to stderr (rank, iteration, phase, start and end ms), 2 = also split the static-hit
+// phase by degree bucket. Either forces per-phase spans in every iteration.
+static int trace_level() {
+    static const int lv = [] { const char* e = std::getenv("ASCETIC_TRACE"); return e ? std::atoi(e) : 0; }();
+    return lv;
+}
+
 // ------------------------------------------------------------------ placer / partition
 Placement place(const uint64_t* off, uint64_t n, uint32_t b_e, uint64_t budget, double frac) {
     Placement p;
@@ -444,15 +452,15 @@ Queues Part::queues(const IterTotals& T) const {
     return q;
 }
 
-cudaEvent_t Part::mark(cudaStream_t s) {
-    if (!timing_) return nullptr;
+cudaEvent_t Part::mark(cudaStream_t s, bool always) {
+    if (!timing_ || (!fine_ && !always)) return nullptr;
     cudaEvent_t e = pool_.get();
     CK(cudaEventRecord(e, s));
     return e;
 }
 
 void Part::span(cudaEvent_t a, cudaStream_t s, uint32_t t, int ph, int sub) {
-    if (!timing_) return;
+    if (!timing_ || !a) return;
     cudaEvent_t e = pool_.get();
     CK(cudaEventRecord(e, s));
     spans_.push_back({a, e, t, ph, sub});
@@ -607,6 +615,7 @@ void Part::begin(int algo, uint32_t source, uint32_t max_iters, bool timing) {
     pool_.reset();
     spans_.clear();
     host_s_ = 0.0;
+    fine_ = true;
     launches0_ = g_launches;
     ev_start_ = pool_.get(); ev_fill0_ = pool_.get(); ev_fill1_ = pool_.get();
     CK(cudaEventRecord(ev_start_, cs_));
@@ -654,7 +663,7 @@ void Part::classify(uint32_t t) {
     ca.tile_agg = d_tile_agg_; ca.tile_incl = d_tile_incl_; ca.tile_flag = d_tile_flag_; ca.epoch = epoch_;
     ca.tot = d_tot_; ca.host_tot = h_tot_;
     ca.host_runs = h_runs_; ca.host_runs_cap = kRunsHostMax;
-    cudaEvent_t e0 = mark(cs_);
+    cudaEvent_t e0 = mark(cs_, true);   // every iteration: its start marks the iteration's wall time
     launch_classify(ca, cs_);
     CK(cudaGetLastError());
     span(e0, cs_, t, PH_CLS);
@@ -693,6 +702,10 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     is.s_static = T.nS;
     const DevState d = dev_state(t);
     const Queues q = queues(T);
+    // per-phase spans only for iterations big enough for them to matter (TIMING = 1): a small
+    // iteration keeps its classify span (its wall time); its ~10 event pairs would cost more device
+    // and host time than its kernels (C1: 0.28 ms device + 0.27 ms host per 1 ms run)
+    fine_ = o_.timing >= 2 || trace_level() > 0 || T.active_arcs >= (1ull << 20) || T.miss_arcs * b_e >= (4ull << 20);
     if (algo_ == ALG_PR) CK(cudaMemsetAsync(d_sum_ + vlo_, 0, (vhi_ - vlo_) * sizeof(unsigned long long), cs_));
     // ---- Static Computing, overlapping the transfer, on its own stream so
     // the on-demand kernels (and through them the chunk buffers' reuse) never queue behind it;
@@ -718,8 +731,7 @@ void Part::expand(uint32_t t, const IterTotals& T) {
         // persistent grid: 4 CTAs/SM leave room for the on-demand kernels; an iteration without
         // misses (resident lists only) takes every slot
         const int cps = o_.static_ctas_per_sm > 0 ? o_.static_ctas_per_sm : (T.miss_arcs ? 4 : 8);
-        static const bool split = [] { const char* e = std::getenv("ASCETIC_TRACE"); return e && e[0] == '2'; }();
-        if (split && timing_) {   // timeline of the three degree buckets (dev: ASCETIC_TRACE=2)
+        if (trace_level() == 2 && timing_) {   // timeline of the three degree buckets
             for (int b = 0; b < 3; ++b) {
                 cudaEvent_t e0 = mark(ss_);
                 launch_static(algo_, d, q, d_static_, b == 0 ? T.n_small : 0, b == 1 ? T.n_med : 0,
@@ -997,13 +1009,13 @@ void Part::end() {
     CK(cudaEventElapsedTime(&ms, ev_start_, ev_end));
     CK(cudaEventElapsedTime(&fill_ms, ev_fill0_, ev_fill1_));
     double ph[PH_N] = {};
-    const char* trace = std::getenv("ASCETIC_TRACE");
+    const bool trace = trace_level() > 0;
     static const char* kPhName[PH_N] = {"classify", "static", "ondemand", "gather", "dma", "finalize", "exchange",
                                         "replace"};
     for (const Span& sp : spans_) {
         float a = 0.f;
         CK(cudaEventElapsedTime(&a, sp.a, sp.b));
-        if (trace && (trace[0] == '1' || trace[0] == '2')) {   // timeline: rank iter kernel-class start end (ms from run start)
+        if (trace) {   // timeline: rank iter kernel-class start end (ms from run start)
             float s0 = 0.f;
             CK(cudaEventElapsedTime(&s0, ev_start_, sp.a));
             static const char* kSub[4] = {"", "_small", "_med", "_hub"};
@@ -1284,7 +1296,10 @@ void Engine::set_option(int opt, int64_t value) {
             if (value < 32 || value > (1ll << 30)) throw Error(ASCETIC_EINVAL, "hub degree must be in [32, 2^30]");
             o_.hub_deg = (uint32_t)value;
             break;
-        case ASCETIC_OPT_TIMING: o_.timing = value ? 1 : 0; break;
+        case ASCETIC_OPT_TIMING:
+            if (value < 0 || value > 2) throw Error(ASCETIC_EINVAL, "timing: 0 = off, 1 = auto, 2 = every phase");
+            o_.timing = (int)value;
+            break;
         case ASCETIC_OPT_GATHER_CTAS:
             if (value < 0 || value > 65535) throw Error(ASCETIC_EINVAL, "gather CTAs must be in [0, 65535]");
             o_.gather_ctas = (int)value;

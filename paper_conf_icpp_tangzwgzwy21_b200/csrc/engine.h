@@ -71,7 +71,8 @@ struct Options {
     int replace_policy = 0;       // hotness counter: 0 = by algorithm, 1 = cumulative, 2 = last iteration
     int relax_mode = 0;           // SSSP/CC min update: 0 = auto, 1 = atomicMin + next bit, 2 = RED.MIN + dense finalize
     uint64_t ce_min_run = 1ull << 20;   // gather-mode iterations: runs >= this many bytes go to the copy engines (0 = off)
-    uint32_t gap_bridge = 256;          // gather: also load host holes <= this many bytes between pieces (0 = off)
+    uint32_t gap_bridge = 0;            // gather: also load host holes <= this many bytes between pieces (0 = off;
+                                        // measured no gain: C2/C4 A/B, profiles/r02/gather_ab_c4.log)
 };
 
 struct HostGraph {
@@ -120,7 +121,7 @@ class Part {
     uint32_t* next_buf(int b) const { return b ? d_next2_ : d_next_; }
     void end();
     void span(cudaEvent_t a, cudaStream_t s, uint32_t t, int ph, int sub = 0);   // close a timed span
-    cudaEvent_t mark(cudaStream_t s);                               // open a timed span
+    cudaEvent_t mark(cudaStream_t s, bool always = false);          // open a timed span
 
     cudaStream_t cs() const { return cs_; }
     const unsigned long long* dev_off() const { return d_off_; }
@@ -156,6 +157,7 @@ class Part {
     int sm_count_;
     int algo_ = 0;
     bool timing_ = true;
+    bool fine_ = true;   // this iteration records per-phase spans
     // device vertex state
     uint32_t nwords_ = 0, ntiles_ = 0;
     unsigned long long* d_off_ = nullptr;

@@ -220,7 +220,7 @@ def test_load_variants_copy_wgt_validate(asc):
 
 @pytest.mark.parametrize("opt,val", [("overlap", 0), ("keep_static", 1), ("chunk_buffers", 2),
                                      ("chunk_buffers", 3), ("chunk_buffers", 8), ("gather_ctas", 1), ("static_ctas_per_sm", 1),
-                                     ("timing", 0), ("relax_mode", 1), ("relax_mode", 2), ("ce_min_run", 0),
+                                     ("timing", 0), ("timing", 2), ("relax_mode", 1), ("relax_mode", 2), ("ce_min_run", 0),
                                      ("ce_min_run", 2048), ("gap_bridge", 0), ("gap_bridge", 4096)])
 def test_options_do_not_change_results(asc, opt, val):
     """Tuning knobs change scheduling only: results, records and bytes stay bit-exact."""
@@ -242,7 +242,7 @@ def test_options_do_not_change_results(asc, opt, val):
         else:
             assert st["h2d_static_fill_bytes"] == p.static_bytes
     defaults = {"overlap": 1, "keep_static": 0, "chunk_buffers": 0, "gather_ctas": 0, "static_ctas_per_sm": 0,
-                "timing": 1, "relax_mode": 0, "ce_min_run": 1 << 20, "gap_bridge": 256}
+                "timing": 1, "relax_mode": 0, "ce_min_run": 1 << 20, "gap_bridge": 0}
     asc.set_option(opt, defaults[opt])
 
 
@@ -455,7 +455,7 @@ def test_hybrid_gather_copy_engine_long_runs(asc, algo, shift):
         asc.run(algo, src, iters)
         st, its = asc.stats()
         res = asc.get_result().copy()
-        for k, v in (("chunk_cap", 0), ("xfer_mode", 0), ("ce_min_run", 1 << 20), ("gap_bridge", 256)):
+        for k, v in (("chunk_cap", 0), ("xfer_mode", 0), ("ce_min_run", 1 << 20), ("gap_bridge", 0)):
             asc.set_option(k, v)
         p = oracle.placer(g.off, g.b_e, g.csr_bytes // 4, 0.3)
         ref = _oracle(algo, g, src, p.s, max_iters=iters)
