@@ -285,7 +285,7 @@ def main():
         asc.set_device(local)
         budget = gg.config_budget(args.config, g)
 
-    asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True)
+    asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True, sorted_rows=True)   # generator rows are sorted
     asc.set_budget(budget)
     asc.set_option("xfer_mode", args.xfer)
     asc.set_option("sparse_exchange", args.sparse_exchange)
@@ -404,7 +404,7 @@ def main():
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record()
         h0 = time.perf_counter()
-        asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True)
+        asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True, sorted_rows=True)
         h1 = time.perf_counter()
         asc.set_budget(budget)
         asc.set_option("xfer_mode", args.xfer)
@@ -441,7 +441,7 @@ def main():
         nbr_pg = np.empty_like(g.nbr)                   # plain (pageable) numpy memory
         np.copyto(nbr_pg, g.nbr)
         t0 = time.perf_counter()
-        asc.load_csr(g.off, nbr_pg, pairs=g.pairs, symmetric=True)
+        asc.load_csr(g.off, nbr_pg, pairs=g.pairs, symmetric=True, sorted_rows=True)
         pin_ms = (time.perf_counter() - t0) * 1e3
         asc.set_budget(budget)
         torch.cuda.synchronize()
@@ -458,7 +458,7 @@ def main():
                                 "pinned_bytes": int(g.nbr.nbytes),
                                 "note": "first call with pageable arrays: load_csr (page-locking the edge "
                                         "array) + one run, GTEPS over both"}
-        asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True)   # unpins nbr_pg
+        asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True, sorted_rows=True)   # unpins nbr_pg
         del nbr_pg
 
     # ---- CPU baseline: the oracle as it stands, bounded sample, rank 0 at N=1 only

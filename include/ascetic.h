@@ -56,7 +56,9 @@ enum {
     ASCETIC_SYMMETRIC = 1u,   /* caller asserts both directions are stored; required for CC and PR */
     ASCETIC_COPY = 2u,        /* copy into library-owned pinned memory instead of pinning in place */
     ASCETIC_VALIDATE = 4u,    /* O(m) check that every neighbour id < n */
-    ASCETIC_PAIRS = 8u        /* nbr holds 2m uint32: interleaved (id, weight) per arc */
+    ASCETIC_PAIRS = 8u,       /* nbr holds 2m uint32: interleaved (id, weight) per arc */
+    ASCETIC_SORTED = 16u      /* caller asserts every row lists its neighbours in ascending id order (checked
+                                 with ASCETIC_VALIDATE); lets PR pull in L2-sized neighbour-id slices */
 };
 
 /* Tuning knobs (ascetic_set_option). None changes what is computed or the
@@ -122,10 +124,14 @@ typedef enum {
     ASCETIC_OPT_CE_MIN_RUN = 21,     /* bytes (default 1 MiB, 0 = off): in gather-mode iterations the miss runs of at
                                       least this many bytes are copied by the copy engines (one cudaMemcpyAsync per
                                       run piece, on a second copy stream) while the SM gather moves the rest */
-    ASCETIC_OPT_GAP_BRIDGE = 22      /* bytes (default 0 = off): the SM gather also loads (and discards) host holes of
+    ASCETIC_OPT_GAP_BRIDGE = 22,     /* bytes (default 0 = off): the SM gather also loads (and discards) host holes of
                                       at most this size between consecutive pieces of a warp's group, so the warp
                                       reads one contiguous block instead of two. Measured: no gain at 64 B, -1 % at
                                       256 B, -2..3 % at 1 KiB on C2/C4 (the link is not charged per block) */
+    ASCETIC_OPT_PR_SEGMENT = 23      /* bytes (default 64 MiB, 0 = off): with ASCETIC_SORTED rows and contrib (4n bytes)
+                                      above 1.5x this, the resident (static) PR pull runs in J = ceil(4n / this)
+                                      passes over neighbour-id slices, capped at the static rows' mean degree / 8,
+                                      so each pass's contrib gathers hit L2 */
 } ascetic_option;
 
 typedef struct {
@@ -179,6 +185,7 @@ typedef struct {
     uint64_t gather_ce_bytes;     /* part of gather_bytes moved by the copy engines (long runs, CE_MIN_RUN) */
     uint64_t gather_load_bytes;   /* host bytes the SM gather loaded: 16-byte cover units incl. bridged holes
                                      (vs gather_bytes - gather_ce_bytes of payload: the over-fetch) */
+    uint64_t pr_segment_passes;   /* PR: neighbour-id slices of the static pull (0 = unsegmented) */
 } ascetic_stats_t;
 
 typedef struct {
@@ -214,8 +221,8 @@ typedef struct {
  * unmodified until ascetic_unload() or the next load_csr. Memory already page-locked
  * (cudaHostAlloc / torch pin_memory) is used as is (pinned off uploads at the link's rate).
  * With ASCETIC_COPY the library keeps private copies of both.
- * Errors: EINVAL (off[0] != 0, non-monotone off, off[n] != m, ids >= n with VALIDATE,
- * wgt with PAIRS), EHOSTMEM (pinning), ENOMEM/ECUDA (device offsets).
+ * Errors: EINVAL (off[0] != 0, non-monotone off, off[n] != m, ids >= n or (with SORTED) a row out of
+ * order with VALIDATE, wgt with PAIRS), EHOSTMEM (pinning), ENOMEM/ECUDA (device offsets).
  */
 int ascetic_load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_t* nbr,
                      const uint32_t* wgt, uint32_t flags);

@@ -32,13 +32,13 @@ OK, EINVAL, ESTATE, ENOMEM, EHOSTMEM, ECUDA, ENCCL, EUNSUPPORTED = 0, -1, -2, -3
 STATUS = {0: "OK", -1: "EINVAL", -2: "ESTATE", -3: "ENOMEM", -4: "EHOSTMEM", -5: "ECUDA", -6: "ENCCL",
           -7: "EUNSUPPORTED"}
 ALGOS = {"bfs": 0, "sssp": 1, "cc": 2, "pr": 3, "prd": 4}
-SYMMETRIC, COPY, VALIDATE, PAIRS = 1, 2, 4, 8
+SYMMETRIC, COPY, VALIDATE, PAIRS, SORTED = 1, 2, 4, 8, 16
 OPTIONS = {"chunk_cap": 1, "xfer_mode": 2, "dma_min_run": 3, "overlap": 4, "keep_static": 5,
            "hub_degree": 6, "timing": 7, "gather_ctas": 8, "chunk_buffers": 9, "static_ctas_per_sm": 10,
            "prefetch": 11, "repartition": 12, "static_placement": 13, "replace_chunks": 14,
            "replace_policy": 15, "placement_seed": 16, "prd_tol_ppm": 17,
            "fused_exchange": 18, "sparse_exchange": 19, "relax_mode": 20,
-           "ce_min_run": 21, "gap_bridge": 22}
+           "ce_min_run": 21, "gap_bridge": 22, "pr_segment": 23}
 INF = 0xFFFFFFFF
 
 
@@ -66,7 +66,8 @@ class Stats(ctypes.Structure):
                 ("swaps_total", ctypes.c_uint64), ("time_replace_s", ctypes.c_double),
                 ("sparse_exchanges", ctypes.c_uint64), ("sparse_exchange_bytes", ctypes.c_uint64),
                 ("chunk_buffers", ctypes.c_uint32), ("reserved0", ctypes.c_uint32),
-                ("gather_ce_bytes", ctypes.c_uint64), ("gather_load_bytes", ctypes.c_uint64)]
+                ("gather_ce_bytes", ctypes.c_uint64), ("gather_load_bytes", ctypes.c_uint64),
+                ("pr_segment_passes", ctypes.c_uint64)]
 
 
 class IterStats(ctypes.Structure):
@@ -125,8 +126,9 @@ def set_device(device: int) -> None:
 
 
 def load_csr(off: np.ndarray, nbr: np.ndarray, wgt: np.ndarray | None = None, *, symmetric: bool = True,
-             pairs: bool = False, copy: bool = False, validate: bool = False) -> None:
-    """off: uint64[n+1]; nbr: uint32[m] (or [2m] (id,w) pairs with pairs=True); wgt: uint32[m] or None."""
+             pairs: bool = False, copy: bool = False, validate: bool = False, sorted_rows: bool = False) -> None:
+    """off: uint64[n+1]; nbr: uint32[m] (or [2m] (id,w) pairs with pairs=True); wgt: uint32[m] or None.
+    sorted_rows asserts ascending neighbour ids in every row (ASCETIC_SORTED)."""
     if off.dtype != np.uint64 or not off.flags.c_contiguous:
         raise TypeError("off must be a C-contiguous uint64 array")
     if nbr.dtype != np.uint32 or not nbr.flags.c_contiguous:
@@ -134,7 +136,7 @@ def load_csr(off: np.ndarray, nbr: np.ndarray, wgt: np.ndarray | None = None, *,
     n = off.size - 1
     m = nbr.size // 2 if pairs else nbr.size
     flags = (SYMMETRIC if symmetric else 0) | (COPY if copy else 0) | (VALIDATE if validate else 0) | \
-            (PAIRS if pairs else 0)
+            (PAIRS if pairs else 0) | (SORTED if sorted_rows else 0)
     wp = None
     if wgt is not None:
         if wgt.dtype != np.uint32 or wgt.size != m:

@@ -135,6 +135,11 @@ void launch_init(int algo, const DevState& d, uint32_t source, cudaStream_t s);
 void launch_static(int algo, const DevState& d, const Queues& q, const void* static_base,
                    uint32_t n_small, uint32_t n_med, uint32_t n_hub, uint32_t n_pieces,
                    uint32_t piece_arcs, int max_ctas, cudaStream_t s);
+// PR static pull in `passes` neighbour-id slices (contrib slice L2-resident per pass); small rows unsegmented;
+// cur_med[n_med], cur_hub[npieces]: per-row / per-piece cursors (scratch). Front prefix only (no slot remap).
+void launch_static_pr_seg(const DevState& d, const Queues& q, const void* sbase, uint32_t ns, uint32_t nm, uint32_t nh,
+                          uint32_t npieces, uint32_t piece, uint32_t passes, uint32_t* cur_med, uint32_t* cur_hub,
+                          int max_ctas, cudaStream_t s);
 void launch_ondemand(int algo, const DevState& d, const Queues& q,
                      const void* chunk, unsigned long long lo, unsigned long long hi, cudaStream_t s);
 // zero-copy gather of miss-stream arcs [lo, hi) into chunk; skips the vertices inside the sorted long

@@ -16,6 +16,7 @@
 //    queue's 64-bit prefix (one global binary search per CTA).
 //  * the gather is a zero-copy SM copy: host arcs are read through the mapped pinned
 //    CSR with the same arc->source map, so the host never needs the request list.
+#include <algorithm>
 #include <cstdlib>
 #include <type_traits>
 
@@ -484,6 +485,84 @@ __global__ void __launch_bounds__(256) k_static_hub(DevState d, const uint32_t* 
             }
             __syncthreads();
         }
+    }
+}
+
+// ------------------------------------------------------------------ PR pull, column-segmented
+// When contrib (4n bytes) is larger than L2, a pull row's 4-byte contrib gathers each fetch a 32-byte
+// DRAM sector (friendster-shaped resident PR: ~7x sector amplification, DRAM-saturated at 111 G
+// arcs/s). Segmented pull: J passes, pass j gathers only neighbours in [lo_id, hi_id), a slice of
+// contrib that stays L2-resident, so its gathers hit. Rows are sorted by neighbour id, so each row's
+// pass-j arcs are the next contiguous stretch of its list: a per-row cursor (indexed by hit-queue
+// position; per piece for hubs) resumes where pass j-1 stopped — every arc is read once over all
+// passes, plus one boundary probe per row and pass. Partial sums are added in 2^-62 fixed point
+// (rows: owner-exclusive; hub pieces: integer atomics), so the order of passes and pieces does not
+// change a bit of the result. Small rows (< 32 arcs) keep the unsegmented kernel.
+template <bool FIRST>
+__global__ void __launch_bounds__(256) k_static_med_pr_seg(DevState d, const uint32_t* __restrict__ q, uint32_t nq,
+                                                           const uint32_t* __restrict__ sbase, uint32_t* __restrict__ cur,
+                                                           uint32_t hi_id) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    for (uint32_t w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < nq; w += nwarps) {
+        const uint32_t u = __ldg(q + w);
+        const unsigned long long a0 = __ldg(d.off + u) - d.static_arc0, a1 = __ldg(d.off + u + 1) - d.static_arc0;
+        unsigned long long p = a0 + (FIRST ? 0u : cur[w]);
+        double acc = 0.0;
+        while (p < a1) {
+            const unsigned long long e = p + lane;
+            const uint32_t id = e < a1 ? ld_stream(sbase + e) : 0xFFFFFFFFu;
+            const bool in = id < hi_id;                  // ids ascend: the segment's arcs are a prefix
+            if (in) acc += pr_in(d, id);
+            const uint32_t taken = __popc(__ballot_sync(FULL, in));
+            p += taken;
+            if (taken < 32) break;
+        }
+        acc = warp_sum_d(acc);
+        if (lane == 0) {
+            cur[w] = (uint32_t)(p - a0);
+            if (acc != 0.0) d.sum[u] += to_fx(acc);
+        }
+    }
+}
+
+template <bool FIRST>
+__global__ void __launch_bounds__(256) k_static_hub_pr_seg(DevState d, const uint32_t* __restrict__ hq,
+                                                           const uint32_t* __restrict__ pre, uint32_t nh,
+                                                           uint32_t npieces, uint32_t piece_arcs,
+                                                           const uint32_t* __restrict__ sbase, uint32_t* __restrict__ cur,
+                                                           uint32_t hi_id) {
+    __shared__ double s_red[8];
+    __shared__ uint32_t s_taken;
+    for (uint32_t b = blockIdx.x; b < npieces; b += gridDim.x) {
+        const uint32_t h = ub_u32(pre, nh, b) - 1;
+        const uint32_t u = __ldg(hq + h);
+        const uint32_t pidx = b - __ldg(pre + h);
+        const unsigned long long o0 = __ldg(d.off + u) - d.static_arc0, o1 = __ldg(d.off + u + 1) - d.static_arc0;
+        const unsigned long long a0 = o0 + (unsigned long long)pidx * piece_arcs;
+        const unsigned long long a1 = min(o1, a0 + piece_arcs);
+        unsigned long long p = a0 + (FIRST ? 0u : cur[b]);
+        double acc = 0.0;
+        while (p < a1) {
+            const unsigned long long e = p + threadIdx.x;
+            const uint32_t id = e < a1 ? ld_stream(sbase + e) : 0xFFFFFFFFu;
+            const bool in = id < hi_id;
+            if (in) acc += pr_in(d, id);
+            const uint32_t taken = (uint32_t)__syncthreads_count(in);
+            p += taken;
+            if (taken < blockDim.x) break;
+        }
+        acc = warp_sum_d(acc);
+        if ((threadIdx.x & 31) == 0) s_red[threadIdx.x >> 5] = acc;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            double t = 0.0;
+            for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += s_red[w];
+            cur[b] = (uint32_t)(p - a0);
+            if (t != 0.0) atomicAdd(d.sum + u, to_fx(t));
+        }
+        (void)s_taken;
+        __syncthreads();
     }
 }
 
@@ -1365,6 +1444,30 @@ void launch_static(int algo, const DevState& d, const Queues& q, const void* sba
         case SSSP: static_launch<SSSP>(d, q, sbase, ns, nm, nh, npieces, piece, max_ctas, s); break;
         case CC: static_launch<CC>(d, q, sbase, ns, nm, nh, npieces, piece, max_ctas, s); break;
         default: static_launch<PR>(d, q, sbase, ns, nm, nh, npieces, piece, max_ctas, s); break;
+    }
+}
+
+void launch_static_pr_seg(const DevState& d, const Queues& q, const void* sbase, uint32_t ns, uint32_t nm, uint32_t nh,
+                          uint32_t npieces, uint32_t piece, uint32_t passes, uint32_t* cur_med, uint32_t* cur_hub,
+                          int max_ctas, cudaStream_t s) {
+    auto cap = [&](unsigned long long b) { return (unsigned)(b < (unsigned long long)max_ctas ? b : max_ctas); };
+    const uint32_t* sb = reinterpret_cast<const uint32_t*>(sbase);
+    if (ns) { k_static_small<PR, false><<<cap((ns + 255) / 256), 256, 0, s>>>(d, q.hq_small, ns, sbase); ++g_launches; }
+    const uint64_t slice = (d.n + passes - 1) / passes;
+    for (uint32_t j = 0; j < passes; ++j) {
+        const uint32_t hi_id = (uint32_t)std::min<uint64_t>(d.n, (j + 1) * slice);
+        if (nm) {
+            if (j == 0) k_static_med_pr_seg<true><<<cap((nm + 7) / 8), 256, 0, s>>>(d, q.hq_med, nm, sb, cur_med, hi_id);
+            else k_static_med_pr_seg<false><<<cap((nm + 7) / 8), 256, 0, s>>>(d, q.hq_med, nm, sb, cur_med, hi_id);
+            ++g_launches;
+        }
+        if (nh) {
+            if (j == 0)
+                k_static_hub_pr_seg<true><<<cap(npieces), 256, 0, s>>>(d, q.hq_hub, q.hub_pre, nh, npieces, piece, sb, cur_hub, hi_id);
+            else
+                k_static_hub_pr_seg<false><<<cap(npieces), 256, 0, s>>>(d, q.hq_hub, q.hub_pre, nh, npieces, piece, sb, cur_hub, hi_id);
+            ++g_launches;
+        }
     }
 }
 

@@ -142,7 +142,7 @@ Part::~Part() {
     if (h_long_) cudaFreeHost(h_long_);
     if (h_long_flag_) cudaFreeHost(h_long_flag_);
     for (int i = 0; i < 2; ++i) { if (h_lint_[i]) cudaFreeHost(h_lint_[i]); dfree(d_lint_[i]); }
-    dfree(d_long_cnt_); dfree(d_cover_);
+    dfree(d_long_cnt_); dfree(d_cover_); dfree(d_seg_cur_);
     for (int i = 0; i < kMaxBuffers; ++i) {
         if (ce_done_[i]) cudaEventDestroy(ce_done_[i]);
         if (xfer_go_[i]) cudaEventDestroy(xfer_go_[i]);
@@ -418,6 +418,7 @@ bool Part::maybe_repartition(const IterTotals& T) {
     const uint64_t lim = off[0] + ms_new / g_.b_e;
     const uint64_t s_new = (uint64_t)(std::upper_bound(off, off + (vhi_ - vlo_) + 1, lim) - off) - 1;
     CK(cudaStreamSynchronize(xs_));   // no transfer may still target the old chunk layout
+    CK(cudaStreamSynchronize(xs2_));
     static_valid_ = false;            // chunk buffers now overlay the old static tail
     ms_cur_ = ms_new;
     s_cur_ = s_new;
@@ -468,7 +469,8 @@ void Part::span(cudaEvent_t a, cudaStream_t s, uint32_t t, int ph, int sub) {
 
 // ---- transfer engine: chunk = miss-stream arcs [lo, hi). mode 1: zero-copy SM gather over
 // the miss queue; mode 2: copy-engine DMA of the run pieces intersecting the window.
-void Part::transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsigned long long hi, int mode) {
+void Part::transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsigned long long hi, int mode,
+                          cudaStream_t xs) {
     if (mode == 1) {
         const uint32_t b_e = g_.b_e;
         // the long runs of the window go to the copy engines on the second copy stream, concurrently
@@ -502,7 +504,7 @@ void Part::transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsig
         // (measured: 64 CTAs at b_e = 8 -> same 47 GB/s, 3x faster on-demand kernels than 296)
         const int ctas = o_.gather_ctas ? o_.gather_ctas : (int)(64u * 8u / b_e);
         launch_gather(q, g_.nbr_dev, g_.m, b_e, d_chunk_[buf], lo, hi, ctas, nlint_ ? d_lint_[lint_buf_] : nullptr,
-                      nlint_, o_.gap_bridge, d_cover_, xs_);
+                      nlint_, o_.gap_bridge, d_cover_, xs);
         if (ce) {
             CK(cudaEventRecord(ce_done_[buf], xs2_));
             CK(cudaStreamWaitEvent(xs_, ce_done_[buf], 0));
@@ -521,7 +523,7 @@ void Part::transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsig
         const unsigned long long p0 = std::max(s0, lo), p1 = std::min(s1, hi);
         if (p1 <= p0) continue;
         CK(cudaMemcpyAsync(dst + (p0 - lo) * b_e, host + (a0 + (p0 - s0)) * b_e, (p1 - p0) * b_e,
-                           cudaMemcpyHostToDevice, xs_));
+                           cudaMemcpyHostToDevice, xs));
     }
 }
 
@@ -731,7 +733,29 @@ void Part::expand(uint32_t t, const IterTotals& T) {
         // persistent grid: 4 CTAs/SM leave room for the on-demand kernels; an iteration without
         // misses (resident lists only) takes every slot
         const int cps = o_.static_ctas_per_sm > 0 ? o_.static_ctas_per_sm : (T.miss_arcs ? 4 : 8);
-        if (trace_level() == 2 && timing_) {   // timeline of the three degree buckets
+        // PR with contrib beyond L2: pull in neighbour-id slices (rows must be sorted; front prefix only)
+        uint32_t passes = 1;
+        if (algo_ == ALG_PR && o_.pr_segment && (g_.flags & ASCETIC_SORTED) && !hot_ && 4ull * g_.n > o_.pr_segment * 3 / 2) {
+            const uint64_t by_l2 = (4ull * g_.n + o_.pr_segment - 1) / o_.pr_segment;
+            const uint64_t by_deg = T.nH ? T.hit_arcs / T.nH / 8 : 0;   // a pass must not cost more than it saves
+            passes = (uint32_t)std::min<uint64_t>(by_l2, by_deg);
+            if (passes >= 2) {
+                const uint64_t need = (uint64_t)T.n_med + T.n_pieces + 2;
+                if (need > seg_cur_n_) {
+                    dfree(d_seg_cur_);
+                    dalloc(&d_seg_cur_, need, &vertex_bytes_);
+                    seg_cur_n_ = need;
+                }
+            }
+        }
+        if (passes >= 2) {
+            cudaEvent_t e0 = mark(ss_);
+            launch_static_pr_seg(d, q, d_static_, T.n_small, T.n_med, T.n_hub, T.n_pieces, kPieceArcs, passes, d_seg_cur_,
+                                 d_seg_cur_ + T.n_med, cps * sm_count_, ss_);
+            CK(cudaGetLastError());
+            span(e0, ss_, t, PH_STATIC);
+            st.pr_segment_passes = passes;
+        } else if (trace_level() == 2 && timing_) {   // timeline of the three degree buckets
             for (int b = 0; b < 3; ++b) {
                 cudaEvent_t e0 = mark(ss_);
                 launch_static(algo_, d, q, d_static_, b == 0 ? T.n_small : 0, b == 1 ? T.n_med : 0,
@@ -777,25 +801,33 @@ void Part::expand(uint32_t t, const IterTotals& T) {
             for (uint32_t r = 0; r < T.n_runs; ++r) { rdst_[r] = acc; acc += g_.off[re_[r]] - g_.off[rb_[r]]; }
         }
         if (mode == 1 && o_.ce_min_run && T.n_runs && miss * b_e >= 2 * o_.ce_min_run) plan_long_runs(T);
-        if (!o_.overlap && static_pending_) CK(cudaStreamWaitEvent(xs_, static_done_, 0));   // ablation
+        if (!o_.overlap && static_pending_) {   // ablation: the transfer waits for static computing
+            CK(cudaStreamWaitEvent(xs_, static_done_, 0));
+            CK(cudaStreamWaitEvent(xs2_, static_done_, 0));
+        }
     }
     // chunks already transferred at the end of the previous iteration (PR prefetch) must be
     // exactly this iteration's first windows
     if (prefetched_ && (mode != 2 || miss != prefetch_miss_ || T.n_runs != prefetch_runs_))
         throw Error(ASCETIC_ECUDA, "internal: prefetched chunks do not match the iteration's miss stream");
     const uint64_t g0 = gchunk_;   // global chunk number of this iteration's chunk 0
+    // small chunks (two buffers of < 4 MiB) are latency-bound transfers: alternate them over both copy
+    // streams so chunk k+1's transfer runs while chunk k's is still in flight (each waits only for
+    // its own buffer's consumer); large chunks stay on one stream (each gets the whole link)
+    const bool alt = mode == 1 && nlint_ == 0 && nbuf_ == 2 && cap_ < (4ull << 20);
     for (uint32_t k = 0; k < nchunks; ++k) {
         const uint64_t gk = g0 + k;
         const int buf = (int)(gk % (uint64_t)nbuf_);
         const unsigned long long lo = (unsigned long long)k * cap_arcs;
         const unsigned long long hi = std::min(miss, lo + cap_arcs);
+        cudaStream_t xk = (alt && (gk & 1u)) ? xs2_ : xs_;
         if (k >= prefetched_) {
-            if (gk >= (uint64_t)nbuf_) CK(cudaStreamWaitEvent(xs_, consumed_[buf], 0));   // buffer reuse
-            cudaEvent_t e0 = mark(xs_);
-            transfer_chunk(q, buf, lo, hi, mode);
+            if (gk >= (uint64_t)nbuf_) CK(cudaStreamWaitEvent(xk, consumed_[buf], 0));   // buffer reuse
+            cudaEvent_t e0 = mark(xk);
+            transfer_chunk(q, buf, lo, hi, mode, xk);
             CK(cudaGetLastError());
-            span(e0, xs_, t, mode == 2 ? PH_DMA : PH_GATHER);
-            CK(cudaEventRecord(ready_[buf], xs_));
+            span(e0, xk, t, mode == 2 ? PH_DMA : PH_GATHER);
+            CK(cudaEventRecord(ready_[buf], xk));
         }
         if (mode == 2) st.dma_bytes += (hi - lo) * b_e; else st.gather_bytes += (hi - lo) * b_e;
         cudaEvent_t e0 = nullptr;
@@ -821,7 +853,7 @@ void Part::expand(uint32_t t, const IterTotals& T) {
             const unsigned long long hi = std::min(miss, lo + cap_arcs);
             if (gk >= (uint64_t)nbuf_) CK(cudaStreamWaitEvent(xs_, consumed_[buf], 0));
             cudaEvent_t e0 = mark(xs_);
-            transfer_chunk(q, buf, lo, hi, mode);
+            transfer_chunk(q, buf, lo, hi, mode, xs_);
             CK(cudaGetLastError());
             span(e0, xs_, t + 1, PH_DMA);
             CK(cudaEventRecord(ready_[buf], xs_));
@@ -1004,6 +1036,7 @@ void Part::end() {
     CK(cudaEventRecord(ev_end, cs_));
     CK(cudaStreamSynchronize(cs_));
     CK(cudaStreamSynchronize(xs_));
+    CK(cudaStreamSynchronize(xs2_));
     CK(cudaStreamSynchronize(ss_));
     float ms = 0.f, fill_ms = 0.f;
     CK(cudaEventElapsedTime(&ms, ev_start_, ev_end));
@@ -1137,6 +1170,11 @@ void Engine::load_csr(uint64_t n, uint64_t m, const uint64_t* off, const uint32_
         const uint64_t step = (flags & ASCETIC_PAIRS) ? 2 : 1;
         for (uint64_t e = 0; e < m; ++e)
             if (nbr[e * step] >= n) throw Error(ASCETIC_EINVAL, "neighbour id >= n at arc " + std::to_string(e));
+        if (flags & ASCETIC_SORTED)
+            for (uint64_t v = 0; v < n; ++v)
+                for (uint64_t e = off[v] + 1; e < off[v + 1]; ++e)
+                    if (nbr[e * step] < nbr[(e - 1) * step])
+                        throw Error(ASCETIC_EINVAL, "row " + std::to_string(v) + " is not sorted (ASCETIC_SORTED)");
     }
     if (device_ < 0) CK(cudaGetDevice(&device_));
     CK(cudaSetDevice(device_));
@@ -1344,6 +1382,10 @@ void Engine::set_option(int opt, int64_t value) {
         case ASCETIC_OPT_CE_MIN_RUN:
             if (value < 0) throw Error(ASCETIC_EINVAL, "copy-engine minimum run must be >= 0 bytes");
             o_.ce_min_run = (uint64_t)value;
+            break;
+        case ASCETIC_OPT_PR_SEGMENT:
+            if (value < 0) throw Error(ASCETIC_EINVAL, "PR segment bytes must be >= 0");
+            o_.pr_segment = (uint64_t)value;
             break;
         case ASCETIC_OPT_GAP_BRIDGE:
             if (value < 0 || value > 65536) throw Error(ASCETIC_EINVAL, "gap bridge must be in [0, 65536] bytes");

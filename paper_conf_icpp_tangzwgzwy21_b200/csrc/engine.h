@@ -71,6 +71,7 @@ struct Options {
     int replace_policy = 0;       // hotness counter: 0 = by algorithm, 1 = cumulative, 2 = last iteration
     int relax_mode = 0;           // SSSP/CC min update: 0 = auto, 1 = atomicMin + next bit, 2 = RED.MIN + dense finalize
     uint64_t ce_min_run = 1ull << 20;   // gather-mode iterations: runs >= this many bytes go to the copy engines (0 = off)
+    uint64_t pr_segment = 64ull << 20;  // PR static pull: neighbour-id slice of contrib per pass (0 = off)
     uint32_t gap_bridge = 0;            // gather: also load host holes <= this many bytes between pieces (0 = off;
                                         // measured no gain: C2/C4 A/B, profiles/r02/gather_ab_c4.log)
 };
@@ -144,7 +145,8 @@ class Part {
     std::vector<ascetic_iter_stats_t> iters;
 
   private:
-    void transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsigned long long hi, int mode);
+    void transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsigned long long hi, int mode,
+                        cudaStream_t xs);
     uint32_t plan_long_runs(const IterTotals& T);   // gather mode: the long runs for the copy engines
     Queues queues(const IterTotals& T) const;
     void free_regions();
@@ -244,6 +246,8 @@ class Part {
     cudaStream_t xs2_ = nullptr;
     cudaEvent_t ce_done_[kMaxBuffers] = {}, xfer_go_[kMaxBuffers] = {}, ev_long_ = nullptr;
     unsigned long long* d_cover_ = nullptr;          // gather: 16-byte units loaded (link bytes / 16)
+    uint32_t* d_seg_cur_ = nullptr;                  // PR segmented pull: cursors (medium rows, then hub pieces)
+    uint64_t seg_cur_n_ = 0;
     static constexpr uint32_t kPieceArcs = 4096;
     static constexpr uint32_t kRunsHostMax = 8192;
 };

@@ -63,7 +63,7 @@ def test_c3_full_pr_43_iterations(asc):
     g = gg.config_graph("c3")
     budget = gg.config_budget("c3", g)
     iters = gg.CONFIGS["c3"]["iters"]
-    asc.load_csr(g.off, g.nbr)
+    asc.load_csr(g.off, g.nbr, sorted_rows=True)          # as bench.py: the static pull runs in id slices
     asc.set_budget(budget)
     p = oracle.placer(g.off, 4, budget)
     asc.run("pr", 0, iters)
@@ -80,6 +80,7 @@ def test_c3_full_pr_43_iterations(asc):
     assert _records(its) == _records(ref.records)
     assert st["h2d_payload_bytes"] == ref.h2d_payload == iters * 4 * (g.m - int(g.off[p.s]))
     assert st["h2d_static_fill_bytes"] == p.static_bytes
+    assert st["pr_segment_passes"] >= 2
     # the run is bitwise reproducible (fixed-point sums, DESIGN R31)
     asc.run("pr", 0, iters)
     assert np.array_equal(asc.get_result().view(np.uint32), res.astype(np.float32).view(np.uint32))
@@ -89,7 +90,7 @@ def test_c4_full_cc(asc):
     """bench.py's default workload: CC on the uk-shaped graph (105 M vertices, 6.4 B arcs) at 30 %."""
     g = gg.config_graph("c4")
     budget = gg.config_budget("c4", g)
-    asc.load_csr(g.off, g.nbr)
+    asc.load_csr(g.off, g.nbr, sorted_rows=True)
     asc.set_budget(budget)
     asc.run("cc")
     st, its = asc.stats()

@@ -469,3 +469,47 @@ def test_hybrid_gather_copy_engine_long_runs(asc, algo, shift):
         # the SM gather loads at least the payload it moves (cover units, bridged holes)
         assert st["gather_load_bytes"] >= st["gather_bytes"] - st["gather_ce_bytes"]
     assert ce_total > 0
+
+
+@pytest.mark.parametrize("resident", [True, False])
+def test_pr_segmented_pull(asc, resident):
+    """PR static pull in neighbour-id slices (ASCETIC_OPT_PR_SEGMENT, sorted rows): a small slice size
+    forces several passes with per-row / per-piece cursors; ranks within tolerance of the oracle,
+    records and bytes unchanged, bitwise reproducible, and close to the unsegmented pull."""
+    g = gg.rmat(14, seed=33)
+    budget = 10 * g.csr_bytes if resident else g.csr_bytes // 3
+    res = {}
+    for seg in (0, 64 << 10):
+        asc.load_csr(g.off, g.nbr, sorted_rows=True)
+        asc.set_option("pr_segment", seg)
+        asc.set_option("hub_degree", 256)                  # hub pieces get cursors too
+        asc.set_budget(budget)
+        asc.run("pr", 0, 8)
+        st, its = asc.stats()
+        res[seg] = asc.get_result().copy()
+        if seg:
+            assert st["pr_segment_passes"] >= 2
+            asc.run("pr", 0, 8)
+            assert np.array_equal(asc.get_result().view(np.uint32), res[seg].view(np.uint32))
+        else:
+            assert st["pr_segment_passes"] == 0
+    asc.set_option("pr_segment", 64 << 20)
+    asc.set_option("hub_degree", 2048)
+    p = oracle.placer(g.off, 4, budget)
+    ref = _oracle("pr", g, 0, p.s, max_iters=8)
+    _check_records(its, ref)
+    _pr_ok(res[64 << 10], ref.values)
+    assert np.abs(res[64 << 10].astype(np.float64) - res[0]).max() <= 1e-6 * res[0].max()
+
+
+def test_sorted_flag_validated(asc):
+    g = gg.rmat(10, seed=5)
+    asc.load_csr(g.off, g.nbr, sorted_rows=True, validate=True)       # generator rows are sorted
+    bad = g.nbr.copy()
+    deg = np.diff(g.off.astype(np.int64))
+    v = int(np.argmax(deg))
+    a = int(g.off[v])
+    bad[a], bad[a + 1] = bad[a + 1], bad[a]
+    with pytest.raises(asc.AsceticError):
+        asc.load_csr(g.off, bad, sorted_rows=True, validate=True)
+    asc.unload()

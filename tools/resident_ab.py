@@ -33,11 +33,14 @@ def main():
                 graphs[w] = gg.rmat(int(a.graph[4:]), seed=2, weights=w)
         g = graphs[w]
         src = int(np.argmax(np.diff(g.off.astype(np.int64))))
-        asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True)
+        asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True, sorted_rows=True)
         asc.set_budget(int(1.2 * g.csr_bytes))
-        modes = [1, 2] if algo in ("sssp", "cc") else [0]
+        modes = [1, 2] if algo in ("sssp", "cc") else ([0, 64 << 20] if algo == "pr" else [0])
         for mode in modes:
-            asc.set_option("relax_mode", mode)
+            if algo == "pr":
+                asc.set_option("pr_segment", mode)
+            else:
+                asc.set_option("relax_mode", mode)
             best = None
             for _ in range(a.reps):
                 asc.run(algo, src, a.pr_iters if algo == "pr" else 0)
@@ -47,12 +50,13 @@ def main():
             st = best
             ex = st["time_run_s"] - st["time_fill_s"]
             rate = st["static_arcs"] / max(1e-12, st["time_static_s"])
-            print(f"{a.graph} {algo:4s} relax={mode} n={g.n} m={g.m} iters={st['iterations']} run {st['time_run_s']*1e3:8.2f} ms "
+            print(f"{a.graph} {algo:4s} {'pr_segment' if algo == 'pr' else 'relax'}={mode} passes={st['pr_segment_passes']} n={g.n} m={g.m} iters={st['iterations']} run {st['time_run_s']*1e3:8.2f} ms "
                   f"excl fill {ex*1e3:8.2f} ms static {st['time_static_s']*1e3:8.2f} ms finalize {st['time_finalize_s']*1e3:6.2f} ms "
                   f"classify {st['time_classify_s']*1e3:6.2f} ms  static {rate/1e9:6.1f} G arcs/s = "
                   f"{rate * (g.b_e + 4) / 1e12:5.2f} TB/s algorithmic  whole {st['active_arcs_total']/ex/1e9:6.1f} GTEPS excl fill",
                   flush=True)
         asc.set_option("relax_mode", 0)
+        asc.set_option("pr_segment", 64 << 20)
     asc.unload()
 
 
