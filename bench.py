@@ -372,15 +372,31 @@ def main():
         d["share_of_step"] = d["time_s"] * 1e3 / total_ms if total_ms else 0.0
     dom = max(kern, key=lambda k_: kern[k_]["time_s"])
     dk = kern[dom]
-    traffic = None
+    # the gather class = the transfer engine in gather mode: SM zero-copy gather + the copy-engine
+    # long runs beside it (same chunk windows, union time)
+    sm_b = sum(s["gather_bytes"] - s["gather_ce_bytes"] for s in per)
+    kern["gather"].update(sm_bytes=sm_b, ce_bytes=sum(s["gather_ce_bytes"] for s in per),
+                          sm_load_bytes=sum(s["gather_load_bytes"] for s in per),
+                          launches=sum(s["gather_chunks"] for s in per))
+    traffic, traffic_note = None, None
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tp):
         try:
-            traffic = json.load(open(tp)).get(args.config, {}).get(dom)
+            t_ = json.load(open(tp)).get(args.config, {}).get(dom)
         except Exception:
-            traffic = None
+            t_ = None
+        if isinstance(t_, dict) and "pcie_read_per_payload" in t_ and kern["gather"]["launches"]:
+            # host-link kernel: PCIe read bytes per launch = ncu's measured PCIe bytes per payload byte
+            # (a capture of full-window launches) x this run's SM payload per gather launch
+            traffic = t_["pcie_read_per_payload"] * sm_b / kern["gather"]["launches"]
+            traffic_note = (f"pcie__read_bytes per SM-gathered payload byte = {t_['pcie_read_per_payload']:.3f} "
+                            f"({t_.get('source', 'ncu')}) x {sm_b / kern['gather']['launches'] / 1e6:.1f} MB "
+                            "of SM payload per gather launch")
+        elif isinstance(t_, (int, float)):
+            traffic = t_
+            traffic_note = "dram__bytes_read.sum + dram__bytes_write.sum of one launch (ncu --set full)"
     roofline = {"kernel": dom, "bound": dk["bound"], "achieved": dk["achieved"], "peak": dk["peak"],
-                "unit": "GB/s", "frac": dk["frac"], "traffic": traffic,
+                "unit": "GB/s", "frac": dk["frac"], "traffic": traffic, "traffic_note": traffic_note,
                 "peak_source": ("pinned H2D cudaMemcpyAsync 1 GiB best-of-5 measured in this run"
                                 if dk["bound"] == "host_link" else f"MEASURED_PEAKS.json hbm_gbs ({hbm_src})"),
                 "per_kernel": {k_: {kk: (round(vv, 6) if isinstance(vv, float) else vv) for kk, vv in d.items()}

@@ -65,7 +65,10 @@ enum {
  * per-iteration payload bytes; they change chunking and the transfer mechanism. */
 typedef enum {
     ASCETIC_OPT_CHUNK_CAP = 1,     /* bytes; 0 = from the placer (C/2). Clamped to the placer's cap, multiple of 16 */
-    ASCETIC_OPT_XFER_MODE = 2,     /* 0 = auto, 1 = zero-copy SM gather only, 2 = copy-engine DMA of runs only */
+    ASCETIC_OPT_XFER_MODE = 2,     /* 0 = auto, 1 = zero-copy SM gather only, 2 = copy-engine DMA of runs only,
+                                      3 = span DMA where the miss stream's host span is at most 2x its payload
+                                      (windows of cap host bytes; dense ones DMA'd whole and read in place,
+                                      sparse ones gathered), else as 0 */
     ASCETIC_OPT_DMA_MIN_RUN = 3,   /* bytes: auto mode uses DMA when every run piece averages >= this */
     ASCETIC_OPT_OVERLAP = 4,       /* 1 (default) = static compute overlaps the transfer; 0 = serialize (ablation, Fig. 8) */
     ASCETIC_OPT_KEEP_STATIC = 5,   /* 1 = keep the Static Region filled across runs (fill counted once) ; default 0 */
@@ -128,10 +131,16 @@ typedef enum {
                                       at most this size between consecutive pieces of a warp's group, so the warp
                                       reads one contiguous block instead of two. Measured: no gain at 64 B, -1 % at
                                       256 B, -2..3 % at 1 KiB on C2/C4 (the link is not charged per block) */
-    ASCETIC_OPT_PR_SEGMENT = 23      /* bytes (default 64 MiB, 0 = off): with ASCETIC_SORTED rows and contrib (4n bytes)
+    ASCETIC_OPT_PR_SEGMENT = 23,     /* bytes (default 64 MiB, 0 = off): with ASCETIC_SORTED rows and contrib (4n bytes)
                                       above 1.5x this, the resident (static) PR pull runs in J = ceil(4n / this)
                                       passes over neighbour-id slices, capped at the static rows' mean degree / 8,
                                       so each pass's contrib gathers hit L2 */
+    ASCETIC_OPT_SPAN_DENSITY = 24    /* percent (default 85, 0 = off): in auto mode an iteration with >= 64 MiB of
+                                      misses whose host span is <= 2x the payload moves each window of cap host
+                                      bytes with ONE copy-engine DMA when its payload is >= this share of those
+                                      bytes (the holes ride along, ~55 GB/s for the whole window), and
+                                      gathers the sparser windows; the on-demand kernels read a DMA'd window in
+                                      place. Payload accounting is unchanged; span_link_bytes counts the holes. */
 } ascetic_option;
 
 typedef struct {
@@ -186,6 +195,9 @@ typedef struct {
     uint64_t gather_load_bytes;   /* host bytes the SM gather loaded: 16-byte cover units incl. bridged holes
                                      (vs gather_bytes - gather_ce_bytes of payload: the over-fetch) */
     uint64_t pr_segment_passes;   /* PR: neighbour-id slices of the static pull (0 = unsegmented) */
+    uint64_t span_chunks;         /* span-DMA windows (XFER_MODE 3 / auto): one DMA of a window's host bytes */
+    uint64_t span_link_bytes;     /* host bytes those DMAs moved (payload + the holes between the missed lists) */
+    uint64_t span_payload_bytes;  /* payload inside them (counted in dma_bytes / h2d_payload_bytes) */
 } ascetic_stats_t;
 
 typedef struct {

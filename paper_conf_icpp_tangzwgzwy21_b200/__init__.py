@@ -38,7 +38,8 @@ OPTIONS = {"chunk_cap": 1, "xfer_mode": 2, "dma_min_run": 3, "overlap": 4, "keep
            "prefetch": 11, "repartition": 12, "static_placement": 13, "replace_chunks": 14,
            "replace_policy": 15, "placement_seed": 16, "prd_tol_ppm": 17,
            "fused_exchange": 18, "sparse_exchange": 19, "relax_mode": 20,
-           "ce_min_run": 21, "gap_bridge": 22, "pr_segment": 23}
+           "ce_min_run": 21, "gap_bridge": 22, "pr_segment": 23,
+           "span_density": 24}
 INF = 0xFFFFFFFF
 
 
@@ -67,7 +68,8 @@ class Stats(ctypes.Structure):
                 ("sparse_exchanges", ctypes.c_uint64), ("sparse_exchange_bytes", ctypes.c_uint64),
                 ("chunk_buffers", ctypes.c_uint32), ("reserved0", ctypes.c_uint32),
                 ("gather_ce_bytes", ctypes.c_uint64), ("gather_load_bytes", ctypes.c_uint64),
-                ("pr_segment_passes", ctypes.c_uint64)]
+                ("pr_segment_passes", ctypes.c_uint64), ("span_chunks", ctypes.c_uint64),
+                ("span_link_bytes", ctypes.c_uint64), ("span_payload_bytes", ctypes.c_uint64)]
 
 
 class IterStats(ctypes.Structure):

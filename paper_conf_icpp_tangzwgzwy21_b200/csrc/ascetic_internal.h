@@ -43,6 +43,7 @@ struct IterTotals {
     uint32_t ready;          // set to 1 last (host spin target)
     uint32_t pad;
     unsigned long long nS;   // |S ∩ owned range| (static vertices of this rank in this iteration)
+    unsigned long long miss_h0, miss_h1;   // host arc span of the miss stream: off[first miss], off[last miss + 1]
 };
 
 struct ClassifyArgs {
@@ -140,8 +141,13 @@ void launch_static(int algo, const DevState& d, const Queues& q, const void* sta
 void launch_static_pr_seg(const DevState& d, const Queues& q, const void* sbase, uint32_t ns, uint32_t nm, uint32_t nh,
                           uint32_t npieces, uint32_t piece, uint32_t passes, uint32_t* cur_med, uint32_t* cur_hub,
                           int max_ctas, cudaStream_t s);
-void launch_ondemand(int algo, const DevState& d, const Queues& q,
-                     const void* chunk, unsigned long long lo, unsigned long long hi, cudaStream_t s);
+// on-demand computing of miss-stream arcs [lo, hi): chunk = the compacted stream (span_base = ~0) or
+// the host arcs [span_base, ...) verbatim (span DMA)
+void launch_ondemand(int algo, const DevState& d, const Queues& q, const void* chunk, unsigned long long lo,
+                     unsigned long long hi, unsigned long long span_base, cudaStream_t s);
+// span windows: for k in [0, nwin], the miss-stream position of host arc h0 + k * win (h1 for k = nwin)
+void launch_span_windows(const Queues& q, unsigned long long h0, unsigned long long h1, unsigned long long win,
+                         uint32_t nwin, unsigned long long* out, uint32_t* flag, cudaStream_t s);
 // zero-copy gather of miss-stream arcs [lo, hi) into chunk; skips the vertices inside the sorted long
 // stream intervals lint[2i, 2i+1) (copied by the copy engines), bridges host holes <= gap_bytes;
 // adds the number of 16-byte host units it loads to *cover

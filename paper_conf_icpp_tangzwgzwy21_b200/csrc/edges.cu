@@ -616,23 +616,34 @@ __device__ __forceinline__ uint32_t warp_map(const unsigned long long* s_pre, ui
 // Tile metadata is read straight from the queues (L1-cached), no shared memory: the kernel can
 // co-reside with any kernel whatever the SM's L1/shared split (a 33 KB/CTA staged variant could
 // not start on SMs configured for the shared-memory-free static kernels).
+// A chunk holds either the compacted miss stream [lo, hi) (arc a at a - lo), or, for a span DMA, the
+// host arcs [span_base, ...) verbatim (arc a of queue vertex k at off[v_k] + (a - pre_k) - span_base).
 template <int ALGO>
 struct TileView {
     const unsigned long long* pre;
+    const unsigned long long* src;
     const uint32_t* u;
     const DevState* d;
+    unsigned long long lo, span_base;
     __device__ __forceinline__ uint32_t vtx(uint32_t k) const { return __ldg(u + k); }
     __device__ __forceinline__ SrcVal<ALGO> val(uint32_t k) const { return src_val<ALGO>(*d, __ldg(u + k)); }
+    __device__ __forceinline__ unsigned long long at(uint32_t k, unsigned long long a) const {
+        return span_base == ~0ull ? a - lo : __ldg(src + k) + (a - __ldg(pre + k)) - span_base;
+    }
 };
 
 template <int ALGO>
 __device__ __forceinline__ void ondemand_tile(const DevState& d, const Queues& q, const void* __restrict__ chunk,
-                                              unsigned long long lo, unsigned long long hi, unsigned long long t) {
+                                              unsigned long long lo, unsigned long long hi, unsigned long long t,
+                                              unsigned long long span_base) {
     const Tile x = tile_of(q, t, lo, hi);
     TileView<ALGO> tv;
     tv.pre = q.mq_pre + x.i0;
+    tv.src = q.mq_src + x.i0;
     tv.u = q.mq + x.i0;
     tv.d = &d;
+    tv.lo = lo;
+    tv.span_base = span_base;
     const unsigned long long* s_pre = tv.pre;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const unsigned long long pw = x.t_lo + (unsigned long long)warp * 256ull;
@@ -651,11 +662,26 @@ __device__ __forceinline__ void ondemand_tile(const DevState& d, const Queues& q
             const unsigned long long a = p + lane;
             id[g] = kInf;
             c[g] = tv.val(mk);
-            if (a < pe) id[g] = ld_stream(reinterpret_cast<const uint32_t*>(chunk) + (a - lo));
+            if (a < pe) id[g] = ld_stream(reinterpret_cast<const uint32_t*>(chunk) + tv.at(mk, a));
         }
 #pragma unroll
         for (int g = 0; g < 8; ++g)
             if (id[g] != kInf) prd_push(d, id[g], c[g]);
+    } else if constexpr (ALGO == BFS) {
+        // span chunks only (compacted BFS chunks use k_ondemand_bfs): map, load ids, then visit
+        uint32_t id[8], w8[8];
+        SrcVal<ALGO> sv[8];
+        uint32_t vm = 0;
+#pragma unroll
+        for (int g = 0; g < 8; ++g) {
+            const unsigned long long p = pw + 32ull * g;
+            const uint32_t mk = warp_map(s_pre, x.cnt, k, p, lane);
+            k = __shfl_sync(FULL, mk, 31);
+            const unsigned long long a = p + lane;
+            id[g] = 0u; w8[g] = 0u; sv[g] = 0u;
+            if (a < pe) { id[g] = ld_stream(reinterpret_cast<const uint32_t*>(chunk) + tv.at(mk, a)); vm |= 1u << g; }
+        }
+        push_batch<BFS, 8>(d, sv, id, w8, vm);
     } else if constexpr (ALGO == SSSP || ALGO == CC) {
         // 3 phases over the warp's 8 groups of 32 arcs: map + chunk loads, state loads, atomics
         uint32_t id[8], cand[8], cur[8];
@@ -668,11 +694,11 @@ __device__ __forceinline__ void ondemand_tile(const DevState& d, const Queues& q
             id[g] = kInf;
             if (a < pe) {
                 if (ALGO == SSSP) {
-                    const uint2 e = ld_stream(reinterpret_cast<const uint2*>(chunk) + (a - lo));
+                    const uint2 e = ld_stream(reinterpret_cast<const uint2*>(chunk) + tv.at(mk, a));
                     id[g] = e.x;
                     cand[g] = sat_add(tv.val(mk), e.y);
                 } else {
-                    id[g] = ld_stream(reinterpret_cast<const uint32_t*>(chunk) + (a - lo));
+                    id[g] = ld_stream(reinterpret_cast<const uint32_t*>(chunk) + tv.at(mk, a));
                     cand[g] = tv.val(mk);
                 }
             }
@@ -695,7 +721,7 @@ __device__ __forceinline__ void ondemand_tile(const DevState& d, const Queues& q
             mk8[g] = warp_map(s_pre, x.cnt, k, p, lane);
             k = __shfl_sync(FULL, mk8[g], 31);
             const unsigned long long a = p + lane;
-            id8[g] = a < pe ? ld_stream(reinterpret_cast<const uint32_t*>(chunk) + (a - lo)) : kInf;
+            id8[g] = a < pe ? ld_stream(reinterpret_cast<const uint32_t*>(chunk) + tv.at(mk8[g], a)) : kInf;
         }
 #pragma unroll
         for (int g = 0; g < 8; ++g) v8[g] = id8[g] != kInf ? pr_in(d, id8[g]) : 0.0;
@@ -719,9 +745,11 @@ __device__ __forceinline__ void ondemand_tile(const DevState& d, const Queues& q
 // one CTA per 2048-arc tile of the chunk window
 template <int ALGO>
 __global__ void __launch_bounds__(256) k_ondemand_g(DevState d, Queues q, const void* __restrict__ chunk,
-                                                    unsigned long long lo, unsigned long long hi) {
+                                                    unsigned long long lo, unsigned long long hi,
+                                                    unsigned long long span_base) {
     const unsigned long long t0 = lo >> kEdgeTileShift, t1 = (hi - 1) >> kEdgeTileShift;
-    for (unsigned long long t = t0 + blockIdx.x; t <= t1; t += gridDim.x) ondemand_tile<ALGO>(d, q, chunk, lo, hi, t);
+    for (unsigned long long t = t0 + blockIdx.x; t <= t1; t += gridDim.x)
+        ondemand_tile<ALGO>(d, q, chunk, lo, hi, t, span_base);
 }
 
 // BFS needs no source: 128-bit loads straight over the chunk.
@@ -924,6 +952,38 @@ __global__ void __launch_bounds__(256) k_long_runs(const uint32_t* __restrict__ 
             __threadfence_system();
             *reinterpret_cast<volatile uint32_t*>(flag) = 1u;
         }
+    }
+}
+
+// Span windows (span-DMA iterations): window k is the host arc range [h0 + k win, h0 + (k+1) win) ∩
+// [h0, h1); out[k] = the miss-stream position of its first missed arc (lists are host-ordered like
+// the stream, so it is the first queue vertex whose list ends after the boundary, entered at the
+// boundary). One CTA; the host spins on flag (mapped memory).
+__global__ void __launch_bounds__(1024) k_span_windows(Queues q, unsigned long long h0, unsigned long long h1,
+                                                       unsigned long long win, uint32_t nwin,
+                                                       unsigned long long* out, uint32_t* flag) {
+    const uint32_t nq = q.n_missq;
+    for (uint32_t k = threadIdx.x; k <= nwin; k += blockDim.x) {
+        const unsigned long long H = k == nwin ? h1 : min(h1, h0 + (unsigned long long)k * win);
+        uint32_t L = 0, R = nq;                            // first j with end_j > H
+        while (L < R) {
+            const uint32_t mid = (L + R) >> 1;
+            const unsigned long long pre = __ldg(q.mq_pre + mid);
+            const unsigned long long end = __ldg(q.mq_src + mid) +
+                                           ((mid + 1 < nq ? __ldg(q.mq_pre + mid + 1) : q.miss_arcs) - pre);
+            if (end > H) R = mid; else L = mid + 1;
+        }
+        unsigned long long pos = q.miss_arcs;
+        if (L < nq) {
+            const unsigned long long s = __ldg(q.mq_src + L);
+            pos = __ldg(q.mq_pre + L) + (H > s ? H - s : 0ull);
+        }
+        out[k] = pos;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence_system();
+        *reinterpret_cast<volatile uint32_t*>(flag) = 1u;
     }
 }
 
@@ -1507,20 +1567,25 @@ void launch_static_bits(const DevState& d, const uint32_t* slot_of, uint32_t b_e
 }
 
 void launch_ondemand(int algo, const DevState& d, const Queues& q, const void* chunk,
-                     unsigned long long lo, unsigned long long hi, cudaStream_t s) {
+                     unsigned long long lo, unsigned long long hi, unsigned long long span_base, cudaStream_t s) {
     if (hi <= lo) return;
     const unsigned long long len = hi - lo;
+    const unsigned tiles = (unsigned)(((hi - 1) >> kEdgeTileShift) - (lo >> kEdgeTileShift) + 1);
+    if (algo == BFS && span_base != ~0ull) {
+        k_ondemand_g<BFS><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi, span_base);
+        ++g_launches;
+        return;
+    }
     if (algo == BFS) {
         k_ondemand_bfs<<<blocks_for(len, 256 * 4), 256, 0, s>>>(d, reinterpret_cast<const uint32_t*>(chunk), len);
         ++g_launches;
         return;
     }
-    const unsigned tiles = (unsigned)(((hi - 1) >> kEdgeTileShift) - (lo >> kEdgeTileShift) + 1);
     switch (algo) {
-        case SSSP: k_ondemand_g<SSSP><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
-        case CC: k_ondemand_g<CC><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
-        case PRD: k_ondemand_g<PRD><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
-        default: k_ondemand_g<PR><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi); break;
+        case SSSP: k_ondemand_g<SSSP><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi, span_base); break;
+        case CC: k_ondemand_g<CC><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi, span_base); break;
+        case PRD: k_ondemand_g<PRD><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi, span_base); break;
+        default: k_ondemand_g<PR><<<tiles, 256, 0, s>>>(d, q, chunk, lo, hi, span_base); break;
     }
     ++g_launches;
 }
@@ -1552,6 +1617,12 @@ void launch_long_runs(const uint32_t* run_b, const uint32_t* run_e, const unsign
     cudaMemsetAsync(done, 0, 4, s);
     k_long_runs<<<blocks_for(n_runs ? n_runs : 1, 256, 148u * 4u), 256, 0, s>>>(run_b, run_e, run_dst, n_runs, off,
                                                                                 min_arcs, out, cap, count, done, flag);
+    ++g_launches;
+}
+
+void launch_span_windows(const Queues& q, unsigned long long h0, unsigned long long h1, unsigned long long win,
+                         uint32_t nwin, unsigned long long* out, uint32_t* flag, cudaStream_t s) {
+    k_span_windows<<<1, 1024, 0, s>>>(q, h0, h1, win, nwin, out, flag);
     ++g_launches;
 }
 

@@ -140,6 +140,8 @@ Part::~Part() {
     if (h_tot_) cudaFreeHost(h_tot_);
     if (h_runs_) cudaFreeHost(h_runs_);
     if (h_long_) cudaFreeHost(h_long_);
+    if (h_win_) cudaFreeHost(h_win_);
+    if (h_span_flag_) cudaFreeHost(h_span_flag_);
     if (h_long_flag_) cudaFreeHost(h_long_flag_);
     for (int i = 0; i < 2; ++i) { if (h_lint_[i]) cudaFreeHost(h_lint_[i]); dfree(d_lint_[i]); }
     dfree(d_long_cnt_); dfree(d_cover_); dfree(d_seg_cur_);
@@ -222,6 +224,9 @@ void Part::alloc_vertex_state() {
     if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_EHOSTMEM, "cudaHostAlloc totals"); }
     e = cudaHostAlloc((void**)&h_runs_, 2ull * kRunsHostMax * sizeof(uint32_t), cudaHostAllocMapped | cudaHostAllocPortable);
     if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_EHOSTMEM, "cudaHostAlloc run list"); }
+    e = cudaHostAlloc((void**)&h_win_, 8ull * (kSpanWinMax + 1), cudaHostAllocMapped | cudaHostAllocPortable);
+    if (e == cudaSuccess) e = cudaHostAlloc((void**)&h_span_flag_, 8, cudaHostAllocMapped | cudaHostAllocPortable);
+    if (e != cudaSuccess) { cudaGetLastError(); throw Error(ASCETIC_EHOSTMEM, "cudaHostAlloc span windows"); }
     e = cudaHostAlloc((void**)&h_long_, 3ull * kLongMax * 8, cudaHostAllocMapped | cudaHostAllocPortable);
     if (e == cudaSuccess) e = cudaHostAlloc((void**)&h_long_flag_, 8, cudaHostAllocMapped | cudaHostAllocPortable);
     for (int i = 0; i < 2 && e == cudaSuccess; ++i) e = cudaHostAlloc((void**)&h_lint_[i], 2ull * kLongMax * 8, cudaHostAllocPortable);
@@ -579,6 +584,35 @@ uint32_t Part::plan_long_runs(const IterTotals& T) {
     return cnt;
 }
 
+// Span-DMA iteration (mode 3): windows are host ranges of cap bytes over the miss stream's host span
+// [miss_h0, miss_h1); a small kernel finds each window's first miss-stream position (mapped memory).
+// False (stay in gather mode) when the span needs more windows than the table holds.
+bool Part::plan_span_windows(const IterTotals& T) {
+    const unsigned long long cap_arcs = cap_ / g_.b_e;
+    const unsigned long long span = T.miss_h1 - T.miss_h0;
+    const uint64_t nwin = (span + cap_arcs - 1) / cap_arcs;
+    if (nwin == 0 || nwin > kSpanWinMax) return false;
+    *reinterpret_cast<volatile uint32_t*>(&h_span_flag_[0]) = 0;
+    Queues q = queues(T);
+    launch_span_windows(q, T.miss_h0, T.miss_h1, cap_arcs, (uint32_t)nwin, h_win_, h_span_flag_, cs_);
+    CK(cudaGetLastError());
+    CK(cudaEventRecord(ev_long_, cs_));
+    const volatile uint32_t* flag = h_span_flag_;
+    uint32_t spins = 0;
+    while (!flag[0]) {
+        if ((++spins & 1023u) == 0) {
+            const cudaError_t e = cudaEventQuery(ev_long_);
+            if (e == cudaSuccess) break;
+            if (e != cudaErrorNotReady) CK(e);
+        }
+    }
+    if (!flag[0]) CK(cudaEventSynchronize(ev_long_));
+    std::atomic_thread_fence(std::memory_order_acquire);
+    st.d2h_bytes += 8ull * (nwin + 1);
+    span_nwin_ = (uint32_t)nwin;
+    return true;
+}
+
 void Part::begin(int algo, uint32_t source, uint32_t max_iters, bool timing) {
     algo_ = algo;
     if (algo == ALG_PRD) {   // tau = floor(res0 * ppm / 1e6), res0 = floor(3 * 2^56 / (20 n))  (DESIGN R29)
@@ -779,12 +813,19 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     // ---- On-demand request, fragmented into chunks
     const unsigned long long cap_arcs = cap_ / b_e;
     const unsigned long long miss = T.miss_arcs;
-    const uint32_t nchunks = miss ? (uint32_t)((miss + cap_arcs - 1) / cap_arcs) : 0;
+    uint32_t nchunks = miss ? (uint32_t)((miss + cap_arcs - 1) / cap_arcs) : 0;
     int mode = 1;
     if (nchunks) {
         if (o_.xfer_mode == 2) mode = 2;
-        else if (o_.xfer_mode == 1) mode = 1;
+        else if (o_.xfer_mode == 1 || o_.xfer_mode == 3) mode = 1;
         else mode = (T.n_runs <= kRunsHostMax && miss * b_e / std::max<uint32_t>(1, T.n_runs) >= o_.dma_min_run) ? 2 : 1;
+        // span DMA: the miss stream is nearly contiguous on the host (few, small holes between its runs)
+        // (forced with XFER_MODE 3 whatever the span, for tests: sparse windows are then gathered)
+        if (mode == 1 && (o_.xfer_mode == 3 || (o_.xfer_mode == 0 && o_.span_density > 0 &&
+                                                 miss * b_e >= o_.span_min_bytes &&
+                                                 T.miss_h1 - T.miss_h0 <= 2 * miss)) &&
+            plan_span_windows(T))
+            mode = 3;
         if (mode == 2) {
             // the run list is already in mapped host memory (classify writes the first
             // kRunsHostMax runs there): no device round trip before the DMAs can be planned
@@ -815,29 +856,61 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     // streams so chunk k+1's transfer runs while chunk k's is still in flight (each waits only for
     // its own buffer's consumer); large chunks stay on one stream (each gets the whole link)
     const bool alt = mode == 1 && nlint_ == 0 && nbuf_ == 2 && cap_ < (4ull << 20);
-    for (uint32_t k = 0; k < nchunks; ++k) {
-        const uint64_t gk = g0 + k;
+    // windows: [k cap, (k+1) cap) of the miss stream, or (span mode) the host ranges of cap bytes
+    // over the miss stream's span; a dense span window is one DMA of its host bytes and the
+    // on-demand kernel reads it in place (span_base), a sparse one is gathered like mode 1
+    uint32_t nwin = nchunks;
+    if (mode == 3) nwin = span_nwin_;
+    uint32_t done = 0;
+    for (uint32_t k = 0; k < nwin; ++k) {
+        unsigned long long lo, hi, base = ~0ull, hbytes = 0;
+        int wmode = mode;
+        if (mode == 3) {
+            lo = h_win_[k];
+            hi = h_win_[k + 1];
+            if (hi <= lo) continue;                                  // a hole-only window
+            const unsigned long long H0 = T.miss_h0 + (unsigned long long)k * cap_arcs;
+            const unsigned long long H1 = std::min<unsigned long long>(T.miss_h1, H0 + cap_arcs);
+            if ((double)(hi - lo) >= o_.span_density * (double)(H1 - H0)) {
+                wmode = 3;
+                base = H0;
+                hbytes = (H1 - H0) * b_e;
+            } else {
+                wmode = 1;
+            }
+        } else {
+            lo = (unsigned long long)k * cap_arcs;
+            hi = std::min(miss, lo + cap_arcs);
+        }
+        const uint64_t gk = g0 + done;
         const int buf = (int)(gk % (uint64_t)nbuf_);
-        const unsigned long long lo = (unsigned long long)k * cap_arcs;
-        const unsigned long long hi = std::min(miss, lo + cap_arcs);
         cudaStream_t xk = (alt && (gk & 1u)) ? xs2_ : xs_;
-        if (k >= prefetched_) {
+        if (done >= prefetched_) {
             if (gk >= (uint64_t)nbuf_) CK(cudaStreamWaitEvent(xk, consumed_[buf], 0));   // buffer reuse
             cudaEvent_t e0 = mark(xk);
-            transfer_chunk(q, buf, lo, hi, mode, xk);
+            if (wmode == 3) {
+                CK(cudaMemcpyAsync(d_chunk_[buf], (const char*)g_.nbr + base * b_e, hbytes, cudaMemcpyHostToDevice, xk));
+            } else {
+                transfer_chunk(q, buf, lo, hi, wmode, xk);
+            }
             CK(cudaGetLastError());
-            span(e0, xk, t, mode == 2 ? PH_DMA : PH_GATHER);
+            span(e0, xk, t, wmode == 1 ? PH_GATHER : PH_DMA);
             CK(cudaEventRecord(ready_[buf], xk));
         }
-        if (mode == 2) st.dma_bytes += (hi - lo) * b_e; else st.gather_bytes += (hi - lo) * b_e;
+        if (wmode == 1) st.gather_bytes += (hi - lo) * b_e;
+        else st.dma_bytes += (hi - lo) * b_e;
+        if (wmode == 3) { st.span_link_bytes += hbytes; st.span_payload_bytes += (hi - lo) * b_e; ++st.span_chunks; }
         cudaEvent_t e0 = nullptr;
         CK(cudaStreamWaitEvent(cs_, ready_[buf], 0));
         e0 = mark(cs_);
-        launch_ondemand(algo_, d, q, d_chunk_[buf], lo, hi, cs_);   // On-demand Computing
+        launch_ondemand(algo_, d, q, d_chunk_[buf], lo, hi, base, cs_);   // On-demand Computing
         CK(cudaGetLastError());
         span(e0, cs_, t, PH_OND);
         CK(cudaEventRecord(consumed_[buf], cs_));
+        if (wmode == 1) ++st.gather_chunks; else ++st.dma_chunks;
+        ++done;
     }
+    nchunks = done;
     gchunk_ = g0 + nchunks;
     prefetched_ = 0;
     // ---- PR: A_t = V every iteration, so the next iteration's miss stream is this one and its
@@ -865,7 +938,6 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     is.chunks = nchunks;
     is.mode = nchunks ? (uint32_t)mode : 0u;
     st.chunks_total += nchunks;
-    if (nchunks && mode == 2) st.dma_chunks += nchunks; else if (nchunks) st.gather_chunks += nchunks;
     st.h2d_payload_bytes += is.miss_bytes;
     st.active_arcs_total += is.active_arcs;
     iters.push_back(is);
@@ -1321,7 +1393,7 @@ void Engine::set_option(int opt, int64_t value) {
             o_.chunk_cap = (uint64_t)value;
             break;
         case ASCETIC_OPT_XFER_MODE:
-            if (value < 0 || value > 2) throw Error(ASCETIC_EINVAL, "xfer mode must be 0, 1 or 2");
+            if (value < 0 || value > 3) throw Error(ASCETIC_EINVAL, "xfer mode must be 0, 1, 2 or 3");
             o_.xfer_mode = (int)value;
             break;
         case ASCETIC_OPT_DMA_MIN_RUN: o_.dma_min_run = (uint64_t)std::max<int64_t>(0, value); break;
@@ -1382,6 +1454,10 @@ void Engine::set_option(int opt, int64_t value) {
         case ASCETIC_OPT_CE_MIN_RUN:
             if (value < 0) throw Error(ASCETIC_EINVAL, "copy-engine minimum run must be >= 0 bytes");
             o_.ce_min_run = (uint64_t)value;
+            break;
+        case ASCETIC_OPT_SPAN_DENSITY:
+            if (value < 0 || value > 100) throw Error(ASCETIC_EINVAL, "span density must be a percentage in [0, 100]");
+            o_.span_density = value / 100.0;
             break;
         case ASCETIC_OPT_PR_SEGMENT:
             if (value < 0) throw Error(ASCETIC_EINVAL, "PR segment bytes must be >= 0");

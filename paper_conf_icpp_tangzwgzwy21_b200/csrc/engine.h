@@ -72,6 +72,8 @@ struct Options {
     int relax_mode = 0;           // SSSP/CC min update: 0 = auto, 1 = atomicMin + next bit, 2 = RED.MIN + dense finalize
     uint64_t ce_min_run = 1ull << 20;   // gather-mode iterations: runs >= this many bytes go to the copy engines (0 = off)
     uint64_t pr_segment = 64ull << 20;  // PR static pull: neighbour-id slice of contrib per pass (0 = off)
+    double span_density = 0.85;         // span DMA of a window when payload >= this share of its host bytes (0 = off)
+    uint64_t span_min_bytes = 64ull << 20;   // ... in iterations with at least this much payload
     uint32_t gap_bridge = 0;            // gather: also load host holes <= this many bytes between pieces (0 = off;
                                         // measured no gain: C2/C4 A/B, profiles/r02/gather_ab_c4.log)
 };
@@ -148,6 +150,7 @@ class Part {
     void transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsigned long long hi, int mode,
                         cudaStream_t xs);
     uint32_t plan_long_runs(const IterTotals& T);   // gather mode: the long runs for the copy engines
+    bool plan_span_windows(const IterTotals& T);    // span-DMA mode: the windows' miss-stream positions
     Queues queues(const IterTotals& T) const;
     void free_regions();
     void layout_regions(uint64_t Ms);
@@ -246,6 +249,10 @@ class Part {
     cudaStream_t xs2_ = nullptr;
     cudaEvent_t ce_done_[kMaxBuffers] = {}, xfer_go_[kMaxBuffers] = {}, ev_long_ = nullptr;
     unsigned long long* d_cover_ = nullptr;          // gather: 16-byte units loaded (link bytes / 16)
+    static constexpr uint32_t kSpanWinMax = 4096;
+    unsigned long long* h_win_ = nullptr;            // mapped: span windows' first miss-stream positions (nwin + 1)
+    uint32_t* h_span_flag_ = nullptr;                // mapped: [0] ready
+    uint32_t span_nwin_ = 0;
     uint32_t* d_seg_cur_ = nullptr;                  // PR segmented pull: cursors (medium rows, then hub pieces)
     uint64_t seg_cur_n_ = 0;
     static constexpr uint32_t kPieceArcs = 4096;

@@ -346,6 +346,16 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
             a.tot->miss_arcs = fin.miss_arcs;
             a.tot->n_small = fin.small; a.tot->n_med = fin.med; a.tot->n_hub = fin.hub;
             a.tot->n_missq = fin.missq; a.tot->n_runs = fin.runs; a.tot->n_pieces = fin.pieces;
+            // host span of the miss stream (the queue is in ascending id, so host order): first list's
+            // start, last list's end; the other CTAs' queue writes are visible after the done count
+            unsigned long long h0 = 0, h1 = 0;
+            if (fin.missq) {
+                const volatile unsigned long long* src = a.mq_src;
+                const volatile unsigned long long* pre = a.mq_pre;
+                h0 = src[0];
+                h1 = src[fin.missq - 1] + (fin.miss_arcs - pre[fin.missq - 1]);
+            }
+            h->miss_h0 = h0; h->miss_h1 = h1;
             __threadfence_system();
             *reinterpret_cast<volatile uint32_t*>(&h->ready) = 1u;
         }

@@ -513,3 +513,40 @@ def test_sorted_flag_validated(asc):
     with pytest.raises(asc.AsceticError):
         asc.load_csr(g.off, bad, sorted_rows=True, validate=True)
     asc.unload()
+
+
+@pytest.mark.parametrize("density", [0, 50, 85])
+@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pr", "prd"])
+def test_span_dma_windows(asc, algo, density):
+    """Span-DMA iterations (XFER_MODE 3): windows are host ranges of cap bytes over the miss stream's
+    span; windows at least `density` % full are one DMA of their host bytes read in place by the
+    on-demand kernels (span_base addressing), sparser ones are gathered. density 0 = every window
+    DMA'd. Values, records and payload bytes equal the oracle's; the span path must run."""
+    g = gg.rmat(12, seed=27, weights=(algo == "sssp"))
+    src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+    iters = 6 if algo in ("pr",) else 0
+    asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True)
+    asc.set_option("chunk_cap", 4096)
+    asc.set_option("xfer_mode", 3)
+    asc.set_option("span_density", density)
+    try:
+        asc.set_budget(g.csr_bytes // 4, 0.3)
+        asc.run(algo, src, iters)
+        st, its = asc.stats()
+        res = asc.get_result().copy()
+    finally:
+        asc.set_option("chunk_cap", 0)
+        asc.set_option("xfer_mode", 0)
+        asc.set_option("span_density", 85)
+    p = oracle.placer(g.off, g.b_e, g.csr_bytes // 4, 0.3)
+    ref = _oracle(algo, g, src, p.s, max_iters=iters)
+    _check_records(its, ref)
+    assert st["h2d_payload_bytes"] == ref.h2d_payload
+    if algo == "pr":
+        _pr_ok(res, ref.values)
+    elif algo == "prd":
+        np.testing.assert_array_equal(res, ref.values.astype(np.float32))
+    else:
+        np.testing.assert_array_equal(res, ref.values)
+    assert st["span_chunks"] > 0 and st["span_link_bytes"] >= st["span_payload_bytes"] > 0
+    assert any(i["mode"] == 3 for i in its)
