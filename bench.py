@@ -163,9 +163,10 @@ def shared_graph(config: str, barrier, local_rank: int, tag: str, alloc_local=No
     barrier()
     meta = json.load(open(base + ".json"))
     n, m, pairs = meta["n"], meta["m"], meta["pairs"]
-    off = np.memmap(meta["files"][0], dtype=np.uint64, mode="r")[: n + 1]
+    # read-write shared mappings (never written): page-locking a read-only mapping can be refused
+    off = np.memmap(meta["files"][0], dtype=np.uint64, mode="r+")[: n + 1]
     cnt = (2 if pairs else 1) * m
-    nbr = np.memmap(meta["files"][1], dtype=np.uint32, mode="r")[:cnt]
+    nbr = np.memmap(meta["files"][1], dtype=np.uint32, mode="r+")[:cnt]
     g = gg.Graph(n=n, m=m, off=off, nbr=nbr, pairs=pairs, name=config)
 
     def cleanup():
