@@ -4,7 +4,7 @@ Two processes (torch.distributed, gloo, 127.0.0.1) each take one 1D edge-balance
 range from the library's own host partitioner (ascetic_partition) and place their Static
 Region with the library's host placer (ascetic_place) under their own budget. They then
 run the per-iteration protocol of SURVEY §8(e) — classify the OWNED active vertices, push
-along owned out-lists, exchange (BFS: OR of next bitmaps by all-gather; CC: MIN all-reduce
+along owned out-lists, exchange (BFS: OR of next bitmaps by reduce-scatter-OR + all-gather; CC: MIN all-reduce
 of labels; PR: SUM of dangling partials + all-gather of contrib slices; PRD: SUM of the
 integer residual increments), finalize on the
 replicated state — with numpy standing in for the kernels and gloo for NCCL. Per-rank
@@ -46,13 +46,41 @@ def _record(t, rank, A, stat, lo, hi, deg, b_e, digest):
 
 
 def _or_allgather(mask):
-    packed = torch.from_numpy(np.packbits(mask.astype(np.uint8)))
-    parts = [torch.empty_like(packed) for _ in range(dist.get_world_size())]
-    dist.all_gather(parts, packed)
-    acc = parts[0].clone()
-    for p in parts[1:]:
-        acc |= p
-    return np.unpackbits(acc.numpy())[: mask.size].astype(bool)
+    """The BFS exchange of Comm::or_words: reduce-scatter-OR of the 32-bit bitmap words by
+    point-to-point slices (rank r owns words [r S, min((r+1) S, nw)), S = ceil(nw / P)), then an
+    all-gather of the ORed slices padded to S words."""
+    P, me = dist.get_world_size(), dist.get_rank()
+    n = mask.size
+    nw = (n + 31) // 32
+    words = np.zeros(nw * 32, dtype=np.uint8)
+    words[:n] = mask
+    words = np.packbits(words.reshape(-1, 32)[:, ::-1], axis=1)[:, ::-1].copy().view(np.uint32).reshape(-1)
+    S = (nw + P - 1) // P
+
+    def ln(r):
+        return 0 if r * S >= nw else min(S, nw - r * S)
+
+    reqs, recv = [], {}
+    for r in range(P):
+        if r == me:
+            continue
+        if ln(r):
+            reqs.append(dist.isend(torch.from_numpy(words[r * S: r * S + ln(r)].astype(np.int64)), r))
+        if ln(me):
+            recv[r] = torch.empty(ln(me), dtype=torch.int64)
+            reqs.append(dist.irecv(recv[r], r))
+    for rq in reqs:
+        rq.wait()
+    mine = words[me * S: me * S + ln(me)].astype(np.int64)
+    for r, t in recv.items():
+        mine |= t.numpy()
+    pad = np.zeros(S, dtype=np.int64)
+    pad[: ln(me)] = mine
+    parts = [torch.empty(S, dtype=torch.int64) for _ in range(P)]
+    dist.all_gather(parts, torch.from_numpy(pad))
+    allw = np.concatenate([p.numpy() for p in parts])[:nw].astype(np.uint32)
+    bits = np.unpackbits(allw.view(np.uint8).reshape(-1, 4)[:, ::-1], axis=1)[:, ::-1].reshape(-1)
+    return bits[:n].astype(bool)
 
 
 def _worker(rank, world, port, algo, q):
