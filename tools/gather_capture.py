@@ -1,4 +1,4 @@
-"""One C4 CC run with the SM gather only (no copy-engine runs), for an ncu capture of gather launches
+"""One C4 CC run with the SM gather only (no copy-engine runs, no span DMA), for an ncu capture of gather launches
 whose payload is known: iteration 1's windows are full chunks of chunk_cap bytes (dev tool).
     ncu --set full -k regex:k_gather16 -s 1 -c 2 -o prof python tools/gather_capture.py"""
 import os
@@ -14,6 +14,7 @@ g = gg.config_graph(cfg)
 asc.set_device(0)
 asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True, sorted_rows=True)
 asc.set_option("ce_min_run", 0)
+asc.set_option("span_density", 0)
 asc.set_budget(gg.config_budget(cfg, g))
 src = gg.sources(g, 1, seed=c["seed"])[0]
 asc.run(c["algo"], src, 0)
