@@ -135,12 +135,14 @@ typedef enum {
                                       above 1.5x this, the resident (static) PR pull runs in J = ceil(4n / this)
                                       passes over neighbour-id slices, capped at the static rows' mean degree / 8,
                                       so each pass's contrib gathers hit L2 */
-    ASCETIC_OPT_SPAN_DENSITY = 24    /* percent (default 85, 0 = off): in auto mode an iteration with >= 64 MiB of
-                                      misses whose host span is <= 2x the payload moves each window of cap host
+    ASCETIC_OPT_SPAN_DENSITY = 24,   /* percent (default 85, 0 = off): in auto mode an iteration with >= 64 MiB of
+                                      misses whose host span is <= SPAN_MAX_RATIO x the payload moves each window of cap host
                                       bytes with ONE copy-engine DMA when its payload is >= this share of those
                                       bytes (the holes ride along, ~55 GB/s for the whole window), and
                                       gathers the sparser windows; the on-demand kernels read a DMA'd window in
                                       place. Payload accounting is unchanged; span_link_bytes counts the holes. */
+    ASCETIC_OPT_SPAN_MAX_RATIO = 25  /* percent (default 200): auto span planning only when the miss stream's host
+                                      span is at most this share of its payload (windows then decided one by one) */
 } ascetic_option;
 
 typedef struct {

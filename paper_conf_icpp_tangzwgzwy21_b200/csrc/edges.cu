@@ -24,7 +24,7 @@
 
 // Batching factors of the static-hit kernels, per algorithm: 16-byte loads per lane per round
 // (8-byte arcs: SSSP; 4-byte arcs: the others) and 32-arc rounds per warp for short lists.
-// Measured on B200, resident RMAT-24 at 8 CTAs/SM (tools/gpu_ab2.sh, profiles/r01/static_batching_ab.md):
+// Measured on B200, resident RMAT-24 at 8 CTAs/SM (profiles/r01/static_batching_ab.md):
 // BFS gains nothing from batching (most arcs stop at the visited word), SSSP is best at 2/2
 // (-14 %), CC/PRD at 2/4 (-10 %). ASC_* override them for tuning builds.
 namespace ascetic { namespace {

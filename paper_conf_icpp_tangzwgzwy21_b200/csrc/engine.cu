@@ -823,7 +823,7 @@ void Part::expand(uint32_t t, const IterTotals& T) {
         // (forced with XFER_MODE 3 whatever the span, for tests: sparse windows are then gathered)
         if (mode == 1 && (o_.xfer_mode == 3 || (o_.xfer_mode == 0 && o_.span_density > 0 &&
                                                  miss * b_e >= o_.span_min_bytes &&
-                                                 T.miss_h1 - T.miss_h0 <= 2 * miss)) &&
+                                                 (double)(T.miss_h1 - T.miss_h0) <= o_.span_max_ratio * (double)miss)) &&
             plan_span_windows(T))
             mode = 3;
         if (mode == 2) {
@@ -1458,6 +1458,10 @@ void Engine::set_option(int opt, int64_t value) {
         case ASCETIC_OPT_SPAN_DENSITY:
             if (value < 0 || value > 100) throw Error(ASCETIC_EINVAL, "span density must be a percentage in [0, 100]");
             o_.span_density = value / 100.0;
+            break;
+        case ASCETIC_OPT_SPAN_MAX_RATIO:
+            if (value < 100 || value > 100000) throw Error(ASCETIC_EINVAL, "span ratio must be a percentage in [100, 100000]");
+            o_.span_max_ratio = value / 100.0;
             break;
         case ASCETIC_OPT_PR_SEGMENT:
             if (value < 0) throw Error(ASCETIC_EINVAL, "PR segment bytes must be >= 0");

@@ -74,6 +74,7 @@ struct Options {
     uint64_t pr_segment = 64ull << 20;  // PR static pull: neighbour-id slice of contrib per pass (0 = off)
     double span_density = 0.85;         // span DMA of a window when payload >= this share of its host bytes (0 = off)
     uint64_t span_min_bytes = 64ull << 20;   // ... in iterations with at least this much payload
+    double span_max_ratio = 2.0;        // ... whose host span is at most this many times the payload
     uint32_t gap_bridge = 0;            // gather: also load host holes <= this many bytes between pieces (0 = off;
                                         // measured no gain: C2/C4 A/B, profiles/r02/gather_ab_c4.log)
 };

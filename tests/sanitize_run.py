@@ -5,7 +5,7 @@ and PageRank-delta. Checks results against the oracle."""
 import os
 import sys
 
-sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))   # repo root
 
 import numpy as np  # noqa: E402
 

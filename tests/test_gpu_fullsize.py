@@ -9,7 +9,7 @@ C4 (CC, uk-shaped, 6.4 B arcs, 30 % budget — bench.py's default workload): eve
 per-iteration record (digest, |A|, |H|, |M|, runs, arcs, miss bytes) bit-exact, static set,
 fill and payload bytes equal to the oracle's placer and simulation.
 C5 on one GPU (RMAT-29, 72 GB CSR, 40 GB budget) needs ~150 GB of host RAM and ~10 minutes of
-generation: it runs only with ASCETIC_FULL_C5=1 (tools/c5_run.py has the same checks).
+generation: it runs only with ASCETIC_FULL_C5=1 (round 1 ran the same checks by hand, profiles/r01/c5_single_gpu.log).
 """
 import os
 

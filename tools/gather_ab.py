@@ -17,6 +17,7 @@ def main():
     ap.add_argument("--ce", default="0,1048576")
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--span", default="0,85", help="span_density percentages (0 = no span DMA)")
+    ap.add_argument("--ratio", default="200", help="span_max_ratio percentages")
     a = ap.parse_args()
     c = gg.CONFIGS[a.config]
     algo = c["algo"]
@@ -29,9 +30,10 @@ def main():
     asc.set_budget(budget)
     asc.run(algo, src, iters)
     for rnd in range(2):                                  # two interleaved rounds
-        for ce, gap, sp in [(int(c_), int(g_), int(s_)) for s_ in a.span.split(",") for c_ in a.ce.split(",")
-                            for g_ in a.gaps.split(",")]:
+        for ce, gap, sp, ra in [(int(c_), int(g_), int(s_), int(r_)) for s_ in a.span.split(",") for c_ in a.ce.split(",")
+                                for g_ in a.gaps.split(",") for r_ in a.ratio.split(",")]:
             if True:
+                asc.set_option("span_max_ratio", ra)
                 asc.set_option("ce_min_run", ce)
                 asc.set_option("gap_bridge", gap)
                 asc.set_option("span_density", sp)
@@ -43,7 +45,7 @@ def main():
                         best = st
                 st = best
                 sm = st["gather_bytes"] - st["gather_ce_bytes"]
-                print(f"round {rnd} {a.config} span={sp:3d} ce_min_run={ce:8d} gap={gap:5d} run {st['time_run_s']*1e3:8.1f} ms "
+                print(f"round {rnd} {a.config} span={sp:3d} ratio={ra:4d} ce_min_run={ce:8d} gap={gap:5d} run {st['time_run_s']*1e3:8.1f} ms "
                       f"{st['gteps']:6.2f} GTEPS  gather {st['gather_bytes']/1e9:6.2f} GB in {st['time_gather_s']*1e3:7.1f} ms "
                       f"= {st['gather_bytes']/max(1e-9, st['time_gather_s'])/1e9:5.1f} GB/s (CE {st['gather_ce_bytes']/1e9:5.2f} GB)  "
                       f"SM load/payload {st['gather_load_bytes']/max(1, sm):.3f}  dma {st['dma_bytes']/1e9:5.2f} GB "

@@ -21,7 +21,6 @@ def main():
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--iters", type=int, default=0)
     ap.add_argument("--config", default="")
-    ap.add_argument("--oracle", action="store_true")
     ap.add_argument("--gather-ctas", type=int, default=0)
     ap.add_argument("--chunk-cap", type=int, default=0)
     ap.add_argument("--sweep", action="store_true")
@@ -96,19 +95,6 @@ def main():
               f"static_Garcs/s={st['static_arcs'] / max(st['time_static_s'], 1e-9) / 1e9:.1f}", flush=True)
     for i in ([] if a.quiet else its):
         print({k: (round(v, 3) if isinstance(v, float) else v) for k, v in i.items() if k != "digest"})
-    if a.oracle:
-        import oracle
-        p = oracle.placer(g.off, g.b_e, budget)
-        t0 = time.time()
-        ref = oracle.run(algo, g.off, g.nbr, src=src, max_iters=iters, is_static=oracle.static_prefix(g.n, p.s))
-        print(f"oracle {time.time()-t0:.2f}s threads={oracle.threads()}")
-        res = asc.get_result()
-        if algo == "pr":
-            print("max rel", float(np.max(np.abs(res - ref.values) / ref.values)))
-        else:
-            print("equal", bool(np.array_equal(res, ref.values)))
-        print("records equal", [ {k: x[k] for k in asc.PARITY_FIELDS} for x in its] ==
-              [{k: x[k] for k in asc.PARITY_FIELDS} for x in ref.records])
 
 
 if __name__ == "__main__":
