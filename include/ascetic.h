@@ -73,8 +73,8 @@ typedef enum {
     ASCETIC_OPT_OVERLAP = 4,       /* 1 (default) = static compute overlaps the transfer; 0 = serialize (ablation, Fig. 8) */
     ASCETIC_OPT_KEEP_STATIC = 5,   /* 1 = keep the Static Region filled across runs (fill counted once) ; default 0 */
     ASCETIC_OPT_HUB_DEGREE = 6,    /* hit-queue degree at/above which a list is split across CTAs (default 2048) */
-    ASCETIC_OPT_TIMING = 7,        /* CUDA-event phase timing: 1 (default) = per-phase spans in iterations with >= 2^20
-                                      active arcs or >= 4 MiB of misses, one span (the iteration) otherwise;
+    ASCETIC_OPT_TIMING = 7,        /* CUDA-event phase timing: 1 (default) = per-phase spans in iterations with >= 2^23
+                                      active arcs or >= 32 MiB of misses, one span (the iteration) otherwise;
                                       2 = every phase of every iteration; 0 = off */
     ASCETIC_OPT_GATHER_CTAS = 8,   /* persistent CTAs of the zero-copy gather; 0 (default) = 512 / b_e (~1 MiB in flight) */
     ASCETIC_OPT_CHUNK_BUFFERS = 9, /* On-demand Region C split into N buffers of C/N (2..8; 0 = auto (default): 3, or 2

@@ -739,9 +739,10 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     const DevState d = dev_state(t);
     const Queues q = queues(T);
     // per-phase spans only for iterations big enough for them to matter (TIMING = 1): a small
-    // iteration keeps its classify span (its wall time); its ~10 event pairs would cost more device
-    // and host time than its kernels (C1: 0.28 ms device + 0.27 ms host per 1 ms run)
-    fine_ = o_.timing >= 2 || trace_level() > 0 || T.active_arcs >= (1ull << 20) || T.miss_arcs * b_e >= (4ull << 20);
+    // iteration keeps its classify span (its wall time); its event pairs would cost more device and
+    // host time than its kernels (C1: 0.28 ms device + 0.27 ms host per 1 ms run; its chunk pipeline
+    // is bound by the host's enqueue rate, ~6 API calls per 0.3 MB chunk, ASCETIC_TRACE timeline)
+    fine_ = o_.timing >= 2 || trace_level() > 0 || T.active_arcs >= (8ull << 20) || T.miss_arcs * b_e >= (32ull << 20);
     if (algo_ == ALG_PR) CK(cudaMemsetAsync(d_sum_ + vlo_, 0, (vhi_ - vlo_) * sizeof(unsigned long long), cs_));
     // ---- Static Computing, overlapping the transfer, on its own stream so
     // the on-demand kernels (and through them the chunk buffers' reuse) never queue behind it;
