@@ -68,6 +68,42 @@ def main():
             ok = np.array_equal(res, exp)
             bad += 0 if ok else 1
             print(f"world={world} {algo} placement={placement} K={K}: {'ok' if ok else 'MISMATCH'}", flush=True)
+    # round-2 paths: span-DMA windows (forced), copy-engine long runs beside the gather, the PR slice pull,
+    # RED.MIN updates (default), one and two ranks
+    for world in (1, 2):
+        asc.unload()
+        asc.emulate_ranks(world)
+        for algo, opts in [("bfs", {"xfer_mode": 3, "span_density": 50}), ("sssp", {"xfer_mode": 3, "span_density": 0}),
+                           ("cc", {"xfer_mode": 1, "ce_min_run": 512}), ("pr", {"xfer_mode": 1, "ce_min_run": 512}),
+                           ("pr", {"pr_segment": 2048}), ("prd", {"xfer_mode": 3, "span_density": 85})]:
+            g = gg.rmat(10, seed=7, weights=(algo == "sssp"))
+            src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+            it = 4 if algo == "pr" else 0
+            asc.unload()
+            asc.load_csr(g.off, g.nbr, pairs=g.pairs, sorted_rows=True)
+            asc.set_option("chunk_cap", 2048)
+            asc.set_option("hub_degree", 64)
+            for k, v in opts.items():
+                asc.set_option(k, v)
+            budget = (20 * g.csr_bytes) if "pr_segment" in opts else g.csr_bytes // (3 * world)
+            asc.set_budget(budget, 0.4)
+            asc.run(algo, src, it)
+            res = asc.get_result()
+            bounds = oracle.partition(g.off, world)
+            st = np.zeros(g.n, dtype=np.uint8)
+            for k in range(world):
+                lo, hi = int(bounds[k]), int(bounds[k + 1])
+                p = oracle.placer(g.off[lo:hi + 1] - g.off[lo], g.b_e, budget, 0.4)
+                st[lo:lo + p.s] = 1
+            ref = oracle.run(algo, g.off, g.nbr, src=src, max_iters=it, is_static=st)
+            if algo == "pr":
+                ok = np.max(np.abs(res - ref.values) / ref.values) < 1e-5
+            else:
+                ok = np.array_equal(res, ref.values.astype(np.float32) if algo == "prd" else ref.values)
+            bad += 0 if ok else 1
+            print(f"world={world} {algo} {opts}: {'ok' if ok else 'MISMATCH'}", flush=True)
+            for k, v in [("xfer_mode", 0), ("span_density", 85), ("ce_min_run", 1 << 20), ("pr_segment", 64 << 20)]:
+                asc.set_option(k, v)
     for k, v in [("static_placement", 0), ("replace_chunks", 0), ("chunk_cap", 0), ("hub_degree", 2048)]:
         asc.set_option(k, v)
     asc.unload()
