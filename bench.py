@@ -120,11 +120,19 @@ def _workload(cfg_key: str):
 def _config(args, c, g) -> dict:
     """The workload, identical in both arms (the driver compares the two config dicts)."""
     import graphgen as gg
-    return {"workload": f"{args.config}: {c['desc']}", "algo": c["algo"], "n": g.n, "m": g.m,
+    algo, iters = _algo(args, c)
+    return {"workload": f"{args.config}: {c['desc']}", "algo": algo, "n": g.n, "m": g.m,
             "budget_bytes": gg.config_budget(args.config, g), "csr_bytes": g.csr_bytes,
-            "pr_iterations": c.get("iters") if c["algo"] == "pr" else None,
+            "pr_iterations": iters if algo == "pr" else None,
             "sources": "8 seeded sources with deg > 0 (seed = config seed), cycled over the steps"
-            if c["algo"] in ("bfs", "sssp") else None}
+            if algo in ("bfs", "sssp") else None}
+
+
+def _algo(args, c):
+    """(algorithm, PR iterations) of a config; C5 ("BFS + PageRank") runs one of them per bench line."""
+    algo = c["algo"] if c["algo"] != "bfs+pr" else args.c5_algo
+    iters = (c.get("iters") or args.c5_pr_iters) if algo == "pr" else 0
+    return algo, iters
 
 
 def shared_graph(config: str, barrier, local_rank: int, tag: str, alloc_local=None):
@@ -190,8 +198,7 @@ def run_reference(args, ws, rank):
     budget = gg.config_budget(args.config, g)
     p = oracle.placer(g.off, g.b_e, budget)
     st = oracle.static_prefix(g.n, p.s)
-    algo = c["algo"]
-    iters = c.get("iters", 0) if algo == "pr" else 0
+    algo, iters = _algo(args, c)
     if algo == "pr":
         iters = min(iters, args.ref_pr_iters)
     srcs = gg.sources(g, 8, seed=c["seed"])
@@ -229,6 +236,8 @@ def main():
     ap.add_argument("--config", default="c4", choices=["c1", "c2", "c3", "c4", "c5"])
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-pageable", action="store_true", help="skip the pageable-input load_csr measurement")
+    ap.add_argument("--c5-algo", default="bfs", choices=["bfs", "pr"], help="C5 (BFS + PageRank): which one a step runs")
+    ap.add_argument("--c5-pr-iters", type=int, default=43, help="C5 PageRank iterations per step")
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="bounded oracle sample for cpu_baseline")
     ap.add_argument("--ref-pr-iters", type=int, default=2, help="PR iterations per reference step (bounded)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -251,8 +260,7 @@ def main():
         dist.init_process_group("nccl", device_id=dev)
     import paper_conf_icpp_tangzwgzwy21_b200 as asc
     gg, c = _workload(args.config)
-    algo = c["algo"]
-    iters = c.get("iters", 0) if algo == "pr" else 0
+    algo, iters = _algo(args, c)
 
     h2d_peak = _h2d_peak(torch, dev)
     hbm_peak, hbm_src = _peaks()

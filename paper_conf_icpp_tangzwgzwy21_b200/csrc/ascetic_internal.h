@@ -71,7 +71,8 @@ struct ClassifyArgs {
     ScanVal* tile_incl;
     uint32_t* tile_flag;
     uint32_t epoch;
-    IterTotals* tot;                   // device
+    IterTotals* tot;                   // device, zero on entry
+    IterTotals* tot_next;              // device: zeroed by the last CTA for the next classify (no memset launch)
     IterTotals* host_tot;              // mapped pinned
     uint32_t* host_runs;               // mapped pinned: (b, e) of the first host_runs_cap runs
     uint32_t host_runs_cap;

@@ -156,6 +156,7 @@ Part::~Part() {
     }
     if (ev_classified_) cudaEventDestroy(ev_classified_);
     if (ev_long_) cudaEventDestroy(ev_long_);
+    if (ev_pipe_) cudaEventDestroy(ev_pipe_);
     free_hot();
     if (ev_acc_) cudaEventDestroy(ev_acc_);
     if (ev_swapped_) cudaEventDestroy(ev_swapped_);
@@ -190,6 +191,7 @@ void Part::alloc_vertex_state() {
     CK(cudaEventCreateWithFlags(&sync_ev_, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&ev_classified_, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&ev_long_, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&ev_pipe_, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&ev_acc_, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&ev_swapped_, cudaEventDisableTiming));
     const uint64_t n = g_.n, m = g_.m;
@@ -216,7 +218,9 @@ void Part::alloc_vertex_state() {
     dalloc(&d_tile_agg_, ntiles_, &vertex_bytes_);
     dalloc(&d_tile_incl_, ntiles_, &vertex_bytes_);
     dalloc(&d_tile_flag_, ntiles_, &vertex_bytes_);
-    dalloc(&d_tot_, 1, &vertex_bytes_);
+    dalloc(&d_tot_, 2, &vertex_bytes_);   // double-buffered: classify t zeroes the buffer of t+1
+    CK(cudaMemset(d_tot_, 0, 2 * sizeof(IterTotals)));
+    tot_buf_ = 0;
     CK(cudaMemset(d_tile_flag_, 0, (size_t)std::max<uint32_t>(ntiles_, 1) * 4));
     CK(cudaMemset(d_S_, 0, (size_t)std::max<uint32_t>(nwords_, 1) * 4));
     epoch_ = 0;
@@ -683,7 +687,6 @@ void Part::begin(int algo, uint32_t source, uint32_t max_iters, bool timing) {
 void Part::classify(uint32_t t) {
     // ---- GenDataMap + compaction
     *reinterpret_cast<volatile uint32_t*>(&h_tot_->ready) = 0;
-    CK(cudaMemsetAsync(d_tot_, 0, sizeof(IterTotals), cs_));
     ++epoch_;
     if (epoch_ >= (1u << 30)) {
         CK(cudaMemsetAsync(d_tile_flag_, 0, (size_t)ntiles_ * 4, cs_));
@@ -697,7 +700,10 @@ void Part::classify(uint32_t t) {
     ca.mq = d_mq_; ca.mq_pre = d_mq_pre_; ca.mq_src = d_mq_src_; ca.tile_first = d_tile_first_;
     ca.run_b = d_run_b_; ca.run_e = d_run_e_; ca.run_dst = d_run_dst_;
     ca.tile_agg = d_tile_agg_; ca.tile_incl = d_tile_incl_; ca.tile_flag = d_tile_flag_; ca.epoch = epoch_;
-    ca.tot = d_tot_; ca.host_tot = h_tot_;
+    ca.tot = d_tot_ + tot_buf_;            // zeroed by the previous classify's last CTA
+    ca.tot_next = d_tot_ + (tot_buf_ ^ 1u);
+    tot_buf_ ^= 1u;
+    ca.host_tot = h_tot_;
     ca.host_runs = h_runs_; ca.host_runs_cap = kRunsHostMax;
     cudaEvent_t e0 = mark(cs_, true);   // every iteration: its start marks the iteration's wall time
     launch_classify(ca, cs_);
@@ -853,10 +859,19 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     if (prefetched_ && (mode != 2 || miss != prefetch_miss_ || T.n_runs != prefetch_runs_))
         throw Error(ASCETIC_ECUDA, "internal: prefetched chunks do not match the iteration's miss stream");
     const uint64_t g0 = gchunk_;   // global chunk number of this iteration's chunk 0
-    // small chunks (two buffers of < 4 MiB) are latency-bound transfers: alternate them over both copy
-    // streams so chunk k+1's transfer runs while chunk k's is still in flight (each waits only for
-    // its own buffer's consumer); large chunks stay on one stream (each gets the whole link)
-    const bool alt = mode == 1 && nlint_ == 0 && nbuf_ == 2 && cap_ < (4ull << 20);
+    // small chunks (two buffers of < 4 MiB, e.g. C1's 0.3 MB) are latency-bound and their pipeline is
+    // bound by the host's enqueue rate (ASCETIC_TRACE: ~6 API calls per chunk): each buffer gets its
+    // own stream that runs the buffer's transfers AND its on-demand kernels in order, so buffer reuse
+    // and transfer -> compute need no events (2 launches per chunk) and chunk k+1's transfer runs
+    // beside chunk k's compute; the two streams join the compute stream at the end. Large chunks keep
+    // the event pipeline (copy stream at the highest priority, compute on its own stream).
+    const bool alt = mode == 1 && nlint_ == 0 && nbuf_ == 2 && cap_ < (4ull << 20) && prefetched_ == 0;
+    cudaStream_t bst[2] = {xs_, xs2_};
+    if (alt && nchunks) {
+        CK(cudaEventRecord(ev_pipe_, cs_));   // after the previous iteration's compute and this one's memsets
+        CK(cudaStreamWaitEvent(xs_, ev_pipe_, 0));
+        CK(cudaStreamWaitEvent(xs2_, ev_pipe_, 0));
+    }
     // windows: [k cap, (k+1) cap) of the miss stream, or (span mode) the host ranges of cap bytes
     // over the miss stream's span; a dense span window is one DMA of its host bytes and the
     // on-demand kernel reads it in place (span_base), a sparse one is gathered like mode 1
@@ -885,7 +900,22 @@ void Part::expand(uint32_t t, const IterTotals& T) {
         }
         const uint64_t gk = g0 + done;
         const int buf = (int)(gk % (uint64_t)nbuf_);
-        cudaStream_t xk = (alt && (gk & 1u)) ? xs2_ : xs_;
+        if (alt) {
+            cudaStream_t sb = bst[buf];
+            cudaEvent_t e0 = mark(sb);
+            transfer_chunk(q, buf, lo, hi, 1, sb);
+            CK(cudaGetLastError());
+            span(e0, sb, t, PH_GATHER);
+            e0 = mark(sb);
+            launch_ondemand(algo_, d, q, d_chunk_[buf], lo, hi, ~0ull, sb);
+            CK(cudaGetLastError());
+            span(e0, sb, t, PH_OND);
+            st.gather_bytes += (hi - lo) * b_e;
+            ++st.gather_chunks;
+            ++done;
+            continue;
+        }
+        cudaStream_t xk = xs_;
         if (done >= prefetched_) {
             if (gk >= (uint64_t)nbuf_) CK(cudaStreamWaitEvent(xk, consumed_[buf], 0));   // buffer reuse
             cudaEvent_t e0 = mark(xk);
@@ -910,6 +940,12 @@ void Part::expand(uint32_t t, const IterTotals& T) {
         CK(cudaEventRecord(consumed_[buf], cs_));
         if (wmode == 1) ++st.gather_chunks; else ++st.dma_chunks;
         ++done;
+    }
+    if (alt && done) {   // the buffers' last users, for whoever uses them next; finalize waits for both
+        for (int b = 0; b < 2; ++b) {
+            CK(cudaEventRecord(consumed_[b], bst[b]));
+            CK(cudaStreamWaitEvent(cs_, consumed_[b], 0));
+        }
     }
     nchunks = done;
     gchunk_ = g0 + nchunks;

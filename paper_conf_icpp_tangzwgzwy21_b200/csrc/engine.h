@@ -187,7 +187,8 @@ class Part {
     ScanVal *d_tile_agg_ = nullptr, *d_tile_incl_ = nullptr;
     uint32_t* d_tile_flag_ = nullptr;
     uint32_t epoch_ = 0;
-    IterTotals* d_tot_ = nullptr;
+    IterTotals* d_tot_ = nullptr;   // [2]
+    uint32_t tot_buf_ = 0;
     IterTotals* h_tot_ = nullptr;   // mapped pinned
     uint32_t* h_runs_ = nullptr;    // mapped pinned (b, e) pairs of the first kRunsHostMax runs
     uint64_t vertex_bytes_ = 0;
@@ -248,7 +249,7 @@ class Part {
     std::vector<uint32_t> lb_, le_;                  // this iteration's long runs, by stream position
     std::vector<unsigned long long> ldst_;
     cudaStream_t xs2_ = nullptr;
-    cudaEvent_t ce_done_[kMaxBuffers] = {}, xfer_go_[kMaxBuffers] = {}, ev_long_ = nullptr;
+    cudaEvent_t ce_done_[kMaxBuffers] = {}, xfer_go_[kMaxBuffers] = {}, ev_long_ = nullptr, ev_pipe_ = nullptr;
     unsigned long long* d_cover_ = nullptr;          // gather: 16-byte units loaded (link bytes / 16)
     static constexpr uint32_t kSpanWinMax = 4096;
     unsigned long long* h_win_ = nullptr;            // mapped: span windows' first miss-stream positions (nwin + 1)

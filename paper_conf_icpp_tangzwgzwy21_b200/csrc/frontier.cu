@@ -356,6 +356,10 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
                 h1 = src[fin.missq - 1] + (fin.miss_arcs - pre[fin.missq - 1]);
             }
             h->miss_h0 = h0; h->miss_h1 = h1;
+            {   // the next classify's totals start from zero
+                unsigned long long* z = reinterpret_cast<unsigned long long*>(a.tot_next);
+                for (size_t i = 0; i < sizeof(IterTotals) / 8; ++i) z[i] = 0ull;
+            }
             __threadfence_system();
             *reinterpret_cast<volatile uint32_t*>(&h->ready) = 1u;
         }

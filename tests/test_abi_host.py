@@ -76,3 +76,18 @@ def test_place_rejects_bad_fraction():
         with pytest.raises(asc.AsceticError) as e:
             asc.place(off, 4, 1 << 20, f)
         assert e.value.code == asc.EINVAL
+
+
+def test_binding_mirrors_header_enums_and_structs():
+    """The ctypes binding's option ids, load flags and stats fields follow include/ascetic.h."""
+    asc = _lib()
+    hdr = open(os.path.join(ROOT, "include", "ascetic.h")).read()
+    opts = {m.group(1).lower(): int(m.group(2)) for m in re.finditer(r"ASCETIC_OPT_([A-Z_0-9]+)\s*=\s*(\d+)", hdr)}
+    assert opts == asc.OPTIONS
+    flags = {m.group(1): int(m.group(2)) for m in re.finditer(r"ASCETIC_([A-Z]+)\s*=\s*(\d+)u", hdr)}
+    assert flags == {"SYMMETRIC": asc.SYMMETRIC, "COPY": asc.COPY, "VALIDATE": asc.VALIDATE, "PAIRS": asc.PAIRS,
+                     "SORTED": asc.SORTED}
+    body = hdr[hdr.index("typedef struct {\n    int32_t algo;"):hdr.index("} ascetic_stats_t;")]
+    names = re.findall(r"^\s*(?:u?int(?:32|64)_t|double)\s+([a-z_0-9, ]+);", body, re.M)
+    fields = [f.strip() for grp in names for f in grp.split(",")]
+    assert fields == [f for f, _ in asc.Stats._fields_]
