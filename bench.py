@@ -257,7 +257,10 @@ def main():
     dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)
     if ws > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        import datetime
+        # generous timeout: the other ranks wait in a barrier while local rank 0 generates the shared
+        # graph (C4 ~3 min, C5 ~8 min on 16 host cores)
+        dist.init_process_group("nccl", device_id=dev, timeout=datetime.timedelta(minutes=60))
     import paper_conf_icpp_tangzwgzwy21_b200 as asc
     gg, c = _workload(args.config)
     algo, iters = _algo(args, c)
