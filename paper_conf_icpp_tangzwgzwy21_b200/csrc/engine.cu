@@ -746,8 +746,8 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     const Queues q = queues(T);
     // per-phase spans only for iterations big enough for them to matter (TIMING = 1): a small
     // iteration keeps its classify span (its wall time); its event pairs would cost more device and
-    // host time than its kernels (C1: 0.28 ms device + 0.27 ms host per 1 ms run; its chunk pipeline
-    // is bound by the host's enqueue rate, ~6 API calls per 0.3 MB chunk, ASCETIC_TRACE timeline)
+    // host time than its kernels (C1: 0.28 ms device + 0.27 ms host per 1 ms run in round 1; bench
+    // step 1.07 -> 0.87 ms when the threshold went from 2^20 arcs / 4 MiB to 2^23 arcs / 32 MiB)
     fine_ = o_.timing >= 2 || trace_level() > 0 || T.active_arcs >= (8ull << 20) || T.miss_arcs * b_e >= (32ull << 20);
     if (algo_ == ALG_PR) CK(cudaMemsetAsync(d_sum_ + vlo_, 0, (vhi_ - vlo_) * sizeof(unsigned long long), cs_));
     // ---- Static Computing, overlapping the transfer, on its own stream so
@@ -859,12 +859,13 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     if (prefetched_ && (mode != 2 || miss != prefetch_miss_ || T.n_runs != prefetch_runs_))
         throw Error(ASCETIC_ECUDA, "internal: prefetched chunks do not match the iteration's miss stream");
     const uint64_t g0 = gchunk_;   // global chunk number of this iteration's chunk 0
-    // small chunks (two buffers of < 4 MiB, e.g. C1's 0.3 MB) are latency-bound and their pipeline is
-    // bound by the host's enqueue rate (ASCETIC_TRACE: ~6 API calls per chunk): each buffer gets its
-    // own stream that runs the buffer's transfers AND its on-demand kernels in order, so buffer reuse
-    // and transfer -> compute need no events (2 launches per chunk) and chunk k+1's transfer runs
-    // beside chunk k's compute; the two streams join the compute stream at the end. Large chunks keep
-    // the event pipeline (copy stream at the highest priority, compute on its own stream).
+    // small chunks (two buffers of < 4 MiB, e.g. C1's 0.3 MB; ~14 us gathers, latency-bound): each
+    // buffer gets its own stream that runs the buffer's transfers AND its on-demand kernels in order,
+    // so buffer reuse and transfer -> compute need no events (2 launches per chunk instead of 2 + 4
+    // event calls) and chunk k+1's transfer runs beside chunk k's compute; the two streams join the
+    // compute stream at the end. (C1: 0.868 -> 0.871 ms per step, i.e. the chunk pipeline is not
+    // host-bound once the per-phase events are off.) Large chunks keep the event pipeline (copy
+    // stream at the highest priority, compute on its own stream).
     const bool alt = mode == 1 && nlint_ == 0 && nbuf_ == 2 && cap_ < (4ull << 20) && prefetched_ == 0;
     cudaStream_t bst[2] = {xs_, xs2_};
     if (alt && nchunks) {
