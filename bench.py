@@ -188,6 +188,89 @@ def shared_graph(config: str, barrier, local_rank: int, tag: str, alloc_local=No
     return g, cleanup, gen_s
 
 
+def roofline_of(per: list, steps: int, total_ms: float, b_e: int, n: int, h2d_peak: float, hbm_peak: float,
+                hbm_src: str, config: str) -> dict:
+    """Roofline entry of a bench line from the library's per-step stats (pure: unit-tested on CPU)."""
+    # ---- per-kernel-class breakdown (library CUDA events on the launching streams)
+    kern = {
+        "gather": dict(time_s=sum(s["time_gather_s"] for s in per), bytes=sum(s["gather_bytes"] for s in per),
+                       bound="host_link", peak=h2d_peak),
+        "dma": dict(time_s=sum(s["time_dma_s"] + s["time_fill_s"] for s in per),
+                    bytes=sum(s["dma_bytes"] + s["h2d_static_fill_bytes"] for s in per), bound="host_link",
+                    peak=h2d_peak),
+        "ondemand": dict(time_s=sum(s["time_ondemand_s"] for s in per),
+                         bytes=sum(s["ondemand_arcs"] for s in per) * (b_e + 4), bound="hbm", peak=hbm_peak),
+        "static": dict(time_s=sum(s["time_static_s"] for s in per),
+                       bytes=sum(s["static_arcs"] for s in per) * (b_e + 4), bound="hbm", peak=hbm_peak),
+        "classify": dict(time_s=sum(s["time_classify_s"] for s in per),
+                         bytes=sum(s["iterations"] for s in per) * (n // 4) + 0, bound="hbm", peak=hbm_peak),
+    }
+    # the transfer path as a whole (the step's bound when out of core): every H2D byte of the step (static
+    # fill + per-iteration miss payload, whichever engine moved it) over the copy streams' busy time
+    kern["transfer"] = dict(time_s=sum(s["time_h2d_busy_s"] for s in per),
+                            bytes=sum(s["h2d_static_fill_bytes"] + s["h2d_payload_bytes"] for s in per),
+                            bound="host_link", peak=h2d_peak)
+    for k_, d in kern.items():
+        d["achieved"] = d["bytes"] / d["time_s"] / 1e9 if d["time_s"] > 0 else 0.0
+        d["frac"] = d["achieved"] / d["peak"] if d["peak"] else 0.0
+        d["share_of_step"] = d["time_s"] * 1e3 / total_ms if total_ms else 0.0
+    # headline entry: the transfer path when it fills most of the step (out of core), else the
+    # longest kernel class; "dominant_kernel" is always the longest class of our own kernels
+    own = ("gather", "ondemand", "static", "classify")
+    dom_kernel = max(own, key=lambda k_: kern[k_]["time_s"])
+    dom = "transfer" if kern["transfer"]["share_of_step"] >= 0.5 else max(
+        ("gather", "dma", "ondemand", "static", "classify"), key=lambda k_: kern[k_]["time_s"])
+    dk = kern[dom]
+    # the gather class = the transfer engine in gather mode: SM zero-copy gather + the copy-engine
+    # long runs beside it (same chunk windows, union time)
+    sm_b = sum(s["gather_bytes"] - s["gather_ce_bytes"] for s in per)
+    kern["gather"].update(sm_bytes=sm_b, ce_bytes=sum(s["gather_ce_bytes"] for s in per),
+                          sm_load_bytes=sum(s["gather_load_bytes"] for s in per),
+                          launches=sum(s["gather_chunks"] for s in per))
+    traffic, traffic_note = None, None
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    tj = {}
+    if os.path.exists(tp):
+        try:
+            tj = json.load(open(tp)).get(config, {})
+        except Exception:
+            tj = {}
+    tg = tj.get("gather")
+    if isinstance(tg, dict) and "pcie_read_per_payload" in tg and kern["gather"]["launches"]:
+        # gather launches: PCIe read bytes = ncu's measured PCIe bytes per payload byte (a capture of
+        # full-window launches) x this run's SM payload per gather launch
+        kern["gather"]["pcie_read_bytes_per_launch"] = tg["pcie_read_per_payload"] * sm_b / kern["gather"]["launches"]
+    if dom == "transfer":
+        # link bytes of the step: copy-engine bytes as moved (static fill, DMA'd runs, span windows
+        # with their holes) + the SM gather's payload scaled by its measured PCIe bytes per payload byte
+        ratio = tg.get("pcie_read_per_payload") if isinstance(tg, dict) else None
+        ce = sum(s["h2d_static_fill_bytes"] + s["dma_bytes"] - s["span_payload_bytes"] + s["span_link_bytes"]
+                 + s["gather_ce_bytes"] for s in per)
+        if ratio or sm_b == 0:
+            ratio = ratio or 0.0
+            traffic = (ce + ratio * sm_b) / steps
+            traffic_note = (f"per step: copy-engine bytes as moved ({ce / steps / 1e9:.2f} GB incl. span holes) + "
+                            f"SM-gathered payload x {ratio:.3f} PCIe read bytes per payload byte "
+                            f"(ncu pcie__read_bytes, {tg.get('source', 'ncu') if isinstance(tg, dict) else 'no SM gather'}); algorithmic bytes per step "
+                            f"{dk['bytes'] / steps / 1e9:.2f} GB")
+    else:
+        t_ = tj.get(dom)
+        if isinstance(t_, (int, float)):
+            traffic = t_
+            traffic_note = "dram__bytes_read.sum + dram__bytes_write.sum of one launch (ncu --set full)"
+    roofline = {"kernel": dom, "bound": dk["bound"], "achieved": dk["achieved"], "peak": dk["peak"],
+                "unit": "GB/s", "frac": dk["frac"], "traffic": traffic, "traffic_note": traffic_note,
+                "dominant_kernel": {"name": dom_kernel, "achieved": kern[dom_kernel]["achieved"],
+                                    "peak": kern[dom_kernel]["peak"], "frac": kern[dom_kernel]["frac"],
+                                    "bound": kern[dom_kernel]["bound"],
+                                    "share_of_step": kern[dom_kernel]["share_of_step"]},
+                "peak_source": ("pinned H2D cudaMemcpyAsync 1 GiB best-of-5 measured in this run"
+                                if dk["bound"] == "host_link" else f"MEASURED_PEAKS.json hbm_gbs ({hbm_src})"),
+                "per_kernel": {k_: {kk: (round(vv, 6) if isinstance(vv, float) else vv) for kk, vv in d.items()}
+                               for k_, d in kern.items()}}
+    return roofline
+
+
 def run_reference(args, ws, rank):
     """--impl reference: the oracle as it stands, on the host cores, same config/metric/unit."""
     if rank != 0:
@@ -363,83 +446,7 @@ def main():
         fill_ms = float(tt.item())
     value_excl_fill = arcs_all / ((total_ms - fill_ms) / 1e3) / 1e9 if total_ms > fill_ms else None
 
-    # ---- per-kernel-class breakdown (library CUDA events on the launching streams)
-    b_e = g.b_e
-    kern = {
-        "gather": dict(time_s=sum(s["time_gather_s"] for s in per), bytes=sum(s["gather_bytes"] for s in per),
-                       bound="host_link", peak=h2d_peak),
-        "dma": dict(time_s=sum(s["time_dma_s"] + s["time_fill_s"] for s in per),
-                    bytes=sum(s["dma_bytes"] + s["h2d_static_fill_bytes"] for s in per), bound="host_link",
-                    peak=h2d_peak),
-        "ondemand": dict(time_s=sum(s["time_ondemand_s"] for s in per),
-                         bytes=sum(s["ondemand_arcs"] for s in per) * (b_e + 4), bound="hbm", peak=hbm_peak),
-        "static": dict(time_s=sum(s["time_static_s"] for s in per),
-                       bytes=sum(s["static_arcs"] for s in per) * (b_e + 4), bound="hbm", peak=hbm_peak),
-        "classify": dict(time_s=sum(s["time_classify_s"] for s in per),
-                         bytes=sum(s["iterations"] for s in per) * (g.n // 4) + 0, bound="hbm", peak=hbm_peak),
-    }
-    # the transfer path as a whole (the step's bound when out of core): every H2D byte of the step (static
-    # fill + per-iteration miss payload, whichever engine moved it) over the copy streams' busy time
-    kern["transfer"] = dict(time_s=sum(s["time_h2d_busy_s"] for s in per),
-                            bytes=sum(s["h2d_static_fill_bytes"] + s["h2d_payload_bytes"] for s in per),
-                            bound="host_link", peak=h2d_peak)
-    for k_, d in kern.items():
-        d["achieved"] = d["bytes"] / d["time_s"] / 1e9 if d["time_s"] > 0 else 0.0
-        d["frac"] = d["achieved"] / d["peak"] if d["peak"] else 0.0
-        d["share_of_step"] = d["time_s"] * 1e3 / total_ms if total_ms else 0.0
-    # headline entry: the transfer path when it fills most of the step (out of core), else the
-    # longest kernel class; "dominant_kernel" is always the longest class of our own kernels
-    own = ("gather", "ondemand", "static", "classify")
-    dom_kernel = max(own, key=lambda k_: kern[k_]["time_s"])
-    dom = "transfer" if kern["transfer"]["share_of_step"] >= 0.5 else max(
-        ("gather", "dma", "ondemand", "static", "classify"), key=lambda k_: kern[k_]["time_s"])
-    dk = kern[dom]
-    # the gather class = the transfer engine in gather mode: SM zero-copy gather + the copy-engine
-    # long runs beside it (same chunk windows, union time)
-    sm_b = sum(s["gather_bytes"] - s["gather_ce_bytes"] for s in per)
-    kern["gather"].update(sm_bytes=sm_b, ce_bytes=sum(s["gather_ce_bytes"] for s in per),
-                          sm_load_bytes=sum(s["gather_load_bytes"] for s in per),
-                          launches=sum(s["gather_chunks"] for s in per))
-    traffic, traffic_note = None, None
-    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    tj = {}
-    if os.path.exists(tp):
-        try:
-            tj = json.load(open(tp)).get(args.config, {})
-        except Exception:
-            tj = {}
-    tg = tj.get("gather")
-    if isinstance(tg, dict) and "pcie_read_per_payload" in tg and kern["gather"]["launches"]:
-        # gather launches: PCIe read bytes = ncu's measured PCIe bytes per payload byte (a capture of
-        # full-window launches) x this run's SM payload per gather launch
-        kern["gather"]["pcie_read_bytes_per_launch"] = tg["pcie_read_per_payload"] * sm_b / kern["gather"]["launches"]
-    if dom == "transfer":
-        # link bytes of the step: copy-engine bytes as moved (static fill, DMA'd runs, span windows
-        # with their holes) + the SM gather's payload scaled by its measured PCIe bytes per payload byte
-        ratio = tg.get("pcie_read_per_payload") if isinstance(tg, dict) else None
-        ce = sum(s["h2d_static_fill_bytes"] + s["dma_bytes"] - s["span_payload_bytes"] + s["span_link_bytes"]
-                 + s["gather_ce_bytes"] for s in per)
-        if ratio:
-            traffic = (ce + ratio * sm_b) / args.steps
-            traffic_note = (f"per step: copy-engine bytes as moved ({ce / args.steps / 1e9:.2f} GB incl. span holes) + "
-                            f"SM-gathered payload x {ratio:.3f} PCIe read bytes per payload byte "
-                            f"(ncu pcie__read_bytes, {tg.get('source', 'ncu')}); algorithmic bytes per step "
-                            f"{dk['bytes'] / args.steps / 1e9:.2f} GB")
-    else:
-        t_ = tj.get(dom)
-        if isinstance(t_, (int, float)):
-            traffic = t_
-            traffic_note = "dram__bytes_read.sum + dram__bytes_write.sum of one launch (ncu --set full)"
-    roofline = {"kernel": dom, "bound": dk["bound"], "achieved": dk["achieved"], "peak": dk["peak"],
-                "unit": "GB/s", "frac": dk["frac"], "traffic": traffic, "traffic_note": traffic_note,
-                "dominant_kernel": {"name": dom_kernel, "achieved": kern[dom_kernel]["achieved"],
-                                    "peak": kern[dom_kernel]["peak"], "frac": kern[dom_kernel]["frac"],
-                                    "bound": kern[dom_kernel]["bound"],
-                                    "share_of_step": kern[dom_kernel]["share_of_step"]},
-                "peak_source": ("pinned H2D cudaMemcpyAsync 1 GiB best-of-5 measured in this run"
-                                if dk["bound"] == "host_link" else f"MEASURED_PEAKS.json hbm_gbs ({hbm_src})"),
-                "per_kernel": {k_: {kk: (round(vv, 6) if isinstance(vv, float) else vv) for kk, vv in d.items()}
-                               for k_, d in kern.items()}}
+    roofline = roofline_of(per, args.steps, total_ms, g.b_e, g.n, h2d_peak, hbm_peak, hbm_src, args.config)
     h2d_total = fill + payload
     link = {"h2d_bytes": h2d_total, "h2d_busy_s": sum(s["time_h2d_busy_s"] for s in per),
             "achieved_gbs": h2d_total / (sum(s["time_h2d_busy_s"] for s in per) or 1) / 1e9,
