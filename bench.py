@@ -448,6 +448,7 @@ def main():
 
     roofline = roofline_of(per, args.steps, total_ms, g.b_e, g.n, h2d_peak, hbm_peak, hbm_src, args.config)
     h2d_total = fill + payload
+    span_holes = _sum_ranks(sum(s["span_link_bytes"] - s["span_payload_bytes"] for s in per))
     link = {"h2d_bytes": h2d_total, "h2d_busy_s": sum(s["time_h2d_busy_s"] for s in per),
             "achieved_gbs": h2d_total / (sum(s["time_h2d_busy_s"] for s in per) or 1) / 1e9,
             "whole_step_gbs": h2d_total / (total_ms / 1e3) / 1e9, "peak_gbs": h2d_peak}
@@ -564,6 +565,9 @@ def main():
                    "h2d_gb_per_run": h2d_total / args.steps / 1e9,
                    "h2d_fill_gb_per_run": fill / args.steps / 1e9,
                    "h2d_payload_gb_per_run": payload / args.steps / 1e9,
+                   # bytes the copy engines and the SM gather actually requested: payload + the holes
+                   # that span-DMA windows carry between missed lists (PCIe protocol overhead excluded)
+                   "h2d_requested_gb_per_run": (h2d_total + span_holes) / args.steps / 1e9,
                    "iterations_per_run": statistics.mean(s["iterations"] for s in per),
                    "sources": srcs if algo in ("bfs", "sssp") else None,
                    "l2": "flushed (512 MiB write) between timed steps; graph > L2",
