@@ -86,6 +86,27 @@ def main():
         print("   payload share by run bytes " + " ".join(f"<{BUCKETS[i + 1]}:{hist[i]:.3f}" for i in range(len(hist) - 1)))
         print("   gap fraction below 16/64/128/256/1024 B: " + " ".join(f"{x:.3f}" for x in gh)
               + f"  gap bytes / payload {gaps.sum() / max(1, rb.sum()):.3f}")
+        # how much of the payload sits in host windows of W bytes that are >= 85 % payload (span-DMA
+        # candidates at that window size)
+        if b.size:
+            hb = b_e * off[b]
+            he = b_e * off[e]
+            h0 = int(hb[0])
+            parts = []
+            for W in (1 << 20, 4 << 20, 16 << 20, 64 << 20, 256 << 20):
+                nwin = int((int(he[-1]) - h0 + W - 1) // W)
+                pay = np.zeros(nwin + 1, dtype=np.int64)
+                # payload per window: split each run at window boundaries (runs are sorted and disjoint)
+                cb = np.cumsum(np.concatenate([[0], (he - hb)]))          # payload before run i
+                edges = h0 + W * np.arange(nwin + 1, dtype=np.int64)
+                # payload below host position x = cb[j] + clip(x - hb[j], 0, len_j), j = last run with hb <= x
+                j = np.searchsorted(hb, edges, side="right") - 1
+                jj = np.clip(j, 0, hb.size - 1)
+                below = np.where(j < 0, 0, cb[jj] + np.clip(edges - hb[jj], 0, he[jj] - hb[jj]))
+                pay = np.diff(below)
+                dense = pay >= 0.85 * W
+                parts.append(f"W={W >> 20}MiB:{pay[dense].sum() / max(1, pay.sum()):.3f}")
+            print("   payload share in >=85%-dense host windows " + " ".join(parts))
     asc.unload()
 
 
