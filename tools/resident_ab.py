@@ -20,6 +20,7 @@ def main():
     ap.add_argument("--algos", default="bfs,sssp,cc,pr")
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--pr-iters", type=int, default=5)
+    ap.add_argument("--pr-segments", default="0,67108864", help="PR: pr_segment values to A/B")
     a = ap.parse_args()
     asc.set_device(0)
     graphs = {}
@@ -35,7 +36,7 @@ def main():
         src = int(np.argmax(np.diff(g.off.astype(np.int64))))
         asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True, sorted_rows=True)
         asc.set_budget(int(1.2 * g.csr_bytes))
-        modes = [1, 2] if algo in ("sssp", "cc") else ([0, 64 << 20] if algo == "pr" else [0])
+        modes = [1, 2] if algo in ("sssp", "cc") else ([int(x) for x in a.pr_segments.split(",")] if algo == "pr" else [0])
         for mode in modes:
             if algo == "pr":
                 asc.set_option("pr_segment", mode)
