@@ -498,6 +498,26 @@ __global__ void __launch_bounds__(256) k_static_hub(DevState d, const uint32_t* 
 // passes, plus one boundary probe per row and pass. Partial sums are added in 2^-62 fixed point
 // (rows: owner-exclusive; hub pieces: integer atomics), so the order of passes and pieces does not
 // change a bit of the result. Small rows (< 32 arcs) keep the unsegmented kernel.
+// first index in [lo, hi) whose id is >= key (ids ascend), found by the warp with 32-ary probing
+__device__ __forceinline__ unsigned long long warp_lower_bound(const uint32_t* __restrict__ ids, unsigned long long lo,
+                                                               unsigned long long hi, uint32_t key, int lane) {
+    while (hi - lo > 32) {
+        const unsigned long long step = (hi - lo + 31) / 32;
+        const unsigned long long i = lo + (unsigned long long)lane * step;
+        const bool below = i < hi && __ldg(ids + i) < key;
+        const uint32_t c = __popc(__ballot_sync(FULL, below));   // probes below key: a prefix of the lanes
+        if (c == 0) return lo;
+        const unsigned long long nlo = lo + (unsigned long long)(c - 1) * step + 1;
+        hi = min(hi, lo + (unsigned long long)c * step);
+        lo = nlo;
+    }
+    const unsigned long long i = lo + lane;
+    const bool below = i < hi && __ldg(ids + i) < key;
+    return lo + __popc(__ballot_sync(FULL, below));
+}
+
+// pass j of a medium row: [cursor, first arc with id >= hi_id), found by a warp search, then the
+// same vectorised pull as the unsegmented kernel over that stretch
 template <bool FIRST>
 __global__ void __launch_bounds__(256) k_static_med_pr_seg(DevState d, const uint32_t* __restrict__ q, uint32_t nq,
                                                            const uint32_t* __restrict__ sbase, uint32_t* __restrict__ cur,
@@ -507,25 +527,18 @@ __global__ void __launch_bounds__(256) k_static_med_pr_seg(DevState d, const uin
     for (uint32_t w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < nq; w += nwarps) {
         const uint32_t u = __ldg(q + w);
         const unsigned long long a0 = __ldg(d.off + u) - d.static_arc0, a1 = __ldg(d.off + u + 1) - d.static_arc0;
-        unsigned long long p = a0 + (FIRST ? 0u : cur[w]);
-        double acc = 0.0;
-        while (p < a1) {
-            const unsigned long long e = p + lane;
-            const uint32_t id = e < a1 ? ld_stream(sbase + e) : 0xFFFFFFFFu;
-            const bool in = id < hi_id;                  // ids ascend: the segment's arcs are a prefix
-            if (in) acc += pr_in(d, id);
-            const uint32_t taken = __popc(__ballot_sync(FULL, in));
-            p += taken;
-            if (taken < 32) break;
-        }
+        const unsigned long long p = a0 + (FIRST ? 0u : cur[w]);
+        const unsigned long long e = warp_lower_bound(sbase, p, a1, hi_id, lane);
+        double acc = e > p ? expand_list<PR, false>(d, sbase, p, e, 0u, lane, 32) : 0.0;
         acc = warp_sum_d(acc);
         if (lane == 0) {
-            cur[w] = (uint32_t)(p - a0);
+            cur[w] = (uint32_t)(e - a0);
             if (acc != 0.0) d.sum[u] += to_fx(acc);
         }
     }
 }
 
+// pass j of a hub piece: warp 0 finds the stretch, the CTA pulls it
 template <bool FIRST>
 __global__ void __launch_bounds__(256) k_static_hub_pr_seg(DevState d, const uint32_t* __restrict__ hq,
                                                            const uint32_t* __restrict__ pre, uint32_t nh,
@@ -533,7 +546,7 @@ __global__ void __launch_bounds__(256) k_static_hub_pr_seg(DevState d, const uin
                                                            const uint32_t* __restrict__ sbase, uint32_t* __restrict__ cur,
                                                            uint32_t hi_id) {
     __shared__ double s_red[8];
-    __shared__ uint32_t s_taken;
+    __shared__ unsigned long long s_end;
     for (uint32_t b = blockIdx.x; b < npieces; b += gridDim.x) {
         const uint32_t h = ub_u32(pre, nh, b) - 1;
         const uint32_t u = __ldg(hq + h);
@@ -541,27 +554,23 @@ __global__ void __launch_bounds__(256) k_static_hub_pr_seg(DevState d, const uin
         const unsigned long long o0 = __ldg(d.off + u) - d.static_arc0, o1 = __ldg(d.off + u + 1) - d.static_arc0;
         const unsigned long long a0 = o0 + (unsigned long long)pidx * piece_arcs;
         const unsigned long long a1 = min(o1, a0 + piece_arcs);
-        unsigned long long p = a0 + (FIRST ? 0u : cur[b]);
-        double acc = 0.0;
-        while (p < a1) {
-            const unsigned long long e = p + threadIdx.x;
-            const uint32_t id = e < a1 ? ld_stream(sbase + e) : 0xFFFFFFFFu;
-            const bool in = id < hi_id;
-            if (in) acc += pr_in(d, id);
-            const uint32_t taken = (uint32_t)__syncthreads_count(in);
-            p += taken;
-            if (taken < blockDim.x) break;
+        const unsigned long long p = a0 + (FIRST ? 0u : cur[b]);
+        if (threadIdx.x < 32) {
+            const unsigned long long e = warp_lower_bound(sbase, p, a1, hi_id, threadIdx.x);
+            if (threadIdx.x == 0) s_end = e;
         }
+        __syncthreads();
+        const unsigned long long e = s_end;
+        double acc = e > p ? expand_list<PR, false>(d, sbase, p, e, 0u, threadIdx.x, blockDim.x) : 0.0;
         acc = warp_sum_d(acc);
         if ((threadIdx.x & 31) == 0) s_red[threadIdx.x >> 5] = acc;
         __syncthreads();
         if (threadIdx.x == 0) {
             double t = 0.0;
             for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += s_red[w];
-            cur[b] = (uint32_t)(p - a0);
+            cur[b] = (uint32_t)(e - a0);
             if (t != 0.0) atomicAdd(d.sum + u, to_fx(t));
         }
-        (void)s_taken;
         __syncthreads();
     }
 }
