@@ -131,7 +131,7 @@ typedef enum {
                                       at most this size between consecutive pieces of a warp's group, so the warp
                                       reads one contiguous block instead of two. Measured: no gain at 64 B, -1 % at
                                       256 B, -2..3 % at 1 KiB on C2/C4 (the link is not charged per block) */
-    ASCETIC_OPT_PR_SEGMENT = 23,     /* bytes (default 64 MiB, 0 = off): with ASCETIC_SORTED rows and contrib (4n bytes)
+    ASCETIC_OPT_PR_SEGMENT = 23,     /* bytes (default 128 MiB, 0 = off): with ASCETIC_SORTED rows and contrib (4n bytes)
                                       above 1.5x this, the resident (static) PR pull runs in J = ceil(4n / this)
                                       passes over neighbour-id slices, capped at the static rows' mean degree / 8,
                                       so each pass's contrib gathers hit L2 */

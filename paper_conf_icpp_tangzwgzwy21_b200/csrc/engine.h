@@ -71,7 +71,8 @@ struct Options {
     int replace_policy = 0;       // hotness counter: 0 = by algorithm, 1 = cumulative, 2 = last iteration
     int relax_mode = 0;           // SSSP/CC min update: 0 = auto, 1 = atomicMin + next bit, 2 = RED.MIN + dense finalize
     uint64_t ce_min_run = 1ull << 20;   // gather-mode iterations: runs >= this many bytes go to the copy engines (0 = off)
-    uint64_t pr_segment = 64ull << 20;  // PR static pull: neighbour-id slice of contrib per pass (0 = off)
+    uint64_t pr_segment = 128ull << 20; // PR static pull: neighbour-id slice of contrib per pass (0 = off; 128 MiB:
+                                        // friendster-shaped resident pull -22 %, profiles/r02/prseg_ab_c3.log)
     double span_density = 0.85;         // span DMA of a window when payload >= this share of its host bytes (0 = off)
     uint64_t span_min_bytes = 64ull << 20;   // ... in iterations with at least this much payload
     double span_max_ratio = 2.0;        // ... whose host span is at most this many times the payload

@@ -102,7 +102,7 @@ def main():
                 ok = np.array_equal(res, ref.values.astype(np.float32) if algo == "prd" else ref.values)
             bad += 0 if ok else 1
             print(f"world={world} {algo} {opts}: {'ok' if ok else 'MISMATCH'}", flush=True)
-            for k, v in [("xfer_mode", 0), ("span_density", 85), ("ce_min_run", 1 << 20), ("pr_segment", 64 << 20)]:
+            for k, v in [("xfer_mode", 0), ("span_density", 85), ("ce_min_run", 1 << 20), ("pr_segment", 128 << 20)]:
                 asc.set_option(k, v)
     for k, v in [("static_placement", 0), ("replace_chunks", 0), ("chunk_cap", 0), ("hub_degree", 2048)]:
         asc.set_option(k, v)

@@ -493,7 +493,7 @@ def test_pr_segmented_pull(asc, resident):
             assert np.array_equal(asc.get_result().view(np.uint32), res[seg].view(np.uint32))
         else:
             assert st["pr_segment_passes"] == 0
-    asc.set_option("pr_segment", 64 << 20)
+    asc.set_option("pr_segment", 128 << 20)
     asc.set_option("hub_degree", 2048)
     p = oracle.placer(g.off, 4, budget)
     ref = _oracle("pr", g, 0, p.s, max_iters=8)

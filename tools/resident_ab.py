@@ -57,7 +57,7 @@ def main():
                   f"{rate * (g.b_e + 4) / 1e12:5.2f} TB/s algorithmic  whole {st['active_arcs_total']/ex/1e9:6.1f} GTEPS excl fill",
                   flush=True)
         asc.set_option("relax_mode", 0)
-        asc.set_option("pr_segment", 64 << 20)
+        asc.set_option("pr_segment", 128 << 20)
     asc.unload()
 
 
