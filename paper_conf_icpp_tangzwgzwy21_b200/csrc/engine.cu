@@ -848,7 +848,9 @@ void Part::expand(uint32_t t, const IterTotals& T) {
             unsigned long long acc = 0;
             for (uint32_t r = 0; r < T.n_runs; ++r) { rdst_[r] = acc; acc += g_.off[re_[r]] - g_.off[rb_[r]]; }
         }
-        if (mode == 1 && o_.ce_min_run && T.n_runs && miss * b_e >= 2 * o_.ce_min_run) plan_long_runs(T);
+        // long runs can only matter when the iteration moves many of them (32 x the threshold): a
+        // small iteration would pay the listing kernel and its host round trip for nothing (C1)
+        if (mode == 1 && o_.ce_min_run && T.n_runs && miss * b_e >= 32 * o_.ce_min_run) plan_long_runs(T);
         if (!o_.overlap && static_pending_) {   // ablation: the transfer waits for static computing
             CK(cudaStreamWaitEvent(xs_, static_done_, 0));
             CK(cudaStreamWaitEvent(xs2_, static_done_, 0));

@@ -142,19 +142,37 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
     const uint32_t anyA = __ballot_sync(FULL, myA != 0);
     const uint32_t piece = a.piece_arcs;
 
+    // Both phases walk the warp's 32 words one at a time (prefix order), but the offsets of the active
+    // vertices are loaded kBatch words ahead: with few CTAs (small graphs) each dependent off[] load
+    // chain costs ~0.5 us, so one load round trip per word made a C1 classify ~20 us.
+    constexpr int kBatch = 8;
     // ---------------- phase A: per-warp counts
     ScanVal mine = sv_zero();
     unsigned long long aArcs = 0, hArcs = 0;
+    unsigned long long degA[kBatch];
     for (int j = 0; j < 32; ++j) {
+        if ((j & (kBatch - 1)) == 0) {
+            const uint32_t any8 = (anyA >> j) & ((1u << kBatch) - 1u);
+#pragma unroll
+            for (int u = 0; u < kBatch; ++u) {
+                degA[u] = 0;
+                if ((any8 >> u) & 1u) {                      // warp-uniform
+                    const uint32_t awu = __shfl_sync(FULL, myA, j + u);
+                    const unsigned long long vu = (unsigned long long)(w0 + j + u) * 32ull + lane;
+                    if ((awu >> lane) & 1u) degA[u] = __ldg(a.off + vu + 1) - __ldg(a.off + vu);
+                }
+            }
+        }
         if (!((anyA >> j) & 1u)) continue;                    // warp-uniform
         const uint32_t aw = __shfl_sync(FULL, myA, j);
         const uint32_t sw = __shfl_sync(FULL, myS, j);
         const uint32_t pm = __shfl_sync(FULL, myMiss, (j + 31) & 31);
         const uint32_t carry_in = (j == 0 ? prevMiss : pm) >> 31;
-        const unsigned long long v = (unsigned long long)(w0 + j) * 32ull + lane;
         const bool act = (aw >> lane) & 1u;
         unsigned long long deg = 0;
-        if (act) deg = __ldg(a.off + v + 1) - __ldg(a.off + v);
+#pragma unroll
+        for (int u = 0; u < kBatch; ++u)
+            if ((j & (kBatch - 1)) == u) deg = degA[u];
         const bool st = (sw >> lane) & 1u;
         const bool hit = act && st, miss = act && !st;
         aArcs += deg;
@@ -246,7 +264,20 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
     const ScanVal wb = sv_add(s_excl, s_warp[warp]);
     uint32_t bS = wb.small, bM = wb.med, bH = wb.hub, bQ = wb.missq, bR = wb.runs, bP = wb.pieces;
     unsigned long long bArcs = wb.miss_arcs;
+    unsigned long long o0B[kBatch], degB[kBatch];
     for (int j = 0; j < 32; ++j) {
+        if ((j & (kBatch - 1)) == 0) {
+            const uint32_t any8 = (anyA >> j) & ((1u << kBatch) - 1u);
+#pragma unroll
+            for (int u = 0; u < kBatch; ++u) {
+                o0B[u] = 0; degB[u] = 0;
+                if ((any8 >> u) & 1u) {                      // warp-uniform
+                    const uint32_t awu = __shfl_sync(FULL, myA, j + u);
+                    const unsigned long long vu = (unsigned long long)(w0 + j + u) * 32ull + lane;
+                    if ((awu >> lane) & 1u) { o0B[u] = __ldg(a.off + vu); degB[u] = __ldg(a.off + vu + 1) - o0B[u]; }
+                }
+            }
+        }
         if (!((anyA >> j) & 1u)) continue;
         const uint32_t aw = __shfl_sync(FULL, myA, j);
         const uint32_t sw = __shfl_sync(FULL, myS, j);
@@ -257,7 +288,9 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
         const unsigned long long v = (unsigned long long)(w0 + j) * 32ull + lane;
         const bool act = (aw >> lane) & 1u;
         unsigned long long deg = 0, o0 = 0;
-        if (act) { o0 = __ldg(a.off + v); deg = __ldg(a.off + v + 1) - o0; }
+#pragma unroll
+        for (int u = 0; u < kBatch; ++u)
+            if ((j & (kBatch - 1)) == u) { deg = degB[u]; o0 = o0B[u]; }
         const bool st = (sw >> lane) & 1u;
         const bool hit = act && st, miss = act && !st;
         const uint32_t hw = aw & sw;
