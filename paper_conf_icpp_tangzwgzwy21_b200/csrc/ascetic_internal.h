@@ -41,7 +41,7 @@ struct IterTotals {
     uint32_t n_small, n_med, n_hub, n_missq, n_runs, n_pieces;
     uint32_t tile_counter, done_counter;
     uint32_t ready;          // set to 1 last (host spin target)
-    uint32_t pad;
+    uint32_t host_runs;      // runs copied to the mapped run list (0 = not copied)
     unsigned long long nS;   // |S ∩ owned range| (static vertices of this rank in this iteration)
     unsigned long long miss_h0, miss_h1;   // host arc span of the miss stream: off[first miss], off[last miss + 1]
 };
@@ -74,8 +74,10 @@ struct ClassifyArgs {
     IterTotals* tot;                   // device, zero on entry
     IterTotals* tot_next;              // device: zeroed by the last CTA for the next classify (no memset launch)
     IterTotals* host_tot;              // mapped pinned
-    uint32_t* host_runs;               // mapped pinned: (b, e) of the first host_runs_cap runs
-    uint32_t host_runs_cap;
+    uint32_t* host_runs;               // mapped pinned: (b, e) of the first host_runs_cap runs, written (by the
+    uint32_t host_runs_cap;            // last CTA) only when the host will plan DMAs: force_host_runs, or at
+    uint32_t force_host_runs;          // most host_runs_cap runs averaging >= dma_min_run_arcs arcs
+    unsigned long long dma_min_run_arcs;
 };
 
 // Device state handed to the edge / finalize kernels.

@@ -705,6 +705,8 @@ void Part::classify(uint32_t t) {
     tot_buf_ ^= 1u;
     ca.host_tot = h_tot_;
     ca.host_runs = h_runs_; ca.host_runs_cap = kRunsHostMax;
+    ca.force_host_runs = o_.xfer_mode == 2 ? 1u : 0u;
+    ca.dma_min_run_arcs = o_.xfer_mode == 0 ? std::max<uint64_t>(1, o_.dma_min_run / g_.b_e) : ~0ull;
     cudaEvent_t e0 = mark(cs_, true);   // every iteration: its start marks the iteration's wall time
     launch_classify(ca, cs_);
     CK(cudaGetLastError());
@@ -834,13 +836,14 @@ void Part::expand(uint32_t t, const IterTotals& T) {
             plan_span_windows(T))
             mode = 3;
         if (mode == 2) {
-            // the run list is already in mapped host memory (classify writes the first
-            // kRunsHostMax runs there): no device round trip before the DMAs can be planned
+            // the run list is already in mapped host memory (classify's last CTA copies the first
+            // kRunsHostMax runs there when the iteration qualifies for DMAs): no device round trip
+            // before the DMAs can be planned
             rb_.resize(T.n_runs); re_.resize(T.n_runs); rdst_.resize(T.n_runs);
             const volatile uint32_t* hr = h_runs_;
-            const uint32_t nh = std::min<uint32_t>(T.n_runs, kRunsHostMax);
+            const uint32_t nh = std::min<uint32_t>(T.host_runs, T.n_runs);
             for (uint32_t r = 0; r < nh; ++r) { rb_[r] = hr[2 * r]; re_[r] = hr[2 * r + 1]; }
-            if (T.n_runs > nh) {   // forced DMA mode with a long run list: fetch the rest
+            if (T.n_runs > nh) {   // forced DMA mode with a long run list (or none copied): fetch the rest
                 CK(cudaMemcpy(rb_.data() + nh, d_run_b_ + nh, (T.n_runs - nh) * 4ull, cudaMemcpyDeviceToHost));
                 CK(cudaMemcpy(re_.data() + nh, d_run_e_ + nh, (T.n_runs - nh) * 4ull, cudaMemcpyDeviceToHost));
             }

@@ -339,12 +339,10 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
                 const uint32_t r = bR + __popc(starts & lt);
                 a.run_b[r] = (uint32_t)v;
                 a.run_dst[r] = bArcs + ex;
-                if (r < a.host_runs_cap) a.host_runs[2 * r] = (uint32_t)v;        // DMA planning copy
             }
             if ((ends >> lane) & 1u) {
                 const uint32_t r = bR + __popc(starts & le) - 1u;
                 a.run_e[r] = (uint32_t)(v + 1);
-                if (r < a.host_runs_cap) a.host_runs[2 * r + 1] = (uint32_t)(v + 1);
             }
             bQ += __popc(balQ);
             bR += __popc(starts);
@@ -353,6 +351,9 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
     }
 
     // ---------------- non-scan totals, completion, totals to host
+    // Only the last CTA writes host (mapped) memory, so the others need only a GPU-scope fence before
+    // their completion count (a system-scope fence in every CTA cost a PCIe round trip each).
+    __shared__ uint32_t s_last;
     __syncthreads();
     if (threadIdx.x == 0) {
         unsigned long long t[6] = {0, 0, 0, 0, 0, 0};
@@ -364,38 +365,55 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
         if (t[3]) atomicAdd(&a.tot->active_arcs, t[3]);
         if (t[4]) atomicAdd(&a.tot->hit_arcs, t[4]);
         atomicAdd(&a.tot->digest, t[5]);                 // Σ mod 2^64
-        __threadfence_system();   // this CTA's mapped-memory run writes before its completion count
-        const uint32_t done = atomicAdd(&a.tot->done_counter, 1u);
-        if (done == a.ntiles - 1) {
-            __threadfence();
-            const ScanVal fin = sv_load_volatile(&a.tile_incl[a.ntiles - 1]);
-            volatile IterTotals* vt = a.tot;
-            IterTotals* h = a.host_tot;
-            h->nA = vt->nA; h->nH = vt->nH; h->nM = vt->nM; h->nS = vt->nS;
-            h->active_arcs = vt->active_arcs; h->hit_arcs = vt->hit_arcs; h->digest = vt->digest;
-            h->miss_arcs = fin.miss_arcs;
-            h->n_small = fin.small; h->n_med = fin.med; h->n_hub = fin.hub;
-            h->n_missq = fin.missq; h->n_runs = fin.runs; h->n_pieces = fin.pieces;
-            a.tot->miss_arcs = fin.miss_arcs;
-            a.tot->n_small = fin.small; a.tot->n_med = fin.med; a.tot->n_hub = fin.hub;
-            a.tot->n_missq = fin.missq; a.tot->n_runs = fin.runs; a.tot->n_pieces = fin.pieces;
-            // host span of the miss stream (the queue is in ascending id, so host order): first list's
-            // start, last list's end; the other CTAs' queue writes are visible after the done count
-            unsigned long long h0 = 0, h1 = 0;
-            if (fin.missq) {
-                const volatile unsigned long long* src = a.mq_src;
-                const volatile unsigned long long* pre = a.mq_pre;
-                h0 = src[0];
-                h1 = src[fin.missq - 1] + (fin.miss_arcs - pre[fin.missq - 1]);
-            }
-            h->miss_h0 = h0; h->miss_h1 = h1;
-            {   // the next classify's totals start from zero
-                unsigned long long* z = reinterpret_cast<unsigned long long*>(a.tot_next);
-                for (size_t i = 0; i < sizeof(IterTotals) / 8; ++i) z[i] = 0ull;
-            }
-            __threadfence_system();
-            *reinterpret_cast<volatile uint32_t*>(&h->ready) = 1u;
+        __threadfence();          // this CTA's queue / run writes before its completion count
+        s_last = atomicAdd(&a.tot->done_counter, 1u) == a.ntiles - 1;
+    }
+    __syncthreads();
+    if (!s_last) return;
+    __threadfence();
+    const ScanVal fin = sv_load_volatile(&a.tile_incl[a.ntiles - 1]);
+    // the run list goes to the host only when the host will plan copy-engine DMAs from it (few,
+    // long runs, or DMA forced): the first host_runs_cap runs, copied by the whole CTA
+    const bool dma = fin.runs && (a.force_host_runs ||
+                                  (fin.runs <= a.host_runs_cap && fin.miss_arcs >= (unsigned long long)fin.runs * a.dma_min_run_arcs));
+    if (dma) {
+        const uint32_t nr = min(fin.runs, a.host_runs_cap);
+        const volatile uint32_t* rb = a.run_b;
+        const volatile uint32_t* re = a.run_e;
+        for (uint32_t r = threadIdx.x; r < nr; r += blockDim.x) {
+            a.host_runs[2 * r] = rb[r];
+            a.host_runs[2 * r + 1] = re[r];
         }
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) {
+        volatile IterTotals* vt = a.tot;
+        IterTotals* h = a.host_tot;
+        h->nA = vt->nA; h->nH = vt->nH; h->nM = vt->nM; h->nS = vt->nS;
+        h->active_arcs = vt->active_arcs; h->hit_arcs = vt->hit_arcs; h->digest = vt->digest;
+        h->miss_arcs = fin.miss_arcs;
+        h->n_small = fin.small; h->n_med = fin.med; h->n_hub = fin.hub;
+        h->n_missq = fin.missq; h->n_runs = fin.runs; h->n_pieces = fin.pieces;
+        h->host_runs = dma ? min(fin.runs, a.host_runs_cap) : 0u;
+        a.tot->miss_arcs = fin.miss_arcs;
+        a.tot->n_small = fin.small; a.tot->n_med = fin.med; a.tot->n_hub = fin.hub;
+        a.tot->n_missq = fin.missq; a.tot->n_runs = fin.runs; a.tot->n_pieces = fin.pieces;
+        // host span of the miss stream (the queue is in ascending id, so host order): first list's
+        // start, last list's end; the other CTAs' queue writes are visible after the done count
+        unsigned long long h0 = 0, h1 = 0;
+        if (fin.missq) {
+            const volatile unsigned long long* src = a.mq_src;
+            const volatile unsigned long long* pre = a.mq_pre;
+            h0 = src[0];
+            h1 = src[fin.missq - 1] + (fin.miss_arcs - pre[fin.missq - 1]);
+        }
+        h->miss_h0 = h0; h->miss_h1 = h1;
+        {   // the next classify's totals start from zero
+            unsigned long long* z = reinterpret_cast<unsigned long long*>(a.tot_next);
+            for (size_t i = 0; i < sizeof(IterTotals) / 8; ++i) z[i] = 0ull;
+        }
+        __threadfence_system();   // the CTA's host writes (runs, totals) before the ready flag
+        *reinterpret_cast<volatile uint32_t*>(&h->ready) = 1u;
     }
 }
 
