@@ -54,6 +54,7 @@ struct ClassifyArgs {
     uint64_t vlo, vhi;                 // owned vertex range of this rank
     uint32_t nwords;
     uint32_t ntiles;
+    uint32_t words_per_warp;           // 32, or 4 for small bitmaps (tile = kClassifyWarps * words_per_warp words)
     uint32_t hub_deg;
     uint32_t piece_arcs;
     uint32_t* hq_small;

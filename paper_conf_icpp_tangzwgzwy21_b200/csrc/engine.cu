@@ -197,7 +197,9 @@ void Part::alloc_vertex_state() {
     const uint64_t n = g_.n, m = g_.m;
     vertex_bytes_ = 0;
     nwords_ = (uint32_t)((n + 31) / 32);
-    ntiles_ = (nwords_ + kTileWords - 1) / kTileWords;
+    // classify tiles: 32 words per warp, or 4 when that would leave more than half the SMs idle
+    wpw_ = (nwords_ + kTileWords - 1) / kTileWords < (uint32_t)(2 * sm_count_) ? 4u : 32u;
+    ntiles_ = (nwords_ + kClassifyWarps * wpw_ - 1) / (kClassifyWarps * wpw_);
     dalloc(&d_off_, n + 1, &vertex_bytes_);
     dalloc(&d_A_, nwords_, &vertex_bytes_);
     dalloc(&d_S_, nwords_, &vertex_bytes_);
@@ -694,7 +696,7 @@ void Part::classify(uint32_t t) {
     }
     ClassifyArgs ca;
     ca.A = d_A_; ca.S = d_S_; ca.off = d_off_; ca.n = g_.n; ca.vlo = vlo_; ca.vhi = vhi_;
-    ca.nwords = nwords_; ca.ntiles = ntiles_;
+    ca.nwords = nwords_; ca.ntiles = ntiles_; ca.words_per_warp = wpw_;
     ca.hub_deg = o_.hub_deg; ca.piece_arcs = kPieceArcs;
     ca.hq_small = d_hq_small_; ca.hq_med = d_hq_med_; ca.hq_hub = d_hq_hub_; ca.hub_pre = d_hub_pre_;
     ca.mq = d_mq_; ca.mq_pre = d_mq_pre_; ca.mq_src = d_mq_src_; ca.tile_first = d_tile_first_;

@@ -166,7 +166,7 @@ class Part {
     bool timing_ = true;
     bool fine_ = true;   // this iteration records per-phase spans
     // device vertex state
-    uint32_t nwords_ = 0, ntiles_ = 0;
+    uint32_t nwords_ = 0, ntiles_ = 0, wpw_ = 32;
     unsigned long long* d_off_ = nullptr;
     uint32_t *d_A_ = nullptr, *d_S_ = nullptr, *d_next_ = nullptr, *d_visited_ = nullptr;
     uint32_t *d_val_ = nullptr, *d_snap_ = nullptr;

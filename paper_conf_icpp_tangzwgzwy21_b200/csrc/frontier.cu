@@ -113,6 +113,10 @@ __device__ __forceinline__ ScanVal sv_load_volatile(const ScanVal* p) {
     return v;
 }
 
+// WPW = bitmap words per warp: 32 (a tile = 8192 vertices) or, for small bitmaps that would leave most
+// SMs idle, 4 (a tile = 1024 vertices: each warp's serial walk over its words is 8x shorter, which is
+// what bounds a small graph's classify, ~30 us at C1's 8 tiles of 32 words)
+template <int WPW>
 __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a) {
     __shared__ uint32_t s_tile;
     __shared__ ScanVal s_warp[kClassifyWarps];
@@ -125,32 +129,33 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
     if (threadIdx.x == 0) s_tile = atomicAdd(&a.tot->tile_counter, 1u);
     __syncthreads();
     const uint32_t tile = s_tile;
-    const uint32_t w0 = tile * kTileWords + warp * 32;
+    const uint32_t w0 = tile * (kClassifyWarps * WPW) + warp * WPW;
     const uint32_t myw = w0 + lane;
+    const bool mine_w = lane < WPW && myw < a.nwords;
 
     // A is replicated across ranks; this rank classifies only its owned range [vlo, vhi)
     // while |A| and the digest are taken over the whole bitmap.
     uint32_t myAll = 0, myS = 0;
-    if (myw < a.nwords) { myAll = __ldg(a.A + myw); myS = __ldg(a.S + myw); }
+    if (mine_w) { myAll = __ldg(a.A + myw); myS = __ldg(a.S + myw); }
     const uint32_t myA = myAll & own_mask(myw, a.vlo, a.vhi);
     const uint32_t myMiss = myA & ~myS;
     uint32_t prevMiss = 0, nextMiss = 0;
     if (w0 > 0 && w0 - 1 < a.nwords)
         prevMiss = __ldg(a.A + w0 - 1) & ~__ldg(a.S + w0 - 1) & own_mask(w0 - 1, a.vlo, a.vhi);
-    if (w0 + 32 < a.nwords)
-        nextMiss = __ldg(a.A + w0 + 32) & ~__ldg(a.S + w0 + 32) & own_mask(w0 + 32, a.vlo, a.vhi);
+    if (w0 + WPW < a.nwords)
+        nextMiss = __ldg(a.A + w0 + WPW) & ~__ldg(a.S + w0 + WPW) & own_mask(w0 + WPW, a.vlo, a.vhi);
     const uint32_t anyA = __ballot_sync(FULL, myA != 0);
     const uint32_t piece = a.piece_arcs;
 
     // Both phases walk the warp's 32 words one at a time (prefix order), but the offsets of the active
     // vertices are loaded kBatch words ahead: with few CTAs (small graphs) each dependent off[] load
     // chain costs ~0.5 us, so one load round trip per word made a C1 classify ~20 us.
-    constexpr int kBatch = 8;
+    constexpr int kBatch = WPW < 8 ? WPW : 8;
     // ---------------- phase A: per-warp counts
     ScanVal mine = sv_zero();
     unsigned long long aArcs = 0, hArcs = 0;
     unsigned long long degA[kBatch];
-    for (int j = 0; j < 32; ++j) {
+    for (int j = 0; j < WPW; ++j) {
         if ((j & (kBatch - 1)) == 0) {
             const uint32_t any8 = (anyA >> j) & ((1u << kBatch) - 1u);
 #pragma unroll
@@ -197,7 +202,7 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
         unsigned long long nA = __popc(myAll), nH = __popc(myA & myS), nM = __popc(myMiss);
         unsigned long long nS = wsum64((unsigned long long)__popc(myS & own_mask(myw, a.vlo, a.vhi)));
         if (lane == 0 && nS) atomicAdd(&a.tot->nS, nS);
-        unsigned long long dg = (myw < a.nwords) ? mix64((unsigned long long)myw ^ ((unsigned long long)myAll * PHI)) : 0ull;
+        unsigned long long dg = mine_w ? mix64((unsigned long long)myw ^ ((unsigned long long)myAll * PHI)) : 0ull;
         nA = wsum64(nA); nH = wsum64(nH); nM = wsum64(nM); dg = wsum64(dg);
         aArcs = wsum64(aArcs); hArcs = wsum64(hArcs);
         if (lane == 0) {
@@ -265,7 +270,7 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
     uint32_t bS = wb.small, bM = wb.med, bH = wb.hub, bQ = wb.missq, bR = wb.runs, bP = wb.pieces;
     unsigned long long bArcs = wb.miss_arcs;
     unsigned long long o0B[kBatch], degB[kBatch];
-    for (int j = 0; j < 32; ++j) {
+    for (int j = 0; j < WPW; ++j) {
         if ((j & (kBatch - 1)) == 0) {
             const uint32_t any8 = (anyA >> j) & ((1u << kBatch) - 1u);
 #pragma unroll
@@ -284,7 +289,7 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
         const uint32_t pm = __shfl_sync(FULL, myMiss, (j + 31) & 31);
         const uint32_t nm = __shfl_sync(FULL, myMiss, (j + 1) & 31);
         const uint32_t carry_in = (j == 0 ? prevMiss : pm) >> 31;
-        const uint32_t carry_out = (j == 31 ? nextMiss : nm) & 1u;
+        const uint32_t carry_out = (j == WPW - 1 ? nextMiss : nm) & 1u;
         const unsigned long long v = (unsigned long long)(w0 + j) * 32ull + lane;
         const bool act = (aw >> lane) & 1u;
         unsigned long long deg = 0, o0 = 0;
@@ -421,7 +426,8 @@ __global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a
 
 void launch_classify(const ClassifyArgs& a, cudaStream_t s) {
     if (a.ntiles == 0) return;
-    k_classify<<<a.ntiles, kClassifyWarps * 32, 0, s>>>(a);
+    if (a.words_per_warp == 4) k_classify<4><<<a.ntiles, kClassifyWarps * 32, 0, s>>>(a);
+    else k_classify<32><<<a.ntiles, kClassifyWarps * 32, 0, s>>>(a);
     ++g_launches;
 }
 
