@@ -168,7 +168,8 @@ typedef struct {
     uint64_t dma_chunks, gather_chunks;
     double time_run_s;            /* ascetic_run wall time incl. fill, all H2D, all exchange */
     double time_fill_s;
-    double time_h2d_busy_s;       /* copy-stream busy time (sum of chunk transfers) */
+    double time_h2d_busy_s;       /* copy-stream busy time (sum of chunk transfers, fill and swaps; per-phase
+                                     spans exist only in iterations TIMING selects) */
     double gteps;                 /* active_arcs_total / time_run_s / 1e9 */
     double gteps_excl_fill;
     uint64_t vertex_state_bytes;  /* device bytes outside the edge budget */
@@ -179,10 +180,11 @@ typedef struct {
     uint64_t static_arcs;         /* arcs they processed */
     double time_ondemand_s;       /* on-demand chunk edge kernels */
     uint64_t ondemand_arcs;
-    double time_gather_s;         /* zero-copy gather kernels (transfer engine, SM path) */
-    uint64_t gather_bytes;
-    double time_dma_s;            /* copy-engine chunk DMAs */
-    uint64_t dma_bytes;
+    double time_gather_s;         /* gather-mode chunk transfers: the zero-copy SM gather (with the copy-engine
+                                     long runs beside it); CUDA events on the copy stream(s) */
+    uint64_t gather_bytes;        /* payload of those chunks */
+    double time_dma_s;            /* copy-engine chunk DMAs (runs and span windows) */
+    uint64_t dma_bytes;           /* payload of those chunks (span windows: without their holes) */
     double time_finalize_s;
     double time_host_s;           /* host planning + waits between classify and the next launches */
     uint64_t repartitions;        /* Eq. 3 re-partitions performed (ASCETIC_OPT_REPARTITION) */
