@@ -683,7 +683,9 @@ void Part::begin(int algo, uint32_t source, uint32_t max_iters, bool timing) {
     CK(cudaEventRecord(ev_fill1_, xs_));
     launch_init(algo, dev_state(0), source, cs_);
     CK(cudaGetLastError());
-    CK(cudaStreamWaitEvent(cs_, ev_fill1_, 0));
+    // only the static-hit kernels read the Static Region: iteration 0's classify and its chunk
+    // transfers (queued on the copy stream right behind the fill) need not wait for the fill
+    CK(cudaStreamWaitEvent(ss_, ev_fill1_, 0));
 }
 
 void Part::classify(uint32_t t) {
