@@ -91,6 +91,75 @@ __global__ void __launch_bounds__(256) ld_gather(const uint64_t* __restrict__ sr
     }
 }
 
+// baseline 2: the product gather's load shape -- 16-byte loads of the piece's 16-byte-aligned cover
+// (k_gather16), one warp per piece, NG units in flight per lane; each lane stores the 8-byte words
+// of its unit that fall inside the piece
+template <int NG>
+__global__ void __launch_bounds__(256) ld16_gather(const uint4* __restrict__ src, const uint64_t* __restrict__ pa,
+                                                   const uint32_t* __restrict__ plen, const uint64_t* __restrict__ pdst,
+                                                   uint32_t npieces, uint64_t* __restrict__ dst) {
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t nw = gridDim.x * 8;
+    for (uint32_t i = blockIdx.x * 8 + warp; i < npieces; i += nw) {
+        const uint64_t a = pa[i], b = a + plen[i];
+        const uint64_t u0 = a >> 4, u1 = (b + 15) >> 4;
+        uint64_t* d8 = dst + pdst[i] / 8;
+        for (uint64_t u = u0; u < u1; u += 32 * NG) {
+            uint4 v[NG];
+#pragma unroll
+            for (int g = 0; g < NG; ++g) {
+                const uint64_t uu = u + 32 * g + lane;
+                if (uu < u1) v[g] = src[uu];
+            }
+#pragma unroll
+            for (int g = 0; g < NG; ++g) {
+                const uint64_t uu = u + 32 * g + lane;
+                if (uu >= u1) continue;
+                const uint64_t w0 = uu * 16, w1 = w0 + 8;
+                if (w0 >= a && w0 < b) d8[(w0 - a) / 8] = ((uint64_t)v[g].y << 32) | v[g].x;
+                if (w1 >= a && w1 < b) d8[(w1 - a) / 8] = ((uint64_t)v[g].w << 32) | v[g].z;
+            }
+        }
+    }
+}
+
+// TMA gather with two slots per warp: the bulk copy of piece i+1 is in flight while the warp
+// stores piece i
+template <int SLOT>
+__global__ void __launch_bounds__(256) tma_gather2(const char* __restrict__ src, const uint64_t* __restrict__ pa,
+                                                   const uint32_t* __restrict__ plen, const uint64_t* __restrict__ pdst,
+                                                   uint32_t npieces, uint64_t* __restrict__ dst) {
+    extern __shared__ __align__(128) char smem[];
+    __shared__ __align__(8) uint64_t bar[16];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    char* slot[2] = {smem + (2 * warp) * (SLOT + 32), smem + (2 * warp + 1) * (SLOT + 32)};
+    if (lane == 0) {
+        mbar_init(&bar[2 * warp], 1); mbar_init(&bar[2 * warp + 1], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncwarp();
+    uint32_t phase[2] = {0, 0};
+    const uint32_t nw = gridDim.x * 8;
+    auto issue = [&](uint32_t i, int k) {
+        const uint64_t a = pa[i], len = plen[i];
+        const uint64_t a16 = a & ~15ull, b16 = (a + len + 15) & ~15ull;
+        if (lane == 0) { mbar_expect(&bar[2 * warp + k], (uint32_t)(b16 - a16)); bulk_g2s(slot[k], src + a16, (uint32_t)(b16 - a16), &bar[2 * warp + k]); }
+    };
+    uint32_t i = blockIdx.x * 8 + warp;
+    int k = 0;
+    if (i < npieces) issue(i, 0);
+    for (; i < npieces; i += nw, k ^= 1) {
+        if (i + nw < npieces) issue(i + nw, k ^ 1);
+        mbar_wait(&bar[2 * warp + k], phase[k]);
+        phase[k] ^= 1;
+        const uint64_t a = pa[i], len = plen[i];
+        const uint64_t* s8 = reinterpret_cast<const uint64_t*>(slot[k] + (a - (a & ~15ull)));
+        uint64_t* d8 = dst + pdst[i] / 8;
+        for (uint32_t q = lane; q < len / 8; q += 32) d8[q] = s8[q];
+        __syncwarp();
+    }
+}
+
 int main() {
     const size_t bytes = 512ull << 20;
     char* h; CK(cudaHostAlloc((void**)&h, bytes + 4096, cudaHostAllocMapped | cudaHostAllocPortable));
@@ -121,6 +190,7 @@ int main() {
         }
     }
     CK(cudaFuncSetAttribute(tma_gather<4096>, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * (4096 + 32)));
+    CK(cudaFuncSetAttribute(tma_gather2<4096>, cudaFuncAttributeMaxDynamicSharedMemorySize, 16 * (4096 + 32)));
     for (int avg_bytes : {256, 768, 1100, 2048, 8192, 65536}) {
         std::mt19937_64 rng(avg_bytes);
         std::vector<uint64_t> pa, pd; std::vector<uint32_t> pl;
@@ -146,6 +216,10 @@ int main() {
             timeit([&] { tma_gather<4096><<<grid, 256, 8 * (4096 + 32)>>>(hd, dpa, dpl, dpd, (uint32_t)pa.size(), (uint64_t*)d); }, nm, (double)total);
             snprintf(nm, sizeof nm, "ld  gather runs avg %dB grid=%d", avg_bytes, grid);
             timeit([&] { ld_gather<<<grid, 256>>>((const uint64_t*)hd, dpa, dpl, dpd, (uint32_t)pa.size(), (uint64_t*)d); }, nm, (double)total);
+            snprintf(nm, sizeof nm, "ld16 cover gather (k_gather16 shape) avg %dB grid=%d", avg_bytes, grid);
+            timeit([&] { ld16_gather<4><<<grid, 256>>>((const uint4*)hd, dpa, dpl, dpd, (uint32_t)pa.size(), (uint64_t*)d); }, nm, (double)total);
+            snprintf(nm, sizeof nm, "TMA gather 2 slots/warp avg %dB grid=%d", avg_bytes, grid);
+            timeit([&] { tma_gather2<4096><<<grid, 256, 16 * (4096 + 32)>>>(hd, dpa, dpl, dpd, (uint32_t)pa.size(), (uint64_t*)d); }, nm, (double)total);
         }
         cudaFree(dpa); cudaFree(dpd); cudaFree(dpl);
     }
