@@ -188,6 +188,23 @@ def shared_graph(config: str, barrier, local_rank: int, tag: str, alloc_local=No
     return g, cleanup, gen_s
 
 
+def spans_cover(per: list) -> bool:
+    """True when the library's per-phase CUDA-event spans cover every class of work in these steps
+    (TIMING=1 gives small iterations one span, leaving their per-kernel times at 0)."""
+    for s in per:
+        if s["gather_bytes"] and not s["time_gather_s"]:
+            return False
+        if s["ondemand_arcs"] and not s["time_ondemand_s"]:
+            return False
+        if s["static_arcs"] and not s["time_static_s"]:
+            return False
+        if (s["h2d_payload_bytes"] + s["h2d_static_fill_bytes"]) and not s["time_h2d_busy_s"]:
+            return False
+        if s["iterations"] and not s["time_classify_s"]:
+            return False
+    return True
+
+
 def roofline_of(per: list, steps: int, total_ms: float, b_e: int, n: int, h2d_peak: float, hbm_peak: float,
                 hbm_src: str, config: str) -> dict:
     """Roofline entry of a bench line from the library's per-step stats (pure: unit-tested on CPU)."""
@@ -318,6 +335,9 @@ def main():
     ap.add_argument("--impl", default="ascetic", choices=["ascetic", "reference"])
     ap.add_argument("--config", default="c4", choices=["c1", "c2", "c3", "c4", "c5"])
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--profile-steps", type=int, default=3,
+                    help="extra steps with every phase timed, for the roofline breakdown when the timed steps "
+                         "left small iterations as one span (after the timed region)")
     ap.add_argument("--no-pageable", action="store_true", help="skip the pageable-input load_csr measurement")
     ap.add_argument("--c5-algo", default="bfs", choices=["bfs", "pr"], help="C5 (BFS + PageRank): which one a step runs")
     ap.add_argument("--c5-pr-iters", type=int, default=43, help="C5 PageRank iterations per step")
@@ -325,6 +345,8 @@ def main():
     ap.add_argument("--ref-pr-iters", type=int, default=2, help="PR iterations per reference step (bounded)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--xfer", type=int, default=0)
+    ap.add_argument("--opt", action="append", default=[], metavar="NAME=VALUE",
+                    help="extra library option for A/B runs (ascetic_set_option), repeatable")
     ap.add_argument("--sparse-exchange", type=int, default=0,
                     help="N > 1, BFS/SSSP/CC: ASCETIC_OPT_SPARSE_EXCHANGE divisor d (0 = dense exchange)")
     args = ap.parse_args()
@@ -384,6 +406,9 @@ def main():
     asc.set_budget(budget)
     asc.set_option("xfer_mode", args.xfer)
     asc.set_option("sparse_exchange", args.sparse_exchange)
+    for kv in args.opt:
+        k_, v_ = kv.split("=", 1)
+        asc.set_option(k_, int(v_))
     l2_flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
 
     def step(i):
@@ -447,6 +472,28 @@ def main():
     value_excl_fill = arcs_all / ((total_ms - fill_ms) / 1e3) / 1e9 if total_ms > fill_ms else None
 
     roofline = roofline_of(per, args.steps, total_ms, g.b_e, g.n, h2d_peak, hbm_peak, hbm_src, args.config)
+    if not spans_cover(per) and args.profile_steps > 0:
+        # small iterations ran with one span each (TIMING=1 keeps per-phase events off the latency path),
+        # so the per-kernel classes above are incomplete: take them from extra steps with every phase
+        # timed, run AFTER the timed region (their event overhead never reaches `value`)
+        asc.set_option("timing", 2)
+        prof, prof_ms = [], 0.0
+        for k in range(args.profile_steps):
+            l2_flush.fill_(k & 0xFF)
+            torch.cuda.synchronize()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record()
+            prof.append(step(args.warmup + k))
+            e1.record()
+            torch.cuda.synchronize()
+            prof_ms += e0.elapsed_time(e1)
+        asc.set_option("timing", 1)
+        roofline = roofline_of(prof, args.profile_steps, prof_ms, g.b_e, g.n, h2d_peak, hbm_peak, hbm_src,
+                               args.config)
+        roofline["phase_spans"] = (f"{args.profile_steps} extra steps with every phase timed (TIMING=2), after "
+                                   f"the timed region: {prof_ms / args.profile_steps:.3f} ms per step with the "
+                                   f"events vs {total_ms / args.steps:.3f} timed")
     h2d_total = fill + payload
     span_holes = _sum_ranks(sum(s["span_link_bytes"] - s["span_payload_bytes"] for s in per))
     link = {"h2d_bytes": h2d_total, "h2d_busy_s": sum(s["time_h2d_busy_s"] for s in per),
@@ -572,6 +619,7 @@ def main():
                    "sources": srcs if algo in ("bfs", "sssp") else None,
                    "l2": "flushed (512 MiB write) between timed steps; graph > L2",
                    "graph_gen_s": round(gen_s, 2),
+                   "options": args.opt or None,
                    "parallelism": f"{ws} process(es), one GPU each" + ("" if ws == 1 else
                                   ": 1D edge-balanced vertex ranges, per-rank static region and budget, "
                                   "NCCL exchange per iteration (OR / MIN / SUM + slice broadcast)"

@@ -141,8 +141,12 @@ typedef enum {
                                       bytes (the holes ride along, ~55 GB/s for the whole window), and
                                       gathers the sparser windows; the on-demand kernels read a DMA'd window in
                                       place. Payload accounting is unchanged; span_link_bytes counts the holes. */
-    ASCETIC_OPT_SPAN_MAX_RATIO = 25  /* percent (default 200): auto span planning only when the miss stream's host
+    ASCETIC_OPT_SPAN_MAX_RATIO = 25, /* percent (default 200): auto span planning only when the miss stream's host
                                       span is at most this share of its payload (windows then decided one by one) */
+    ASCETIC_OPT_FUSED_VISIT = 26     /* BFS, SM-gathered chunks: the gather visits the ids it lands (On-demand
+                                      Computing P:694 fused into the transfer; the chunk is still written).
+                                      1 (default) = for small chunks (two buffers of < 4 MiB, where the
+                                      gather -> on-demand chain is the latency), 2 = every gathered chunk, 0 = off */
 } ascetic_option;
 
 typedef struct {

@@ -39,7 +39,8 @@ OPTIONS = {"chunk_cap": 1, "xfer_mode": 2, "dma_min_run": 3, "overlap": 4, "keep
            "replace_policy": 15, "placement_seed": 16, "prd_tol_ppm": 17,
            "fused_exchange": 18, "sparse_exchange": 19, "relax_mode": 20,
            "ce_min_run": 21, "gap_bridge": 22, "pr_segment": 23,
-           "span_density": 24, "span_max_ratio": 25}
+           "span_density": 24, "span_max_ratio": 25,
+           "fused_visit": 26}
 INF = 0xFFFFFFFF
 
 

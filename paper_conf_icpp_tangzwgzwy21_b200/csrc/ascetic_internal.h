@@ -157,7 +157,8 @@ void launch_span_windows(const Queues& q, unsigned long long h0, unsigned long l
 // adds the number of 16-byte host units it loads to *cover
 void launch_gather(const Queues& q, const void* host_nbr, uint64_t m, uint32_t b_e, void* chunk,
                    unsigned long long lo, unsigned long long hi, int max_ctas, const unsigned long long* lint,
-                   uint32_t nlint, uint32_t gap_bytes, unsigned long long* cover, cudaStream_t s);
+                   uint32_t nlint, uint32_t gap_bytes, unsigned long long* cover, cudaStream_t s,
+                   const DevState* visit = nullptr);   // BFS: visit the landed ids in the gather (fused)
 // long miss runs (>= min_arcs arcs): append (b, e, dst) of each into out[3*i] (mapped host memory,
 // unordered, at most cap), count into *count; `flag` set to 1 by the last CTA (host spin target)
 void launch_long_runs(const uint32_t* run_b, const uint32_t* run_e, const unsigned long long* run_dst, uint32_t n_runs,

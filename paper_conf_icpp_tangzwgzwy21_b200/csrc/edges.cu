@@ -803,12 +803,20 @@ __device__ __forceinline__ uint4 ld_host16(const uint4* p) {
 // instruction are not what the link charges for.
 // Long runs: stream intervals lint[2i, 2i+1) (sorted, disjoint; whole vertices) go through the copy
 // engines instead (Part::transfer_chunk); their vertices are skipped here.
-template <int BE, int NG>
+// VISIT (BFS, 4-byte arcs): On-demand Computing fused into the landing of the chunk -- each word
+// the gather stores is a neighbour id, visited right there (visited-word loads of the lane's words
+// batched, then a fire-and-forget OR into next for the unvisited ones), so the chunk needs no
+// separate on-demand kernel. The chunk is still written (the On-demand Region holds the data as
+// before); what goes is one kernel launch per chunk and the chunk re-read. Used for small chunks,
+// where the gather -> on-demand launch chain is the latency of the iteration (C1).
+template <int BE, int NG, bool VISIT>
 __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restrict__ host, uint32_t hoff,
                                                   unsigned long long w_end, uint32_t* __restrict__ chunk,
                                                   unsigned long long lo, unsigned long long hi,
                                                   const unsigned long long* __restrict__ lint, uint32_t nlint,
-                                                  uint32_t gap_words, unsigned long long* __restrict__ cover) {
+                                                  uint32_t gap_words, unsigned long long* __restrict__ cover,
+                                                  DevState d) {
+    static_assert(!VISIT || BE == 4, "fused visit: BFS arcs are bare 4-byte ids");
     // tile metadata staged in shared memory (reading it through L1 instead gathers at the same rate,
     // but its L1 traffic slows the concurrent static-hit kernels)
     __shared__ unsigned long long s_pre[kEdgeTile + 1];
@@ -930,6 +938,28 @@ __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restr
                     for (int c = 0; c < 4; ++c) {
                         const unsigned long long w = uw[g] * 4 + c;
                         if (w >= pw0[g] && w < pw1[g]) chunk[pd0[g] + (w - pw0[g])] = wv[c];
+                    }
+                }
+                if constexpr (VISIT) {
+                    // the lane's NG x 4 landed ids: all visited-word loads first, then the ORs
+                    uint32_t vw[NG][4];
+#pragma unroll
+                    for (int g = 0; g < NG; ++g) {
+#pragma unroll
+                        for (int c = 0; c < 4; ++c) {
+                            const unsigned long long w = uw[g] * 4 + c;
+                            const uint32_t id = c == 0 ? val[g].x : c == 1 ? val[g].y : c == 2 ? val[g].z : val[g].w;
+                            vw[g][c] = (uw[g] != ~0ull && w >= pw0[g] && w < pw1[g]) ? ld_state_ro(d.visited + (id >> 5)) : ~0u;
+                        }
+                    }
+#pragma unroll
+                    for (int g = 0; g < NG; ++g) {
+#pragma unroll
+                        for (int c = 0; c < 4; ++c) {
+                            const uint32_t id = c == 0 ? val[g].x : c == 1 ? val[g].y : c == 2 ? val[g].z : val[g].w;
+                            const uint32_t bit = 1u << (id & 31);
+                            if (!(vw[g][c] & bit)) atomicOr(d.next + (id >> 5), bit);   // result unused: RED.OR
+                        }
                     }
                 }
             }
@@ -1601,7 +1631,8 @@ void launch_ondemand(int algo, const DevState& d, const Queues& q, const void* c
 
 void launch_gather(const Queues& q, const void* host_nbr, uint64_t m, uint32_t b_e, void* chunk,
                    unsigned long long lo, unsigned long long hi, int max_ctas, const unsigned long long* lint,
-                   uint32_t nlint, uint32_t gap_bytes, unsigned long long* cover, cudaStream_t s) {
+                   uint32_t nlint, uint32_t gap_bytes, unsigned long long* cover, cudaStream_t s,
+                   const DevState* visit) {
     if (hi <= lo) return;
     const unsigned long long tiles = ((hi - 1) >> kEdgeTileShift) - (lo >> kEdgeTileShift) + 1;
     const unsigned grid = (unsigned)(tiles < (unsigned long long)max_ctas ? tiles : (unsigned long long)max_ctas);
@@ -1614,8 +1645,10 @@ void launch_gather(const Queues& q, const void* host_nbr, uint64_t m, uint32_t b
     // one per piece boundary, so 4 per lane (128) usually needs a second, nearly empty round; 6 took
     // C2's gather from 44.6-44.7 to 45.0 GB/s (profiles/r01/gather_ng_ab.log; 5 and 8 within noise of
     // 6). 4-byte arcs: 64 units per segment, 4 per lane fits.
-    if (b_e == 8) k_gather16<8, 6><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi, lint, nlint, gap_bytes / 4, cover);
-    else k_gather16<4, 4><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi, lint, nlint, gap_bytes / 4, cover);
+    const DevState none{};
+    if (b_e == 8) k_gather16<8, 6, false><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi, lint, nlint, gap_bytes / 4, cover, none);
+    else if (visit) k_gather16<4, 4, true><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi, lint, nlint, gap_bytes / 4, cover, *visit);
+    else k_gather16<4, 4, false><<<grid, 256, 0, s>>>(q, base, hoff, w_end, c, lo, hi, lint, nlint, gap_bytes / 4, cover, none);
     ++g_launches;
 }
 

@@ -481,7 +481,7 @@ void Part::span(cudaEvent_t a, cudaStream_t s, uint32_t t, int ph, int sub) {
 // ---- transfer engine: chunk = miss-stream arcs [lo, hi). mode 1: zero-copy SM gather over
 // the miss queue; mode 2: copy-engine DMA of the run pieces intersecting the window.
 void Part::transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsigned long long hi, int mode,
-                          cudaStream_t xs) {
+                          cudaStream_t xs, const DevState* visit) {
     if (mode == 1) {
         const uint32_t b_e = g_.b_e;
         // the long runs of the window go to the copy engines on the second copy stream, concurrently
@@ -515,7 +515,7 @@ void Part::transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsig
         // (measured: 64 CTAs at b_e = 8 -> same 47 GB/s, 3x faster on-demand kernels than 296)
         const int ctas = o_.gather_ctas ? o_.gather_ctas : (int)(64u * 8u / b_e);
         launch_gather(q, g_.nbr_dev, g_.m, b_e, d_chunk_[buf], lo, hi, ctas, nlint_ ? d_lint_[lint_buf_] : nullptr,
-                      nlint_, o_.gap_bridge, d_cover_, xs);
+                      nlint_, o_.gap_bridge, d_cover_, xs, visit);
         if (ce) {
             CK(cudaEventRecord(ce_done_[buf], xs2_));
             CK(cudaStreamWaitEvent(xs_, ce_done_[buf], 0));
@@ -885,6 +885,10 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     // windows: [k cap, (k+1) cap) of the miss stream, or (span mode) the host ranges of cap bytes
     // over the miss stream's span; a dense span window is one DMA of its host bytes and the
     // on-demand kernel reads it in place (span_base), a sparse one is gathered like mode 1
+    // BFS: On-demand Computing of a gathered chunk fused into its gather (the ids are visited as they
+    // land); not with copy-engine long runs beside the gather (their vertices are not in its lanes)
+    const bool fuse = algo_ == ALG_BFS && b_e == 4 && nlint_ == 0 &&
+                      (o_.fused_visit == 2 || (o_.fused_visit == 1 && alt));
     uint32_t nwin = nchunks;
     if (mode == 3) nwin = span_nwin_;
     uint32_t done = 0;
@@ -913,13 +917,15 @@ void Part::expand(uint32_t t, const IterTotals& T) {
         if (alt) {
             cudaStream_t sb = bst[buf];
             cudaEvent_t e0 = mark(sb);
-            transfer_chunk(q, buf, lo, hi, 1, sb);
+            transfer_chunk(q, buf, lo, hi, 1, sb, fuse ? &d : nullptr);
             CK(cudaGetLastError());
             span(e0, sb, t, PH_GATHER);
-            e0 = mark(sb);
-            launch_ondemand(algo_, d, q, d_chunk_[buf], lo, hi, ~0ull, sb);
-            CK(cudaGetLastError());
-            span(e0, sb, t, PH_OND);
+            if (!fuse) {
+                e0 = mark(sb);
+                launch_ondemand(algo_, d, q, d_chunk_[buf], lo, hi, ~0ull, sb);
+                CK(cudaGetLastError());
+                span(e0, sb, t, PH_OND);
+            }
             st.gather_bytes += (hi - lo) * b_e;
             ++st.gather_chunks;
             ++done;
@@ -932,7 +938,7 @@ void Part::expand(uint32_t t, const IterTotals& T) {
             if (wmode == 3) {
                 CK(cudaMemcpyAsync(d_chunk_[buf], (const char*)g_.nbr + base * b_e, hbytes, cudaMemcpyHostToDevice, xk));
             } else {
-                transfer_chunk(q, buf, lo, hi, wmode, xk);
+                transfer_chunk(q, buf, lo, hi, wmode, xk, fuse && wmode == 1 ? &d : nullptr);
             }
             CK(cudaGetLastError());
             span(e0, xk, t, wmode == 1 ? PH_GATHER : PH_DMA);
@@ -943,10 +949,12 @@ void Part::expand(uint32_t t, const IterTotals& T) {
         if (wmode == 3) { st.span_link_bytes += hbytes; st.span_payload_bytes += (hi - lo) * b_e; ++st.span_chunks; }
         cudaEvent_t e0 = nullptr;
         CK(cudaStreamWaitEvent(cs_, ready_[buf], 0));
-        e0 = mark(cs_);
-        launch_ondemand(algo_, d, q, d_chunk_[buf], lo, hi, base, cs_);   // On-demand Computing
-        CK(cudaGetLastError());
-        span(e0, cs_, t, PH_OND);
+        if (!(fuse && wmode == 1)) {   // (fused: the gather already computed the chunk)
+            e0 = mark(cs_);
+            launch_ondemand(algo_, d, q, d_chunk_[buf], lo, hi, base, cs_);   // On-demand Computing
+            CK(cudaGetLastError());
+            span(e0, cs_, t, PH_OND);
+        }
         CK(cudaEventRecord(consumed_[buf], cs_));
         if (wmode == 1) ++st.gather_chunks; else ++st.dma_chunks;
         ++done;
@@ -1517,6 +1525,10 @@ void Engine::set_option(int opt, int64_t value) {
         case ASCETIC_OPT_GAP_BRIDGE:
             if (value < 0 || value > 65536) throw Error(ASCETIC_EINVAL, "gap bridge must be in [0, 65536] bytes");
             o_.gap_bridge = (uint32_t)value;
+            break;
+        case ASCETIC_OPT_FUSED_VISIT:
+            if (value < 0 || value > 2) throw Error(ASCETIC_EINVAL, "fused visit must be 0, 1 or 2");
+            o_.fused_visit = (int)value;
             break;
         case ASCETIC_OPT_CHUNK_BUFFERS:
             if (value != 0 && (value < 2 || value > 8)) throw Error(ASCETIC_EINVAL, "chunk buffers must be 0 (auto) or in [2, 8]");

@@ -76,6 +76,7 @@ struct Options {
     double span_density = 0.85;         // span DMA of a window when payload >= this share of its host bytes (0 = off)
     uint64_t span_min_bytes = 64ull << 20;   // ... in iterations with at least this much payload
     double span_max_ratio = 2.0;        // ... whose host span is at most this many times the payload
+    int fused_visit = 1;                // BFS gathered chunks: visit in the gather (1 = small chunks, 2 = all, 0 = off)
     uint32_t gap_bridge = 0;            // gather: also load host holes <= this many bytes between pieces (0 = off;
                                         // measured no gain: C2/C4 A/B, profiles/r02/gather_ab_c4.log)
 };
@@ -150,7 +151,8 @@ class Part {
 
   private:
     void transfer_chunk(const Queues& q, int buf, unsigned long long lo, unsigned long long hi, int mode,
-                        cudaStream_t xs);
+                        cudaStream_t xs,
+                        const DevState* visit = nullptr);
     uint32_t plan_long_runs(const IterTotals& T);   // gather mode: the long runs for the copy engines
     bool plan_span_windows(const IterTotals& T);    // span-DMA mode: the windows' miss-stream positions
     Queues queues(const IterTotals& T) const;

@@ -48,3 +48,15 @@ def test_hbm_bound_step_picks_longest_class_and_dma_only_config_traffic():
                h2d_payload_bytes=144.3e9, time_h2d_busy_s=2.8, iterations=43)
     r = bench.roofline_of([st], 1, 2872.0, 4, 65_608_366, 55.6, 6553.6, "measured", "c3")
     assert r["kernel"] == "transfer" and abs(r["traffic"] - (10.7e9 + 144.3e9)) < 1.0
+
+
+def test_spans_cover_detects_single_span_iterations():
+    # every class with work has event time: the timed steps carry the breakdown
+    full = _step(time_gather_s=0.1, gather_bytes=1e9, time_h2d_busy_s=0.1, h2d_payload_bytes=1e9, iterations=3,
+                 time_classify_s=0.001, ondemand_arcs=1e6, time_ondemand_s=0.01, static_arcs=1e6, time_static_s=0.01)
+    assert bench.spans_cover([full])
+    # a C1-like step (TIMING=1: small iterations ran as one span each): work without per-phase time
+    c1 = _step(gather_bytes=6e6, h2d_payload_bytes=6e6, iterations=7, time_classify_s=0.0002, ondemand_arcs=1e6)
+    assert not bench.spans_cover([full, c1])
+    # no work, no time needed
+    assert bench.spans_cover([_step()])

@@ -108,10 +108,12 @@ def test_c4_full_cc(asc):
 
 @pytest.mark.skipif(os.environ.get("ASCETIC_FULL_C5") != "1", reason="C5 needs ~150 GB host RAM, set ASCETIC_FULL_C5=1")
 def test_c5_one_gpu(asc):
-    """C5 (RMAT-29, 40 GB budget) on one GPU: BFS bit-exact with every record, PR-2 within tolerance."""
+    """C5 (RMAT-29, 40 GB budget) on one GPU: BFS bit-exact with every record, PR within tolerance after
+    ASCETIC_FULL_C5_PR_ITERS iterations (default 2; 43 = the configured PR run, ~8 more oracle minutes)."""
+    pr_iters = int(os.environ.get("ASCETIC_FULL_C5_PR_ITERS", "2"))
     g = gg.config_graph("c5")
     budget = gg.config_budget("c5", g)
-    asc.load_csr(g.off, g.nbr)
+    asc.load_csr(g.off, g.nbr, sorted_rows=True)          # as bench.py (PR: static pull in id slices)
     asc.set_budget(budget)
     p = oracle.placer(g.off, 4, budget)
     stat = oracle.static_prefix(g.n, p.s)
@@ -123,10 +125,14 @@ def test_c5_one_gpu(asc):
     np.testing.assert_array_equal(res, ref.values)
     assert _records(its) == _records(ref.records)
     assert st["h2d_payload_bytes"] == ref.h2d_payload
-    asc.run("pr", 0, 2)
+    asc.run("pr", 0, pr_iters)
     st, its = asc.stats()
     res = asc.get_result().astype(np.float64)
-    ref = oracle.run("pr", g.off, g.nbr, max_iters=2, is_static=stat)
+    ref = oracle.run("pr", g.off, g.nbr, max_iters=pr_iters, is_static=stat)
+    assert st["iterations"] == pr_iters
+    print(f"c5 pr-{pr_iters}: max rel {(np.abs(res - ref.values) / ref.values).max():.3e} "
+          f"L1 {np.abs(res - ref.values).sum():.3e} sum-1 {res.sum() - 1.0:.3e}")
+    assert abs(res.sum() - 1.0) <= 1e-5
     rel = np.abs(res - ref.values) / ref.values
     assert rel.max() <= 1e-5 and np.abs(res - ref.values).sum() <= 1e-6
     assert _records(its) == _records(ref.records)

@@ -550,3 +550,31 @@ def test_span_dma_windows(asc, algo, density):
         np.testing.assert_array_equal(res, ref.values)
     assert st["span_chunks"] > 0 and st["span_link_bytes"] >= st["span_payload_bytes"] > 0
     assert any(i["mode"] == 3 for i in its)
+
+
+@pytest.mark.parametrize("fv", [0, 1, 2])
+@pytest.mark.parametrize("nbuf,xfer", [(0, 0), (3, 0), (2, 1), (4, 1)])
+def test_bfs_fused_visit(asc, fv, nbuf, xfer):
+    """ASCETIC_OPT_FUSED_VISIT: BFS's On-demand Computing done by the gather as the ids land (small-chunk
+    pipeline with fv = 1, every gathered chunk with fv = 2) gives the same levels, records and bytes
+    as the separate on-demand kernel (fv = 0). Small chunk caps give many chunks per level."""
+    g = gg.rmat(13, seed=31)
+    src = int(np.argmax(np.diff(g.off.astype(np.int64))))
+    asc.load_csr(g.off, g.nbr)
+    asc.set_option("fused_visit", fv)
+    asc.set_option("chunk_buffers", nbuf)
+    asc.set_option("xfer_mode", xfer)
+    asc.set_option("chunk_cap", 8192)
+    asc.set_budget(g.csr_bytes // 4)
+    p = oracle.placer(g.off, 4, g.csr_bytes // 4)
+    ref = _oracle("bfs", g, src, p.s)
+    for rep in range(2):
+        asc.run("bfs", src)
+        st, its = asc.stats()
+        np.testing.assert_array_equal(asc.get_result(), ref.values)
+        _check_records(its, ref)
+        assert st["h2d_payload_bytes"] == ref.h2d_payload
+    asc.set_option("fused_visit", 1)
+    asc.set_option("chunk_buffers", 0)
+    asc.set_option("xfer_mode", 0)
+    asc.set_option("chunk_cap", 0)
