@@ -403,12 +403,12 @@ def main():
         budget = gg.config_budget(args.config, g)
 
     asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True, sorted_rows=True)   # generator rows are sorted
+    for kv in args.opt:                               # before set_budget: some shape the On-demand Region
+        k_, v_ = kv.split("=", 1)
+        asc.set_option(k_, int(v_))
     asc.set_budget(budget)
     asc.set_option("xfer_mode", args.xfer)
     asc.set_option("sparse_exchange", args.sparse_exchange)
-    for kv in args.opt:
-        k_, v_ = kv.split("=", 1)
-        asc.set_option(k_, int(v_))
     l2_flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
 
     def step(i):

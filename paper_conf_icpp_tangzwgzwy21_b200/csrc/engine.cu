@@ -150,6 +150,7 @@ Part::~Part() {
         if (xfer_go_[i]) cudaEventDestroy(xfer_go_[i]);
     }
     if (xs2_) { cudaStreamSynchronize(xs2_); cudaStreamDestroy(xs2_); }
+    for (cudaStream_t& x : xs34_) if (x) { cudaStreamSynchronize(x); cudaStreamDestroy(x); x = nullptr; }
     for (int i = 0; i < kMaxBuffers; ++i) {
         if (ready_[i]) cudaEventDestroy(ready_[i]);
         if (consumed_[i]) cudaEventDestroy(consumed_[i]);
@@ -180,6 +181,7 @@ void Part::alloc_vertex_state() {
     CK(cudaStreamCreateWithPriority(&xs_, cudaStreamNonBlocking, hi_pri));
     CK(cudaStreamCreateWithPriority(&ss_, cudaStreamNonBlocking, lo_pri));
     CK(cudaStreamCreateWithPriority(&xs2_, cudaStreamNonBlocking, hi_pri));
+    for (cudaStream_t& x : xs34_) CK(cudaStreamCreateWithPriority(&x, cudaStreamNonBlocking, hi_pri));
     for (int i = 0; i < kMaxBuffers; ++i) {
         CK(cudaEventCreateWithFlags(&ready_[i], cudaEventDisableTiming));
         CK(cudaEventCreateWithFlags(&consumed_[i], cudaEventDisableTiming));
@@ -430,6 +432,7 @@ bool Part::maybe_repartition(const IterTotals& T) {
     const uint64_t s_new = (uint64_t)(std::upper_bound(off, off + (vhi_ - vlo_) + 1, lim) - off) - 1;
     CK(cudaStreamSynchronize(xs_));   // no transfer may still target the old chunk layout
     CK(cudaStreamSynchronize(xs2_));
+    for (cudaStream_t x : xs34_) CK(cudaStreamSynchronize(x));
     static_valid_ = false;            // chunk buffers now overlay the old static tail
     ms_cur_ = ms_new;
     s_cur_ = s_new;
@@ -875,12 +878,13 @@ void Part::expand(uint32_t t, const IterTotals& T) {
     // compute stream at the end. (C1: 0.868 -> 0.871 ms per step, i.e. the chunk pipeline is not
     // host-bound once the per-phase events are off.) Large chunks keep the event pipeline (copy
     // stream at the highest priority, compute on its own stream).
-    const bool alt = mode == 1 && nlint_ == 0 && nbuf_ == 2 && cap_ < (4ull << 20) && prefetched_ == 0;
-    cudaStream_t bst[2] = {xs_, xs2_};
+    // (up to 4 buffers: with BFS's fused visit a buffer's stream holds only gathers, so more buffers of
+    // smaller chunks put more chunk transfers in flight at once)
+    const bool alt = mode == 1 && nlint_ == 0 && nbuf_ <= 4 && cap_ < (4ull << 20) && prefetched_ == 0;
+    cudaStream_t bst[4] = {xs_, xs2_, xs34_[0], xs34_[1]};
     if (alt && nchunks) {
         CK(cudaEventRecord(ev_pipe_, cs_));   // after the previous iteration's compute and this one's memsets
-        CK(cudaStreamWaitEvent(xs_, ev_pipe_, 0));
-        CK(cudaStreamWaitEvent(xs2_, ev_pipe_, 0));
+        for (int b = 0; b < nbuf_; ++b) CK(cudaStreamWaitEvent(bst[b], ev_pipe_, 0));
     }
     // windows: [k cap, (k+1) cap) of the miss stream, or (span mode) the host ranges of cap bytes
     // over the miss stream's span; a dense span window is one DMA of its host bytes and the
@@ -959,8 +963,8 @@ void Part::expand(uint32_t t, const IterTotals& T) {
         if (wmode == 1) ++st.gather_chunks; else ++st.dma_chunks;
         ++done;
     }
-    if (alt && done) {   // the buffers' last users, for whoever uses them next; finalize waits for both
-        for (int b = 0; b < 2; ++b) {
+    if (alt && done) {   // the buffers' last users, for whoever uses them next; finalize waits for all
+        for (int b = 0; b < nbuf_; ++b) {
             CK(cudaEventRecord(consumed_[b], bst[b]));
             CK(cudaStreamWaitEvent(cs_, consumed_[b], 0));
         }
@@ -1164,6 +1168,7 @@ void Part::end() {
     CK(cudaStreamSynchronize(cs_));
     CK(cudaStreamSynchronize(xs_));
     CK(cudaStreamSynchronize(xs2_));
+    for (cudaStream_t x : xs34_) CK(cudaStreamSynchronize(x));
     CK(cudaStreamSynchronize(ss_));
     float ms = 0.f, fill_ms = 0.f;
     CK(cudaEventElapsedTime(&ms, ev_start_, ev_end));

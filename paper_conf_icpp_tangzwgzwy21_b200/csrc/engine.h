@@ -252,6 +252,7 @@ class Part {
     std::vector<uint32_t> lb_, le_;                  // this iteration's long runs, by stream position
     std::vector<unsigned long long> ldst_;
     cudaStream_t xs2_ = nullptr;
+    cudaStream_t xs34_[2] = {nullptr, nullptr};   // small-chunk pipeline: buffers 2 and 3's own streams
     cudaEvent_t ce_done_[kMaxBuffers] = {}, xfer_go_[kMaxBuffers] = {}, ev_long_ = nullptr, ev_pipe_ = nullptr;
     unsigned long long* d_cover_ = nullptr;          // gather: 16-byte units loaded (link bytes / 16)
     static constexpr uint32_t kSpanWinMax = 4096;
