@@ -145,6 +145,7 @@ Part::~Part() {
     if (h_long_flag_) cudaFreeHost(h_long_flag_);
     for (int i = 0; i < 2; ++i) { if (h_lint_[i]) cudaFreeHost(h_lint_[i]); dfree(d_lint_[i]); }
     dfree(d_long_cnt_); dfree(d_cover_); dfree(d_seg_cur_);
+    if (h_cover_) { cudaFreeHost(h_cover_); h_cover_ = nullptr; }
     for (int i = 0; i < kMaxBuffers; ++i) {
         if (ce_done_[i]) cudaEventDestroy(ce_done_[i]);
         if (xfer_go_[i]) cudaEventDestroy(xfer_go_[i]);
@@ -242,6 +243,7 @@ void Part::alloc_vertex_state() {
     dalloc(&d_long_cnt_, 2, &vertex_bytes_);
     for (int i = 0; i < 2; ++i) dalloc(&d_lint_[i], 2ull * kLongMax, &vertex_bytes_);
     dalloc(&d_cover_, 1, &vertex_bytes_);
+    CK(cudaMallocHost(&h_cover_, sizeof(unsigned long long)));
 }
 
 void Part::alloc_algo_state(int algo, bool multi) {
@@ -714,7 +716,9 @@ void Part::classify(uint32_t t) {
     ca.host_runs = h_runs_; ca.host_runs_cap = kRunsHostMax;
     ca.force_host_runs = o_.xfer_mode == 2 ? 1u : 0u;
     ca.dma_min_run_arcs = o_.xfer_mode == 0 ? std::max<uint64_t>(1, o_.dma_min_run / g_.b_e) : ~0ull;
-    cudaEvent_t e0 = mark(cs_, true);   // every iteration: its start marks the iteration's wall time
+    // the iteration's start marks its wall time, with TIMING = 1 only when the previous iteration was
+    // big enough for per-phase spans (a small run's event pairs cost more than its classify kernels)
+    cudaEvent_t e0 = mark(cs_);
     launch_classify(ca, cs_);
     CK(cudaGetLastError());
     span(e0, cs_, t, PH_CLS);
@@ -1165,6 +1169,7 @@ void Part::end() {
     cudaEvent_t ev_end = pool_.get();
     join_static();
     CK(cudaEventRecord(ev_end, cs_));
+    CK(cudaMemcpyAsync(h_cover_, d_cover_, 8, cudaMemcpyDeviceToHost, cs_));   // after every gather (cs_ joins them)
     CK(cudaStreamSynchronize(cs_));
     CK(cudaStreamSynchronize(xs_));
     CK(cudaStreamSynchronize(xs2_));
@@ -1212,11 +1217,12 @@ void Part::end() {
         }
     }
     for (size_t i = 0; i < iters.size(); ++i) {
-        cudaEvent_t a = cls_start[i], b = cls_start[i + 1] ? cls_start[i + 1] : ev_end;
+        // to the next iteration's start (unmarked after a small iteration: no wall time then)
+        cudaEvent_t a = cls_start[i], b = cls_start[i + 1] ? cls_start[i + 1] : (i + 1 < iters.size() ? nullptr : ev_end);
         float w = 0.f;
-        if (a) CK(cudaEventElapsedTime(&w, a, b));
+        if (a && b) CK(cudaEventElapsedTime(&w, a, b));
         iters[i].ms_total = w;
-        if (a && x_first[i]) {
+        if (a && b && x_first[i]) {
             float h = 0.f, span_ms = 0.f, tl = 0.f;
             CK(cudaEventElapsedTime(&h, a, x_first[i]));
             CK(cudaEventElapsedTime(&span_ms, x_first[i], x_last[i]));
@@ -1239,9 +1245,7 @@ void Part::end() {
     st.chunk_buffers = (uint32_t)nbuf_;
     st.static_fraction_used = pl_.R;
     {
-        unsigned long long units = 0;
-        CK(cudaMemcpy(&units, d_cover_, 8, cudaMemcpyDeviceToHost));
-        st.gather_load_bytes = units * 16ull;
+        st.gather_load_bytes = *h_cover_ * 16ull;
     }
     st.time_run_s = ms / 1e3;
     st.time_fill_s = fill_ms / 1e3;

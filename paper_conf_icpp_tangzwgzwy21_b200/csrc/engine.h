@@ -255,6 +255,7 @@ class Part {
     cudaStream_t xs34_[2] = {nullptr, nullptr};   // small-chunk pipeline: buffers 2 and 3's own streams
     cudaEvent_t ce_done_[kMaxBuffers] = {}, xfer_go_[kMaxBuffers] = {}, ev_long_ = nullptr, ev_pipe_ = nullptr;
     unsigned long long* d_cover_ = nullptr;          // gather: 16-byte units loaded (link bytes / 16)
+    unsigned long long* h_cover_ = nullptr;          // its pinned host copy, read after the run's end
     static constexpr uint32_t kSpanWinMax = 4096;
     unsigned long long* h_win_ = nullptr;            // mapped: span windows' first miss-stream positions (nwin + 1)
     uint32_t* h_span_flag_ = nullptr;                // mapped: [0] ready
