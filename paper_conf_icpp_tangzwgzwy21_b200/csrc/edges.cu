@@ -776,6 +776,25 @@ __global__ void __launch_bounds__(256) k_ondemand_bfs(DevState d, const uint32_t
 }
 
 // ------------------------------------------------------------------ zero-copy gather (transfer engine)
+// TMA bulk copy (cp.async.bulk, global -> shared, completion on an mbarrier) of the tile metadata
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(unsigned long long* b, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(b)), "r"(count) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(unsigned long long* b, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, unsigned long long* b) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long* b, uint32_t phase) {
+    uint32_t done = 0;
+    while (!done)
+        asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+                     : "=r"(done) : "r"(smem_u32(b)), "r"(phase) : "memory");
+}
 // host (mapped pinned) 16-byte load, not allocated in L1: read once, and keeping it out of L1
 // leaves the concurrent static-hit kernels their L1 hits on vertex state (C2 static 14.9 -> 12.1 ms,
 // C4-shaped 13.8 -> 11.0 ms; the gather rate is unchanged)
@@ -817,22 +836,36 @@ __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restr
                                                   uint32_t gap_words, unsigned long long* __restrict__ cover,
                                                   DevState d) {
     static_assert(!VISIT || BE == 4, "fused visit: BFS arcs are bare 4-byte ids");
-    // tile metadata staged in shared memory (reading it through L1 instead gathers at the same rate,
-    // but its L1 traffic slows the concurrent static-hit kernels)
-    __shared__ unsigned long long s_pre[kEdgeTile + 1];
-    __shared__ unsigned long long s_src[kEdgeTile + 1];
+    // tile metadata (the miss-queue prefix and host offsets of the tile's vertices) staged in shared
+    // memory by TMA: one elected thread bulk-copies both contiguous slices (16-byte aligned, so from
+    // the even index at or below i0; the queues carry 2 elements of padding) and every thread waits
+    // on the mbarrier. (Reading the metadata through L1 instead gathers at the same rate, but its L1
+    // traffic slows the concurrent static-hit kernels.)
+    __shared__ alignas(16) unsigned long long s_pre_raw[kEdgeTile + 4];
+    __shared__ alignas(16) unsigned long long s_src_raw[kEdgeTile + 4];
+    __shared__ alignas(8) unsigned long long s_bar;
     constexpr unsigned long long AW = BE / 4;                 // words per arc
     const unsigned long long w_off = hoff / 4;                // host word index of arc 0
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const unsigned long long t0 = lo >> kEdgeTileShift, t1 = (hi - 1) >> kEdgeTileShift;
+    if (threadIdx.x == 0) mbar_init(&s_bar, 1);
+    __syncthreads();
+    uint32_t phase = 0;
     for (unsigned long long t = t0 + blockIdx.x; t <= t1; t += gridDim.x) {
         const Tile x = tile_of(q, t, lo, hi);
-        __syncthreads();
-        for (uint32_t k = threadIdx.x; k < x.cnt; k += blockDim.x) {
-            s_pre[k] = __ldg(q.mq_pre + x.i0 + k);
-            s_src[k] = __ldg(q.mq_src + x.i0 + k);
+        const uint32_t sh = x.i0 & 1u;
+        __syncthreads();                                      // the previous tile's readers are done
+        if (threadIdx.x == 0) {
+            const uint32_t bytes = ((x.cnt + sh + 1u) & ~1u) * 8u;
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic reads before async writes
+            mbar_expect_tx(&s_bar, 2u * bytes);
+            bulk_g2s(s_pre_raw, q.mq_pre + (x.i0 - sh), bytes, &s_bar);
+            bulk_g2s(s_src_raw, q.mq_src + (x.i0 - sh), bytes, &s_bar);
         }
-        __syncthreads();
+        mbar_wait(&s_bar, phase);
+        phase ^= 1u;
+        const unsigned long long* s_pre = s_pre_raw + sh;
+        const unsigned long long* s_src = s_src_raw + sh;
         const unsigned long long pw = x.t_lo + (unsigned long long)warp * 256ull;
         if (pw >= x.t_hi) continue;
         const unsigned long long pe = min(x.t_hi, pw + 256ull);

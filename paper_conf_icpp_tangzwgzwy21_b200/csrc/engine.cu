@@ -214,8 +214,8 @@ void Part::alloc_vertex_state() {
     dalloc(&d_hq_hub_, hub_cap_, &vertex_bytes_);
     dalloc(&d_hub_pre_, hub_cap_, &vertex_bytes_);
     dalloc(&d_mq_, own, &vertex_bytes_);
-    dalloc(&d_mq_pre_, own, &vertex_bytes_);
-    dalloc(&d_mq_src_, own, &vertex_bytes_);
+    dalloc(&d_mq_pre_, own + 2, &vertex_bytes_);   // +2: the gather's TMA copies whole 16-byte pairs
+    dalloc(&d_mq_src_, own + 2, &vertex_bytes_);
     dalloc(&d_tile_first_, (m >> kEdgeTileShift) + 2, &vertex_bytes_);
     dalloc(&d_run_b_, own / 2 + 1, &vertex_bytes_);
     dalloc(&d_run_e_, own / 2 + 1, &vertex_bytes_);
