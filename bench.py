@@ -491,7 +491,7 @@ def main():
             torch.cuda.synchronize()
             prof_ms += e0.elapsed_time(e1)
             prof.append(stats())
-        asc.set_option("timing", 1)
+        asc.set_option("timing", int(dict(kv.split("=", 1) for kv in args.opt).get("timing", 1)))
         roofline = roofline_of(prof, args.profile_steps, prof_ms, g.b_e, g.n, h2d_peak, hbm_peak, hbm_src,
                                args.config)
         roofline["phase_spans"] = (f"{args.profile_steps} extra steps with every phase timed (TIMING=2), after "
