@@ -924,9 +924,28 @@ __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restr
                 const uint32_t y = __shfl_up_sync(FULL, incl, o);
                 if (lane >= o) incl += y;
             }
+            const uint32_t units = __shfl_sync(FULL, incl, 31);
+            if (lane == 0 && units) atomicAdd(cover, (unsigned long long)units);   // 16-byte units read
+            // a piece of >= 32 units (512 B) starts at an enumeration slot congruent to its first host
+            // unit mod 32, so each of its warp loads covers exactly one 512-byte host block: random
+            // runs read at 51 GB/s that way vs 49 with 2 KB warp segments at arbitrary offsets
+            // (tools/zc_seg.cu, profiles/r02/zc_seg.log). Up to 31 idle slots per long piece; short
+            // pieces stay packed. Pads of the warp's long pieces are resolved in lane order.
+            {
+                const bool lstart = start && cnt && ((W1 + 3) >> 2) - (W0 >> 2) >= 32ull;
+                uint32_t m = __ballot_sync(FULL, lstart), S = 0, shift = 0;
+                while (m) {
+                    const int l = __ffs(m) - 1;
+                    m &= m - 1u;
+                    const uint32_t e_l = __shfl_sync(FULL, incl - cnt, l) + S;
+                    const uint32_t pad = ((uint32_t)__shfl_sync(FULL, (uint32_t)u0, l) - e_l) & 31u;
+                    S += pad;
+                    if (lane >= l) shift += pad;
+                }
+                incl += shift;
+            }
             const uint32_t excl = incl - cnt;
-            const uint32_t total = __shfl_sync(FULL, incl, 31);
-            if (lane == 0 && total) atomicAdd(cover, (unsigned long long)total);   // 16-byte units read
+            const uint32_t total = __shfl_sync(FULL, incl, 31);   // enumeration slots incl. the pads
             for (uint32_t b = 0; b < total; b += 32u * NG) {
                 // NG groups of 32 units: all loads first (NG x 16 B in flight per lane), then the stores
                 uint4 val[NG];
@@ -946,7 +965,7 @@ __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restr
                     pw1[g] = __shfl_sync(FULL, W1, i);
                     pd0[g] = __shfl_sync(FULL, D0, i);
                     uw[g] = ~0ull;
-                    if (tt < total) {
+                    if (tt < total && tt >= eo) {                 // (below eo: a pad slot, idle)
                         uw[g] = uo + (tt - eo);
                         // the array's first / last unit may stick out of [w_off, w_end): read those
                         // word by word in the store phase, never outside the caller's array
