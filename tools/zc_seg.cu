@@ -4,6 +4,9 @@
 // long run is read as consecutive warp segments whose boundaries sit at arbitrary host offsets.
 //   mode 0: segments of SEG bytes at stream offsets (host boundaries at the run's random alignment)
 //   mode 1: segment boundaries moved to the next 512-byte host block boundary (first segment shorter)
+//   mode 2: segments at stream offsets, but each warp load of a segment covers one 512-byte host block
+//           (the segment's first load starts at its block, lanes before the segment idle): k_gather16
+//           since the long-piece alignment
 // One warp per segment, 16-byte cover loads, NG units in flight per lane, each lane stores its words.
 // nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -o tools/zc_seg tools/zc_seg.cu
 #include <algorithm>
@@ -19,6 +22,7 @@
 #define CK(x) do { cudaError_t e_ = (x); if (e_ != cudaSuccess) { printf("%s: %s\n", #x, cudaGetErrorString(e_)); exit(1);} } while (0)
 
 // segment i: host bytes [ha[i], hb[i]) (16-byte multiples), stream offset d[i]
+template <bool ALIGN>
 __global__ void __launch_bounds__(256) seg_gather(const uint4* __restrict__ host, const uint64_t* __restrict__ ha,
                                                   const uint64_t* __restrict__ hb, const uint64_t* __restrict__ dd,
                                                   uint32_t nseg, uint4* __restrict__ dst) {
@@ -27,17 +31,17 @@ __global__ void __launch_bounds__(256) seg_gather(const uint4* __restrict__ host
     for (uint32_t i = blockIdx.x * 8 + (threadIdx.x >> 5); i < nseg; i += nw) {
         const uint64_t u0 = ha[i] >> 4, u1 = hb[i] >> 4;
         uint4* d = dst + (dd[i] >> 4);
-        for (uint64_t u = u0; u < u1; u += 32 * 6) {
+        for (uint64_t u = ALIGN ? (u0 & ~31ull) : u0; u < u1; u += 32 * 6) {
             uint4 v[6];
 #pragma unroll
             for (int g = 0; g < 6; ++g) {
                 const uint64_t uu = u + 32 * g + lane;
-                if (uu < u1) v[g] = host[uu];
+                if (uu >= u0 && uu < u1) v[g] = host[uu];
             }
 #pragma unroll
             for (int g = 0; g < 6; ++g) {
                 const uint64_t uu = u + 32 * g + lane;
-                if (uu < u1) d[uu - u0] = v[g];
+                if (uu >= u0 && uu < u1) d[uu - u0] = v[g];
             }
         }
     }
@@ -57,8 +61,8 @@ int main() {
     cudaEventCreate(&e0); cudaEventCreate(&e1);
     for (uint64_t run : {(uint64_t)4096, (uint64_t)16384, (uint64_t)65536}) {
         for (uint64_t seg : {(uint64_t)1024, (uint64_t)2048, (uint64_t)4096, (uint64_t)8192, (uint64_t)1 << 30}) {
-            for (int mode : {0, 1}) {
-                if (seg >= run && mode == 1) continue;
+            for (int mode : {0, 1, 2}) {
+                if (seg >= run && mode >= 1) continue;
                 std::mt19937_64 rng(run * 7 + seg);
                 std::vector<uint64_t> ha, hb, dd;
                 uint64_t total = 0;
@@ -82,7 +86,8 @@ int main() {
                 float best = 1e9;
                 for (int r = 0; r < 4; ++r) {
                     cudaEventRecord(e0);
-                    seg_gather<<<64, 256>>>((const uint4*)hd, dha, dhb, ddd, (uint32_t)ha.size(), dst);
+                    if (mode == 2) seg_gather<true><<<64, 256>>>((const uint4*)hd, dha, dhb, ddd, (uint32_t)ha.size(), dst);
+                    else seg_gather<false><<<64, 256>>>((const uint4*)hd, dha, dhb, ddd, (uint32_t)ha.size(), dst);
                     cudaEventRecord(e1);
                     CK(cudaEventSynchronize(e1));
                     float ms; cudaEventElapsedTime(&ms, e0, e1);
@@ -90,7 +95,7 @@ int main() {
                 }
                 CK(cudaGetLastError());
                 printf("run %6llu B  seg %10llu B  %s  %zu segments  %6.2f GB/s\n", (unsigned long long)run,
-                       (unsigned long long)seg, mode ? "512B-aligned ends" : "stream offsets   ", ha.size(),
+                       (unsigned long long)seg, mode == 1 ? "512B-aligned ends      " : mode == 2 ? "stream offs, loads alnd" : "stream offsets         ", ha.size(),
                        total / (best / 1e3) / 1e9);
                 cudaFree(dha); cudaFree(dhb); cudaFree(ddd);
             }
