@@ -938,7 +938,9 @@ __global__ void __launch_bounds__(256) k_gather16(Queues q, const uint4* __restr
                     const int l = __ffs(m) - 1;
                     m &= m - 1u;
                     const uint32_t e_l = __shfl_sync(FULL, incl - cnt, l) + S;
-                    const uint32_t pad = ((uint32_t)__shfl_sync(FULL, (uint32_t)u0, l) - e_l) & 31u;
+                    // (units count from the 16-byte-aligned array base: add its phase in the 512 B block)
+                    const uint32_t blk = (uint32_t)(reinterpret_cast<uintptr_t>(host) >> 4);
+                    const uint32_t pad = ((uint32_t)__shfl_sync(FULL, (uint32_t)u0, l) + blk - e_l) & 31u;
                     S += pad;
                     if (lane >= l) shift += pad;
                 }
