@@ -425,6 +425,7 @@ def main():
     deg64 = np.diff(g.off.astype(np.int64)) if algo == "bfs" else None
     clocks = Clocks(local)
     clocks.start()
+    time.sleep(1.0)                                   # the sampler's own start-up (NVML init) stays out of the steps
     per = []
     total_ms = 0.0
     for k in range(args.steps):
