@@ -333,19 +333,20 @@ def test_eq3_repartition_parity(asc, algo):
     asc.set_option("repartition", 0)
 
 
-@pytest.mark.parametrize("shift", [1, 2, 3])
+@pytest.mark.parametrize("shift", [1, 2, 3, 37, 102])
 @pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pr"])
 def test_gather_unaligned_host_arrays(asc, algo, shift):
-    """The zero-copy gather reads 16-byte-aligned cover units of the host CSR: host arrays that
-    start 4, 8 or 12 bytes past a 16-byte boundary (and chunk windows that cut runs anywhere)
-    must still deliver exactly the missed lists."""
+    """The zero-copy gather reads 16-byte-aligned cover units of the host CSR, and enumerates long
+    pieces by 512-byte host block: host arrays that start 4, 8 or 12 bytes past a 16-byte boundary
+    and at other phases of a 512-byte block (shift in words from a 16-byte boundary), with chunk
+    windows that cut runs anywhere, must still deliver exactly the missed lists."""
     cfg = ALGO_GRAPHS[algo]
     g = gg.rmat(cfg["scale"], seed=11, weights=cfg["weights"])
-    buf = np.zeros(g.nbr.size + 8, dtype=np.uint32)
+    buf = np.zeros(g.nbr.size + 136, dtype=np.uint32)
     base = (-(buf.ctypes.data // 4)) % 4             # word offset of a 16-byte boundary
     nbr = buf[base + shift: base + shift + g.nbr.size]
     nbr[:] = g.nbr
-    assert nbr.ctypes.data % 16 == 4 * shift
+    assert nbr.ctypes.data % 16 == 4 * (shift % 4)
     src = int(np.argmax(np.diff(g.off.astype(np.int64))))
     iters = 6 if algo == "pr" else 0
     for cap in (4096, 200):
