@@ -117,7 +117,7 @@ __device__ __forceinline__ ScanVal sv_load_volatile(const ScanVal* p) {
 // SMs idle, 4 (a tile = 1024 vertices: each warp's serial walk over its words is 8x shorter, which is
 // what bounds a small graph's classify, ~30 us at C1's 8 tiles of 32 words)
 template <int WPW>
-__global__ void __launch_bounds__(kClassifyWarps * 32) k_classify(ClassifyArgs a) {
+__global__ void __launch_bounds__(kClassifyWarps * 32, 4) k_classify(ClassifyArgs a) {
     __shared__ uint32_t s_tile;
     __shared__ ScanVal s_warp[kClassifyWarps];
     __shared__ ScanVal s_excl;

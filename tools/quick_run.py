@@ -49,7 +49,7 @@ def main():
         algo, iters = a.algo, a.iters
     print(f"gen {time.time()-t0:.1f}s n={g.n} m={g.m}", flush=True)
     t0 = time.time()
-    asc.load_csr(g.off, g.nbr, pairs=g.pairs)
+    asc.load_csr(g.off, g.nbr, pairs=g.pairs, symmetric=True, sorted_rows=True)   # as bench.py
     print(f"load {time.time()-t0:.2f}s", flush=True)
     asc.set_budget(budget)
     asc.set_option("xfer_mode", a.xfer)
